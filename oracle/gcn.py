@@ -1,0 +1,166 @@
+"""fp64 CPU oracle of PCGCN's hot path — TEST INFRASTRUCTURE ONLY.
+
+Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s cpu_baseline /
+``--impl reference`` legs may import this module.  It shares no code with the
+CUDA path (``paper_conf_ipps_tianmyd20_b200``) and never imports it.
+
+What it computes is the *plain definition* with no partitioning: PCGCN only
+reorders a commutative/associative sum (§III-A.c, "PCGCN is equal
+to the original GCN and can produce the same numerical results"), so the oracle
+for the partition-centric propagation is the un-partitioned GCN layer.
+
+  Eq. (1):   Z = D̃^-1/2 A D̃^-1/2 X Θ
+  with Kipf's renormalisation Ã = A + I, d̃ = Ã·1 (reading #1 in DESIGN.md:
+  the paper writes A but uses D̃ and cites [1]).
+  Alg. 1, PAPER.md L101-L125 (transform, then propagate, per layer), with
+  ℓ = 2 and ReLU between the layers (Kipf's model, L203; reading #14).
+  Backward: not described by the paper (reading A4); derived by the chain rule,
+  using Âᵀ = Â (symmetric input, reading #2).
+
+Pins (tests/test_oracle.py): dense brute force, K_n, cycles, the P3/P4 path
+worked example (tests/golden/path_graph.txt), stars, the universal eigenvector
+s = sqrt(d̃), disjoint cliques, the empty graph, adjoint identity, finite
+differences and torch-fp64 autograd of the same model, the uniform-logit
+closed form of softmax-CE.
+"""
+from __future__ import annotations
+
+import numpy as np
+import scipy.sparse as sp
+
+
+# ---------------------------------------------------------------------------
+# Graph and normalisation  (Eq. 1; readings #1-#4)
+# ---------------------------------------------------------------------------
+
+def binary_adjacency(n: int, rowptr, col) -> sp.csr_matrix:
+    """A: binary, symmetric, no self-loops, duplicates collapsed (reading #3).
+
+    Row v holds the in-neighbours of v (CSR convention of Fig. 5(a)).
+    Raises ValueError if the input is not symmetric (reading #2)."""
+    rowptr = np.asarray(rowptr, dtype=np.int64)
+    col = np.asarray(col, dtype=np.int64)
+    rows = np.repeat(np.arange(n, dtype=np.int64), np.diff(rowptr))
+    keep = rows != col
+    A = sp.csr_matrix((np.ones(int(keep.sum())), (rows[keep], col[keep])), shape=(n, n))
+    A.sum_duplicates()
+    A.data[:] = 1.0
+    if (A != A.T).nnz != 0:
+        raise ValueError("input graph is not symmetric")
+    A.sort_indices()
+    return A
+
+
+def normalized_adjacency(n: int, rowptr, col, norm: str = "sym"):
+    """Return (Â, d̃, r) with Â = D̃^-1/2 (A+I) D̃^-1/2 (norm='sym') or
+    Â = A + I (norm='none', used by the integer-exact pin), d̃ = 1 + deg and
+    r = d̃^-1/2, all fp64."""
+    A = binary_adjacency(n, rowptr, col)
+    At = (A + sp.identity(n, format="csr")).tocsr()
+    At.sort_indices()
+    dt = np.asarray(At.sum(axis=1)).ravel()
+    r = 1.0 / np.sqrt(dt)
+    if norm == "none":
+        return At, dt, r
+    D = sp.diags(r)
+    Ahat = (D @ At @ D).tocsr()
+    Ahat.sort_indices()
+    return Ahat, dt, r
+
+
+def aggregate(Ahat: sp.csr_matrix, Y: np.ndarray) -> np.ndarray:
+    """Z = Â·Y in fp64 — the propagation h_k = Σ_i f(E_{k,i}, a_i) of Alg. 1
+    (L118-L121) summed over all k at once."""
+    return np.asarray(Ahat @ np.asarray(Y, dtype=np.float64))
+
+
+def aggregate_rows(n: int, rowptr, col, Y: np.ndarray, rows, norm: str = "sym") -> np.ndarray:
+    """Z_i for selected rows only, straight from the edge definition
+    (pin P15 at full scale): Z_i = r_i Σ_{j∈N(i)∪{i}} r_j Y_j."""
+    rowptr = np.asarray(rowptr, dtype=np.int64)
+    col = np.asarray(col, dtype=np.int64)
+    # neighbour sets after dropping self-loops and duplicates, computed lazily
+    cache = {}
+
+    def nbrs(v):
+        if v not in cache:
+            s = col[rowptr[v]:rowptr[v + 1]]
+            cache[v] = np.unique(s[s != v])
+        return cache[v]
+
+    out = np.zeros((len(rows), Y.shape[1]), dtype=np.float64)
+    for t, i in enumerate(rows):
+        nb = np.concatenate([nbrs(i), [i]])
+        if norm == "none":
+            out[t] = np.asarray(Y[nb], dtype=np.float64).sum(axis=0)
+            continue
+        dj = np.array([len(nbrs(j)) + 1 for j in nb], dtype=np.float64)
+        wj = 1.0 / np.sqrt(dj)
+        ri = 1.0 / np.sqrt(len(nbrs(i)) + 1.0)
+        out[t] = ri * (wj[:, None] * np.asarray(Y[nb], dtype=np.float64)).sum(axis=0)
+    return out
+
+
+# ---------------------------------------------------------------------------
+# 2-layer GCN (Alg. 1 with L = 2; Kipf's model)  — forward, loss, backward
+# ---------------------------------------------------------------------------
+
+def forward(Ahat, X, Th0, Th1):
+    """a¹ = X Θ0, P1 = Â a¹, H1 = ReLU(P1), a² = H1 Θ1, L = Â a²  (Alg. 1)."""
+    X = np.asarray(X, dtype=np.float64)
+    P1 = aggregate(Ahat, X @ np.asarray(Th0, dtype=np.float64))
+    H1 = np.maximum(P1, 0.0)
+    L = aggregate(Ahat, H1 @ np.asarray(Th1, dtype=np.float64))
+    return P1, H1, L
+
+
+def softmax_ce(L, labels, train):
+    """loss = (1/|T|) Σ_{i∈T} [logsumexp(L_i) − L_{i,y_i}],
+    dL = (softmax(L) − onehot(y)) ⊙ [i∈T] / |T|   (reading #14)."""
+    L = np.asarray(L, dtype=np.float64)
+    train = np.asarray(train, dtype=bool)
+    m = L.max(axis=1, keepdims=True)
+    e = np.exp(L - m)
+    s = e.sum(axis=1, keepdims=True)
+    lse = (m + np.log(s)).ravel()
+    nT = int(train.sum())
+    idx = np.arange(L.shape[0])
+    loss = float(((lse - L[idx, labels]) * train).sum() / nT)
+    dL = e / s
+    dL[idx, labels] -= 1.0
+    dL *= (train[:, None] / nT)
+    return loss, dL
+
+
+def backward(Ahat, X, Th0, Th1, P1, H1, dL):
+    """Chain rule through Alg. 1 (the paper is silent on the backward, reading A4):
+    G1 = Âᵀ dL = Â dL, ∇Θ1 = H1ᵀ G1, dP1 = (G1 Θ1ᵀ) ⊙ [P1 > 0],
+    G0 = Â dP1, ∇Θ0 = Xᵀ G0."""
+    X = np.asarray(X, dtype=np.float64)
+    G1 = aggregate(Ahat.T.tocsr(), dL)
+    gTh1 = H1.T @ G1
+    dP1 = (G1 @ np.asarray(Th1, dtype=np.float64).T) * (P1 > 0)
+    G0 = aggregate(Ahat.T.tocsr(), dP1)
+    gTh0 = X.T @ G0
+    return dict(G1=G1, dP1=dP1, G0=G0, gTh0=gTh0, gTh1=gTh1)
+
+
+def epoch(Ahat, X, Th0, Th1, labels, train):
+    """One full-batch epoch (fwd + loss + bwd), returning every intermediate."""
+    P1, H1, L = forward(Ahat, X, Th0, Th1)
+    loss, dL = softmax_ce(L, labels, train)
+    g = backward(Ahat, X, Th0, Th1, P1, H1, dL)
+    return dict(P1=P1, H1=H1, L=L, loss=loss, dL=dL, **g)
+
+
+def sgd(Th, g, lr):
+    return np.asarray(Th, dtype=np.float64) - lr * g
+
+
+def adam(Th, g, m, v, t, lr=0.01, b1=0.9, b2=0.999, eps=1e-8):
+    """Adam (Kingma & Ba, Alg. 1) with bias correction; t starts at 1."""
+    m = b1 * m + (1 - b1) * g
+    v = b2 * v + (1 - b2) * g * g
+    mh = m / (1 - b1 ** t)
+    vh = v / (1 - b2 ** t)
+    return Th - lr * mh / (np.sqrt(vh) + eps), m, v

@@ -1,0 +1,98 @@
+"""The BASELINE.json workloads as seeded synthetic recipes.
+
+Input infrastructure only.  Sizes follow the paper's counting convention
+(Table I): nnz(A+I) = 2*m + n.
+  C1 Cora-shaped   n=2,708   m=5,278       1433 -> 16 -> 7    P=8
+  C2 Pubmed-shaped n=19,717  m=44,324      500  -> 16 -> 3    P=32  (nnz 108,365 = Table I)
+  C3 Reddit-shaped n=232,965 m=57,307,946  602  -> 128 -> 41  P=128
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass
+
+import numpy as np
+
+from . import rng as R
+from .graphs import Graph, SBMSpec, sbm
+
+
+@dataclass
+class Workload:
+    name: str
+    spec: SBMSpec
+    f_in: int
+    hidden: int
+    classes: int
+    P: int
+    feat_kind: str  # "binary" | "tfidf" | "normal"
+    feat_seed: int
+    theta_seed: int
+
+
+def _zipf_sizes(n: int, k: int, s: float) -> list:
+    w = (np.arange(1, k + 1, dtype=np.float64)) ** (-s)
+    raw = w / w.sum() * n
+    base = np.floor(raw).astype(np.int64)
+    rem = n - int(base.sum())
+    order = np.argsort(-(raw - base), kind="stable")
+    base[order[:rem]] += 1
+    return [int(x) for x in base]
+
+
+CORA = Workload(
+    "cora", SBMSpec([351, 217, 418, 818, 426, 298, 180], sub_size=64, p_sub=0.60, p_class=0.20,
+                    m_target=5_278, alpha=2.5, cap=125.0, seed=1001),
+    f_in=1433, hidden=16, classes=7, P=8, feat_kind="binary", feat_seed=1002, theta_seed=1003)
+
+PUBMED = Workload(
+    "pubmed", SBMSpec([4_103, 7_739, 7_875], sub_size=128, p_sub=0.60, p_class=0.20,
+                      m_target=44_324, alpha=2.5, cap=110.0, seed=2001),
+    f_in=500, hidden=16, classes=3, P=32, feat_kind="tfidf", feat_seed=2002, theta_seed=2003)
+
+REDDIT = Workload(
+    "reddit", SBMSpec(_zipf_sizes(232_965, 41, 0.8), sub_size=0, p_sub=0.0, p_class=0.75,
+                      m_target=57_307_946, alpha=2.5, cap=200.0, seed=3001),
+    f_in=602, hidden=128, classes=41, P=128, feat_kind="normal", feat_seed=3002, theta_seed=3003)
+
+WORKLOADS = {w.name: w for w in (CORA, PUBMED, REDDIT)}
+
+
+def scaled(w: Workload, frac: float, name: str | None = None) -> Workload:
+    """Same recipe at a fraction of the vertices and edges (test sizes)."""
+    sizes = [max(2, int(round(c * frac))) for c in w.spec.class_sizes]
+    spec = SBMSpec(sizes, w.spec.sub_size, w.spec.p_sub, w.spec.p_class,
+                   max(1, int(round(w.spec.m_target * frac))), w.spec.alpha, w.spec.cap, w.spec.seed)
+    return Workload(name or f"{w.name}@{frac}", spec, w.f_in, w.hidden, w.classes,
+                    max(1, int(round(w.P * frac ** 0.5))), w.feat_kind, w.feat_seed, w.theta_seed)
+
+
+def graph(w: Workload, impl: str = "auto") -> Graph:
+    return sbm(w.spec, impl=impl)
+
+
+def features(w: Workload, n: int) -> np.ndarray:
+    """X [n x f_in] float32, row i belongs to vertex id i."""
+    g = np.random.default_rng([w.feat_seed, 0])
+    if w.feat_kind == "binary":
+        return (g.random((n, w.f_in), dtype=np.float32) < 0.0127).astype(np.float32)
+    if w.feat_kind == "tfidf":
+        idf = g.uniform(0.5, 3.0, size=w.f_in).astype(np.float32)
+        mask = g.random((n, w.f_in), dtype=np.float32) < 0.10
+        return (mask * g.random((n, w.f_in), dtype=np.float32) * idf).astype(np.float32)
+    return g.standard_normal((n, w.f_in), dtype=np.float32)
+
+
+def train_mask(n: int, seed: int) -> np.ndarray:
+    """80% of vertices, chosen by hash(id, seed)."""
+    h = R.draws(R.stream_key(seed, 13), np.arange(n, dtype=np.uint64))
+    return (h % np.uint64(10)) < np.uint64(8)
+
+
+def glorot(fan_in: int, fan_out: int, seed: int, idx: int) -> np.ndarray:
+    a = np.sqrt(6.0 / (fan_in + fan_out))
+    g = np.random.default_rng([seed, idx])
+    return g.uniform(-a, a, size=(fan_in, fan_out)).astype(np.float32)
+
+
+def thetas(w: Workload):
+    return glorot(w.f_in, w.hidden, w.theta_seed, 0), glorot(w.hidden, w.classes, w.theta_seed, 1)
