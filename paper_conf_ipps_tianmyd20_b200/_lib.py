@@ -1,0 +1,227 @@
+"""Thin ctypes binding of libpcgcn.so (include/pcgcn.h) — argument marshalling only.
+
+Every compute step runs in the library's sm_100a kernels; there is no CPU
+fallback.  Importing this module fails loudly if the shared library is missing.
+Device buffers are torch CUDA tensors (PyTorch is used for device memory,
+streams and process groups only).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libpcgcn.so")
+
+if not os.path.exists(LIB_PATH):
+    raise ImportError(f"{LIB_PATH} is missing: build it with `python -m paper_conf_ipps_tianmyd20_b200.build`"
+                      " (no CPU fallback exists)")
+lib = ctypes.CDLL(LIB_PATH)
+
+c_i32, c_i64, c_f32, c_u32, c_vp = ctypes.c_int32, ctypes.c_int64, ctypes.c_float, ctypes.c_uint32, ctypes.c_void_p
+
+# status codes
+OK, EINVAL, ENOTSYM, ECUDA, ENOMEM, ENCCL, EUNSUP = range(7)
+NORM_SYM, NORM_NONE = 0, 1
+DENSE_TF32X2, DENSE_FP32_SIMT = 0, 1
+IN_PRESCALED, RELU, MASK_OUT, OUT_PRESCALED = 1, 2, 4, 8
+X_NAMES = ["part", "perm", "pstart", "r", "blk_k", "blk_i", "blk_nnz", "blk_dense", "sp_rowptr", "sp_col",
+           "rt_row0", "rt_nrows", "rt_cptr", "ch_col0", "bits", "zd_index", "sweeps"]
+X_DTYPES = [np.int32, np.int32, np.int64, np.float32, np.int32, np.int32, np.int64, np.uint8, np.int64,
+            np.int32, np.int32, np.int32, np.int64, np.int32, np.uint32, np.int32, np.int32]
+CE_WORK_FLOATS = 1024
+
+
+class Csr(ctypes.Structure):
+    _fields_ = [("n", c_i64), ("nnz", c_i64), ("rowptr", c_vp), ("col", c_vp)]
+
+
+class Opts(ctypes.Structure):
+    _fields_ = [("norm", c_i32), ("dense_prec", c_i32), ("f_max", c_i32), ("lp_sweeps", c_i32),
+                ("part", c_vp), ("build_device", c_i32), ("rank", c_i32), ("world", c_i32)]
+
+
+class Stats(ctypes.Structure):
+    _fields_ = [("n", c_i64), ("nnz", c_i64), ("P", c_i32), ("lp_sweeps", c_i32), ("clusters", c_i64),
+                ("blocks_nonempty", c_i64), ("blocks_dense", c_i64), ("nnz_sparse", c_i64),
+                ("nnz_dense", c_i64), ("intra_edges", c_i64), ("row_tiles", c_i64), ("chunks", c_i64),
+                ("row_lo", c_i64), ("row_hi", c_i64), ("shard_nnz_sparse", c_i64), ("shard_chunks", c_i64),
+                ("theta", ctypes.c_double), ("partition_ms", ctypes.c_double), ("plan_ms", ctypes.c_double),
+                ("device_bytes", c_i64)]
+
+    def as_dict(self):
+        return {k: getattr(self, k) for k, _ in self._fields_}
+
+
+def _sig(name, res, *args):
+    f = getattr(lib, name)
+    f.restype = res
+    f.argtypes = list(args)
+    return f
+
+
+_sig("pcgcn_opts_default", None, ctypes.POINTER(Opts))
+_sig("pcgcn_plan", c_i32, ctypes.POINTER(Csr), c_i32, c_f32, ctypes.POINTER(Opts), ctypes.POINTER(c_vp))
+_sig("pcgcn_destroy", None, c_vp)
+_sig("pcgcn_forward", c_i32, c_vp, c_vp, c_i64, c_vp, c_i64, c_i32, c_u32, c_vp, c_vp)
+_sig("pcgcn_backward", c_i32, c_vp, c_vp, c_i64, c_vp, c_i64, c_i32, c_u32, c_vp)
+_sig("pcgcn_gemm_xw", c_i32, c_vp, c_i64, c_vp, c_i64, c_vp, c_vp, c_i64, c_i64, c_i32, c_i32, c_vp)
+_sig("pcgcn_gemm_xtg_work_floats", c_i64, c_i64, c_i32, c_i32)
+_sig("pcgcn_gemm_xtg", c_i32, c_vp, c_i64, c_vp, c_i64, c_vp, c_i64, c_i32, c_i32, c_vp, c_vp)
+_sig("pcgcn_gemm_dwt", c_i32, c_vp, c_i64, c_vp, c_vp, c_vp, c_vp, c_i64, c_i64, c_i32, c_i32, c_vp)
+_sig("pcgcn_softmax_ce", c_i32, c_vp, c_i64, c_vp, c_vp, c_i64, c_i32, c_f32, c_vp, c_vp, c_vp, c_vp, c_vp)
+_sig("pcgcn_adam", c_i32, c_vp, c_vp, c_vp, c_vp, c_i64, c_f32, c_f32, c_f32, c_f32, c_vp, c_vp)
+_sig("pcgcn_sgd", c_i32, c_vp, c_vp, c_i64, c_f32, c_vp)
+_sig("pcgcn_plan_perm", c_i32, c_vp, c_vp)
+_sig("pcgcn_plan_stats", c_i32, c_vp, ctypes.POINTER(Stats))
+_sig("pcgcn_plan_rowscale", c_vp, c_vp)
+_sig("pcgcn_plan_export_bytes", c_i64, c_vp, c_i32)
+_sig("pcgcn_plan_export", c_i32, c_vp, c_i32, c_vp, c_i64)
+_sig("pcgcn_calibrate", c_i32, c_i32, c_i32, c_f32, ctypes.POINTER(c_f32), ctypes.POINTER(c_f32),
+     ctypes.POINTER(c_f32))
+_sig("pcgcn_last_error", ctypes.c_char_p)
+_sig("pcgcn_abi_version", c_i32)
+
+
+class PcgcnError(RuntimeError):
+    def __init__(self, code, where):
+        msg = lib.pcgcn_last_error().decode(errors="replace")
+        super().__init__(f"{where} failed with status {code}: {msg}")
+        self.code = code
+
+
+def check(code, where):
+    if code != OK:
+        raise PcgcnError(code, where)
+
+
+def _ptr(t):
+    """device pointer of a torch tensor (or None)."""
+    return None if t is None else ctypes.c_void_p(t.data_ptr())
+
+
+def _stream(stream):
+    if stream is None:
+        import torch
+        stream = torch.cuda.current_stream()
+    return ctypes.c_void_p(stream.cuda_stream if hasattr(stream, "cuda_stream") else int(stream))
+
+
+class Plan:
+    """pcgcn_plan / pcgcn_forward / pcgcn_backward / pcgcn_destroy."""
+
+    def __init__(self, n, rowptr, col, P, theta, *, norm=NORM_SYM, dense_prec=DENSE_TF32X2, f_max=128,
+                 lp_sweeps=10, part=None, build_device=True, rank=0, world=1):
+        self._h = None
+        self.n = int(n)
+        rowptr = np.ascontiguousarray(rowptr, dtype=np.int64)
+        col = np.ascontiguousarray(col, dtype=np.int32)
+        A = Csr(self.n, int(rowptr[-1]), rowptr.ctypes.data, col.ctypes.data)
+        o = Opts()
+        lib.pcgcn_opts_default(ctypes.byref(o))
+        o.norm, o.dense_prec, o.f_max, o.lp_sweeps = norm, dense_prec, f_max, lp_sweeps
+        if part is not None:
+            part = np.ascontiguousarray(part, dtype=np.int32)
+            o.part = part.ctypes.data
+        o.build_device = 1 if build_device else 0
+        o.rank, o.world = rank, world
+        h = c_vp()
+        check(lib.pcgcn_plan(ctypes.byref(A), int(P), float(theta), ctypes.byref(o), ctypes.byref(h)), "pcgcn_plan")
+        self._h = h
+        self.P = int(P)
+        self.f_max = f_max
+        st = self.stats()
+        self.row_lo, self.row_hi = st["row_lo"], st["row_hi"]
+
+    def __del__(self):
+        self.destroy()
+
+    def destroy(self):
+        if getattr(self, "_h", None):
+            lib.pcgcn_destroy(self._h)
+            self._h = None
+
+    def stats(self):
+        s = Stats()
+        check(lib.pcgcn_plan_stats(self._h, ctypes.byref(s)), "pcgcn_plan_stats")
+        return s.as_dict()
+
+    def perm(self):
+        out = np.empty(self.n, dtype=np.int32)
+        check(lib.pcgcn_plan_perm(self._h, out.ctypes.data), "pcgcn_plan_perm")
+        return out
+
+    def export(self, name):
+        w = X_NAMES.index(name)
+        nbytes = lib.pcgcn_plan_export_bytes(self._h, w)
+        out = np.empty(nbytes // np.dtype(X_DTYPES[w]).itemsize, dtype=X_DTYPES[w])
+        if nbytes:
+            check(lib.pcgcn_plan_export(self._h, w, out.ctypes.data, nbytes), "pcgcn_plan_export")
+        return out
+
+    def rowscale_ptr(self):
+        return lib.pcgcn_plan_rowscale(self._h)
+
+    def forward(self, Y, Z, F=None, flags=0, mask=None, stream=None):
+        F = Y.shape[1] if F is None else F
+        check(lib.pcgcn_forward(self._h, _ptr(Y), Y.stride(0), _ptr(Z), Z.stride(0), F, flags, _ptr(mask),
+                                _stream(stream)), "pcgcn_forward")
+
+    def backward(self, dZ, dY, F=None, flags=0, stream=None):
+        F = dZ.shape[1] if F is None else F
+        check(lib.pcgcn_backward(self._h, _ptr(dZ), dZ.stride(0), _ptr(dY), dY.stride(0), F, flags,
+                                 _stream(stream)), "pcgcn_backward")
+
+
+def gemm_xw(X, W, s, Y, M=None, K=None, N=None, stream=None):
+    M = X.shape[0] if M is None else M
+    K = X.shape[1] if K is None else K
+    N = W.shape[1] if N is None else N
+    check(lib.pcgcn_gemm_xw(_ptr(X), X.stride(0), _ptr(W), W.stride(0), s, _ptr(Y), Y.stride(0), M, K, N,
+                            _stream(stream)), "pcgcn_gemm_xw")
+
+
+def gemm_xtg_work_floats(M, K, N):
+    return int(lib.pcgcn_gemm_xtg_work_floats(M, K, N))
+
+
+def gemm_xtg(X, D, G, work, M=None, K=None, N=None, stream=None):
+    M = X.shape[0] if M is None else M
+    K = X.shape[1] if K is None else K
+    N = G.shape[1] if N is None else N
+    check(lib.pcgcn_gemm_xtg(_ptr(X), X.stride(0), _ptr(D), D.stride(0), _ptr(G), M, K, N, _ptr(work),
+                             _stream(stream)), "pcgcn_gemm_xtg")
+
+
+def gemm_dwt(D, W, mask, s, O, M=None, N=None, K=None, stream=None):
+    M = D.shape[0] if M is None else M
+    K = W.shape[0] if K is None else K
+    N = W.shape[1] if N is None else N
+    check(lib.pcgcn_gemm_dwt(_ptr(D), D.stride(0), _ptr(W), _ptr(mask), s, _ptr(O), O.stride(0), M, N, K,
+                             _stream(stream)), "pcgcn_gemm_dwt")
+
+
+def softmax_ce(L, labels, train, inv_nT, s, dL, loss, work, M=None, C=None, stream=None):
+    M = L.shape[0] if M is None else M
+    C = L.shape[1] if C is None else C
+    assert dL.stride(0) == L.stride(0)
+    check(lib.pcgcn_softmax_ce(_ptr(L), L.stride(0), _ptr(labels), _ptr(train), M, C, float(inv_nT), s,
+                               _ptr(dL), _ptr(loss), _ptr(work), _stream(stream)), "pcgcn_softmax_ce")
+
+
+def adam(theta, grad, m, v, lr, step, b1=0.9, b2=0.999, eps=1e-8, stream=None):
+    check(lib.pcgcn_adam(_ptr(theta), _ptr(grad), _ptr(m), _ptr(v), theta.numel(), lr, b1, b2, eps, _ptr(step),
+                         _stream(stream)), "pcgcn_adam")
+
+
+def sgd(theta, grad, lr, stream=None):
+    check(lib.pcgcn_sgd(_ptr(theta), _ptr(grad), theta.numel(), lr, _stream(stream)), "pcgcn_sgd")
+
+
+def calibrate(F, block_rows=2048, p_ref=0.05):
+    th, tf, ts = c_f32(), c_f32(), c_f32()
+    check(lib.pcgcn_calibrate(F, block_rows, p_ref, ctypes.byref(th), ctypes.byref(tf), ctypes.byref(ts)),
+          "pcgcn_calibrate")
+    return th.value, tf.value, ts.value

@@ -1,0 +1,109 @@
+// θ calibration (row a3): the paper's procedure of L161 (§III-B.c) on the
+// B200 itself.  "We profile the runtime of full and selective modes for a
+// block of sparsity p, denoted by T_f and T_s ... θ = T_f·p/T_s."
+//
+// Synthetic workload: a bipartite random block between two vertex blocks of
+// `block_rows` vertices each, edge density p_ref (seeded splitmix64, so the
+// block is the same on every call), plus the n self-loops of Ã.  The plan is
+// built twice with an explicit partition override (θ >= 1 -> every block
+// selective, θ = 0 -> every block full) and each mode's forward at width F is
+// timed with CUDA events (median of 15 after 3 warm-ups).
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdint>
+#include <vector>
+
+#include "plan_internal.h"
+
+namespace {
+
+uint64_t mix64(uint64_t x) {
+  x ^= x >> 30; x *= 0xBF58476D1CE4E5B9ull;
+  x ^= x >> 27; x *= 0x94D049BB133111EBull;
+  x ^= x >> 31;
+  return x;
+}
+
+float time_forward(pcgcn_plan_t p, const float* Y, float* Z, int F, int64_t ld, cudaStream_t s) {
+  cudaEvent_t a, b;
+  cudaEventCreate(&a);
+  cudaEventCreate(&b);
+  std::vector<float> ts;
+  for (int it = 0; it < 18; ++it) {
+    cudaEventRecord(a, s);
+    pcgcn_forward(p, Y, ld, Z, ld, F, PCGCN_IN_PRESCALED, nullptr, s);
+    cudaEventRecord(b, s);
+    cudaEventSynchronize(b);
+    float ms = 0;
+    cudaEventElapsedTime(&ms, a, b);
+    if (it >= 3) ts.push_back(ms);
+  }
+  cudaEventDestroy(a);
+  cudaEventDestroy(b);
+  std::sort(ts.begin(), ts.end());
+  return ts[ts.size() / 2];
+}
+
+}  // namespace
+
+extern "C" pcgcn_status pcgcn_calibrate(int32_t F, int32_t block_rows, float p_ref, float* theta_out,
+                                        float* t_full_ms, float* t_sel_ms) {
+  if (F < 1 || F > 256 || block_rows < 32 || !(p_ref > 0.f && p_ref <= 1.f) || !theta_out) {
+    pcgcn::set_error("calibrate: bad arguments");
+    return PCGCN_EINVAL;
+  }
+  const int64_t B = block_rows, n = 2 * B;
+  // symmetric bipartite block: edge (u in V0, v in V1) present iff hash < p
+  const uint64_t thr = uint64_t(double(p_ref) * 18446744073709551615.0);
+  std::vector<std::vector<int32_t>> adj(n);
+  for (int64_t u = 0; u < B; ++u)
+    for (int64_t v = 0; v < B; ++v)
+      if (mix64(0x5eedull * 0x9E3779B97F4A7C15ull + uint64_t(u * B + v)) < thr) {
+        adj[u].push_back(int32_t(B + v));
+        adj[B + v].push_back(int32_t(u));
+      }
+  std::vector<int64_t> rowptr(n + 1, 0);
+  for (int64_t v = 0; v < n; ++v) rowptr[v + 1] = rowptr[v] + int64_t(adj[v].size());
+  std::vector<int32_t> col(rowptr[n]);
+  for (int64_t v = 0; v < n; ++v) std::copy(adj[v].begin(), adj[v].end(), col.begin() + rowptr[v]);
+  std::vector<int32_t> part(n);
+  for (int64_t v = 0; v < n; ++v) part[v] = v < B ? 0 : 1;
+  pcgcn_csr A{n, rowptr[n], rowptr.data(), col.data()};
+  pcgcn_opts o;
+  pcgcn_opts_default(&o);
+  o.part = part.data();
+  o.f_max = F;
+  pcgcn_plan_t ps = nullptr, pf = nullptr;
+  pcgcn_status st = pcgcn_plan(&A, 2, 2.0f, &o, &ps);
+  if (st != PCGCN_OK) return st;
+  st = pcgcn_plan(&A, 2, 0.0f, &o, &pf);
+  if (st != PCGCN_OK) { pcgcn_destroy(ps); return st; }
+  const int64_t ld = (F + 3) / 4 * 4;
+  float *Y = nullptr, *Z = nullptr;
+  cudaStream_t s = nullptr;
+  if (cudaMalloc(&Y, sizeof(float) * n * ld) != cudaSuccess || cudaMalloc(&Z, sizeof(float) * n * ld) != cudaSuccess ||
+      cudaStreamCreate(&s) != cudaSuccess) {
+    pcgcn_destroy(ps);
+    pcgcn_destroy(pf);
+    pcgcn::set_error("calibrate: allocation failed");
+    return PCGCN_ENOMEM;
+  }
+  cudaMemsetAsync(Y, 0, sizeof(float) * n * ld, s);
+  float ts = time_forward(ps, Y, Z, F, ld, s);
+  float tf = time_forward(pf, Y, Z, F, ld, s);
+  cudaError_t e = cudaStreamSynchronize(s);
+  cudaFree(Y);
+  cudaFree(Z);
+  cudaStreamDestroy(s);
+  pcgcn_destroy(ps);
+  pcgcn_destroy(pf);
+  if (e != cudaSuccess) {
+    pcgcn::set_error(std::string("calibrate: ") + cudaGetErrorString(e));
+    return PCGCN_ECUDA;
+  }
+  *theta_out = tf * p_ref / ts;  // θ = T_f·p/T_s (L161)
+  if (t_full_ms) *t_full_ms = tf;
+  if (t_sel_ms) *t_sel_ms = ts;
+  return PCGCN_OK;
+}

@@ -1,0 +1,156 @@
+// Feature-transform GEMMs of the 2-layer GCN step (Alg. 1 a^l = h^{l-1} w^l,
+// L114; the paper runs these as TF MatMul / cuBLAS, L203) and their backward
+// counterparts (the paper is silent on the backward, reading A4).
+//
+// Round-1 implementation: fp32 CUDA-core tiles (64x64 output tile per CTA,
+// 4x4 register micro-tiles, BK=16 smem double-staging) with fused epilogues:
+//   xw : Y = diag(s)·(X·W)                      (a4, a7: source prescaling)
+//   dwt: O = diag(s)·((D·Wᵀ) ⊙ mask)            (a11: ReLU' via the bit mask)
+//   xtg: G = Xᵀ·D, split over M into fixed slices + fixed-order reduction
+//        (a11, a13: deterministic, no atomics)
+// The tcgen05 3xTF32 path for xw/xtg is the next step.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdint>
+
+#include "kernels.h"
+
+namespace pcgcn {
+namespace {
+
+constexpr int BM = 64, BN = 64, BK = 16;
+
+// C[m][n] = Σ_k opA(m,k)·opB(k,n) over k in [k0,k1)
+//   opA(m,k) = AT ? A[k*lda+m] : A[m*lda+k]
+//   opB(k,n) = BT ? B[n*ldb+k] : B[k*ldb+n]
+// Epilogue: optional row scale s[m], optional mask bits (row stride mw), store
+// to C[m*ldc+n] (+ z*zstride for split partials).
+template <bool AT, bool BT>
+__global__ void __launch_bounds__(256) gemm_simt_kernel(
+    const float* __restrict__ A, int64_t lda, const float* __restrict__ B, int64_t ldb,
+    float* __restrict__ C, int64_t ldc, int64_t M, int N, int64_t K, int64_t kslice,
+    const float* __restrict__ s, const uint32_t* __restrict__ mask, int mw, int64_t zstride) {
+  __shared__ float As[BK][BM + 4];
+  __shared__ float Bs[BK][BN + 4];
+  const int tid = threadIdx.x;
+  const int tx = tid % 16, ty = tid / 16;
+  const int64_t m0 = int64_t(blockIdx.x) * BM;
+  const int n0 = blockIdx.y * BN;
+  const int64_t kb = int64_t(blockIdx.z) * kslice;
+  const int64_t ke = (kb + kslice < K) ? kb + kslice : K;
+  float acc[4][4] = {};
+  for (int64_t k0 = kb; k0 < ke; k0 += BK) {
+    // load A tile (BM x BK) -> As[k][m]
+#pragma unroll
+    for (int t = 0; t < (BM * BK) / 256; ++t) {
+      int e = tid + t * 256;
+      int mm, kk;
+      if (AT) { mm = e % BM; kk = e / BM; } else { kk = e % BK; mm = e / BK; }
+      int64_t gm = m0 + mm, gk = k0 + kk;
+      float v = 0.f;
+      if (gm < M && gk < ke) v = AT ? A[gk * lda + gm] : A[gm * lda + gk];
+      As[kk][mm] = v;
+    }
+#pragma unroll
+    for (int t = 0; t < (BN * BK) / 256; ++t) {
+      int e = tid + t * 256;
+      int nn, kk;
+      if (BT) { kk = e % BK; nn = e / BK; } else { nn = e % BN; kk = e / BN; }
+      int gn = n0 + nn;
+      int64_t gk = k0 + kk;
+      float v = 0.f;
+      if (gn < N && gk < ke) v = BT ? B[int64_t(gn) * ldb + gk] : B[gk * ldb + gn];
+      Bs[kk][nn] = v;
+    }
+    __syncthreads();
+#pragma unroll
+    for (int kk = 0; kk < BK; ++kk) {
+      float a[4], b[4];
+#pragma unroll
+      for (int i = 0; i < 4; ++i) a[i] = As[kk][ty + 16 * i];
+#pragma unroll
+      for (int j = 0; j < 4; ++j) b[j] = Bs[kk][tx + 16 * j];
+#pragma unroll
+      for (int i = 0; i < 4; ++i)
+#pragma unroll
+        for (int j = 0; j < 4; ++j) acc[i][j] = fmaf(a[i], b[j], acc[i][j]);
+    }
+    __syncthreads();
+  }
+  float* Cz = C + int64_t(blockIdx.z) * zstride;
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    int64_t gm = m0 + ty + 16 * i;
+    if (gm >= M) continue;
+    float sc = s ? s[gm] : 1.f;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      int gn = n0 + tx + 16 * j;
+      if (gn >= N) continue;
+      float v = acc[i][j];
+      if (mask) v = ((mask[gm * mw + (gn >> 5)] >> (gn & 31)) & 1u) ? v : 0.f;
+      Cz[gm * ldc + gn] = v * sc;
+    }
+  }
+}
+
+__global__ void reduce_slices_kernel(const float* __restrict__ part, int nslices, int64_t count,
+                                     float* __restrict__ out) {
+  for (int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < count;
+       i += int64_t(gridDim.x) * blockDim.x) {
+    float a = 0.f;
+    for (int z = 0; z < nslices; ++z) a += part[int64_t(z) * count + i];
+    out[i] = a;
+  }
+}
+
+// zero the pad columns [N, ldc) of the first M rows (outputs' pad must be 0)
+__global__ void zero_pad_kernel(float* C, int64_t ldc, int64_t M, int N) {
+  const int w = int(ldc) - N;
+  if (w <= 0) return;
+  for (int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < M * w;
+       i += int64_t(gridDim.x) * blockDim.x)
+    C[(i / w) * ldc + N + (i % w)] = 0.f;
+}
+
+int xtg_slices(int64_t M) { return int(std::min<int64_t>(296, std::max<int64_t>(1, (M + 1023) / 1024))); }
+
+}  // namespace
+
+cudaError_t launch_gemm_xw(const float* X, int64_t ldx, const float* W, int64_t ldw, const float* s,
+                           float* Y, int64_t ldy, int64_t M, int K, int N, cudaStream_t st) {
+  dim3 grid(unsigned((M + BM - 1) / BM), unsigned((N + BN - 1) / BN), 1);
+  gemm_simt_kernel<false, false><<<grid, 256, 0, st>>>(X, ldx, W, ldw, Y, ldy, M, N, K, K, s,
+                                                       nullptr, 0, 0);
+  if (ldy > N) zero_pad_kernel<<<256, 256, 0, st>>>(Y, ldy, M, N);
+  return cudaGetLastError();
+}
+
+int64_t gemm_xtg_work_floats(int64_t M, int K, int N) { return int64_t(xtg_slices(M)) * K * N; }
+
+cudaError_t launch_gemm_xtg(const float* X, int64_t ldx, const float* D, int64_t ldd, float* G,
+                            int64_t M, int K, int N, float* work, cudaStream_t st) {
+  // G[K x N] = Xᵀ D : output rows = K (A = X transposed), reduction over M
+  const int ns = xtg_slices(M);
+  int64_t kslice = ((M + ns - 1) / ns + BK - 1) / BK * BK;
+  dim3 grid(unsigned((K + BM - 1) / BM), unsigned((N + BN - 1) / BN), unsigned(ns));
+  gemm_simt_kernel<true, false><<<grid, 256, 0, st>>>(X, ldx, D, ldd, work, N, K, N, M, kslice,
+                                                      nullptr, nullptr, 0, int64_t(K) * N);
+  reduce_slices_kernel<<<std::max<int64_t>(1, std::min<int64_t>(1024, (int64_t(K) * N + 255) / 256)), 256, 0, st>>>(
+      work, ns, int64_t(K) * N, G);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_gemm_dwt(const float* D, int64_t ldd, const float* W, const uint32_t* mask,
+                            const float* s, float* O, int64_t ldo, int64_t M, int N, int K,
+                            cudaStream_t st) {
+  // O[M x K] = D[M x N] · Wᵀ  with W [K x N] row-major: opB(n, k) = W[k*N + n]
+  dim3 grid(unsigned((M + BM - 1) / BM), unsigned((K + BN - 1) / BN), 1);
+  gemm_simt_kernel<false, true><<<grid, 256, 0, st>>>(D, ldd, W, N, O, ldo, M, K, N, N, s, mask,
+                                                      (K + 31) / 32, 0);
+  if (ldo > K) zero_pad_kernel<<<256, 256, 0, st>>>(O, ldo, M, K);
+  return cudaGetLastError();
+}
+
+}  // namespace pcgcn

@@ -1,0 +1,72 @@
+// Launchers of the sm_100a kernels (internal; the ABI is include/pcgcn.h).
+#pragma once
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+namespace pcgcn {
+
+// ---- aggregation (sparse.cu) ----
+struct AggArgs {
+  const float* Y;            // prescaled input (all n rows), ld ldy
+  int64_t ldy;
+  float* Z;                  // shard-local output rows, ld ldz
+  int64_t ldz;
+  uint32_t* mask;            // shard-local [rows x ceil(F/32)] or nullptr
+  const int64_t* rowptr;     // shard-local merged selective CSR
+  const int32_t* col;
+  const float* r;            // [n] plan order
+  int64_t row_lo;            // first plan row of the shard
+  int64_t rows;              // rows in the shard
+  const int32_t* zd_index;   // shard-local, or nullptr if no dense tiles
+  const float* zd;           // dense partial sums, ld ldzd
+  int64_t ldzd;
+  int F;
+  bool relu, out_prescaled;
+};
+cudaError_t launch_sparse_agg(const AggArgs& a, cudaStream_t s);
+
+// diag(r)·Y (optional) and the tf32 hi/lo split of the result (optional)
+cudaError_t launch_prescale_split(const float* Y, int64_t ldy, const float* r, int64_t n, int F,
+                                  float* ypre, int64_t ldpre, float* yhi, float* ylo, int64_t ldhl,
+                                  cudaStream_t s);
+
+// ---- dense-mode tcgen05 tile contraction (dense_tc.cu) ----
+struct DenseArgs {
+  const float* yhi;          // [n x ldhl] tf32 hi part of the prescaled input
+  const float* ylo;          // [n x ldhl] lo part
+  int64_t n, ldhl;
+  const int32_t* rt_row0;    // shard row tiles
+  const int32_t* rt_nrows;
+  const int64_t* rt_cptr;
+  const int32_t* ch_col0;
+  const uint32_t* bits;
+  int64_t nrt;
+  float* zd;                 // [nrt*128 x ldzd]
+  int64_t ldzd;
+  int npad;                  // UMMA N (multiple of 16, >= F)
+};
+cudaError_t launch_dense_tc(const DenseArgs& a, cudaStream_t s);
+// CUDA-core fp32 full mode (§IV-C) on the prescaled input y
+cudaError_t launch_dense_simt_y(const DenseArgs& a, const float* y, int64_t ldy, int F,
+                                cudaStream_t s);
+
+// ---- GEMMs (gemm.cu) ----
+cudaError_t launch_gemm_xw(const float* X, int64_t ldx, const float* W, int64_t ldw, const float* s,
+                           float* Y, int64_t ldy, int64_t M, int K, int N, cudaStream_t st);
+int64_t gemm_xtg_work_floats(int64_t M, int K, int N);
+cudaError_t launch_gemm_xtg(const float* X, int64_t ldx, const float* D, int64_t ldd, float* G,
+                            int64_t M, int K, int N, float* work, cudaStream_t st);
+cudaError_t launch_gemm_dwt(const float* D, int64_t ldd, const float* W, const uint32_t* mask,
+                            const float* s, float* O, int64_t ldo, int64_t M, int N, int K,
+                            cudaStream_t st);
+
+// ---- loss / optimiser (loss_opt.cu) ----
+cudaError_t launch_softmax_ce(const float* L, int64_t ld, const int32_t* labels,
+                              const uint8_t* train, int64_t M, int C, float inv_nT, const float* s,
+                              float* dL, float* loss, float* work, cudaStream_t st);
+cudaError_t launch_adam(float* th, const float* g, float* m, float* v, int64_t n, float lr, float b1,
+                        float b2, float eps, int32_t* step, cudaStream_t st);
+cudaError_t launch_sgd(float* th, const float* g, int64_t n, float lr, cudaStream_t st);
+
+}  // namespace pcgcn

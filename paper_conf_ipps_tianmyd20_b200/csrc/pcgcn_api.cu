@@ -1,0 +1,379 @@
+// C ABI of libpcgcn.so (include/pcgcn.h): plan lifetime, device upload,
+// forward/backward orchestration (prescale/split -> full-mode tiles ->
+// selective rows with the combine epilogue), and the GEMM / loss / optimiser
+// entry points.  No CPU fallback: every device entry fails with PCGCN_ECUDA
+// when no usable GPU is present.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstring>
+#include <new>
+#include <string>
+
+#include "kernels.h"
+#include "plan_internal.h"
+
+namespace pcgcn {
+
+namespace {
+thread_local std::string g_err;
+void* (*g_alloc)(size_t, void*) = nullptr;
+void (*g_free)(void*, void*) = nullptr;
+void* g_ctx = nullptr;
+
+int64_t round_up(int64_t x, int64_t m) { return (x + m - 1) / m * m; }
+
+pcgcn_status cuda_fail(cudaError_t e, const char* where) {
+  set_error(std::string(where) + ": " + cudaGetErrorString(e));
+  return PCGCN_ECUDA;
+}
+
+void* dev_alloc(size_t bytes) {
+  if (bytes == 0) bytes = 16;
+  if (g_alloc) return g_alloc(bytes, g_ctx);
+  void* p = nullptr;
+  if (cudaMalloc(&p, bytes) != cudaSuccess) return nullptr;
+  return p;
+}
+void dev_free(void* p) {
+  if (!p) return;
+  if (g_free) g_free(p, g_ctx);
+  else cudaFree(p);
+}
+
+template <class T>
+pcgcn_status upload(DevicePlan& d, T** dst, const T* src, int64_t count) {
+  *dst = static_cast<T*>(dev_alloc(sizeof(T) * std::max<int64_t>(count, 1)));
+  if (!*dst) { set_error("device allocation failed"); return PCGCN_ENOMEM; }
+  d.owned.push_back(*dst);
+  d.bytes += int64_t(sizeof(T)) * std::max<int64_t>(count, 1);
+  if (count > 0 && src) {
+    cudaError_t e = cudaMemcpy(*dst, src, sizeof(T) * count, cudaMemcpyHostToDevice);
+    if (e != cudaSuccess) return cuda_fail(e, "upload");
+  }
+  return PCGCN_OK;
+}
+
+bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
+}  // namespace
+
+void set_error(const std::string& msg) { g_err = msg; }
+
+void free_device_plan(pcgcn_plan_s* p) {
+  for (void* q : p->d.owned) dev_free(q);
+  p->d = DevicePlan();
+}
+
+pcgcn_status upload_plan(pcgcn_plan_s* p) {
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaGetDevice (no usable GPU)");
+  cudaDeviceProp prop;
+  e = cudaGetDeviceProperties(&prop, dev);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaGetDeviceProperties");
+  if (prop.major < 10) {
+    set_error("libpcgcn requires an sm_100 (B200) device");
+    return PCGCN_ECUDA;
+  }
+  DevicePlan& d = p->d;
+  const int64_t n = p->n;
+  d.rows = p->row_hi - p->row_lo;
+  d.nnz_s = p->sp_rowptr[p->row_hi] - p->sp_rowptr[p->row_lo];
+  d.nrt = p->rt_hi - p->rt_lo;
+  const int64_t ch_lo = p->rt_cptr[p->rt_lo], ch_hi = p->rt_cptr[p->rt_hi];
+  d.nch = ch_hi - ch_lo;
+  d.fpad_max = int(round_up(std::max(p->opts.f_max, 1), 16));
+  d.n_pad = n;
+  pcgcn_status st;
+#define UP(dst, src, cnt) \
+  if ((st = upload(d, dst, src, cnt)) != PCGCN_OK) return st
+  UP(&d.r, p->r.data(), n);
+  std::vector<int64_t> rp(d.rows + 1);
+  for (int64_t v = 0; v <= d.rows; ++v) rp[v] = p->sp_rowptr[p->row_lo + v] - p->sp_rowptr[p->row_lo];
+  UP(&d.sp_rowptr, rp.data(), d.rows + 1);
+  UP(&d.sp_col, p->sp_col.data() + p->sp_rowptr[p->row_lo], d.nnz_s);
+  if (d.nch > 0) {
+    std::vector<int32_t> zi(d.rows);
+    const int64_t base = p->rt_lo * TILE_M;
+    for (int64_t v = 0; v < d.rows; ++v) {
+      int32_t z = p->zd_index[p->row_lo + v];
+      zi[v] = z < 0 ? -1 : int32_t(z - base);
+    }
+    UP(&d.zd_index, zi.data(), d.rows);
+    UP(&d.rt_row0, p->rt_row0.data() + p->rt_lo, d.nrt);
+    UP(&d.rt_nrows, p->rt_nrows.data() + p->rt_lo, d.nrt);
+    std::vector<int64_t> cp(d.nrt + 1);
+    for (int64_t t = 0; t <= d.nrt; ++t) cp[t] = p->rt_cptr[p->rt_lo + t] - ch_lo;
+    UP(&d.rt_cptr, cp.data(), d.nrt + 1);
+    UP(&d.ch_col0, p->ch_col0.data() + ch_lo, d.nch);
+    UP(&d.bits, p->bits.data() + ch_lo * TILE_M, d.nch * TILE_M);
+    UP(&d.zd, (float*)nullptr, d.nrt * TILE_M * d.fpad_max);
+    UP(&d.yhi, (float*)nullptr, d.n_pad * d.fpad_max);
+    UP(&d.ylo, (float*)nullptr, d.n_pad * d.fpad_max);
+  }
+  UP(&d.ypre, (float*)nullptr, n * d.fpad_max);
+#undef UP
+  d.built = true;
+  p->stats.device_bytes = d.bytes;
+  return PCGCN_OK;
+}
+
+namespace {
+
+pcgcn_status aggregate(pcgcn_plan_t p, const float* Y, int64_t ldy, float* Z, int64_t ldz, int32_t F,
+                       uint32_t flags, uint32_t* mask, void* stream) {
+  if (!p || !p->d.built) { set_error("plan has no device structures"); return PCGCN_EINVAL; }
+  if (!Y || !Z || F < 1 || F > p->opts.f_max || ldy < round_up(F, 4) || ldz < round_up(F, 4) ||
+      (ldy & 3) || (ldz & 3) || !aligned16(Y) || !aligned16(Z)) {
+    set_error("forward/backward: bad Y/Z/F/ld (ld >= roundup(F,4), 16-byte aligned rows, F <= f_max)");
+    return PCGCN_EINVAL;
+  }
+  if ((flags & PCGCN_MASK_OUT) && !mask) { set_error("MASK_OUT needs a mask buffer"); return PCGCN_EINVAL; }
+  DevicePlan& d = p->d;
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  cudaError_t e;
+  const bool dense = d.nch > 0;
+  const bool prescaled = (flags & PCGCN_IN_PRESCALED) != 0;
+  const int npad = int(round_up(F, 16));
+  const int64_t ld4 = round_up(F, 4);
+  const float* src = Y;
+  int64_t ldsrc = ldy;
+  const bool tc = p->opts.dense_prec == PCGCN_DENSE_TF32X2;
+  if (!prescaled || (dense && tc)) {
+    float* ypre = prescaled ? nullptr : d.ypre;
+    e = launch_prescale_split(Y, ldy, prescaled ? nullptr : d.r, p->n, F, ypre, ld4,
+                              (dense && tc) ? d.yhi : nullptr, (dense && tc) ? d.ylo : nullptr, npad, s);
+    if (e != cudaSuccess) return cuda_fail(e, "prescale_split");
+    if (!prescaled) { src = d.ypre; ldsrc = ld4; }
+  }
+  if (dense) {
+    DenseArgs da{d.yhi, d.ylo, p->n, npad, d.rt_row0, d.rt_nrows, d.rt_cptr, d.ch_col0, d.bits,
+                 d.nrt, d.zd, npad, npad};
+    e = tc ? launch_dense_tc(da, s) : launch_dense_simt_y(da, src, ldsrc, F, s);
+    if (e != cudaSuccess) return cuda_fail(e, "dense-mode kernel");
+  }
+  AggArgs a;
+  a.Y = src; a.ldy = ldsrc; a.Z = Z; a.ldz = ldz;
+  a.mask = (flags & PCGCN_MASK_OUT) ? mask : nullptr;
+  a.rowptr = d.sp_rowptr; a.col = d.sp_col; a.r = d.r;
+  a.row_lo = p->row_lo; a.rows = d.rows;
+  a.zd_index = dense ? d.zd_index : nullptr;
+  a.zd = d.zd; a.ldzd = npad;
+  a.F = F;
+  a.relu = (flags & PCGCN_RELU) != 0;
+  a.out_prescaled = (flags & PCGCN_OUT_PRESCALED) != 0;
+  e = launch_sparse_agg(a, s);
+  if (e != cudaSuccess) return cuda_fail(e, "selective-mode kernel");
+  return PCGCN_OK;
+}
+
+}  // namespace
+}  // namespace pcgcn
+
+using namespace pcgcn;
+
+extern "C" {
+
+int32_t pcgcn_abi_version(void) { return 1; }
+
+const char* pcgcn_last_error(void) { return g_err.c_str(); }
+
+void pcgcn_set_allocator(void* (*alloc)(size_t, void*), void (*release)(void*, void*), void* ctx) {
+  g_alloc = alloc;
+  g_free = release;
+  g_ctx = ctx;
+}
+
+void pcgcn_opts_default(pcgcn_opts* o) {
+  if (!o) return;
+  std::memset(o, 0, sizeof(*o));
+  o->norm = PCGCN_NORM_SYM;
+  o->dense_prec = PCGCN_DENSE_TF32X2;
+  o->f_max = 128;
+  o->lp_sweeps = 10;
+  o->part = nullptr;
+  o->build_device = 1;
+  o->rank = 0;
+  o->world = 1;
+}
+
+pcgcn_status pcgcn_plan(const pcgcn_csr* A, int32_t P, float theta, const pcgcn_opts* o,
+                        pcgcn_plan_t* out) {
+  if (!A || !out) { set_error("pcgcn_plan: null argument"); return PCGCN_EINVAL; }
+  *out = nullptr;
+  pcgcn_opts def;
+  pcgcn_opts_default(&def);
+  if (!o) o = &def;
+  if (o->f_max < 1 || o->f_max > 256) { set_error("f_max must be in [1, 256]"); return PCGCN_EINVAL; }
+  if (o->dense_prec != PCGCN_DENSE_TF32X2 && o->dense_prec != PCGCN_DENSE_FP32_SIMT) {
+    set_error("unknown dense_prec");
+    return PCGCN_EUNSUP;
+  }
+  if (o->dense_prec == PCGCN_DENSE_FP32_SIMT && o->f_max > 128) {
+    set_error("FP32_SIMT full mode supports F <= 128");
+    return PCGCN_EUNSUP;
+  }
+  pcgcn_plan_s* p = new (std::nothrow) pcgcn_plan_s();
+  if (!p) { set_error("out of host memory"); return PCGCN_ENOMEM; }
+  pcgcn_status st;
+  try {
+    st = build_host_plan(A, P, theta, o, p);
+  } catch (const std::bad_alloc&) {
+    st = PCGCN_ENOMEM;
+    set_error("out of host memory in planner");
+  } catch (...) {
+    st = PCGCN_EINVAL;
+    set_error("planner failure");
+  }
+  if (st == PCGCN_OK && o->build_device) st = upload_plan(p);
+  if (st != PCGCN_OK) {
+    free_device_plan(p);
+    delete p;
+    return st;
+  }
+  p->opts.part = nullptr;  // borrowed pointer: do not keep
+  *out = p;
+  return PCGCN_OK;
+}
+
+void pcgcn_destroy(pcgcn_plan_t p) {
+  if (!p) return;
+  free_device_plan(p);
+  delete p;
+}
+
+pcgcn_status pcgcn_forward(pcgcn_plan_t p, const float* Y, int64_t ldy, float* Z, int64_t ldz,
+                           int32_t F, uint32_t flags, uint32_t* mask, void* stream) {
+  return aggregate(p, Y, ldy, Z, ldz, F, flags, mask, stream);
+}
+
+pcgcn_status pcgcn_backward(pcgcn_plan_t p, const float* dZ, int64_t ldz, float* dY, int64_t ldy,
+                            int32_t F, uint32_t flags, void* stream) {
+  // Âᵀ = Â for a symmetric input: the forward plan serves the backward.
+  return aggregate(p, dZ, ldz, dY, ldy, F, flags & ~uint32_t(PCGCN_MASK_OUT), nullptr, stream);
+}
+
+pcgcn_status pcgcn_plan_perm(pcgcn_plan_t p, int32_t* perm) {
+  if (!p || !perm) { set_error("null argument"); return PCGCN_EINVAL; }
+  std::memcpy(perm, p->perm.data(), sizeof(int32_t) * p->n);
+  return PCGCN_OK;
+}
+
+pcgcn_status pcgcn_plan_stats(pcgcn_plan_t p, pcgcn_stats* s) {
+  if (!p || !s) { set_error("null argument"); return PCGCN_EINVAL; }
+  *s = p->stats;
+  return PCGCN_OK;
+}
+
+const float* pcgcn_plan_rowscale(pcgcn_plan_t p) { return p && p->d.built ? p->d.r : nullptr; }
+
+int64_t pcgcn_plan_export_bytes(pcgcn_plan_t p, int32_t which) {
+  if (!p) return -1;
+  switch (which) {
+    case PCGCN_X_PART: return 4 * int64_t(p->part.size());
+    case PCGCN_X_PERM: return 4 * int64_t(p->perm.size());
+    case PCGCN_X_PSTART: return 8 * int64_t(p->pstart.size());
+    case PCGCN_X_R: return 4 * int64_t(p->r.size());
+    case PCGCN_X_BLK_K: return 4 * int64_t(p->blk_k.size());
+    case PCGCN_X_BLK_I: return 4 * int64_t(p->blk_i.size());
+    case PCGCN_X_BLK_NNZ: return 8 * int64_t(p->blk_nnz.size());
+    case PCGCN_X_BLK_DENSE: return int64_t(p->blk_dense.size());
+    case PCGCN_X_SP_ROWPTR: return 8 * int64_t(p->sp_rowptr.size());
+    case PCGCN_X_SP_COL: return 4 * int64_t(p->sp_col.size());
+    case PCGCN_X_RT_ROW0: return 4 * int64_t(p->rt_row0.size());
+    case PCGCN_X_RT_NROWS: return 4 * int64_t(p->rt_nrows.size());
+    case PCGCN_X_RT_CPTR: return 8 * int64_t(p->rt_cptr.size());
+    case PCGCN_X_CH_COL0: return 4 * int64_t(p->ch_col0.size());
+    case PCGCN_X_BITS: return 4 * int64_t(p->bits.size());
+    case PCGCN_X_ZD_INDEX: return 4 * int64_t(p->zd_index.size());
+    case PCGCN_X_SWEEPS: return 4;
+    default: return -1;
+  }
+}
+
+pcgcn_status pcgcn_plan_export(pcgcn_plan_t p, int32_t which, void* buf, int64_t bytes) {
+  int64_t need = pcgcn_plan_export_bytes(p, which);
+  if (need < 0 || !buf || bytes < need) { set_error("plan_export: bad which / buffer"); return PCGCN_EINVAL; }
+  const void* src = nullptr;
+  switch (which) {
+    case PCGCN_X_PART: src = p->part.data(); break;
+    case PCGCN_X_PERM: src = p->perm.data(); break;
+    case PCGCN_X_PSTART: src = p->pstart.data(); break;
+    case PCGCN_X_R: src = p->r.data(); break;
+    case PCGCN_X_BLK_K: src = p->blk_k.data(); break;
+    case PCGCN_X_BLK_I: src = p->blk_i.data(); break;
+    case PCGCN_X_BLK_NNZ: src = p->blk_nnz.data(); break;
+    case PCGCN_X_BLK_DENSE: src = p->blk_dense.data(); break;
+    case PCGCN_X_SP_ROWPTR: src = p->sp_rowptr.data(); break;
+    case PCGCN_X_SP_COL: src = p->sp_col.data(); break;
+    case PCGCN_X_RT_ROW0: src = p->rt_row0.data(); break;
+    case PCGCN_X_RT_NROWS: src = p->rt_nrows.data(); break;
+    case PCGCN_X_RT_CPTR: src = p->rt_cptr.data(); break;
+    case PCGCN_X_CH_COL0: src = p->ch_col0.data(); break;
+    case PCGCN_X_BITS: src = p->bits.data(); break;
+    case PCGCN_X_ZD_INDEX: src = p->zd_index.data(); break;
+    case PCGCN_X_SWEEPS: src = &p->sweeps; break;
+  }
+  if (need > 0) std::memcpy(buf, src, size_t(need));
+  return PCGCN_OK;
+}
+
+pcgcn_status pcgcn_gemm_xw(const float* X, int64_t ldx, const float* W, int64_t ldw, const float* s,
+                           float* Y, int64_t ldy, int64_t M, int32_t K, int32_t N, void* stream) {
+  if (!X || !W || !Y || M < 0 || K < 1 || N < 1 || ldx < K || ldw < N || ldy < N) {
+    set_error("gemm_xw: bad arguments");
+    return PCGCN_EINVAL;
+  }
+  cudaError_t e = launch_gemm_xw(X, ldx, W, ldw, s, Y, ldy, M, K, N, static_cast<cudaStream_t>(stream));
+  return e == cudaSuccess ? PCGCN_OK : cuda_fail(e, "gemm_xw");
+}
+
+int64_t pcgcn_gemm_xtg_work_floats(int64_t M, int32_t K, int32_t N) { return gemm_xtg_work_floats(M, K, N); }
+
+pcgcn_status pcgcn_gemm_xtg(const float* X, int64_t ldx, const float* D, int64_t ldd, float* G,
+                            int64_t M, int32_t K, int32_t N, float* work, void* stream) {
+  if (!X || !D || !G || !work || M < 0 || K < 1 || N < 1 || ldx < K || ldd < N) {
+    set_error("gemm_xtg: bad arguments");
+    return PCGCN_EINVAL;
+  }
+  cudaError_t e = launch_gemm_xtg(X, ldx, D, ldd, G, M, K, N, work, static_cast<cudaStream_t>(stream));
+  return e == cudaSuccess ? PCGCN_OK : cuda_fail(e, "gemm_xtg");
+}
+
+pcgcn_status pcgcn_gemm_dwt(const float* D, int64_t ldd, const float* W, const uint32_t* mask,
+                            const float* s, float* O, int64_t ldo, int64_t M, int32_t N, int32_t K,
+                            void* stream) {
+  if (!D || !W || !O || M < 0 || K < 1 || N < 1 || ldd < N || ldo < K) {
+    set_error("gemm_dwt: bad arguments");
+    return PCGCN_EINVAL;
+  }
+  cudaError_t e = launch_gemm_dwt(D, ldd, W, mask, s, O, ldo, M, N, K, static_cast<cudaStream_t>(stream));
+  return e == cudaSuccess ? PCGCN_OK : cuda_fail(e, "gemm_dwt");
+}
+
+pcgcn_status pcgcn_softmax_ce(const float* L, int64_t ld, const int32_t* labels, const uint8_t* train,
+                              int64_t M, int32_t C, float inv_nT, const float* s, float* dL,
+                              float* loss, float* work, void* stream) {
+  if (!L || !labels || !train || !dL || !loss || !work || C < 1 || C > 256 || ld < C) {
+    set_error("softmax_ce: bad arguments");
+    return PCGCN_EINVAL;
+  }
+  cudaError_t e = launch_softmax_ce(L, ld, labels, train, M, C, inv_nT, s, dL, loss, work,
+                                    static_cast<cudaStream_t>(stream));
+  return e == cudaSuccess ? PCGCN_OK : cuda_fail(e, "softmax_ce");
+}
+
+pcgcn_status pcgcn_adam(float* theta, const float* grad, float* m, float* v, int64_t n, float lr,
+                        float b1, float b2, float eps, int32_t* step, void* stream) {
+  if (!theta || !grad || !m || !v || !step || n < 0) { set_error("adam: bad arguments"); return PCGCN_EINVAL; }
+  cudaError_t e = launch_adam(theta, grad, m, v, n, lr, b1, b2, eps, step, static_cast<cudaStream_t>(stream));
+  return e == cudaSuccess ? PCGCN_OK : cuda_fail(e, "adam");
+}
+
+pcgcn_status pcgcn_sgd(float* theta, const float* grad, int64_t n, float lr, void* stream) {
+  if (!theta || !grad || n < 0) { set_error("sgd: bad arguments"); return PCGCN_EINVAL; }
+  cudaError_t e = launch_sgd(theta, grad, n, lr, static_cast<cudaStream_t>(stream));
+  return e == cudaSuccess ? PCGCN_OK : cuda_fail(e, "sgd");
+}
+
+}  // extern "C"

@@ -1,0 +1,75 @@
+// Internal plan layout shared by the host planner (planner.cpp) and the
+// device side (pcgcn_api.cu).  Not part of the ABI.
+#pragma once
+#include <cstdint>
+#include <string>
+#include <vector>
+
+#include "../../include/pcgcn.h"
+
+namespace pcgcn {
+
+constexpr int TILE_M = 128;  // dense row tile: destination rows (UMMA M)
+constexpr int TILE_K = 32;   // dense chunk: source columns (one 128-byte tf32 K-major row)
+
+struct DevicePlan {
+  bool built = false;
+  float* r = nullptr;             // [n] plan order
+  int64_t* sp_rowptr = nullptr;   // [rows+1] shard-local, rebased to 0
+  int32_t* sp_col = nullptr;      // [nnz_s shard]
+  int32_t* zd_index = nullptr;    // [rows] shard-local row tile slot (t*128+rr), -1 none
+  int32_t* rt_row0 = nullptr;     // [nrt shard] plan row
+  int32_t* rt_nrows = nullptr;    // [nrt shard]
+  int64_t* rt_cptr = nullptr;     // [nrt+1] rebased
+  int32_t* ch_col0 = nullptr;     // [nch shard]
+  uint32_t* bits = nullptr;       // [nch*128]
+  float* zd = nullptr;            // [nrt*128*fpad_max] dense partial sums
+  float* yhi = nullptr;           // [n_pad*fpad_max] tf32 hi part of the (prescaled) input
+  float* ylo = nullptr;           // [n_pad*fpad_max] lo part
+  float* ypre = nullptr;          // [n*fpad_max] prescaled copy for un-prescaled inputs
+  int64_t rows = 0, nnz_s = 0, nrt = 0, nch = 0;
+  int64_t n_pad = 0;
+  int fpad_max = 0;
+  int64_t bytes = 0;
+  std::vector<void*> owned;
+};
+
+}  // namespace pcgcn
+
+struct pcgcn_plan_s {
+  int64_t n = 0;
+  int64_t nnz_t = 0;  // nnz(Ã)
+  int32_t P = 0;
+  float theta = 0.f;
+  pcgcn_opts opts{};
+  int32_t sweeps = 0;
+  int64_t clusters = 0;
+  std::vector<int32_t> part, perm;
+  std::vector<int64_t> pstart;
+  std::vector<float> r;
+  std::vector<int32_t> blk_k, blk_i;
+  std::vector<int64_t> blk_nnz;
+  std::vector<uint8_t> blk_dense;
+  std::vector<int64_t> sp_rowptr;
+  std::vector<int32_t> sp_col;
+  std::vector<int32_t> rt_row0, rt_nrows;
+  std::vector<int64_t> rt_cptr;
+  std::vector<int32_t> ch_col0;
+  std::vector<uint32_t> bits;
+  std::vector<int32_t> zd_index;
+  // shard
+  int32_t k_lo = 0, k_hi = 0;
+  int64_t row_lo = 0, row_hi = 0, rt_lo = 0, rt_hi = 0;
+  pcgcn_stats stats{};
+  pcgcn::DevicePlan d;
+};
+
+namespace pcgcn {
+// host planner (planner.cpp); fills every host array and stats (not device)
+pcgcn_status build_host_plan(const pcgcn_csr* A, int32_t P, float theta, const pcgcn_opts* o,
+                             pcgcn_plan_s* p);
+// device side (pcgcn_api.cu)
+pcgcn_status upload_plan(pcgcn_plan_s* p);
+void free_device_plan(pcgcn_plan_s* p);
+void set_error(const std::string& msg);
+}  // namespace pcgcn

@@ -1,0 +1,414 @@
+// Host planner of PCGCN (deterministic, multithreaded, result independent of
+// the thread count).  Builds, for one symmetric input graph:
+//   1. Ã = A + I in clean form, d̃ and r = fp32(d̃^-½)      (Eq. 1; reading #1-#4)
+//   2. the vertex partition {V_k}                           (L95-L97 §III-A.a)
+//      — synchronous label propagation + packing, replacing METIS (reading #8)
+//   3. the plan-order permutation (vertex blocks become row ranges, so the
+//      "split a^l -> a_k^l" and "concat h_k^l" of Alg. 1, L115/L123, are free)
+//   4. the K×K edge-block table with densities and mode bits (θ rule, L161)
+//   5. the merged selective CSR (L179) and the full-mode tiles (L175) as
+//      128×32 bit chunks grouped per 128-row destination tile.
+// The plan spec it implements is DESIGN.md "Plan spec"; oracle/plan.py is an
+// independent re-derivation and tests/test_plan_abi.py compares them bit-exactly.
+#include <algorithm>
+#include <chrono>
+#include <cmath>
+#include <cstring>
+#include <numeric>
+#include <thread>
+#include <vector>
+
+#include "plan_internal.h"
+
+namespace pcgcn {
+namespace {
+
+int nthreads() {
+  unsigned h = std::thread::hardware_concurrency();
+  return h == 0 ? 4 : int(std::min(h, 64u));
+}
+
+template <class F>
+void parallel_for(int64_t n, F f) {
+  int T = nthreads();
+  if (n < 4096) T = 1;
+  std::vector<std::thread> th;
+  for (int t = 0; t < T; ++t) {
+    int64_t a = n * t / T, b = n * (t + 1) / T;
+    if (T == 1) { f(t, a, b); return; }
+    th.emplace_back([=, &f] { f(t, a, b); });
+  }
+  for (auto& x : th) x.join();
+}
+
+double ms_since(std::chrono::steady_clock::time_point t0) {
+  return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+}
+
+// Clean binary A (no self-loops, no duplicates, sorted rows).
+struct CleanA {
+  std::vector<int64_t> ptr;
+  std::vector<int32_t> col;
+};
+
+pcgcn_status clean_graph(const pcgcn_csr* A, CleanA& C) {
+  const int64_t n = A->n;
+  std::vector<int64_t> cnt(n, 0);
+  std::vector<int32_t> tmp(A->nnz);
+  bool bad = false;
+  parallel_for(n, [&](int, int64_t a, int64_t b) {
+    for (int64_t v = a; v < b; ++v) {
+      int64_t s = A->rowptr[v], e = A->rowptr[v + 1];
+      int32_t* out = tmp.data() + s;
+      int64_t k = 0;
+      for (int64_t i = s; i < e; ++i) {
+        int32_t j = A->col[i];
+        if (j < 0 || j >= n) { bad = true; continue; }
+        if (j != v) out[k++] = j;
+      }
+      std::sort(out, out + k);
+      cnt[v] = std::unique(out, out + k) - out;
+    }
+  });
+  if (bad) { set_error("column index out of range"); return PCGCN_EINVAL; }
+  C.ptr.assign(n + 1, 0);
+  for (int64_t v = 0; v < n; ++v) C.ptr[v + 1] = C.ptr[v] + cnt[v];
+  C.col.resize(C.ptr[n]);
+  parallel_for(n, [&](int, int64_t a, int64_t b) {
+    for (int64_t v = a; v < b; ++v)
+      std::memcpy(C.col.data() + C.ptr[v], tmp.data() + A->rowptr[v], sizeof(int32_t) * cnt[v]);
+  });
+  // symmetry: every (v, j) must have (j, v)
+  std::vector<uint8_t> asym(nthreads(), 0);
+  parallel_for(n, [&](int t, int64_t a, int64_t b) {
+    for (int64_t v = a; v < b && !asym[t]; ++v)
+      for (int64_t i = C.ptr[v]; i < C.ptr[v + 1]; ++i) {
+        int32_t j = C.col[i];
+        if (!std::binary_search(C.col.data() + C.ptr[j], C.col.data() + C.ptr[j + 1], int32_t(v))) {
+          asym[t] = 1;
+          break;
+        }
+      }
+  });
+  for (auto x : asym)
+    if (x) { set_error("adjacency is not symmetric (A^T != A)"); return PCGCN_ENOTSYM; }
+  return PCGCN_OK;
+}
+
+// Synchronous label propagation on Ã (self vote included), ties -> smallest label.
+int32_t label_propagation(const CleanA& C, int64_t n, int32_t T, std::vector<int32_t>& lab) {
+  lab.resize(n);
+  std::iota(lab.begin(), lab.end(), 0);
+  std::vector<int32_t> nxt(n);
+  int32_t it = 0;
+  for (it = 1; it <= T; ++it) {
+    std::vector<uint8_t> changed(nthreads(), 0);
+    parallel_for(n, [&](int t, int64_t a, int64_t b) {
+      std::vector<int32_t> buf;
+      for (int64_t v = a; v < b; ++v) {
+        int64_t s = C.ptr[v], e = C.ptr[v + 1];
+        buf.resize(e - s + 1);
+        for (int64_t i = s; i < e; ++i) buf[i - s] = lab[C.col[i]];
+        buf[e - s] = lab[v];
+        std::sort(buf.begin(), buf.end());
+        int32_t best = buf[0];
+        int64_t best_c = 0;
+        for (size_t i = 0; i < buf.size();) {
+          size_t j = i;
+          while (j < buf.size() && buf[j] == buf[i]) ++j;
+          if (int64_t(j - i) > best_c) { best_c = int64_t(j - i); best = buf[i]; }
+          i = j;
+        }
+        nxt[v] = best;
+        if (best != lab[v]) changed[t] = 1;
+      }
+    });
+    bool any = false;
+    for (auto c : changed) any |= c != 0;
+    if (!any) return it;
+    lab.swap(nxt);
+  }
+  return T;
+}
+
+// Clusters ordered by (size desc, smallest member asc), members by id, cut
+// into P consecutive chunks (numpy array_split sizes).
+int64_t pack_parts(const std::vector<int32_t>& lab, int64_t n, int32_t P, std::vector<int32_t>& part) {
+  std::vector<int64_t> size(n, 0), minid(n, n);
+  for (int64_t v = 0; v < n; ++v) {
+    size[lab[v]]++;
+    minid[lab[v]] = std::min(minid[lab[v]], v);
+  }
+  std::vector<int32_t> cl;
+  for (int64_t l = 0; l < n; ++l)
+    if (size[l] > 0) cl.push_back(int32_t(l));
+  std::sort(cl.begin(), cl.end(), [&](int32_t a, int32_t b) {
+    if (size[a] != size[b]) return size[a] > size[b];
+    return minid[a] < minid[b];
+  });
+  std::vector<int64_t> off(n, 0);
+  int64_t run = 0;
+  for (int32_t l : cl) { off[l] = run; run += size[l]; }
+  std::vector<int32_t> seq(n);
+  for (int64_t v = 0; v < n; ++v) seq[off[lab[v]]++] = int32_t(v);
+  part.assign(n, 0);
+  const int64_t q = n / P, rem = n % P;
+  int64_t pos = 0;
+  for (int32_t k = 0; k < P; ++k) {
+    int64_t sz = q + (k < rem ? 1 : 0);
+    for (int64_t i = 0; i < sz; ++i) part[seq[pos++]] = k;
+  }
+  return int64_t(cl.size());
+}
+
+}  // namespace
+
+pcgcn_status build_host_plan(const pcgcn_csr* A, int32_t P, float theta, const pcgcn_opts* o,
+                             pcgcn_plan_s* p) {
+  auto t0 = std::chrono::steady_clock::now();
+  const int64_t n = A->n;
+  if (n <= 0 || P < 1 || P > n || !A->rowptr || (A->nnz > 0 && !A->col) || A->rowptr[0] != 0 ||
+      A->rowptr[n] != A->nnz) {
+    set_error("pcgcn_plan: bad graph or P");
+    return PCGCN_EINVAL;
+  }
+  for (int64_t v = 0; v < n; ++v)
+    if (A->rowptr[v + 1] < A->rowptr[v]) { set_error("rowptr not monotone"); return PCGCN_EINVAL; }
+  if (!(theta >= 0.f)) { set_error("theta must be >= 0 (calibrate first)"); return PCGCN_EINVAL; }
+  if (o->world < 1 || o->rank < 0 || o->rank >= o->world) { set_error("bad rank/world"); return PCGCN_EINVAL; }
+  p->n = n; p->P = P; p->theta = theta; p->opts = *o;
+
+  CleanA C;
+  pcgcn_status st = clean_graph(A, C);
+  if (st != PCGCN_OK) return st;
+  p->nnz_t = C.ptr[n] + n;
+
+  // r = fp32(1/sqrt(fp64 d̃)), d̃ = 1 + deg  (correctly rounded => bit-exact)
+  std::vector<float> r_orig(n);
+  for (int64_t v = 0; v < n; ++v) {
+    double d = double(C.ptr[v + 1] - C.ptr[v] + 1);
+    r_orig[v] = o->norm == PCGCN_NORM_NONE ? 1.0f : float(1.0 / std::sqrt(d));
+  }
+
+  // partition
+  auto tp = std::chrono::steady_clock::now();
+  if (o->part) {
+    p->part.assign(o->part, o->part + n);
+    for (int64_t v = 0; v < n; ++v)
+      if (p->part[v] < 0 || p->part[v] >= P) { set_error("part override out of range"); return PCGCN_EINVAL; }
+    p->sweeps = 0;
+    p->clusters = 0;
+  } else {
+    std::vector<int32_t> lab;
+    p->sweeps = label_propagation(C, n, o->lp_sweeps, lab);
+    p->clusters = pack_parts(lab, n, P, p->part);
+  }
+  double part_ms = ms_since(tp);
+
+  // permutation: sort by (part, id)
+  std::vector<int64_t> psize(P, 0);
+  for (int64_t v = 0; v < n; ++v) psize[p->part[v]]++;
+  p->pstart.assign(P + 1, 0);
+  for (int32_t k = 0; k < P; ++k) p->pstart[k + 1] = p->pstart[k] + psize[k];
+  p->perm.resize(n);
+  std::vector<int64_t> inv(n);
+  {
+    std::vector<int64_t> fill(p->pstart.begin(), p->pstart.end() - 1);
+    for (int64_t v = 0; v < n; ++v) {
+      int64_t pos = fill[p->part[v]]++;
+      p->perm[pos] = int32_t(v);
+      inv[v] = pos;
+    }
+  }
+  p->r.resize(n);
+  for (int64_t v = 0; v < n; ++v) p->r[v] = r_orig[p->perm[v]];
+  std::vector<int32_t> pid(n);  // partition of each plan row
+  for (int32_t k = 0; k < P; ++k)
+    for (int64_t v = p->pstart[k]; v < p->pstart[k + 1]; ++v) pid[v] = k;
+
+  // Ã in plan order, rows sorted
+  std::vector<int64_t> tptr(n + 1, 0);
+  for (int64_t v = 0; v < n; ++v) {
+    int32_t old = p->perm[v];
+    tptr[v + 1] = tptr[v] + (C.ptr[old + 1] - C.ptr[old]) + 1;
+  }
+  std::vector<int32_t> tcol(tptr[n]);
+  parallel_for(n, [&](int, int64_t a, int64_t b) {
+    for (int64_t v = a; v < b; ++v) {
+      int32_t old = p->perm[v];
+      int32_t* out = tcol.data() + tptr[v];
+      int64_t k = 0;
+      for (int64_t i = C.ptr[old]; i < C.ptr[old + 1]; ++i) out[k++] = int32_t(inv[C.col[i]]);
+      out[k++] = int32_t(v);
+      std::sort(out, out + k);
+    }
+  });
+  std::vector<int64_t>().swap(C.ptr);
+  std::vector<int32_t>().swap(C.col);
+
+  // block table per destination partition k (rows contiguous)
+  std::vector<std::vector<std::pair<int32_t, int64_t>>> blocks(P);  // (i, nnz) sorted by i
+  parallel_for(P, [&](int, int64_t a, int64_t b) {
+    std::vector<int64_t> cnt(P, 0);
+    std::vector<int32_t> touched;
+    for (int64_t k = a; k < b; ++k) {
+      for (int64_t v = p->pstart[k]; v < p->pstart[k + 1]; ++v)
+        for (int64_t e = tptr[v]; e < tptr[v + 1]; ++e) {
+          int32_t i = pid[tcol[e]];
+          if (cnt[i]++ == 0) touched.push_back(i);
+        }
+      std::sort(touched.begin(), touched.end());
+      for (int32_t i : touched) { blocks[k].push_back({i, cnt[i]}); cnt[i] = 0; }
+      touched.clear();
+    }
+  });
+  std::vector<int64_t> bptr(P + 1, 0);
+  for (int32_t k = 0; k < P; ++k) bptr[k + 1] = bptr[k] + int64_t(blocks[k].size());
+  const int64_t nb = bptr[P];
+  p->blk_k.resize(nb); p->blk_i.resize(nb); p->blk_nnz.resize(nb); p->blk_dense.resize(nb);
+  const double th = double(theta);
+  int64_t nb_dense = 0, intra = 0;
+  for (int32_t k = 0; k < P; ++k)
+    for (size_t j = 0; j < blocks[k].size(); ++j) {
+      int64_t b = bptr[k] + int64_t(j);
+      int32_t i = blocks[k][j].first;
+      int64_t z = blocks[k][j].second;
+      p->blk_k[b] = k; p->blk_i[b] = i; p->blk_nnz[b] = z;
+      double dens = double(z) / (double(psize[k]) * double(psize[i]));
+      p->blk_dense[b] = dens > th ? 1 : 0;
+      nb_dense += p->blk_dense[b];
+      if (i == k) intra += z;
+    }
+
+  // mode of each edge -> merged selective CSR + dense chunks, per partition
+  std::vector<int64_t> sp_cnt(n, 0);
+  struct TileOut {
+    int32_t row0, nrows;
+    std::vector<int32_t> col0;
+    std::vector<uint32_t> bits;
+  };
+  std::vector<std::vector<TileOut>> tiles(P);
+  parallel_for(P, [&](int, int64_t a, int64_t b) {
+    std::vector<uint8_t> dense_i(P, 0);
+    std::vector<std::pair<int32_t, int32_t>> ent;  // (col0, (rr<<5)|bit)
+    for (int64_t k = a; k < b; ++k) {
+      bool any_dense = false;
+      for (int64_t j = bptr[k]; j < bptr[k + 1]; ++j) {
+        dense_i[p->blk_i[j]] = p->blk_dense[j];
+        any_dense |= p->blk_dense[j] != 0;
+      }
+      for (int64_t v = p->pstart[k]; v < p->pstart[k + 1]; ++v) {
+        int64_t c = 0;
+        for (int64_t e = tptr[v]; e < tptr[v + 1]; ++e) c += dense_i[pid[tcol[e]]] ? 0 : 1;
+        sp_cnt[v] = c;
+      }
+      if (any_dense) {
+        for (int64_t r0 = p->pstart[k]; r0 < p->pstart[k + 1]; r0 += TILE_M) {
+          int64_t r1 = std::min<int64_t>(r0 + TILE_M, p->pstart[k + 1]);
+          ent.clear();
+          for (int64_t v = r0; v < r1; ++v)
+            for (int64_t e = tptr[v]; e < tptr[v + 1]; ++e) {
+              int32_t j = tcol[e];
+              int32_t i = pid[j];
+              if (!dense_i[i]) continue;
+              int64_t c0 = p->pstart[i] + ((j - p->pstart[i]) / TILE_K) * TILE_K;
+              ent.push_back({int32_t(c0), int32_t(((v - r0) << 5) | (j - c0))});
+            }
+          if (ent.empty()) continue;
+          std::sort(ent.begin(), ent.end());
+          TileOut T;
+          T.row0 = int32_t(r0);
+          T.nrows = int32_t(r1 - r0);
+          for (size_t q = 0; q < ent.size();) {
+            int32_t c0 = ent[q].first;
+            size_t base = T.bits.size();
+            T.col0.push_back(c0);
+            T.bits.resize(base + TILE_M, 0u);
+            for (; q < ent.size() && ent[q].first == c0; ++q)
+              T.bits[base + (ent[q].second >> 5)] |= 1u << (ent[q].second & 31);
+          }
+          tiles[k].push_back(std::move(T));
+        }
+      }
+      for (int64_t j = bptr[k]; j < bptr[k + 1]; ++j) dense_i[p->blk_i[j]] = 0;
+    }
+  });
+  p->sp_rowptr.assign(n + 1, 0);
+  for (int64_t v = 0; v < n; ++v) p->sp_rowptr[v + 1] = p->sp_rowptr[v] + sp_cnt[v];
+  p->sp_col.resize(p->sp_rowptr[n]);
+  parallel_for(P, [&](int, int64_t a, int64_t b) {
+    std::vector<uint8_t> dense_i(P, 0);
+    for (int64_t k = a; k < b; ++k) {
+      for (int64_t j = bptr[k]; j < bptr[k + 1]; ++j) dense_i[p->blk_i[j]] = p->blk_dense[j];
+      for (int64_t v = p->pstart[k]; v < p->pstart[k + 1]; ++v) {
+        int64_t o2 = p->sp_rowptr[v];
+        for (int64_t e = tptr[v]; e < tptr[v + 1]; ++e)
+          if (!dense_i[pid[tcol[e]]]) p->sp_col[o2++] = tcol[e];
+      }
+      for (int64_t j = bptr[k]; j < bptr[k + 1]; ++j) dense_i[p->blk_i[j]] = 0;
+    }
+  });
+  p->rt_cptr.assign(1, 0);
+  p->zd_index.assign(n, -1);
+  std::vector<int64_t> part_rt(P + 1, 0);  // row-tile range of each partition
+  for (int32_t k = 0; k < P; ++k) {
+    part_rt[k] = int64_t(p->rt_row0.size());
+    for (auto& T : tiles[k]) {
+      int64_t t = int64_t(p->rt_row0.size());
+      p->rt_row0.push_back(T.row0);
+      p->rt_nrows.push_back(T.nrows);
+      p->ch_col0.insert(p->ch_col0.end(), T.col0.begin(), T.col0.end());
+      p->bits.insert(p->bits.end(), T.bits.begin(), T.bits.end());
+      p->rt_cptr.push_back(int64_t(p->ch_col0.size()));
+      for (int32_t rr = 0; rr < T.nrows; ++rr) p->zd_index[T.row0 + rr] = int32_t(t * TILE_M + rr);
+    }
+    std::vector<TileOut>().swap(tiles[k]);
+  }
+  part_rt[P] = int64_t(p->rt_row0.size());
+
+  // shard: contiguous partition ranges balanced by a cost model
+  {
+    std::vector<double> cost(P, 0.0);
+    for (int32_t k = 0; k < P; ++k) {
+      int64_t sp = p->sp_rowptr[p->pstart[k + 1]] - p->sp_rowptr[p->pstart[k]];
+      int64_t ch = p->rt_cptr[part_rt[k + 1]] - p->rt_cptr[part_rt[k]];
+      cost[k] = double(sp) + 16.0 * double(ch) + double(psize[k]);
+    }
+    double tot = 0;
+    for (double c : cost) tot += c;
+    auto bound = [&](int32_t q) -> int32_t {
+      if (q <= 0) return 0;
+      if (q >= o->world) return P;
+      double target = tot * double(q) / double(o->world), run = 0;
+      for (int32_t k = 0; k < P; ++k) {
+        if (run >= target) return k;
+        run += cost[k];
+      }
+      return P;
+    };
+    p->k_lo = bound(o->rank);
+    p->k_hi = bound(o->rank + 1);
+    p->row_lo = p->pstart[p->k_lo];
+    p->row_hi = p->pstart[p->k_hi];
+    p->rt_lo = part_rt[p->k_lo];
+    p->rt_hi = part_rt[p->k_hi];
+  }
+
+  // stats
+  pcgcn_stats& S = p->stats;
+  std::memset(&S, 0, sizeof(S));
+  S.n = n; S.nnz = p->nnz_t; S.P = P; S.lp_sweeps = p->sweeps; S.clusters = p->clusters;
+  S.blocks_nonempty = nb; S.blocks_dense = nb_dense;
+  S.nnz_sparse = p->sp_rowptr[n]; S.nnz_dense = p->nnz_t - p->sp_rowptr[n];
+  S.intra_edges = intra;
+  S.row_tiles = int64_t(p->rt_row0.size()); S.chunks = int64_t(p->ch_col0.size());
+  S.row_lo = p->row_lo; S.row_hi = p->row_hi;
+  S.shard_nnz_sparse = p->sp_rowptr[p->row_hi] - p->sp_rowptr[p->row_lo];
+  S.shard_chunks = p->rt_cptr[p->rt_hi] - p->rt_cptr[p->rt_lo];
+  S.theta = theta;
+  S.partition_ms = part_ms;
+  S.plan_ms = ms_since(t0);
+  return PCGCN_OK;
+}
+
+}  // namespace pcgcn

@@ -1,0 +1,193 @@
+// Selective-mode ("sparse") aggregation of PCGCN on sm_100a, plus the input
+// prescale / tf32-split pass that feeds both modes.
+//
+// Paper: §III-B.a (L137, L149) and §IV-B (L177-L181, Fig. 6).  The selective
+// blocks of all partition pairs are merged into one CSR (L179); per edge the
+// kernel decodes the source index, fetches the source feature row, multiplies
+// by the edge value and accumulates into the destination (L149); "consecutive
+// threads process consecutive dimensions of the feature vector and update the
+// accumulated intermediate data in registers" and each destination row is
+// written once (L181).
+//
+// B200 design:
+//   * one warp per destination row; the 32 lanes split into S = 32/G edge
+//     slots of G lanes, each lane owning one float4 of the row (F <= 128) or
+//     two (F <= 256) — full lane use for narrow F (41 -> G=16, S=2);
+//   * the warp loads 32 source indices with one coalesced load and broadcasts
+//     them by shuffle; the unrolled loop keeps up to 32/S independent 16-byte
+//     row loads in flight per lane (the gather is L2-bandwidth bound);
+//   * edge values are not stored: Â_ij = r_i r_j, with r_j folded into the
+//     producer (IN_PRESCALED) and r_i applied once in the epilogue;
+//   * fused epilogue: + dense-mode partial sum Zd (mode combine, L193),
+//     × r_i, optional second × r_i, ReLU and the bit-packed ReLU mask;
+//   * fixed summation order (4 interleaved accumulators, then a butterfly over
+//     slots): bitwise reproducible run to run.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdint>
+
+#include "kernels.h"
+
+namespace pcgcn {
+namespace {
+
+__device__ __forceinline__ float4 ld_f4(const float* p) {
+  return __ldg(reinterpret_cast<const float4*>(p));
+}
+__device__ __forceinline__ void add4(float4& a, const float4& b) {
+  a.x += b.x; a.y += b.y; a.z += b.z; a.w += b.w;
+}
+
+template <int G, int V, bool HAS_ZD>
+__global__ void __launch_bounds__(256) sparse_agg_kernel(AggArgs a) {
+  constexpr int S = 32 / G;       // edge slots per warp
+  constexpr int STEPS = 32 / S;   // edges per slot per index batch
+  const int64_t row = int64_t(blockIdx.x) * 8 + (threadIdx.x >> 5);
+  if (row >= a.rows) return;
+  const int lane = threadIdx.x & 31;
+  const int slot = lane / G, l = lane % G;
+  const int nvec = (a.F + 3) >> 2;
+  const int64_t e0 = a.rowptr[row], e1 = a.rowptr[row + 1];
+  float4 acc[4][V];
+#pragma unroll
+  for (int u = 0; u < 4; ++u)
+#pragma unroll
+    for (int v = 0; v < V; ++v) acc[u][v] = make_float4(0.f, 0.f, 0.f, 0.f);
+
+  for (int64_t base = e0; base < e1; base += 32) {
+    const int cnt = (e1 - base) < 32 ? int(e1 - base) : 32;
+    const int myidx = lane < cnt ? __ldg(a.col + base + lane) : 0;
+#pragma unroll
+    for (int k = 0; k < STEPS; ++k) {
+      const int eb = k * S + slot;
+      const int j = __shfl_sync(0xffffffffu, myidx, eb);
+      if (eb < cnt) {
+        const float* src = a.Y + int64_t(j) * a.ldy;
+#pragma unroll
+        for (int v = 0; v < V; ++v) {
+          const int q = l + G * v;
+          if (q < nvec) add4(acc[k & 3][v], ld_f4(src + 4 * q));
+        }
+      }
+    }
+  }
+  float4 tot[V];
+#pragma unroll
+  for (int v = 0; v < V; ++v) {
+    tot[v] = acc[0][v];
+    add4(tot[v], acc[1][v]);
+    float4 t2 = acc[2][v];
+    add4(t2, acc[3][v]);
+    add4(tot[v], t2);
+#pragma unroll
+    for (int off = G; off < 32; off <<= 1) {
+      tot[v].x += __shfl_xor_sync(0xffffffffu, tot[v].x, off);
+      tot[v].y += __shfl_xor_sync(0xffffffffu, tot[v].y, off);
+      tot[v].z += __shfl_xor_sync(0xffffffffu, tot[v].z, off);
+      tot[v].w += __shfl_xor_sync(0xffffffffu, tot[v].w, off);
+    }
+  }
+  const float ri = a.r[a.row_lo + row];
+  const int zi = HAS_ZD ? a.zd_index[row] : -1;
+  const int mw = (a.F + 31) >> 5;
+#pragma unroll
+  for (int v = 0; v < V; ++v) {
+    const int q = l + G * v;
+    const bool own = slot == 0 && q < nvec;
+    float4 z = tot[v];
+    if (HAS_ZD && own && zi >= 0) add4(z, ld_f4(a.zd + int64_t(zi) * a.ldzd + 4 * q));
+    z.x *= ri; z.y *= ri; z.z *= ri; z.w *= ri;
+    if (a.out_prescaled) { z.x *= ri; z.y *= ri; z.z *= ri; z.w *= ri; }
+    if (a.mask) {
+      const int c = 4 * q;
+      uint32_t nib = 0;
+      if (own) {
+        nib |= (z.x > 0.f && c + 0 < a.F) ? 1u : 0u;
+        nib |= (z.y > 0.f && c + 1 < a.F) ? 2u : 0u;
+        nib |= (z.z > 0.f && c + 2 < a.F) ? 4u : 0u;
+        nib |= (z.w > 0.f && c + 3 < a.F) ? 8u : 0u;
+      }
+      uint32_t w = nib << (4 * (q & 7));
+      w |= __shfl_xor_sync(0xffffffffu, w, 1);
+      w |= __shfl_xor_sync(0xffffffffu, w, 2);
+      w |= __shfl_xor_sync(0xffffffffu, w, 4);
+      if (own && (q & 7) == 0) a.mask[row * mw + (q >> 3)] = w;
+    }
+    if (a.relu) {
+      z.x = fmaxf(z.x, 0.f); z.y = fmaxf(z.y, 0.f); z.z = fmaxf(z.z, 0.f); z.w = fmaxf(z.w, 0.f);
+    }
+    if (own) *reinterpret_cast<float4*>(a.Z + row * a.ldz + 4 * q) = z;
+  }
+}
+
+template <int G, int V>
+cudaError_t launch_gv(const AggArgs& a, cudaStream_t s) {
+  dim3 grid(unsigned((a.rows + 7) / 8));
+  if (a.zd_index)
+    sparse_agg_kernel<G, V, true><<<grid, 256, 0, s>>>(a);
+  else
+    sparse_agg_kernel<G, V, false><<<grid, 256, 0, s>>>(a);
+  return cudaGetLastError();
+}
+
+__global__ void prescale_split_kernel(const float* __restrict__ Y, int64_t ldy,
+                                      const float* __restrict__ r, int64_t n, int F,
+                                      float* __restrict__ ypre, int64_t ldpre,
+                                      float* __restrict__ yhi, float* __restrict__ ylo,
+                                      int64_t ldhl) {
+  const int nvec = (F + 3) >> 2;
+  const int cvec = yhi ? int(ldhl >> 2) : nvec;  // hi/lo rows are written to their full padded width
+  const int64_t total = n * cvec;
+  for (int64_t idx = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; idx < total;
+       idx += int64_t(gridDim.x) * blockDim.x) {
+    const int64_t i = idx / cvec;
+    const int q = int(idx - i * cvec);
+    float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
+    if (q < nvec) {
+      v = ld_f4(Y + i * ldy + 4 * q);
+      if (r) {
+        const float ri = __ldg(r + i);
+        v.x *= ri; v.y *= ri; v.z *= ri; v.w *= ri;
+      }
+      if (ypre) *reinterpret_cast<float4*>(ypre + i * ldpre + 4 * q) = v;
+    }
+    if (yhi) {
+      float4 h;
+      h.x = __uint_as_float(__float_as_uint(v.x) & 0xffffe000u);
+      h.y = __uint_as_float(__float_as_uint(v.y) & 0xffffe000u);
+      h.z = __uint_as_float(__float_as_uint(v.z) & 0xffffe000u);
+      h.w = __uint_as_float(__float_as_uint(v.w) & 0xffffe000u);
+      float4 lo = make_float4(v.x - h.x, v.y - h.y, v.z - h.z, v.w - h.w);
+      *reinterpret_cast<float4*>(yhi + i * ldhl + 4 * q) = h;
+      *reinterpret_cast<float4*>(ylo + i * ldhl + 4 * q) = lo;
+    }
+  }
+}
+
+}  // namespace
+
+cudaError_t launch_sparse_agg(const AggArgs& a, cudaStream_t s) {
+  if (a.rows <= 0) return cudaSuccess;
+  const int nvec = (a.F + 3) / 4;
+  if (nvec <= 1) return launch_gv<1, 1>(a, s);
+  if (nvec <= 2) return launch_gv<2, 1>(a, s);
+  if (nvec <= 4) return launch_gv<4, 1>(a, s);
+  if (nvec <= 8) return launch_gv<8, 1>(a, s);
+  if (nvec <= 16) return launch_gv<16, 1>(a, s);
+  if (nvec <= 32) return launch_gv<32, 1>(a, s);
+  return launch_gv<32, 2>(a, s);
+}
+
+cudaError_t launch_prescale_split(const float* Y, int64_t ldy, const float* r, int64_t n, int F,
+                                  float* ypre, int64_t ldpre, float* yhi, float* ylo, int64_t ldhl,
+                                  cudaStream_t s) {
+  if (n <= 0) return cudaSuccess;
+  const int cvec = yhi ? int(ldhl / 4) : (F + 3) / 4;
+  int64_t total = n * cvec;
+  int blocks = int(std::min<int64_t>((total + 255) / 256, 148 * 16));
+  prescale_split_kernel<<<blocks, 256, 0, s>>>(Y, ldy, r, n, F, ypre, ldpre, yhi, ylo, ldhl);
+  return cudaGetLastError();
+}
+
+}  // namespace pcgcn

@@ -1,0 +1,159 @@
+"""2-layer GCN training step on the PCGCN C ABI.
+
+Alg. 1 with L = 2 — per layer: transform a^l = h^{l-1} w^l
+(L114, pcgcn_gemm_xw) then partition-centric propagation (L118-L121,
+pcgcn_forward) — followed by the softmax-CE loss, the backward through both
+layers (pcgcn_backward reuses the forward plan since Âᵀ = Â) and the update.
+PyTorch only owns device memory, the stream and (optionally) the CUDA graph;
+every arithmetic step runs in libpcgcn's kernels.
+
+Prescaling: Â = D̃^-½ Ã D̃^-½, so every producer of an aggregation input writes
+diag(r)·Y (r = d̃^-½) and the aggregation applies r_i once in its epilogue:
+    a4  Y0' = diag(r)·X·Θ0                 gemm_xw(rowscale=r)
+    a5/6 H1 = ReLU(Â X Θ0), mask1          forward(IN_PRESCALED|RELU|MASK_OUT)
+    a7  Y1' = diag(r)·H1·Θ1                gemm_xw(rowscale=r)
+    a8  Lg  = Â H1 Θ1                      forward(IN_PRESCALED)
+    a9  loss, dL' = diag(r)·dL             softmax_ce(rowscale=r)
+    a10 G1  = Â dL                          backward(IN_PRESCALED)
+    a11 ∇Θ1 = H1ᵀ G1 ; dP1' = diag(r)((G1Θ1ᵀ)⊙mask1)   gemm_xtg, gemm_dwt
+    a12 G0  = Â dP1                         backward(IN_PRESCALED)
+    a13 ∇Θ0 = Xᵀ G0                         gemm_xtg
+    a14 Θ ← Adam/SGD(Θ, ∇Θ)  (all-reduce of ∇Θ first when sharded)
+"""
+from __future__ import annotations
+
+import numpy as np
+import torch
+
+from . import _lib as L
+
+
+def _ld(F: int) -> int:
+    return (F + 3) // 4 * 4
+
+
+class GCN2:
+    def __init__(self, plan: L.Plan, X_plan: np.ndarray, labels_plan: np.ndarray, train_plan: np.ndarray,
+                 Th0: np.ndarray, Th1: np.ndarray, *, optimizer: str = "adam", lr: float = 0.01,
+                 device: str | torch.device = "cuda", exchange=None):
+        """All row-indexed host arrays are already in plan order (X_plan = X[perm]).
+        ``exchange`` (sharded runs): object with ``gather(local, full)`` and
+        ``allreduce(t)``; rows owned here are plan.row_lo:plan.row_hi."""
+        self.plan = plan
+        self.dev = torch.device(device)
+        self.n = plan.n
+        self.lo, self.hi = plan.row_lo, plan.row_hi
+        self.rows = self.hi - self.lo
+        self.f_in = X_plan.shape[1]
+        self.H = Th0.shape[1]
+        self.C = Th1.shape[1]
+        self.optimizer = optimizer
+        self.lr = lr
+        self.exchange = exchange
+        assert max(self.H, self.C) <= plan.f_max
+        d, f32 = self.dev, torch.float32
+        n, rows, H, C = self.n, self.rows, self.H, self.C
+        self.ldH, self.ldC = _ld(H), _ld(C)
+        self.X = torch.from_numpy(np.ascontiguousarray(X_plan[self.lo:self.hi], dtype=np.float32)).to(d)
+        self.labels = torch.from_numpy(np.ascontiguousarray(labels_plan[self.lo:self.hi], dtype=np.int32)).to(d)
+        self.train = torch.from_numpy(np.ascontiguousarray(train_plan[self.lo:self.hi], dtype=np.uint8)).to(d)
+        self.inv_nT = 1.0 / float(np.count_nonzero(train_plan))
+        # parameters (flat, Θ0 then Θ1) and optimiser state
+        self.theta = torch.from_numpy(np.concatenate([Th0.ravel(), Th1.ravel()]).astype(np.float32)).to(d)
+        self.Th0 = self.theta[: self.f_in * H].view(self.f_in, H)
+        self.Th1 = self.theta[self.f_in * H:].view(H, C)
+        self.grad = torch.zeros_like(self.theta)
+        self.gTh0 = self.grad[: self.f_in * H].view(self.f_in, H)
+        self.gTh1 = self.grad[self.f_in * H:].view(H, C)
+        self.m = torch.zeros_like(self.theta)
+        self.v = torch.zeros_like(self.theta)
+        self.step_ctr = torch.zeros(1, dtype=torch.int32, device=d)
+        # activations: inputs of aggregations span all n rows (sources), outputs the shard
+        self.Y0 = torch.zeros(n, self.ldH, dtype=f32, device=d)
+        self.H1 = torch.zeros(rows, self.ldH, dtype=f32, device=d)
+        self.mask1 = torch.zeros(rows, (H + 31) // 32, dtype=torch.int32, device=d)
+        self.Y1 = torch.zeros(n, self.ldC, dtype=f32, device=d)
+        self.Lg = torch.zeros(rows, self.ldC, dtype=f32, device=d)
+        self.dL = torch.zeros(n, self.ldC, dtype=f32, device=d)
+        self.G1 = torch.zeros(rows, self.ldC, dtype=f32, device=d)
+        self.dP1 = torch.zeros(n, self.ldH, dtype=f32, device=d)
+        self.G0 = torch.zeros(rows, self.ldH, dtype=f32, device=d)
+        self.loss = torch.zeros(1, dtype=f32, device=d)
+        self.ce_work = torch.zeros(L.CE_WORK_FLOATS, dtype=f32, device=d)
+        wk = max(L.gemm_xtg_work_floats(rows, self.f_in, H), L.gemm_xtg_work_floats(rows, H, C))
+        self.xtg_work = torch.zeros(max(wk, 1), dtype=f32, device=d)
+        self.r = plan.rowscale_ptr()  # device [n]
+        self.r_local = None if self.lo == 0 else self.r + 4 * self.lo
+        self._graph = None
+
+    # -- one epoch -------------------------------------------------------
+    def _r_rows(self):
+        import ctypes
+        return ctypes.c_void_p(self.r + 4 * self.lo) if self.lo else ctypes.c_void_p(self.r)
+
+    def _local(self, full):
+        return full[self.lo:self.hi]
+
+    def _gather(self, full):
+        if self.exchange is not None:
+            self.exchange.gather(full, self.lo, self.hi)
+
+    def epoch(self, stream=None):
+        rr = self._r_rows()
+        H, C, p = self.H, self.C, self.plan
+        # layer 1
+        L.gemm_xw(self.X, self.Th0, rr, self._local(self.Y0), M=self.rows, K=self.f_in, N=H, stream=stream)
+        self._gather(self.Y0)
+        p.forward(self.Y0, self.H1, F=H, flags=L.IN_PRESCALED | L.RELU | L.MASK_OUT, mask=self.mask1,
+                  stream=stream)
+        # layer 2
+        L.gemm_xw(self.H1, self.Th1, rr, self._local(self.Y1), M=self.rows, K=H, N=C, stream=stream)
+        self._gather(self.Y1)
+        p.forward(self.Y1, self.Lg, F=C, flags=L.IN_PRESCALED, stream=stream)
+        # loss
+        L.softmax_ce(self.Lg, self.labels, self.train, self.inv_nT, rr, self._local(self.dL), self.loss,
+                     self.ce_work, M=self.rows, C=C, stream=stream)
+        self._gather(self.dL)
+        # backward
+        p.backward(self.dL, self.G1, F=C, flags=L.IN_PRESCALED, stream=stream)
+        L.gemm_xtg(self.H1, self.G1, self.gTh1, self.xtg_work, M=self.rows, K=H, N=C, stream=stream)
+        L.gemm_dwt(self.G1, self.Th1, self.mask1, rr, self._local(self.dP1), M=self.rows, N=C, K=H,
+                   stream=stream)
+        self._gather(self.dP1)
+        p.backward(self.dP1, self.G0, F=H, flags=L.IN_PRESCALED, stream=stream)
+        L.gemm_xtg(self.X, self.G0, self.gTh0, self.xtg_work, M=self.rows, K=self.f_in, N=H, stream=stream)
+        if self.exchange is not None:
+            self.exchange.allreduce(self.grad)
+            self.exchange.allreduce(self.loss)
+        # update
+        if self.optimizer == "adam":
+            L.adam(self.theta, self.grad, self.m, self.v, self.lr, self.step_ctr, stream=stream)
+        elif self.optimizer == "sgd":
+            L.sgd(self.theta, self.grad, self.lr, stream=stream)
+
+    def launches_per_epoch(self) -> int:
+        """Kernel launches of libpcgcn per epoch (for the bench's gpu_launches)."""
+        st = self.plan.stats()
+        dense = st["shard_chunks"] > 0
+        agg = 1 + (2 if dense else 0)          # prescale/split + dense tiles + selective rows
+        gemm_xw = 1 + 1                          # tile kernel + pad zeroing (ld > N) — upper bound
+        n = 2 * gemm_xw + 4 * agg + 2 + 2 * 2 + 2  # + softmax(2) + 2 x xtg(2) + dwt(2)
+        n += 2 if self.optimizer == "adam" else 1
+        return n
+
+    # -- CUDA graph ------------------------------------------------------
+    def capture(self, warmup: int = 2):
+        s = torch.cuda.Stream(device=self.dev)
+        s.wait_stream(torch.cuda.current_stream(self.dev))
+        with torch.cuda.stream(s):
+            for _ in range(warmup):
+                self.epoch(stream=s)
+        torch.cuda.current_stream(self.dev).wait_stream(s)
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=s):
+            self.epoch(stream=s)
+        self._graph = g
+        return g
+
+    def replay(self):
+        self._graph.replay()

@@ -1,0 +1,330 @@
+"""GPU parity: the CUDA path through the C ABI vs the fp64 oracle on the same
+seeded inputs (run on a B200: pytest -m gpu).
+
+Error metric (reading #18): condition-scaled
+    err = max_{i,f} |z - z*| / (|Â|·|Y|)_{i,f}
+which equals the plain relative error for nonnegative inputs and is immune to
+cancellation in mixed-sign sums.  Gates (BASELINE.json north_star):
+sparse fp32 <= 1e-5, dense tcgen05 2xTF32 <= 1e-5, integer-exact regime
+bitwise; plan arrays bit-exact (tests/test_plan_abi.py).
+"""
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+from oracle import gcn as O  # noqa: E402
+from synth import configs as C  # noqa: E402
+from synth import graphs as G  # noqa: E402
+
+L = pytest.importorskip("paper_conf_ipps_tianmyd20_b200._lib")
+
+TOL = 1e-5
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _gpu():
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    torch.cuda.init()
+
+
+def _ld(F):
+    return (F + 3) // 4 * 4
+
+
+def aggregate_gpu(g, Y, P, theta, *, dense=L.DENSE_TF32X2, norm=L.NORM_SYM, part=None, backward=False,
+                  flags=0, f_max=None):
+    F = Y.shape[1]
+    f_max = f_max or max(128, F)
+    pl = L.Plan(g.n, g.rowptr, g.col, P, theta, norm=norm, dense_prec=dense, part=part, f_max=f_max)
+    perm = pl.perm()
+    Yp = np.zeros((g.n, _ld(F)), dtype=np.float32)
+    Yp[:, :F] = Y[perm]
+    Yd = torch.from_numpy(Yp).cuda()
+    Zd = torch.full((g.n, _ld(F)), float("nan"), device="cuda")
+    if backward:
+        pl.backward(Yd, Zd, F=F, flags=flags)
+    else:
+        pl.forward(Yd, Zd, F=F, flags=flags)
+    torch.cuda.synchronize()
+    Z = np.empty((g.n, F), dtype=np.float64)
+    Z[perm] = Zd.cpu().numpy()[:, :F]
+    return Z, pl, Zd
+
+
+def cond_err(g, Y, Z, norm="sym"):
+    Ahat = O.normalized_adjacency(g.n, g.rowptr, g.col, norm)[0]
+    Zs = O.aggregate(Ahat, Y.astype(np.float64))
+    scale = O.aggregate(abs(Ahat), np.abs(Y.astype(np.float64)))
+    scale = np.maximum(scale, 1e-30)
+    return float(np.max(np.abs(Z - Zs) / scale)), Zs
+
+
+def _feat(n, F, seed, nonneg=False):
+    rng = np.random.default_rng(seed)
+    Y = rng.standard_normal((n, F)).astype(np.float32)
+    return np.abs(Y) if nonneg else Y
+
+
+SMALL = {
+    "path": lambda: G.path(37),
+    "cycle": lambda: G.cycle(300),
+    "star": lambda: G.star(260),
+    "complete": lambda: G.complete(150),
+    "cliques": lambda: G.cliques([130, 70, 200, 5, 1], seed=2),
+    "empty": lambda: G.empty(77),
+    "messy": lambda: G.messy_random(700, 4000, 3),
+    "cora": lambda: G.sbm(C.CORA.spec),
+}
+
+
+@pytest.mark.parametrize("name", list(SMALL))
+@pytest.mark.parametrize("mode", ["sparse", "dense_tc", "dense_simt", "hybrid"])
+@pytest.mark.parametrize("F", [1, 7, 16, 41, 128])
+def test_aggregation_parity(name, mode, F):
+    g = SMALL[name]()
+    P = max(1, min(8, g.n // 40))
+    theta = {"sparse": 2.0, "dense_tc": 0.0, "dense_simt": 0.0, "hybrid": 0.05}[mode]
+    dense = L.DENSE_FP32_SIMT if mode == "dense_simt" else L.DENSE_TF32X2
+    Y = _feat(g.n, F, 11)
+    Z, pl, _ = aggregate_gpu(g, Y, P, theta, dense=dense)
+    err, _ = cond_err(g, Y, Z)
+    assert err <= TOL, (name, mode, F, err, pl.stats())
+
+
+def test_closed_forms_complete_and_cycle_dense():
+    g = G.complete(200)
+    Y = _feat(g.n, 64, 3)
+    Z, pl, _ = aggregate_gpu(g, Y, 1, 0.0)
+    assert pl.stats()["nnz_dense"] == 200 * 200
+    np.testing.assert_allclose(Z, np.repeat(Y.astype(np.float64).mean(0, keepdims=True), 200, 0),
+                               rtol=2e-6, atol=2e-6)
+    g = G.cycle(500)
+    Y = _feat(g.n, 16, 4)
+    Z, _, _ = aggregate_gpu(g, Y, 5, 2.0)
+    exp = (np.roll(Y, 1, 0) + Y + np.roll(Y, -1, 0)).astype(np.float64) / 3.0
+    np.testing.assert_allclose(Z, exp, rtol=1e-5, atol=1e-6)
+
+
+@pytest.mark.parametrize("mode", ["sparse", "dense_tc", "dense_simt", "hybrid"])
+def test_integer_exact_bitwise(mode):
+    """Pin P9: Ã unnormalised, small integers -> every order gives the exact
+    sum, so GPU (either mode, any partition) == oracle bitwise."""
+    g = G.cliques([300, 129, 64, 33, 2], seed=5)
+    rng = np.random.default_rng(9)
+    Y = rng.integers(-1000, 1000, size=(g.n, 40)).astype(np.float32)
+    theta = {"sparse": 2.0, "dense_tc": 0.0, "dense_simt": 0.0, "hybrid": 0.3}[mode]
+    dense = L.DENSE_FP32_SIMT if mode == "dense_simt" else L.DENSE_TF32X2
+    Z, _, _ = aggregate_gpu(g, Y, 5, theta, dense=dense, norm=L.NORM_NONE)
+    exp = O.aggregate(O.normalized_adjacency(g.n, g.rowptr, g.col, "none")[0], Y.astype(np.float64))
+    assert np.array_equal(Z, exp)
+
+
+def test_partition_invariance_integer_regime():
+    """L131 §III-A.c: only the summation order changes — bitwise under P9."""
+    g = G.sbm(C.CORA.spec)
+    Y = np.random.default_rng(1).integers(-50, 50, size=(g.n, 16)).astype(np.float32)
+    outs = []
+    for P, theta, part in ((8, 0.05, None), (3, 2.0, None), (8, 0.0, None),
+                           (6, 0.01, np.random.default_rng(2).integers(0, 6, g.n))):
+        Z, _, _ = aggregate_gpu(g, Y, P, theta, norm=L.NORM_NONE, part=part)
+        outs.append(Z)
+    for Z in outs[1:]:
+        assert np.array_equal(Z, outs[0])
+
+
+def test_relabel_invariance_tolerance():
+    g = G.sbm(C.CORA.spec)
+    Y = _feat(g.n, 16, 3)
+    Z1, _, _ = aggregate_gpu(g, Y, 8, 0.05)
+    perm = np.random.default_rng(3).permutation(g.n)
+    inv = np.argsort(perm)
+    # relabel vertex v -> inv[v]
+    rows = np.repeat(np.arange(g.n), np.diff(g.rowptr))
+    g2 = G.from_edges(g.n, list(zip(inv[rows], inv[g.col])), symmetrize=False)
+    Z2, _, _ = aggregate_gpu(g2, Y[perm], 8, 0.05)
+    np.testing.assert_allclose(Z2, Z1[perm], rtol=1e-5, atol=1e-6)
+
+
+def test_backward_equals_forward_and_deterministic():
+    g = G.sbm(C.PUBMED.spec)
+    Y = _feat(g.n, 16, 8)
+    Zf, _, Zf_d = aggregate_gpu(g, Y, 32, 0.02)
+    Zb, _, Zb_d = aggregate_gpu(g, Y, 32, 0.02, backward=True)
+    assert torch.equal(Zf_d, Zb_d)
+    Z2, _, Z2_d = aggregate_gpu(g, Y, 32, 0.02)
+    assert torch.equal(Zf_d, Z2_d)
+
+
+def test_epilogue_flags_relu_mask_prescaled():
+    g = G.sbm(C.CORA.spec)
+    F = 41
+    Y = _feat(g.n, F, 12)
+    pl = L.Plan(g.n, g.rowptr, g.col, 8, 0.03)
+    perm = pl.perm()
+    Ahat, dt, r = O.normalized_adjacency(g.n, g.rowptr, g.col)
+    Zs = O.aggregate(Ahat, Y.astype(np.float64))[perm]
+    rp = r[perm][:, None]
+    Yp = np.zeros((g.n, 44), np.float32)
+    Yp[:, :F] = (Y[perm] * rp).astype(np.float32)  # prescaled input
+    Yd = torch.from_numpy(Yp).cuda()
+    Z = torch.zeros(g.n, 44, device="cuda")
+    mask = torch.zeros(g.n, 2, dtype=torch.int32, device="cuda")
+    pl.forward(Yd, Z, F=F, flags=L.IN_PRESCALED | L.RELU | L.MASK_OUT | L.OUT_PRESCALED, mask=mask)
+    torch.cuda.synchronize()
+    Zc = Z.cpu().numpy()[:, :F].astype(np.float64)
+    np.testing.assert_allclose(Zc, np.maximum(Zs, 0) * rp, rtol=1e-5, atol=1e-6)
+    m = mask.cpu().numpy().view(np.uint32)
+    bits = ((m[:, :, None] >> np.arange(32, dtype=np.uint32)) & 1).reshape(g.n, 64)[:, :F]
+    agree = bits.astype(bool) == (Zs > 0)
+    near0 = np.abs(Zs) < 1e-6
+    assert np.all(agree | near0)
+    assert np.all(bits.reshape(g.n, 64)[:, F:] == 0) if bits.shape[1] > F else True
+
+
+def _np(t):
+    return t.detach().cpu().numpy().astype(np.float64)
+
+
+@pytest.mark.parametrize("M,K,N", [(1000, 602, 128), (2708, 1433, 16), (777, 128, 41), (5, 3, 7)])
+def test_gemms(M, K, N):
+    rng = np.random.default_rng(M + K + N)
+    X = torch.from_numpy(rng.standard_normal((M, K)).astype(np.float32)).cuda()
+    W = torch.from_numpy(rng.standard_normal((K, N)).astype(np.float32)).cuda()
+    s = torch.from_numpy(rng.random(M).astype(np.float32) + 0.5).cuda()
+    ldn = _ld(N)
+    Y = torch.full((M, ldn), float("nan"), device="cuda")
+    import ctypes
+    L.gemm_xw(X, W, ctypes.c_void_p(s.data_ptr()), Y, N=N)
+    torch.cuda.synchronize()
+    exp = _np(s)[:, None] * (_np(X) @ _np(W))
+    scale = _np(s)[:, None] * (np.abs(_np(X)) @ np.abs(_np(W)))
+    assert np.max(np.abs(_np(Y)[:, :N] - exp) / scale) < TOL
+    assert np.all(_np(Y)[:, N:] == 0)
+    # Xᵀ D
+    D = torch.from_numpy(rng.standard_normal((M, N)).astype(np.float32)).cuda()
+    Gm = torch.zeros(K, N, device="cuda")
+    work = torch.zeros(L.gemm_xtg_work_floats(M, K, N), device="cuda")
+    L.gemm_xtg(X, D, Gm, work)
+    torch.cuda.synchronize()
+    exp = _np(X).T @ _np(D)
+    scale = np.abs(_np(X)).T @ np.abs(_np(D))
+    assert np.max(np.abs(_np(Gm) - exp) / scale) < TOL
+    # diag(s)((D Wᵀ) ⊙ mask)  with W [K2 x N]
+    K2 = K
+    W2 = torch.from_numpy(rng.standard_normal((K2, N)).astype(np.float32)).cuda()
+    mw = (K2 + 31) // 32
+    mbits = rng.integers(0, 2**32, size=(M, mw), dtype=np.uint64).astype(np.uint32)
+    mask = torch.from_numpy(mbits.view(np.int32)).cuda()
+    O_ = torch.full((M, _ld(K2)), float("nan"), device="cuda")
+    L.gemm_dwt(D, W2, mask, ctypes.c_void_p(s.data_ptr()), O_)
+    torch.cuda.synchronize()
+    mk = ((mbits[:, :, None] >> np.arange(32, dtype=np.uint32)) & 1).reshape(M, mw * 32)[:, :K2]
+    exp = _np(s)[:, None] * ((_np(D) @ _np(W2).T) * mk)
+    scale = _np(s)[:, None] * (np.abs(_np(D)) @ np.abs(_np(W2)).T) + 1e-30
+    assert np.max(np.abs(_np(O_)[:, :K2] - exp) / scale) < TOL
+
+
+def test_softmax_ce_and_adam():
+    rng = np.random.default_rng(4)
+    M, Cc = 5000, 41
+    Lg = rng.standard_normal((M, Cc)).astype(np.float32) * 3
+    y = rng.integers(0, Cc, M).astype(np.int32)
+    T = rng.random(M) < 0.8
+    Ld = torch.zeros(M, 44, device="cuda")
+    Ld[:, :Cc] = torch.from_numpy(Lg).cuda()
+    dL = torch.zeros_like(Ld)
+    loss = torch.zeros(1, device="cuda")
+    work = torch.zeros(L.CE_WORK_FLOATS, device="cuda")
+    L.softmax_ce(Ld, torch.from_numpy(y).cuda(), torch.from_numpy(T.astype(np.uint8)).cuda(), 1.0 / T.sum(),
+                 None, dL, loss, work, C=Cc)
+    torch.cuda.synchronize()
+    l_ref, dL_ref = O.softmax_ce(Lg, y, T)
+    assert abs(loss.item() - l_ref) <= 1e-5 * abs(l_ref)
+    np.testing.assert_allclose(_np(dL)[:, :Cc], dL_ref, rtol=0, atol=1e-7 / T.sum() * 50)
+    # Adam: two steps vs oracle
+    th = rng.standard_normal(1000).astype(np.float32)
+    gs = [rng.standard_normal(1000).astype(np.float32) for _ in range(2)]
+    td = torch.from_numpy(th.copy()).cuda()
+    m = torch.zeros_like(td)
+    v = torch.zeros_like(td)
+    step = torch.zeros(1, dtype=torch.int32, device="cuda")
+    ref, mr, vr = th.astype(np.float64), np.zeros(1000), np.zeros(1000)
+    for t, g_ in enumerate(gs, 1):
+        L.adam(td, torch.from_numpy(g_).cuda(), m, v, 0.01, step)
+        ref, mr, vr = O.adam(ref, g_.astype(np.float64), mr, vr, t)
+    torch.cuda.synchronize()
+    assert step.item() == 2
+    np.testing.assert_allclose(_np(td), ref, rtol=1e-5, atol=1e-6)
+
+
+@pytest.mark.parametrize("wname,theta", [("cora", 0.05), ("pubmed", 0.02), ("cora", 2.0), ("pubmed", 0.0)])
+def test_epoch_parity(wname, theta):
+    """Rows a4-a13 of one 2-layer GCN epoch + an SGD step vs the fp64 oracle."""
+    from paper_conf_ipps_tianmyd20_b200.gcn import GCN2
+    w = C.WORKLOADS[wname]
+    g = C.graph(w)
+    X = C.features(w, g.n)
+    Th0, Th1 = C.thetas(w)
+    y = g.labels
+    T = C.train_mask(g.n, w.theta_seed)
+    pl = L.Plan(g.n, g.rowptr, g.col, w.P, theta)
+    perm = pl.perm()
+    model = GCN2(pl, X[perm], y[perm], T[perm], Th0, Th1, optimizer="sgd", lr=0.1)
+    model.epoch()
+    torch.cuda.synchronize()
+    Ahat = O.normalized_adjacency(g.n, g.rowptr, g.col)[0]
+    ref = O.epoch(Ahat, X, Th0, Th1, y, T)
+    # The ReLU mask [P1 > 0] is decided in floating point; with these seeded
+    # inputs no P1 entry lies within 1e-6 of its condition scale of zero, so
+    # the fp32 and fp64 decisions cannot differ (checked here, oracle side only).
+    p1_scale = O.aggregate(abs(Ahat), np.abs(X.astype(np.float64)) @ np.abs(Th0.astype(np.float64)))
+    assert not np.any(np.abs(ref["P1"]) <= 1e-6 * p1_scale), "ambiguous ReLU decisions: change the seed"
+    inv = np.argsort(perm)
+
+    def unperm(t, F):
+        return _np(t)[:, :F][inv]
+
+    def rel(a, b):
+        return np.max(np.abs(a - b)) / max(np.max(np.abs(b)), 1e-30)
+
+    assert abs(model.loss.item() - ref["loss"]) <= 1e-5 * abs(ref["loss"])
+    assert rel(unperm(model.H1, w.hidden), ref["H1"]) < 1e-5
+    assert rel(unperm(model.Lg, w.classes), ref["L"]) < 1e-5
+    assert rel(unperm(model.G1, w.classes), ref["G1"]) < 1e-5
+    assert rel(unperm(model.G0, w.hidden), ref["G0"]) < 1e-4
+    # gradients are long fp32 reductions over all n rows: 1e-4 of max |g|
+    new = _np(model.theta)
+    g0 = (Th0.astype(np.float64).ravel() - new[: Th0.size]) / 0.1
+    g1 = (Th1.astype(np.float64).ravel() - new[Th0.size:]) / 0.1
+    assert rel(_np(model.gTh1).ravel(), ref["gTh1"].ravel()) < 1e-4
+    assert rel(_np(model.gTh0).ravel(), ref["gTh0"].ravel()) < 1e-4
+    assert rel(g0, ref["gTh0"].ravel()) < 1e-3 and rel(g1, ref["gTh1"].ravel()) < 1e-3
+
+
+def test_cuda_graph_replay_matches_eager():
+    from paper_conf_ipps_tianmyd20_b200.gcn import GCN2
+    w = C.CORA
+    g = C.graph(w)
+    X = C.features(w, g.n)
+    Th0, Th1 = C.thetas(w)
+    T = C.train_mask(g.n, 1)
+    pl = L.Plan(g.n, g.rowptr, g.col, 8, 0.05)
+    perm = pl.perm()
+    a = GCN2(pl, X[perm], g.labels[perm], T[perm], Th0, Th1)
+    b = GCN2(pl, X[perm], g.labels[perm], T[perm], Th0, Th1)
+    for _ in range(3):
+        a.epoch()
+    b.capture(warmup=1)
+    b.replay()
+    b.replay()
+    torch.cuda.synchronize()
+    assert torch.equal(a.theta, b.theta)
+    assert a.step_ctr.item() == b.step_ctr.item() == 3
+
+
+def test_calibrate_theta():
+    th, tf, ts = L.calibrate(128, 1024, 0.05)
+    assert tf > 0 and ts > 0 and 0 < th < 1
