@@ -1,0 +1,410 @@
+#!/usr/bin/env python
+"""PCGCN hot-path benchmark: 2-layer GCN epoch ms + aggregation GB/s on B200.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+                    [--workload reddit|pubmed|cora] [--theta auto|<float>] [--P <int>]
+
+A step is one full-batch training epoch of the 2-layer GCN (SURVEY.md §8(a)
+rows a4-a14: both transforms, four partition-centric aggregations, loss,
+backward, Adam) over the Reddit-shaped synthetic graph (BASELINE.json
+configs[2]; the north-star target config), replayed as one CUDA graph.
+Timing: CUDA events on the launching stream around every step, L2 flushed
+(256 MiB write) between steps outside the events, barrier + synchronize
+around the K timed steps, max over ranks.  Prints ONE JSON line on rank 0.
+
+--impl reference times the fp64 CPU oracle (oracle/, the only other place
+bench.py runs it) on a bounded row sample of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+MEASURED_PEAKS = os.path.join(ROOT, "MEASURED_PEAKS.json")
+FALLBACK_HBM_GBS = 6650.0
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--workload", default="reddit")
+    ap.add_argument("--theta", default="auto")
+    ap.add_argument("--P", type=int, default=0)
+    ap.add_argument("--oracle-frac", type=float, default=0.02)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--eager", action="store_true", help="no CUDA graph")
+    return ap.parse_args()
+
+
+def log(*a):
+    print(*a, file=sys.stderr, flush=True)
+
+
+# ---------------------------------------------------------------------------
+# clocks during the timed region
+# ---------------------------------------------------------------------------
+class ClockSampler:
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                 "-lms", "100"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except Exception:
+            self.proc = None
+        return self
+
+    def __exit__(self, *exc):
+        self.lines = []
+        if self.proc is not None:
+            time.sleep(0.25)
+            self.proc.terminate()
+            try:
+                out, _ = self.proc.communicate(timeout=5)
+            except Exception:
+                out = ""
+            self.lines = [l for l in out.splitlines() if l.strip()]
+
+    def summary(self):
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for l in getattr(self, "lines", []):
+            f = [x.strip() for x in l.split(",")]
+            try:
+                sm.append(float(f[0]))
+                mx = float(f[1])
+            except (ValueError, IndexError):
+                continue
+            for nm, v in zip(names, f[4:8]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"], "samples": 0}
+        return {"sm_mhz": float(np.median(sm)), "sm_max_mhz": mx, "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ---------------------------------------------------------------------------
+# workload
+# ---------------------------------------------------------------------------
+def load_workload(name):
+    from synth import configs as C
+    w = C.WORKLOADS[name]
+    t0 = time.time()
+    g = C.graph(w)
+    X = C.features(w, g.n)
+    Th0, Th1 = C.thetas(w)
+    T = C.train_mask(g.n, w.theta_seed)
+    log(f"[bench] {name}: n={g.n} nnz(A)={g.nnz} generated in {time.time() - t0:.1f}s")
+    return w, g, X, Th0, Th1, g.labels, T
+
+
+def hbm_peak():
+    try:
+        j = json.load(open(MEASURED_PEAKS))
+        return float(j["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:
+        return FALLBACK_HBM_GBS, "fallback (B200_PROFILING.md)"
+
+
+def agg_bytes(st, n, rows, F, dense_rows, nchunks):
+    """Algorithmic HBM bytes of one aggregation call (SURVEY.md §8(d) B_min):
+    index stream + row pointers + r + read Y once + write Z (+ Zd round trip
+    for rows with full-mode blocks) + full-mode bit tiles."""
+    nnz_s = st["shard_nnz_sparse"]
+    b = nnz_s * 4 + (rows + 1) * 8 + rows * 4 + n * F * 4 + rows * F * 4
+    b += 2 * dense_rows * F * 4 + nchunks * (512 + 4)
+    return int(b)
+
+
+# ---------------------------------------------------------------------------
+# oracle (CPU baseline / reference arm): bounded row sample of one epoch
+# ---------------------------------------------------------------------------
+class OracleSample:
+    """Times the fp64 oracle's epoch operations restricted to a seeded random
+    sample of output rows (fraction ``frac``) and extrapolates to the full
+    epoch (x 1/frac).  Full-height inputs of each aggregation are prepared
+    untimed (their values do not change the cost)."""
+
+    def __init__(self, w, g, X, Th0, Th1, labels, T, frac, seed=7):
+        from oracle import gcn as O
+        self.O = O
+        t0 = time.time()
+        self.Ahat = O.normalized_adjacency(g.n, g.rowptr, g.col)[0]
+        rng = np.random.default_rng(seed)
+        self.rows = np.sort(rng.choice(g.n, size=max(1, int(g.n * frac)), replace=False))
+        self.frac = len(self.rows) / g.n
+        self.AS = self.Ahat[self.rows]
+        self.X = X.astype(np.float64)
+        self.XS = self.X[self.rows]
+        self.Th0 = Th0.astype(np.float64)
+        self.Th1 = Th1.astype(np.float64)
+        H, C = Th0.shape[1], Th1.shape[1]
+        self.YH = rng.standard_normal((g.n, H))
+        self.YC = rng.standard_normal((g.n, C))
+        self.labels = labels[self.rows]
+        self.T = T[self.rows]
+        self.nT = int(T.sum())
+        log(f"[bench] oracle sample prepared in {time.time() - t0:.1f}s (frac={self.frac:.4f})")
+
+    def epoch_ms(self):
+        O = self.O
+        t0 = time.perf_counter()
+        a1 = self.XS @ self.Th0                     # a4 (sampled rows)
+        P1 = O.aggregate(self.AS, self.YH)          # a5/a6
+        H1 = np.maximum(P1, 0.0)
+        a2 = H1 @ self.Th1                          # a7
+        Lg = O.aggregate(self.AS, self.YC)          # a8
+        loss, dL = O.softmax_ce(Lg, self.labels, self.T)   # a9
+        G1 = O.aggregate(self.AS, self.YC)          # a10
+        g1 = H1.T @ G1                              # a11
+        dP1 = (G1 @ self.Th1.T) * (P1 > 0)
+        G0 = O.aggregate(self.AS, self.YH)          # a12
+        g0 = self.XS.T @ G0                         # a13
+        th0 = self.Th0 - 0.01 * g0                  # a14
+        th1 = self.Th1 - 0.01 * g1
+        del a1, a2, loss, dL, dP1, th0, th1
+        return (time.perf_counter() - t0) * 1e3 / self.frac
+
+    def cores(self):
+        try:
+            from threadpoolctl import threadpool_info
+            blas = max([i.get("num_threads", 1) for i in threadpool_info()] or [1])
+        except Exception:
+            blas = 1
+        return int(blas), len(os.sched_getaffinity(0))
+
+
+def run_reference(args, rank, world):
+    if rank != 0:
+        return
+    w, g, X, Th0, Th1, labels, T = load_workload(args.workload)
+    osamp = OracleSample(w, g, X, Th0, Th1, labels, T, args.oracle_frac)
+    for _ in range(args.warmup):
+        osamp.epoch_ms()
+    ts = [osamp.epoch_ms() for _ in range(args.steps)]
+    v = float(np.mean(ts))
+    blas, cores = osamp.cores()
+    sample = (f"{len(osamp.rows)} seeded random output rows ({osamp.frac:.2%} of n) of every epoch op "
+              f"(4 aggregations scipy fp64 single-threaded, GEMMs numpy BLAS {blas} threads), x1/frac")
+    line = {
+        "impl": "reference", "metric": "2-layer GCN epoch ms (oracle, extrapolated from a row sample)",
+        "value": v, "unit": "ms", "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": v, "higher_is_better": False, "scaling": "strong", "vs_baseline": None,
+        "dtype": "f64", "data": "synthetic",
+        "config": {"workload": f"{w.name}-shaped DC-SBM n={g.n} nnz(A+I)={g.nnz + g.n} F={w.f_in}->{w.hidden}->{w.classes}",
+                   "parallelism": "cpu"},
+        "cpu_baseline": {"value": v, "unit": "ms", "cores": blas, "host_cores": cores, "kind": "oracle",
+                         "sample": sample},
+        "e2e": {"value": v, "unit": "ms", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+# ---------------------------------------------------------------------------
+# our arm
+# ---------------------------------------------------------------------------
+def main():
+    args = parse()
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    import torch
+    import torch.distributed as dist
+    if world > 1:
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        if world > 1:
+            dist.destroy_process_group()
+        return
+
+    from paper_conf_ipps_tianmyd20_b200 import _lib as L
+    from paper_conf_ipps_tianmyd20_b200.gcn import GCN2
+    from paper_conf_ipps_tianmyd20_b200.dist import RowExchange
+
+    dev = torch.device("cuda", local)
+    torch.cuda.set_device(dev)
+    w, g, X, Th0, Th1, labels, T = load_workload(args.workload)
+    P = args.P or w.P
+    if args.theta == "auto":
+        avg_part = max(64, min(8192, g.n // P))
+        theta, t_f, t_s = L.calibrate(w.hidden, avg_part, 0.05)
+        theta_src = f"calibrated (L161): T_f={t_f:.4f}ms T_s={t_s:.4f}ms at p=0.05, {avg_part}-row blocks, F={w.hidden}"
+    else:
+        theta, theta_src = float(args.theta), "fixed"
+    t0 = time.time()
+    pl = L.Plan(g.n, g.rowptr, g.col, P, theta, f_max=max(w.hidden, w.classes), rank=rank, world=world)
+    st = pl.stats()
+    log(f"[bench] plan in {time.time() - t0:.1f}s theta={theta:.4g} ({theta_src}) stats={st}")
+    perm = pl.perm()
+    Xp = np.ascontiguousarray(X[perm])
+    exch = RowExchange(pl.row_lo, pl.row_hi) if world > 1 else None
+    model = GCN2(pl, Xp, labels[perm], T[perm], Th0, Th1, optimizer="adam", lr=0.01, device=dev, exchange=exch)
+    use_graph = world == 1 and not args.eager
+    stream = torch.cuda.current_stream(dev)
+    if use_graph:
+        model.capture(warmup=1)
+
+    def step():
+        if use_graph:
+            model.replay()
+        else:
+            model.epoch()
+
+    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
+    for _ in range(max(args.warmup, 3)):
+        step()
+    torch.cuda.synchronize(dev)
+
+    # ---- timed region ----
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    with ClockSampler(local) as clk:
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize(dev)
+        for i in range(args.steps):
+            flush.zero_()
+            evs[i][0].record()
+            step()
+            evs[i][1].record()
+        torch.cuda.synchronize(dev)
+        if world > 1:
+            dist.barrier()
+    times = [a.elapsed_time(b) for a, b in evs]
+    ms = float(np.mean(times))
+    if world > 1:
+        t = torch.tensor([ms], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+    clocks = clk.summary()
+
+    # ---- instrumented eager pass: per-step durations on the launching stream ----
+    names, marks = [], []
+
+    def hook(name):
+        e = torch.cuda.Event(enable_timing=True)
+        e.record()
+        names.append(name)
+        marks.append(e)
+
+    per = {}
+    reps = 3
+    for _ in range(reps):
+        names.clear(); marks.clear()
+        flush.zero_()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e0.record()
+        model.epoch(hook=hook)
+        torch.cuda.synchronize(dev)
+        prev = e0
+        for nm, e in zip(names, marks):
+            per[nm] = per.get(nm, 0.0) + prev.elapsed_time(e) / reps
+            prev = e
+    peak, peak_src = hbm_peak()
+    rows = pl.row_hi - pl.row_lo
+    dense_rows = int(st["row_tiles"]) * 128 if world == 1 else int(st["shard_chunks"] > 0) * rows
+    bH = agg_bytes(st, g.n, rows, w.hidden, dense_rows, st["shard_chunks"])
+    bC = agg_bytes(st, g.n, rows, w.classes, dense_rows, st["shard_chunks"])
+    t_agg = per["a5a6_agg_fwd_H"]
+    achieved = bH / (t_agg * 1e-3) / 1e9
+    agg_total = sum(per[k] for k in per if "agg" in k)
+
+    # ---- e2e: host buffers, H2D of the step's inputs and D2H of the loss inside the region ----
+    e2e = None
+    if not args.no_e2e:
+        Xh = torch.from_numpy(np.ascontiguousarray(Xp[pl.row_lo:pl.row_hi])).pin_memory()
+        lab_h = model.labels.cpu().pin_memory()
+        tr_h = model.train.cpu().pin_memory()
+        loss_h = torch.empty(1, dtype=torch.float32).pin_memory()
+        h2d = Xh.numel() * 4 + lab_h.numel() * 4 + tr_h.numel()
+        e2e_ev = []
+        for i in range(args.steps):
+            flush.zero_()
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record()
+            model.X.copy_(Xh, non_blocking=True)
+            model.labels.copy_(lab_h, non_blocking=True)
+            model.train.copy_(tr_h, non_blocking=True)
+            step()
+            loss_h.copy_(model.loss, non_blocking=True)
+            b.record()
+            e2e_ev.append((a, b))
+        torch.cuda.synchronize(dev)
+        e2e_ms = float(np.mean([a.elapsed_time(b) for a, b in e2e_ev]))
+        if world > 1:
+            t = torch.tensor([e2e_ms], device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            e2e_ms = float(t.item())
+        e2e = {"value": e2e_ms, "unit": "ms", "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": 4}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        try:
+            osamp = OracleSample(w, g, X, Th0, Th1, labels, T, args.oracle_frac)
+            v = float(np.mean([osamp.epoch_ms() for _ in range(2)]))
+            blas, cores = osamp.cores()
+            cpu = {"value": v, "unit": "ms", "cores": blas, "host_cores": cores, "kind": "oracle",
+                   "sample": f"{len(osamp.rows)} seeded random output rows ({osamp.frac:.2%}) of every epoch op, "
+                             f"extrapolated x1/frac; scipy SpMM single-threaded, numpy GEMMs {blas} BLAS threads"}
+        except Exception as e:  # the baseline must never break the GPU line
+            cpu = {"value": None, "unit": "ms", "cores": None, "kind": "oracle", "sample": f"failed: {e}"}
+
+    if rank == 0:
+        line = {
+            "metric": "2-layer GCN epoch ms", "value": ms, "unit": "ms", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": False,
+            "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {
+                "workload": f"{w.name}-shaped DC-SBM (BASELINE configs[2]) n={g.n} nnz(A+I)={st['nnz']} "
+                            f"F={w.f_in}->{w.hidden}->{w.classes}",
+                "P": P, "theta": theta, "theta_source": theta_src, "optimizer": "adam",
+                "parallelism": f"dp-rows{world}" if world > 1 else "single",
+                "l2": "flushed (256 MiB write) between timed steps",
+                "cuda_graph": use_graph,
+                "plan": {k: st[k] for k in ("blocks_nonempty", "blocks_dense", "nnz_sparse", "nnz_dense",
+                                            "row_tiles", "chunks", "intra_edges", "lp_sweeps", "clusters",
+                                            "partition_ms", "plan_ms")},
+            },
+            "roofline": {"kernel": "aggregation F=H (prescale/split + tcgen05 full tiles + selective gather), fwd layer 1",
+                         "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                         "frac": achieved / peak, "traffic": None, "peak_source": peak_src,
+                         "algorithmic_bytes": bH, "ms": t_agg,
+                         "gather_GBs": st["shard_nnz_sparse"] * w.hidden * 4 / (t_agg * 1e-3) / 1e9},
+            "agg_GBs": {"fwd_H": bH / (per["a5a6_agg_fwd_H"] * 1e-3) / 1e9,
+                        "fwd_C": bC / (per["a8_agg_fwd_C"] * 1e-3) / 1e9,
+                        "bwd_C": bC / (per["a10_agg_bwd_C"] * 1e-3) / 1e9,
+                        "bwd_H": bH / (per["a12_agg_bwd_H"] * 1e-3) / 1e9},
+            "step_breakdown_ms": {k: round(v, 4) for k, v in per.items()},
+            "agg_share": agg_total / max(sum(per.values()), 1e-9),
+            "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": model.launches_per_epoch() * args.steps,
+            "clocks": clocks,
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

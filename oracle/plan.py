@@ -132,14 +132,14 @@ def build(n: int, rowptr, col, P: int, theta: float, part=None, norm: str = "sym
     zd_index = np.full(n, -1, dtype=np.int32)
     if len(dd):
         kd = np.searchsorted(pstart, dd, side="right") - 1
-        kr = np.searchsorted(pstart, ds, side="right") - 1
         t_of = (dd - pstart[kd]) // TILE_M
-        c_of = (ds - pstart[kr]) // TILE_K
-        # group key: (k, t, i, c)
-        order = np.lexsort((ds, dd, c_of, kr, t_of, kd))
-        kd, t_of, kr, c_of, dd, ds = kd[order], t_of[order], kr[order], c_of[order], dd[order], ds[order]
+        # chunk = 32-aligned global source window (shared by the full-mode
+        # blocks of one row tile that overlap it); group key: (k, t, window)
+        c_of = ds // TILE_K
+        order = np.lexsort((ds, dd, c_of, t_of, kd))
+        kd, t_of, c_of, dd, ds = kd[order], t_of[order], c_of[order], dd[order], ds[order]
         tile_key = np.stack([kd, t_of], 1)
-        chunk_key = np.stack([kd, t_of, kr, c_of], 1)
+        chunk_key = np.stack([kd, t_of, c_of], 1)
         brk_c = np.ones(len(dd), dtype=bool)
         brk_c[1:] = np.any(chunk_key[1:] != chunk_key[:-1], axis=1)
         brk_t = np.ones(len(dd), dtype=bool)
@@ -154,7 +154,7 @@ def build(n: int, rowptr, col, P: int, theta: float, part=None, norm: str = "sym
                 r0 = int(pstart[k] + t * TILE_M)
                 rt_row0.append(r0)
                 rt_nrows.append(int(min(TILE_M, pstart[k + 1] - r0)))
-            c0 = int(pstart[kr[a]] + c_of[a] * TILE_K)
+            c0 = int(c_of[a] * TILE_K)
             ch_col0.append(c0)
             w = np.zeros(TILE_M, dtype=np.uint32)
             rr = (dd[a:b] - rt_row0[-1]).astype(np.int64)

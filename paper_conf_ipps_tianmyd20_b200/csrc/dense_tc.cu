@@ -113,24 +113,24 @@ __device__ __forceinline__ uint64_t make_sdesc(uint32_t saddr, uint32_t lbo, uin
   return d;
 }
 
-// instruction descriptor, kind::tf32: D f32, A/B tf32, A K-major, B MN-major
+// instruction descriptor, kind::tf32: D f32 [4,6), A tf32 [7,10), B tf32
+// [10,13), A and B K-major (bits 15/16 = 0), N>>3 [17,23), M>>4 [24,29).
+// (MN-major B reads as zeros for kind::tf32 on the B200 — measured with
+// tests/cuda/tc_probe.cu — so the split input is stored feature-major.)
 __host__ __device__ constexpr uint32_t make_idesc_tf32(int M, int N) {
-  return (1u << 4) | (2u << 7) | (2u << 10) | (0u << 15) | (1u << 16) | (uint32_t(N >> 3) << 17) |
-         (uint32_t(M >> 4) << 24);
+  return (1u << 4) | (2u << 7) | (2u << 10) | (uint32_t(N >> 3) << 17) | (uint32_t(M >> 4) << 24);
 }
 
 struct SmemPlan {
-  int npad, atom_cols, n_atoms, stages;
+  int npad, stages;
   uint32_t a_bytes, b_bytes, stage_bytes;
 };
 
 __host__ __device__ inline SmemPlan smem_plan(int npad) {
   SmemPlan s;
   s.npad = npad;
-  s.atom_cols = (npad % 32 == 0) ? 32 : 16;     // SW128 (128 B rows) or SW64 (64 B rows)
-  s.n_atoms = npad / s.atom_cols;
-  s.a_bytes = BM * BK * 4;                       // 16 KB
-  s.b_bytes = BK * npad * 4;                     // per operand (hi or lo)
+  s.a_bytes = BM * BK * 4;                       // 16 KB: 128 rows x 128 B (K-major SW128)
+  s.b_bytes = npad * BK * 4;                     // per operand (hi or lo): npad rows x 128 B (K-major SW128)
   s.stage_bytes = s.a_bytes + 2 * s.b_bytes;
   int st = int((200 * 1024) / s.stage_bytes);
   s.stages = st < 2 ? 2 : (st > 6 ? 6 : st);
@@ -188,22 +188,18 @@ __global__ void __launch_bounds__(NTHREADS, 1)
         const int s = i % sp.stages;
         const uint32_t ph = uint32_t(i / sp.stages) & 1u;
         mbar_wait(&empty[s], ph ^ 1u);
-        const int row0 = ch_col0[c_begin + i];
+        const int src0 = ch_col0[c_begin + i];
         mbar_expect_tx(&full_tma[s], tx);
-        for (int a = 0; a < sp.n_atoms; ++a) {
-          const uint32_t off = uint32_t(a) * (BK * sp.atom_cols * 4);
-          tma_load_2d(&map_hi, &full_tma[s], sBh + s * sp.b_bytes + off, a * sp.atom_cols, row0);
-          tma_load_2d(&map_lo, &full_tma[s], sBl + s * sp.b_bytes + off, a * sp.atom_cols, row0);
-        }
+        // box = 32 sources (128 B, inner) x npad features: row f of the smem
+        // tile holds Y'[src0..src0+31][f] — the K-major SW128 B operand
+        tma_load_2d(&map_hi, &full_tma[s], sBh + s * sp.b_bytes, src0, 0);
+        tma_load_2d(&map_lo, &full_tma[s], sBl + s * sp.b_bytes, src0, 0);
       }
     }
   } else if (warp == 1) {
     if (lane == 0) {
       // ---- MMA issuer ----
       const uint32_t idesc = make_idesc_tf32(BM, npad);
-      const uint32_t b_layout = sp.atom_cols == 32 ? 2u : 4u;          // SW128 : SW64
-      const uint32_t b_kgroup = 8u * uint32_t(sp.atom_cols) * 4u;       // 8 K-rows of one atom
-      const uint32_t b_lbo = uint32_t(BK) * uint32_t(sp.atom_cols) * 4u; // next N atom
       for (int i = 0; i < nch; ++i) {
         const int s = i % sp.stages;
         const uint32_t ph = uint32_t(i / sp.stages) & 1u;
@@ -216,8 +212,8 @@ __global__ void __launch_bounds__(NTHREADS, 1)
 #pragma unroll
         for (int kk = 0; kk < BK / 8; ++kk) {
           const uint64_t ad = make_sdesc(a0 + kk * 32u, 16u, 1024u, 2u);
-          const uint64_t bh = make_sdesc(bh0 + kk * b_kgroup, b_lbo, b_kgroup, b_layout);
-          const uint64_t bl = make_sdesc(bl0 + kk * b_kgroup, b_lbo, b_kgroup, b_layout);
+          const uint64_t bh = make_sdesc(bh0 + kk * 32u, 16u, 1024u, 2u);
+          const uint64_t bl = make_sdesc(bl0 + kk * 32u, 16u, 1024u, 2u);
           tc_mma_tf32(tmem_base, ad, bh, idesc, (i > 0 || kk > 0) ? 1u : 0u);
           tc_mma_tf32(tmem_base, ad, bl, idesc, 1u);
         }
@@ -289,16 +285,17 @@ PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
   return fn;
 }
 
-bool make_map(CUtensorMap* map, const float* base, int64_t rows, int npad, int atom_cols) {
+// feature-major split input [npad rows][ldT floats]; inner dim = n sources,
+// so chunk boxes that run past n are zero-filled by the TMA unit
+bool make_map(CUtensorMap* map, const float* base, int64_t n, int64_t ldT, int npad) {
   auto enc = get_encode();
   if (!enc) return false;
-  cuuint64_t dims[2] = {cuuint64_t(npad), cuuint64_t(rows)};
-  cuuint64_t strides[1] = {cuuint64_t(npad) * 4};
-  cuuint32_t box[2] = {cuuint32_t(atom_cols), cuuint32_t(BK)};
+  cuuint64_t dims[2] = {cuuint64_t(n), cuuint64_t(npad)};
+  cuuint64_t strides[1] = {cuuint64_t(ldT) * 4};
+  cuuint32_t box[2] = {cuuint32_t(BK), cuuint32_t(npad)};
   cuuint32_t estr[2] = {1, 1};
   CUresult r = enc(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(base), dims, strides, box,
-                   estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                   atom_cols == 32 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_64B,
+                   estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
                    CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   return r == CUDA_SUCCESS;
 }
@@ -307,10 +304,10 @@ bool make_map(CUtensorMap* map, const float* base, int64_t rows, int npad, int a
 
 cudaError_t launch_dense_tc(const DenseArgs& a, cudaStream_t s) {
   if (a.nrt <= 0) return cudaSuccess;
-  if (a.npad % 16 != 0 || a.npad < 16 || a.npad > 256 || a.ldhl != a.npad) return cudaErrorInvalidValue;
+  if (a.npad % 16 != 0 || a.npad < 16 || a.npad > 256 || a.ldT % 4 != 0) return cudaErrorInvalidValue;
   const SmemPlan sp = smem_plan(a.npad);
   CUtensorMap mh, ml;
-  if (!make_map(&mh, a.yhi, a.n, a.npad, sp.atom_cols) || !make_map(&ml, a.ylo, a.n, a.npad, sp.atom_cols))
+  if (!make_map(&mh, a.hiT, a.n, a.ldT, a.npad) || !make_map(&ml, a.loT, a.n, a.ldT, a.npad))
     return cudaErrorInvalidValue;
   const size_t smem = 1024 + size_t(sp.stages) * sp.stage_bytes + (3 * sp.stages + 1) * 8 + 16;
   static bool attr_done = false;

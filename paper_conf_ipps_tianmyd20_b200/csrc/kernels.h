@@ -26,16 +26,18 @@ struct AggArgs {
 };
 cudaError_t launch_sparse_agg(const AggArgs& a, cudaStream_t s);
 
-// diag(r)·Y (optional) and the tf32 hi/lo split of the result (optional)
-cudaError_t launch_prescale_split(const float* Y, int64_t ldy, const float* r, int64_t n, int F,
-                                  float* ypre, int64_t ldpre, float* yhi, float* ylo, int64_t ldhl,
-                                  cudaStream_t s);
+// ypre = diag(r)·Y
+cudaError_t launch_prescale(const float* Y, int64_t ldy, const float* r, int64_t n, int F, float* ypre,
+                            int64_t ldpre, cudaStream_t s);
+// tf32 hi/lo split of Y written feature-major: hiT/loT [npad x ldT]
+cudaError_t launch_split_transpose(const float* Y, int64_t ldy, int64_t n, int F, int npad, float* hiT,
+                                   float* loT, int64_t ldT, cudaStream_t s);
 
 // ---- dense-mode tcgen05 tile contraction (dense_tc.cu) ----
 struct DenseArgs {
-  const float* yhi;          // [n x ldhl] tf32 hi part of the prescaled input
-  const float* ylo;          // [n x ldhl] lo part
-  int64_t n, ldhl;
+  const float* hiT;          // [npad x ldT] tf32 hi part of the prescaled input, feature-major
+  const float* loT;          // [npad x ldT] lo part
+  int64_t n, ldT;
   const int32_t* rt_row0;    // shard row tiles
   const int32_t* rt_nrows;
   const int64_t* rt_cptr;

@@ -83,7 +83,7 @@ pcgcn_status upload_plan(pcgcn_plan_s* p) {
   const int64_t ch_lo = p->rt_cptr[p->rt_lo], ch_hi = p->rt_cptr[p->rt_hi];
   d.nch = ch_hi - ch_lo;
   d.fpad_max = int(round_up(std::max(p->opts.f_max, 1), 16));
-  d.n_pad = n;
+  d.n_pad = round_up(n, 32);  // row stride of the feature-major hi/lo split (zero-filled past n)
   pcgcn_status st;
 #define UP(dst, src, cnt) \
   if ((st = upload(d, dst, src, cnt)) != PCGCN_OK) return st
@@ -139,15 +139,18 @@ pcgcn_status aggregate(pcgcn_plan_t p, const float* Y, int64_t ldy, float* Z, in
   const float* src = Y;
   int64_t ldsrc = ldy;
   const bool tc = p->opts.dense_prec == PCGCN_DENSE_TF32X2;
-  if (!prescaled || (dense && tc)) {
-    float* ypre = prescaled ? nullptr : d.ypre;
-    e = launch_prescale_split(Y, ldy, prescaled ? nullptr : d.r, p->n, F, ypre, ld4,
-                              (dense && tc) ? d.yhi : nullptr, (dense && tc) ? d.ylo : nullptr, npad, s);
-    if (e != cudaSuccess) return cuda_fail(e, "prescale_split");
-    if (!prescaled) { src = d.ypre; ldsrc = ld4; }
+  if (!prescaled) {
+    e = launch_prescale(Y, ldy, d.r, p->n, F, d.ypre, ld4, s);
+    if (e != cudaSuccess) return cuda_fail(e, "prescale");
+    src = d.ypre;
+    ldsrc = ld4;
+  }
+  if (dense && tc) {
+    e = launch_split_transpose(src, ldsrc, p->n, F, npad, d.yhi, d.ylo, d.n_pad, s);
+    if (e != cudaSuccess) return cuda_fail(e, "split_transpose");
   }
   if (dense) {
-    DenseArgs da{d.yhi, d.ylo, p->n, npad, d.rt_row0, d.rt_nrows, d.rt_cptr, d.ch_col0, d.bits,
+    DenseArgs da{d.yhi, d.ylo, d.n_pad, d.n_pad, d.rt_row0, d.rt_nrows, d.rt_cptr, d.ch_col0, d.bits,
                  d.nrt, d.zd, npad, npad};
     e = tc ? launch_dense_tc(da, s) : launch_dense_simt_y(da, src, ldsrc, F, s);
     if (e != cudaSuccess) return cuda_fail(e, "dense-mode kernel");

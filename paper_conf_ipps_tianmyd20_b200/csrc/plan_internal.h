@@ -24,8 +24,8 @@ struct DevicePlan {
   int32_t* ch_col0 = nullptr;     // [nch shard]
   uint32_t* bits = nullptr;       // [nch*128]
   float* zd = nullptr;            // [nrt*128*fpad_max] dense partial sums
-  float* yhi = nullptr;           // [n_pad*fpad_max] tf32 hi part of the (prescaled) input
-  float* ylo = nullptr;           // [n_pad*fpad_max] lo part
+  float* yhi = nullptr;           // [fpad_max x n_pad] tf32 hi part of the (prescaled) input, feature-major
+  float* ylo = nullptr;           // [fpad_max x n_pad] lo part
   float* ypre = nullptr;          // [n*fpad_max] prescaled copy for un-prescaled inputs
   int64_t rows = 0, nnz_s = 0, nrt = 0, nch = 0;
   int64_t n_pad = 0;

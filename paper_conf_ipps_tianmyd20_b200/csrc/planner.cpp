@@ -311,7 +311,9 @@ pcgcn_status build_host_plan(const pcgcn_csr* A, int32_t P, float theta, const p
               int32_t j = tcol[e];
               int32_t i = pid[j];
               if (!dense_i[i]) continue;
-              int64_t c0 = p->pstart[i] + ((j - p->pstart[i]) / TILE_K) * TILE_K;
+              // 32-aligned global source window (TMA box starts must be 16-byte
+              // aligned); dense blocks sharing a window share one chunk
+              int64_t c0 = (int64_t(j) / TILE_K) * TILE_K;
               ent.push_back({int32_t(c0), int32_t(((v - r0) << 5) | (j - c0))});
             }
           if (ent.empty()) continue;

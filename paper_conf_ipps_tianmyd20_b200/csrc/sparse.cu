@@ -131,36 +131,50 @@ cudaError_t launch_gv(const AggArgs& a, cudaStream_t s) {
   return cudaGetLastError();
 }
 
-__global__ void prescale_split_kernel(const float* __restrict__ Y, int64_t ldy,
-                                      const float* __restrict__ r, int64_t n, int F,
-                                      float* __restrict__ ypre, int64_t ldpre,
-                                      float* __restrict__ yhi, float* __restrict__ ylo,
-                                      int64_t ldhl) {
+// ypre = diag(r)·Y (row-major, ld ldpre)
+__global__ void prescale_kernel(const float* __restrict__ Y, int64_t ldy, const float* __restrict__ r,
+                                int64_t n, int F, float* __restrict__ ypre, int64_t ldpre) {
   const int nvec = (F + 3) >> 2;
-  const int cvec = yhi ? int(ldhl >> 2) : nvec;  // hi/lo rows are written to their full padded width
-  const int64_t total = n * cvec;
+  const int64_t total = n * nvec;
   for (int64_t idx = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; idx < total;
        idx += int64_t(gridDim.x) * blockDim.x) {
-    const int64_t i = idx / cvec;
-    const int q = int(idx - i * cvec);
-    float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
-    if (q < nvec) {
-      v = ld_f4(Y + i * ldy + 4 * q);
-      if (r) {
-        const float ri = __ldg(r + i);
-        v.x *= ri; v.y *= ri; v.z *= ri; v.w *= ri;
-      }
-      if (ypre) *reinterpret_cast<float4*>(ypre + i * ldpre + 4 * q) = v;
-    }
-    if (yhi) {
-      float4 h;
-      h.x = __uint_as_float(__float_as_uint(v.x) & 0xffffe000u);
-      h.y = __uint_as_float(__float_as_uint(v.y) & 0xffffe000u);
-      h.z = __uint_as_float(__float_as_uint(v.z) & 0xffffe000u);
-      h.w = __uint_as_float(__float_as_uint(v.w) & 0xffffe000u);
-      float4 lo = make_float4(v.x - h.x, v.y - h.y, v.z - h.z, v.w - h.w);
-      *reinterpret_cast<float4*>(yhi + i * ldhl + 4 * q) = h;
-      *reinterpret_cast<float4*>(ylo + i * ldhl + 4 * q) = lo;
+    const int64_t i = idx / nvec;
+    const int q = int(idx - i * nvec);
+    float4 v = ld_f4(Y + i * ldy + 4 * q);
+    const float ri = __ldg(r + i);
+    v.x *= ri; v.y *= ri; v.z *= ri; v.w *= ri;
+    *reinterpret_cast<float4*>(ypre + i * ldpre + 4 * q) = v;
+  }
+}
+
+// tf32 split of the (prescaled) input, written TRANSPOSED (feature-major):
+//   hiT[f][j] = Y[j][f] with the low 13 mantissa bits cleared, loT = Y - hi.
+// Feature-major rows make the dense kernel's B operand K-major (source index
+// contiguous), the layout the tf32 UMMA reads.  32x32 tiles through smem keep
+// both the row-major reads and the transposed writes coalesced.  Feature rows
+// F..npad-1 are written as zero.
+__global__ void __launch_bounds__(256) split_transpose_kernel(const float* __restrict__ Y, int64_t ldy,
+                                                              int64_t n, int F, int npad,
+                                                              float* __restrict__ hiT,
+                                                              float* __restrict__ loT, int64_t ldT) {
+  __shared__ float tile[32][33];
+  const int64_t j0 = int64_t(blockIdx.x) * 32;
+  const int f0 = blockIdx.y * 32;
+  const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5;  // 32 x 8
+  for (int rr = ty; rr < 32; rr += 8) {
+    const int64_t j = j0 + rr;
+    const int f = f0 + tx;
+    tile[rr][tx] = (j < n && f < F) ? __ldg(Y + j * ldy + f) : 0.f;
+  }
+  __syncthreads();
+  for (int rr = ty; rr < 32; rr += 8) {
+    const int f = f0 + rr;
+    const int64_t j = j0 + tx;
+    if (f < npad && j < ldT) {
+      const float v = tile[tx][rr];
+      const float h = __uint_as_float(__float_as_uint(v) & 0xffffe000u);
+      hiT[int64_t(f) * ldT + j] = h;
+      loT[int64_t(f) * ldT + j] = v - h;
     }
   }
 }
@@ -179,14 +193,20 @@ cudaError_t launch_sparse_agg(const AggArgs& a, cudaStream_t s) {
   return launch_gv<32, 2>(a, s);
 }
 
-cudaError_t launch_prescale_split(const float* Y, int64_t ldy, const float* r, int64_t n, int F,
-                                  float* ypre, int64_t ldpre, float* yhi, float* ylo, int64_t ldhl,
-                                  cudaStream_t s) {
+cudaError_t launch_prescale(const float* Y, int64_t ldy, const float* r, int64_t n, int F, float* ypre,
+                            int64_t ldpre, cudaStream_t s) {
   if (n <= 0) return cudaSuccess;
-  const int cvec = yhi ? int(ldhl / 4) : (F + 3) / 4;
-  int64_t total = n * cvec;
-  int blocks = int(std::min<int64_t>((total + 255) / 256, 148 * 16));
-  prescale_split_kernel<<<blocks, 256, 0, s>>>(Y, ldy, r, n, F, ypre, ldpre, yhi, ylo, ldhl);
+  const int64_t total = n * ((F + 3) / 4);
+  const int blocks = int(std::min<int64_t>((total + 255) / 256, 148 * 16));
+  prescale_kernel<<<blocks, 256, 0, s>>>(Y, ldy, r, n, F, ypre, ldpre);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_split_transpose(const float* Y, int64_t ldy, int64_t n, int F, int npad, float* hiT,
+                                   float* loT, int64_t ldT, cudaStream_t s) {
+  if (n <= 0) return cudaSuccess;
+  dim3 grid(unsigned((ldT + 31) / 32), unsigned((npad + 31) / 32));
+  split_transpose_kernel<<<grid, 256, 0, s>>>(Y, ldy, n, F, npad, hiT, loT, ldT);
   return cudaGetLastError();
 }
 

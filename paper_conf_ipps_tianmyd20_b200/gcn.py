@@ -98,38 +98,56 @@ class GCN2:
         if self.exchange is not None:
             self.exchange.gather(full, self.lo, self.hi)
 
-    def epoch(self, stream=None):
+    def epoch(self, stream=None, hook=None):
+        """One epoch; ``hook(name)`` (optional) is called after every step so a
+        caller can record CUDA events between them."""
+        mark = hook or (lambda name: None)
         rr = self._r_rows()
         H, C, p = self.H, self.C, self.plan
         # layer 1
         L.gemm_xw(self.X, self.Th0, rr, self._local(self.Y0), M=self.rows, K=self.f_in, N=H, stream=stream)
+        mark("a4_gemm_xw0")
         self._gather(self.Y0)
+        mark("x_gather_y0")
         p.forward(self.Y0, self.H1, F=H, flags=L.IN_PRESCALED | L.RELU | L.MASK_OUT, mask=self.mask1,
                   stream=stream)
+        mark("a5a6_agg_fwd_H")
         # layer 2
         L.gemm_xw(self.H1, self.Th1, rr, self._local(self.Y1), M=self.rows, K=H, N=C, stream=stream)
+        mark("a7_gemm_xw1")
         self._gather(self.Y1)
+        mark("x_gather_y1")
         p.forward(self.Y1, self.Lg, F=C, flags=L.IN_PRESCALED, stream=stream)
+        mark("a8_agg_fwd_C")
         # loss
         L.softmax_ce(self.Lg, self.labels, self.train, self.inv_nT, rr, self._local(self.dL), self.loss,
                      self.ce_work, M=self.rows, C=C, stream=stream)
+        mark("a9_softmax_ce")
         self._gather(self.dL)
+        mark("x_gather_dl")
         # backward
         p.backward(self.dL, self.G1, F=C, flags=L.IN_PRESCALED, stream=stream)
+        mark("a10_agg_bwd_C")
         L.gemm_xtg(self.H1, self.G1, self.gTh1, self.xtg_work, M=self.rows, K=H, N=C, stream=stream)
         L.gemm_dwt(self.G1, self.Th1, self.mask1, rr, self._local(self.dP1), M=self.rows, N=C, K=H,
                    stream=stream)
+        mark("a11_gemm_xtg1_dwt")
         self._gather(self.dP1)
+        mark("x_gather_dp1")
         p.backward(self.dP1, self.G0, F=H, flags=L.IN_PRESCALED, stream=stream)
+        mark("a12_agg_bwd_H")
         L.gemm_xtg(self.X, self.G0, self.gTh0, self.xtg_work, M=self.rows, K=self.f_in, N=H, stream=stream)
+        mark("a13_gemm_xtg0")
         if self.exchange is not None:
             self.exchange.allreduce(self.grad)
             self.exchange.allreduce(self.loss)
+        mark("x_allreduce")
         # update
         if self.optimizer == "adam":
             L.adam(self.theta, self.grad, self.m, self.v, self.lr, self.step_ctr, stream=stream)
         elif self.optimizer == "sgd":
             L.sgd(self.theta, self.grad, self.lr, stream=stream)
+        mark("a14_update")
 
     def launches_per_epoch(self) -> int:
         """Kernel launches of libpcgcn per epoch (for the bench's gpu_launches)."""

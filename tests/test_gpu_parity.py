@@ -277,11 +277,19 @@ def test_epoch_parity(wname, theta):
     torch.cuda.synchronize()
     Ahat = O.normalized_adjacency(g.n, g.rowptr, g.col)[0]
     ref = O.epoch(Ahat, X, Th0, Th1, y, T)
-    # The ReLU mask [P1 > 0] is decided in floating point; with these seeded
-    # inputs no P1 entry lies within 1e-6 of its condition scale of zero, so
-    # the fp32 and fp64 decisions cannot differ (checked here, oracle side only).
+    # The ReLU mask [P1 > 0] is a decision taken in floating point.  Entries
+    # with |P1| within 1e-6 of their condition scale may legitimately go either
+    # way in fp32; both outcomes are valid, so the oracle computes the backward
+    # for every combination of those (few) decisions and the GPU must match one.
     p1_scale = O.aggregate(abs(Ahat), np.abs(X.astype(np.float64)) @ np.abs(Th0.astype(np.float64)))
-    assert not np.any(np.abs(ref["P1"]) <= 1e-6 * p1_scale), "ambiguous ReLU decisions: change the seed"
+    amb = np.argwhere(np.abs(ref["P1"]) <= 1e-6 * p1_scale)
+    assert len(amb) <= 8, f"{len(amb)} ambiguous ReLU decisions"
+    variants = []
+    for bits in range(2 ** len(amb)):
+        P1v = ref["P1"].copy()
+        for t, (i, f) in enumerate(amb):
+            P1v[i, f] = 1e-300 if (bits >> t) & 1 else -1e-300
+        variants.append(O.backward(Ahat, X, Th0, Th1, P1v, ref["H1"], ref["dL"]))
     inv = np.argsort(perm)
 
     def unperm(t, F):
@@ -294,14 +302,16 @@ def test_epoch_parity(wname, theta):
     assert rel(unperm(model.H1, w.hidden), ref["H1"]) < 1e-5
     assert rel(unperm(model.Lg, w.classes), ref["L"]) < 1e-5
     assert rel(unperm(model.G1, w.classes), ref["G1"]) < 1e-5
-    assert rel(unperm(model.G0, w.hidden), ref["G0"]) < 1e-4
     # gradients are long fp32 reductions over all n rows: 1e-4 of max |g|
+    assert rel(_np(model.gTh1).ravel(), ref["gTh1"].ravel()) < 1e-4
+    G0 = unperm(model.G0, w.hidden)
+    gth0 = _np(model.gTh0).ravel()
+    ok = [v for v in variants if rel(G0, v["G0"]) < 1e-4 and rel(gth0, v["gTh0"].ravel()) < 1e-4]
+    assert ok, min(rel(G0, v["G0"]) for v in variants)
     new = _np(model.theta)
     g0 = (Th0.astype(np.float64).ravel() - new[: Th0.size]) / 0.1
     g1 = (Th1.astype(np.float64).ravel() - new[Th0.size:]) / 0.1
-    assert rel(_np(model.gTh1).ravel(), ref["gTh1"].ravel()) < 1e-4
-    assert rel(_np(model.gTh0).ravel(), ref["gTh0"].ravel()) < 1e-4
-    assert rel(g0, ref["gTh0"].ravel()) < 1e-3 and rel(g1, ref["gTh1"].ravel()) < 1e-3
+    assert rel(g0, ok[0]["gTh0"].ravel()) < 1e-3 and rel(g1, ref["gTh1"].ravel()) < 1e-3
 
 
 def test_cuda_graph_replay_matches_eager():
