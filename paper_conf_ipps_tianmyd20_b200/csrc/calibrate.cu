@@ -2,12 +2,12 @@
 // B200 itself.  "We profile the runtime of full and selective modes for a
 // block of sparsity p, denoted by T_f and T_s ... θ = T_f·p/T_s."
 //
-// Synthetic workload: a bipartite random block between two vertex blocks of
-// `block_rows` vertices each, edge density p_ref (seeded splitmix64, so the
-// block is the same on every call), plus the n self-loops of Ã.  The plan is
-// built twice with an explicit partition override (θ >= 1 -> every block
-// selective, θ = 0 -> every block full) and each mode's forward at width F is
-// timed with CUDA events (median of 15 after 3 warm-ups).
+// Synthetic workload: pairs of vertex blocks of `block_rows` vertices joined
+// by random bipartite blocks of edge density p_ref (seeded splitmix64, so the
+// blocks are the same on every call), plus the n self-loops of Ã.  The plan
+// is built twice with an explicit partition override (θ >= 1 -> every block
+// selective; θ just below p_ref -> the p-blocks full) and each mode's forward
+// at width F is timed with CUDA events (median of 15 after 3 warm-ups).
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -53,31 +53,44 @@ extern "C" pcgcn_status pcgcn_calibrate(int32_t F, int32_t block_rows, float p_r
     pcgcn::set_error("calibrate: bad arguments");
     return PCGCN_EINVAL;
   }
-  const int64_t B = block_rows, n = 2 * B;
-  // symmetric bipartite block: edge (u in V0, v in V1) present iff hash < p
+  // Pc vertex blocks of B rows; blocks (2q, 2q+1) are joined by a symmetric
+  // random bipartite block of density p.  Pc is chosen so the full-mode
+  // kernel sees >= 2 row tiles per SM (a 2-block probe would leave most of
+  // the 148 SMs idle and overstate T_f).
+  const int64_t B = block_rows;
+  const int64_t tiles_per_block = (B + 127) / 128;
+  int64_t Pc = (296 + tiles_per_block - 1) / tiles_per_block;
+  Pc = std::max<int64_t>(2, Pc + (Pc & 1));
+  const int64_t n = Pc * B;
   const uint64_t thr = uint64_t(double(p_ref) * 18446744073709551615.0);
   std::vector<std::vector<int32_t>> adj(n);
-  for (int64_t u = 0; u < B; ++u)
-    for (int64_t v = 0; v < B; ++v)
-      if (mix64(0x5eedull * 0x9E3779B97F4A7C15ull + uint64_t(u * B + v)) < thr) {
-        adj[u].push_back(int32_t(B + v));
-        adj[B + v].push_back(int32_t(u));
-      }
+  for (int64_t q = 0; q < Pc / 2; ++q) {
+    const int64_t b0 = 2 * q * B, b1 = b0 + B;
+    for (int64_t u = 0; u < B; ++u)
+      for (int64_t v = 0; v < B; ++v)
+        if (mix64(0x5eedull * 0x9E3779B97F4A7C15ull + uint64_t((q * B + u) * B + v)) < thr) {
+          adj[b0 + u].push_back(int32_t(b1 + v));
+          adj[b1 + v].push_back(int32_t(b0 + u));
+        }
+  }
   std::vector<int64_t> rowptr(n + 1, 0);
   for (int64_t v = 0; v < n; ++v) rowptr[v + 1] = rowptr[v] + int64_t(adj[v].size());
   std::vector<int32_t> col(rowptr[n]);
   for (int64_t v = 0; v < n; ++v) std::copy(adj[v].begin(), adj[v].end(), col.begin() + rowptr[v]);
   std::vector<int32_t> part(n);
-  for (int64_t v = 0; v < n; ++v) part[v] = v < B ? 0 : 1;
+  for (int64_t v = 0; v < n; ++v) part[v] = int32_t(v / B);
   pcgcn_csr A{n, rowptr[n], rowptr.data(), col.data()};
   pcgcn_opts o;
   pcgcn_opts_default(&o);
   o.part = part.data();
   o.f_max = F;
   pcgcn_plan_t ps = nullptr, pf = nullptr;
-  pcgcn_status st = pcgcn_plan(&A, 2, 2.0f, &o, &ps);
+  // diagonal blocks hold only the self-loops (density 1/B): keep them selective
+  // in both plans so the two timings differ only in the mode of the p-blocks
+  const float theta_full = 2.0f / float(B);
+  pcgcn_status st = pcgcn_plan(&A, int32_t(Pc), 2.0f, &o, &ps);
   if (st != PCGCN_OK) return st;
-  st = pcgcn_plan(&A, 2, 0.0f, &o, &pf);
+  st = pcgcn_plan(&A, int32_t(Pc), std::min(theta_full, 0.5f * p_ref), &o, &pf);
   if (st != PCGCN_OK) { pcgcn_destroy(ps); return st; }
   const int64_t ld = (F + 3) / 4 * 4;
   float *Y = nullptr, *Z = nullptr;

@@ -21,6 +21,7 @@ struct AggArgs {
   const int32_t* zd_index;   // shard-local, or nullptr if no dense tiles
   const float* zd;           // dense partial sums, ld ldzd
   int64_t ldzd;
+  const float* zrow;         // >= 16 zero floats (load sentinel)
   int F;
   bool relu, out_prescaled;
 };

@@ -112,7 +112,10 @@ pcgcn_status upload_plan(pcgcn_plan_s* p) {
     UP(&d.ylo, (float*)nullptr, d.n_pad * d.fpad_max);
   }
   UP(&d.ypre, (float*)nullptr, n * d.fpad_max);
+  UP(&d.zrow, (float*)nullptr, 256);
 #undef UP
+  e = cudaMemset(d.zrow, 0, 256 * sizeof(float));
+  if (e != cudaSuccess) return cuda_fail(e, "memset");
   d.built = true;
   p->stats.device_bytes = d.bytes;
   return PCGCN_OK;
@@ -162,6 +165,7 @@ pcgcn_status aggregate(pcgcn_plan_t p, const float* Y, int64_t ldy, float* Z, in
   a.row_lo = p->row_lo; a.rows = d.rows;
   a.zd_index = dense ? d.zd_index : nullptr;
   a.zd = d.zd; a.ldzd = npad;
+  a.zrow = d.zrow;
   a.F = F;
   a.relu = (flags & PCGCN_RELU) != 0;
   a.out_prescaled = (flags & PCGCN_OUT_PRESCALED) != 0;

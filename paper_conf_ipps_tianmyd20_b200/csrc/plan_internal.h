@@ -27,6 +27,7 @@ struct DevicePlan {
   float* yhi = nullptr;           // [fpad_max x n_pad] tf32 hi part of the (prescaled) input, feature-major
   float* ylo = nullptr;           // [fpad_max x n_pad] lo part
   float* ypre = nullptr;          // [n*fpad_max] prescaled copy for un-prescaled inputs
+  float* zrow = nullptr;          // [256] zeros: gather sentinel
   int64_t rows = 0, nnz_s = 0, nrt = 0, nch = 0;
   int64_t n_pad = 0;
   int fpad_max = 0;

@@ -55,21 +55,32 @@ __global__ void __launch_bounds__(256) sparse_agg_kernel(AggArgs a) {
 #pragma unroll
     for (int v = 0; v < V; ++v) acc[u][v] = make_float4(0.f, 0.f, 0.f, 0.f);
 
+  // Branch-free batches: every lane issues UNR independent 16-byte loads
+  // before consuming any (edges past the row end and lanes past F read a
+  // zero row instead of branching, so ptxas can keep the loads in flight).
+  constexpr int UNR = STEPS < 8 ? STEPS : 8;
+  const float* zrow = a.zrow;
   for (int64_t base = e0; base < e1; base += 32) {
     const int cnt = (e1 - base) < 32 ? int(e1 - base) : 32;
-    const int myidx = lane < cnt ? __ldg(a.col + base + lane) : 0;
+    const int myidx = lane < cnt ? __ldg(a.col + base + lane) : -1;
 #pragma unroll
-    for (int k = 0; k < STEPS; ++k) {
-      const int eb = k * S + slot;
-      const int j = __shfl_sync(0xffffffffu, myidx, eb);
-      if (eb < cnt) {
+    for (int k0 = 0; k0 < STEPS; k0 += UNR) {
+      float4 buf[UNR][V];
+#pragma unroll
+      for (int u = 0; u < UNR; ++u) {
+        const int j = __shfl_sync(0xffffffffu, myidx, (k0 + u) * S + slot);
         const float* src = a.Y + int64_t(j) * a.ldy;
 #pragma unroll
         for (int v = 0; v < V; ++v) {
           const int q = l + G * v;
-          if (q < nvec) add4(acc[k & 3][v], ld_f4(src + 4 * q));
+          buf[u][v] = ld_f4((j >= 0 && q < nvec) ? src + 4 * q : zrow);
         }
       }
+#pragma unroll
+      for (int u = 0; u < UNR; ++u)
+#pragma unroll
+        for (int v = 0; v < V; ++v) add4(acc[(k0 + u) & 3][v], buf[u][v]);
+      if ((k0 + UNR) * S >= cnt) break;  // warp-uniform: rest of the batch is empty
     }
   }
   float4 tot[V];
