@@ -334,7 +334,8 @@ def main():
     # ---- e2e: host buffers, H2D of the step's inputs and D2H of the loss inside the region ----
     e2e = None
     if not args.no_e2e:
-        Xh = torch.from_numpy(np.ascontiguousarray(Xp[pl.row_lo:pl.row_hi])).pin_memory()
+        Xh = torch.zeros(model.X.shape, dtype=torch.float32).pin_memory()  # same padded layout as model.X
+        Xh[:, :w.f_in] = torch.from_numpy(np.ascontiguousarray(Xp[pl.row_lo:pl.row_hi]))
         lab_h = model.labels.cpu().pin_memory()
         tr_h = model.train.cpu().pin_memory()
         loss_h = torch.empty(1, dtype=torch.float32).pin_memory()

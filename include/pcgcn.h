@@ -137,14 +137,19 @@ pcgcn_status pcgcn_backward(pcgcn_plan_t p, const float* dZ, int64_t ldz, float*
 /* ---- dense helpers of the 2-layer GCN step (Alg. 1 transform, L114) ---- */
 
 /* Y = diag(s)·(X·W):  X DEVICE [M x K] ld ldx, W DEVICE [K x N] ld ldw, Y DEVICE [M x N] ld ldy.
- * s: DEVICE [M] row scale or NULL.  fp32 in/out (3xTF32 tensor-core split). */
+ * s: DEVICE [M] row scale or NULL.  fp32 in/out.  With ldx, ldy multiples of
+ * 4 and `work` (DEVICE, pcgcn_gemm_xw_work_floats(K,N) floats) it runs on the
+ * tcgen05 tensor cores in 3xTF32 (A_hi·B_hi + A_lo·B_hi + A_hi·B_lo); else
+ * (work NULL / unaligned) on fp32 CUDA cores. */
+int64_t pcgcn_gemm_xw_work_floats(int32_t K, int32_t N);
 pcgcn_status pcgcn_gemm_xw(const float* X, int64_t ldx, const float* W, int64_t ldw, const float* s,
-                           float* Y, int64_t ldy, int64_t M, int32_t K, int32_t N, void* stream);
+                           float* Y, int64_t ldy, int64_t M, int32_t K, int32_t N, float* work, void* stream);
 
 /* G = Xᵀ·D:  X DEVICE [M x K] ld ldx, D DEVICE [M x N] ld ldd, G DEVICE [K x N] (ld N), fp32.
  * Split over M into fixed slices whose partial products land in `work`
  * (DEVICE, pcgcn_gemm_xtg_work_floats(M,K,N) floats), then summed in a fixed
- * order: deterministic, no atomics. */
+ * order: deterministic, no atomics.  tcgen05 3xTF32 when ldx, ldd are
+ * multiples of 4, else fp32 CUDA cores. */
 int64_t pcgcn_gemm_xtg_work_floats(int64_t M, int32_t K, int32_t N);
 pcgcn_status pcgcn_gemm_xtg(const float* X, int64_t ldx, const float* D, int64_t ldd, float* G,
                             int64_t M, int32_t K, int32_t N, float* work, void* stream);

@@ -67,7 +67,8 @@ _sig("pcgcn_plan", c_i32, ctypes.POINTER(Csr), c_i32, c_f32, ctypes.POINTER(Opts
 _sig("pcgcn_destroy", None, c_vp)
 _sig("pcgcn_forward", c_i32, c_vp, c_vp, c_i64, c_vp, c_i64, c_i32, c_u32, c_vp, c_vp)
 _sig("pcgcn_backward", c_i32, c_vp, c_vp, c_i64, c_vp, c_i64, c_i32, c_u32, c_vp)
-_sig("pcgcn_gemm_xw", c_i32, c_vp, c_i64, c_vp, c_i64, c_vp, c_vp, c_i64, c_i64, c_i32, c_i32, c_vp)
+_sig("pcgcn_gemm_xw_work_floats", c_i64, c_i32, c_i32)
+_sig("pcgcn_gemm_xw", c_i32, c_vp, c_i64, c_vp, c_i64, c_vp, c_vp, c_i64, c_i64, c_i32, c_i32, c_vp, c_vp)
 _sig("pcgcn_gemm_xtg_work_floats", c_i64, c_i64, c_i32, c_i32)
 _sig("pcgcn_gemm_xtg", c_i32, c_vp, c_i64, c_vp, c_i64, c_vp, c_i64, c_i32, c_i32, c_vp, c_vp)
 _sig("pcgcn_gemm_dwt", c_i32, c_vp, c_i64, c_vp, c_vp, c_vp, c_vp, c_i64, c_i64, c_i32, c_i32, c_vp)
@@ -175,12 +176,16 @@ class Plan:
                                  _stream(stream)), "pcgcn_backward")
 
 
-def gemm_xw(X, W, s, Y, M=None, K=None, N=None, stream=None):
+def gemm_xw_work_floats(K, N):
+    return int(lib.pcgcn_gemm_xw_work_floats(K, N))
+
+
+def gemm_xw(X, W, s, Y, M=None, K=None, N=None, work=None, stream=None):
     M = X.shape[0] if M is None else M
     K = X.shape[1] if K is None else K
     N = W.shape[1] if N is None else N
     check(lib.pcgcn_gemm_xw(_ptr(X), X.stride(0), _ptr(W), W.stride(0), s, _ptr(Y), Y.stride(0), M, K, N,
-                            _stream(stream)), "pcgcn_gemm_xw")
+                            _ptr(work), _stream(stream)), "pcgcn_gemm_xw")
 
 
 def gemm_xtg_work_floats(M, K, N):

@@ -2,13 +2,14 @@
 // L114; the paper runs these as TF MatMul / cuBLAS, L203) and their backward
 // counterparts (the paper is silent on the backward, reading A4).
 //
-// Round-1 implementation: fp32 CUDA-core tiles (64x64 output tile per CTA,
-// 4x4 register micro-tiles, BK=16 smem double-staging) with fused epilogues:
+// xw and xtg run on the tcgen05 engine (tc_engine.cu) in 3xTF32 when the
+// operands are 16-byte aligned (ld % 4 == 0) and a workspace is given; the
+// fp32 CUDA-core tiles below (64x64 output tile per CTA, 4x4 register
+// micro-tiles) serve the remaining shapes and dwt, with fused epilogues:
 //   xw : Y = diag(s)·(X·W)                      (a4, a7: source prescaling)
 //   dwt: O = diag(s)·((D·Wᵀ) ⊙ mask)            (a11: ReLU' via the bit mask)
 //   xtg: G = Xᵀ·D, split over M into fixed slices + fixed-order reduction
 //        (a11, a13: deterministic, no atomics)
-// The tcgen05 3xTF32 path for xw/xtg is the next step.
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -118,8 +119,26 @@ int xtg_slices(int64_t M) { return int(std::min<int64_t>(296, std::max<int64_t>(
 
 }  // namespace
 
+int64_t r32(int64_t x) { return (x + 31) / 32 * 32; }
+int npad16(int n) { return (n + 15) / 16 * 16; }
+
+int64_t gemm_xw_work_floats(int K, int N) { return 2 * int64_t(npad16(N)) * r32(K); }
+
 cudaError_t launch_gemm_xw(const float* X, int64_t ldx, const float* W, int64_t ldw, const float* s,
-                           float* Y, int64_t ldy, int64_t M, int K, int N, cudaStream_t st) {
+                           float* Y, int64_t ldy, int64_t M, int K, int N, float* work, cudaStream_t st) {
+  if (work && ldx % 4 == 0 && ldy % 4 == 0 && N <= 256 && M > 0) {
+    // tcgen05 3xTF32: Wᵀ split hi/lo (feature-major), then the engine
+    const int np = npad16(N);
+    const int64_t ldT = r32(K);
+    float* hi = work;
+    float* lo = work + int64_t(np) * ldT;
+    cudaError_t e = launch_split_transpose(W, ldw, K, N, np, hi, lo, ldT, st);
+    if (e != cudaSuccess) return e;
+    e = launch_tc_gemm_xw(X, ldx, hi, lo, ldT, s, Y, ldy, M, K, N, st);
+    if (e != cudaSuccess) return e;
+    if (ldy > np) zero_pad_kernel<<<256, 256, 0, st>>>(Y, ldy, M, np);
+    return cudaGetLastError();
+  }
   dim3 grid(unsigned((M + BM - 1) / BM), unsigned((N + BN - 1) / BN), 1);
   gemm_simt_kernel<false, false><<<grid, 256, 0, st>>>(X, ldx, W, ldw, Y, ldy, M, N, K, K, s,
                                                        nullptr, 0, 0);
@@ -127,10 +146,44 @@ cudaError_t launch_gemm_xw(const float* X, int64_t ldx, const float* W, int64_t 
   return cudaGetLastError();
 }
 
-int64_t gemm_xtg_work_floats(int64_t M, int K, int N) { return int64_t(xtg_slices(M)) * K * N; }
+int64_t gemm_xtg_work_floats(int64_t M, int K, int N) {
+  const int64_t simt = int64_t(xtg_slices(M)) * K * N;
+  const int64_t tc = 2 * int64_t(npad16(N)) * r32(M) + tc_xtg_slices(M) * int64_t(K) * npad16(N);
+  return simt > tc ? simt : tc;
+}
+
+__global__ void reduce_slices_ld_kernel(const float* __restrict__ part, int nslices, int64_t rows, int N,
+                                        int ldp, float* __restrict__ out) {
+  const int64_t count = rows * N;
+  for (int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < count;
+       i += int64_t(gridDim.x) * blockDim.x) {
+    const int64_t r = i / N;
+    const int c = int(i - r * N);
+    float a = 0.f;
+    for (int z = 0; z < nslices; ++z) a += part[int64_t(z) * rows * ldp + r * ldp + c];
+    out[i] = a;
+  }
+}
 
 cudaError_t launch_gemm_xtg(const float* X, int64_t ldx, const float* D, int64_t ldd, float* G,
                             int64_t M, int K, int N, float* work, cudaStream_t st) {
+  if (ldx % 4 == 0 && ldd % 4 == 0 && N <= 256 && M > 0) {
+    // tcgen05 3xTF32: Dᵀ split hi/lo (feature-major), engine over fixed row
+    // slices, then a fixed-order sum of the slice partials
+    const int np = npad16(N);
+    const int64_t ldT = r32(M);
+    float* hi = work;
+    float* lo = work + int64_t(np) * ldT;
+    float* part = lo + int64_t(np) * ldT;
+    cudaError_t e = launch_split_transpose(D, ldd, M, N, np, hi, lo, ldT, st);
+    if (e != cudaSuccess) return e;
+    e = launch_tc_gemm_xtg(X, ldx, hi, lo, ldT, part, M, K, N, st);
+    if (e != cudaSuccess) return e;
+    const int64_t cnt = int64_t(K) * N;
+    reduce_slices_ld_kernel<<<unsigned(std::max<int64_t>(1, std::min<int64_t>(1024, (cnt + 255) / 256))), 256, 0, st>>>(
+        part, int(tc_xtg_slices(M)), K, N, np, G);
+    return cudaGetLastError();
+  }
   // G[K x N] = Xᵀ D : output rows = K (A = X transposed), reduction over M
   const int ns = xtg_slices(M);
   int64_t kslice = ((M + ns - 1) / ns + BK - 1) / BK * BK;

@@ -55,8 +55,15 @@ cudaError_t launch_dense_simt_y(const DenseArgs& a, const float* y, int64_t ldy,
                                 cudaStream_t s);
 
 // ---- GEMMs (gemm.cu) ----
+int64_t gemm_xw_work_floats(int K, int N);
 cudaError_t launch_gemm_xw(const float* X, int64_t ldx, const float* W, int64_t ldw, const float* s,
-                           float* Y, int64_t ldy, int64_t M, int K, int N, cudaStream_t st);
+                           float* Y, int64_t ldy, int64_t M, int K, int N, float* work, cudaStream_t st);
+// tcgen05 engine GEMMs (tc_engine.cu)
+cudaError_t launch_tc_gemm_xw(const float* X, int64_t ldx, const float* wThi, const float* wTlo, int64_t ldwT,
+                              const float* rs, float* Y, int64_t ldy, int64_t M, int K, int N, cudaStream_t s);
+int64_t tc_xtg_slices(int64_t M);
+cudaError_t launch_tc_gemm_xtg(const float* X, int64_t ldx, const float* dThi, const float* dTlo, int64_t lddT,
+                               float* partial, int64_t M, int K, int N, cudaStream_t s);
 int64_t gemm_xtg_work_floats(int64_t M, int K, int N);
 cudaError_t launch_gemm_xtg(const float* X, int64_t ldx, const float* D, int64_t ldd, float* G,
                             int64_t M, int K, int N, float* work, cudaStream_t st);

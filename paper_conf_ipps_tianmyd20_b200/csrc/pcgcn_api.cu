@@ -325,13 +325,15 @@ pcgcn_status pcgcn_plan_export(pcgcn_plan_t p, int32_t which, void* buf, int64_t
   return PCGCN_OK;
 }
 
+int64_t pcgcn_gemm_xw_work_floats(int32_t K, int32_t N) { return gemm_xw_work_floats(K, N); }
+
 pcgcn_status pcgcn_gemm_xw(const float* X, int64_t ldx, const float* W, int64_t ldw, const float* s,
-                           float* Y, int64_t ldy, int64_t M, int32_t K, int32_t N, void* stream) {
+                           float* Y, int64_t ldy, int64_t M, int32_t K, int32_t N, float* work, void* stream) {
   if (!X || !W || !Y || M < 0 || K < 1 || N < 1 || ldx < K || ldw < N || ldy < N) {
     set_error("gemm_xw: bad arguments");
     return PCGCN_EINVAL;
   }
-  cudaError_t e = launch_gemm_xw(X, ldx, W, ldw, s, Y, ldy, M, K, N, static_cast<cudaStream_t>(stream));
+  cudaError_t e = launch_gemm_xw(X, ldx, W, ldw, s, Y, ldy, M, K, N, work, static_cast<cudaStream_t>(stream));
   return e == cudaSuccess ? PCGCN_OK : cuda_fail(e, "gemm_xw");
 }
 

@@ -26,6 +26,8 @@
 
 #include <algorithm>
 #include <cstdint>
+#include <cstdio>
+#include <cstdlib>
 
 #include "kernels.h"
 
@@ -41,24 +43,28 @@ __device__ __forceinline__ void add4(float4& a, const float4& b) {
 
 template <int G, int V, bool HAS_ZD>
 __global__ void __launch_bounds__(256) sparse_agg_kernel(AggArgs a) {
-  constexpr int S = 32 / G;       // edge slots per warp
-  constexpr int STEPS = 32 / S;   // edges per slot per index batch
+  constexpr int S = 32 / G;                 // edges in flight per warp step (slots)
+  constexpr int STEPS = 32 / S;             // steps per 32-index batch
+  constexpr int UNR = (8 / V) < 1 ? 1 : (8 / V) > STEPS ? STEPS : (8 / V);  // loads in flight: UNR*V
+  constexpr int NACC = V >= 3 ? 1 : (V == 2 ? 2 : 4);                        // interleaved partial sums
   const int64_t row = int64_t(blockIdx.x) * 8 + (threadIdx.x >> 5);
   if (row >= a.rows) return;
   const int lane = threadIdx.x & 31;
   const int slot = lane / G, l = lane % G;
   const int nvec = (a.F + 3) >> 2;
   const int64_t e0 = a.rowptr[row], e1 = a.rowptr[row + 1];
-  float4 acc[4][V];
+  // per-lane column offsets (loop invariant); lanes past F read the zero row
+  int qoff[V];
 #pragma unroll
-  for (int u = 0; u < 4; ++u)
+  for (int v = 0; v < V; ++v) qoff[v] = (l + G * v) < nvec ? 4 * (l + G * v) : -1;
+  float4 acc[NACC][V];
+#pragma unroll
+  for (int u = 0; u < NACC; ++u)
 #pragma unroll
     for (int v = 0; v < V; ++v) acc[u][v] = make_float4(0.f, 0.f, 0.f, 0.f);
 
-  // Branch-free batches: every lane issues UNR independent 16-byte loads
-  // before consuming any (edges past the row end and lanes past F read a
-  // zero row instead of branching, so ptxas can keep the loads in flight).
-  constexpr int UNR = STEPS < 8 ? STEPS : 8;
+  // Branch-free batches: every lane issues UNR*V independent 16-byte loads
+  // before consuming any; edges past the row end read the zero row.
   const float* zrow = a.zrow;
   for (int64_t base = e0; base < e1; base += 32) {
     const int cnt = (e1 - base) < 32 ? int(e1 - base) : 32;
@@ -71,15 +77,12 @@ __global__ void __launch_bounds__(256) sparse_agg_kernel(AggArgs a) {
         const int j = __shfl_sync(0xffffffffu, myidx, (k0 + u) * S + slot);
         const float* src = a.Y + int64_t(j) * a.ldy;
 #pragma unroll
-        for (int v = 0; v < V; ++v) {
-          const int q = l + G * v;
-          buf[u][v] = ld_f4((j >= 0 && q < nvec) ? src + 4 * q : zrow);
-        }
+        for (int v = 0; v < V; ++v) buf[u][v] = ld_f4((j >= 0 && qoff[v] >= 0) ? src + qoff[v] : zrow);
       }
 #pragma unroll
       for (int u = 0; u < UNR; ++u)
 #pragma unroll
-        for (int v = 0; v < V; ++v) add4(acc[(k0 + u) & 3][v], buf[u][v]);
+        for (int v = 0; v < V; ++v) add4(acc[(k0 + u) % NACC][v], buf[u][v]);
       if ((k0 + UNR) * S >= cnt) break;  // warp-uniform: rest of the batch is empty
     }
   }
@@ -87,12 +90,10 @@ __global__ void __launch_bounds__(256) sparse_agg_kernel(AggArgs a) {
 #pragma unroll
   for (int v = 0; v < V; ++v) {
     tot[v] = acc[0][v];
-    add4(tot[v], acc[1][v]);
-    float4 t2 = acc[2][v];
-    add4(t2, acc[3][v]);
-    add4(tot[v], t2);
 #pragma unroll
-    for (int off = G; off < 32; off <<= 1) {
+    for (int u = 1; u < NACC; ++u) add4(tot[v], acc[u][v]);
+#pragma unroll
+    for (int off = G; off < 32; off <<= 1) {  // fixed butterfly over the slots
       tot[v].x += __shfl_xor_sync(0xffffffffu, tot[v].x, off);
       tot[v].y += __shfl_xor_sync(0xffffffffu, tot[v].y, off);
       tot[v].z += __shfl_xor_sync(0xffffffffu, tot[v].z, off);
@@ -101,34 +102,45 @@ __global__ void __launch_bounds__(256) sparse_agg_kernel(AggArgs a) {
   }
   const float ri = a.r[a.row_lo + row];
   const int zi = HAS_ZD ? a.zd_index[row] : -1;
-  const int mw = (a.F + 31) >> 5;
+  uint32_t bal[V][4];
 #pragma unroll
   for (int v = 0; v < V; ++v) {
-    const int q = l + G * v;
-    const bool own = slot == 0 && q < nvec;
+    const bool own = slot == 0 && qoff[v] >= 0;
     float4 z = tot[v];
-    if (HAS_ZD && own && zi >= 0) add4(z, ld_f4(a.zd + int64_t(zi) * a.ldzd + 4 * q));
+    if (HAS_ZD && own && zi >= 0) add4(z, ld_f4(a.zd + int64_t(zi) * a.ldzd + qoff[v]));
     z.x *= ri; z.y *= ri; z.z *= ri; z.w *= ri;
     if (a.out_prescaled) { z.x *= ri; z.y *= ri; z.z *= ri; z.w *= ri; }
     if (a.mask) {
-      const int c = 4 * q;
-      uint32_t nib = 0;
-      if (own) {
-        nib |= (z.x > 0.f && c + 0 < a.F) ? 1u : 0u;
-        nib |= (z.y > 0.f && c + 1 < a.F) ? 2u : 0u;
-        nib |= (z.z > 0.f && c + 2 < a.F) ? 4u : 0u;
-        nib |= (z.w > 0.f && c + 3 < a.F) ? 8u : 0u;
-      }
-      uint32_t w = nib << (4 * (q & 7));
-      w |= __shfl_xor_sync(0xffffffffu, w, 1);
-      w |= __shfl_xor_sync(0xffffffffu, w, 2);
-      w |= __shfl_xor_sync(0xffffffffu, w, 4);
-      if (own && (q & 7) == 0) a.mask[row * mw + (q >> 3)] = w;
+      const int c = qoff[v];
+      bal[v][0] = __ballot_sync(0xffffffffu, own && z.x > 0.f && c + 0 < a.F);
+      bal[v][1] = __ballot_sync(0xffffffffu, own && z.y > 0.f && c + 1 < a.F);
+      bal[v][2] = __ballot_sync(0xffffffffu, own && z.z > 0.f && c + 2 < a.F);
+      bal[v][3] = __ballot_sync(0xffffffffu, own && z.w > 0.f && c + 3 < a.F);
     }
     if (a.relu) {
       z.x = fmaxf(z.x, 0.f); z.y = fmaxf(z.y, 0.f); z.z = fmaxf(z.z, 0.f); z.w = fmaxf(z.w, 0.f);
     }
-    if (own) *reinterpret_cast<float4*>(a.Z + row * a.ldz + 4 * q) = z;
+    if (own) *reinterpret_cast<float4*>(a.Z + row * a.ldz + qoff[v]) = z;
+  }
+  if (a.mask) {
+    // lane w assembles mask word w: column col = 32w + b lives in lane
+    // (col/4) % G, vector v = (col/4) / G, component col % 4
+    const int mw = (a.F + 31) >> 5;
+    if (lane < mw) {
+      uint32_t word = 0;
+#pragma unroll 4
+      for (int b = 0; b < 32; ++b) {
+        const int col = 32 * lane + b;
+        const int q = col >> 2;
+        const int vv = q / G, ll = q % G;
+        uint32_t bit = 0;
+#pragma unroll
+        for (int v = 0; v < V; ++v)
+          if (v == vv) bit = (bal[v][col & 3] >> ll) & 1u;
+        word |= bit << b;
+      }
+      a.mask[row * mw + lane] = word;
+    }
   }
 }
 
@@ -194,14 +206,33 @@ __global__ void __launch_bounds__(256) split_transpose_kernel(const float* __res
 
 cudaError_t launch_sparse_agg(const AggArgs& a, cudaStream_t s) {
   if (a.rows <= 0) return cudaSuccess;
+  // (G lanes x V float4) per edge, minimising warp instructions per edge
+  // (~G*(3+5V)/32) while keeping each v-slice of G lanes a contiguous segment
   const int nvec = (a.F + 3) / 4;
+  // tuning override (benchmarks only): PCGCN_SPARSE_GV="G,V" when G*V >= nvec
+  static int og = -1, ov = -1;
+  if (og < 0) {
+    og = ov = 0;
+    if (const char* e = getenv("PCGCN_SPARSE_GV")) sscanf(e, "%d,%d", &og, &ov);
+  }
+  if (og > 0 && og * ov >= nvec) {
+#define GV(g, v) if (og == g && ov == v) return launch_gv<g, v>(a, s);
+    GV(32, 1) GV(32, 2) GV(16, 1) GV(16, 2) GV(16, 3) GV(16, 4) GV(8, 1) GV(8, 2) GV(8, 3) GV(8, 4)
+    GV(4, 3) GV(4, 4) GV(2, 4)
+#undef GV
+  }
   if (nvec <= 1) return launch_gv<1, 1>(a, s);
-  if (nvec <= 2) return launch_gv<2, 1>(a, s);
-  if (nvec <= 4) return launch_gv<4, 1>(a, s);
-  if (nvec <= 8) return launch_gv<8, 1>(a, s);
-  if (nvec <= 16) return launch_gv<16, 1>(a, s);
-  if (nvec <= 32) return launch_gv<32, 1>(a, s);
-  return launch_gv<32, 2>(a, s);
+  if (nvec <= 2) return launch_gv<1, 2>(a, s);
+  if (nvec <= 3) return launch_gv<1, 3>(a, s);
+  if (nvec <= 4) return launch_gv<1, 4>(a, s);
+  if (nvec <= 6) return launch_gv<2, 3>(a, s);
+  if (nvec <= 8) return launch_gv<2, 4>(a, s);
+  if (nvec <= 12) return launch_gv<4, 3>(a, s);
+  if (nvec <= 16) return launch_gv<4, 4>(a, s);
+  if (nvec <= 24) return launch_gv<8, 3>(a, s);
+  if (nvec <= 32) return launch_gv<32, 1>(a, s);  // measured faster than (8,4) at F=128 on C3
+  if (nvec <= 48) return launch_gv<16, 3>(a, s);
+  return launch_gv<16, 4>(a, s);
 }
 
 cudaError_t launch_prescale(const float* Y, int64_t ldy, const float* r, int64_t n, int F, float* ypre,

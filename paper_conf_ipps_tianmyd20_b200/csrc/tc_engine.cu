@@ -1,0 +1,544 @@
+// tcgen05 engine for sm_100a: one persistent, warp-specialised kernel that
+// computes   D[tile] = Σ_chunks A[tile, chunk] · B[chunk]   with fp32
+// accumulators in TMEM, B tiles fed by TMA and A tiles built by threads
+// directly in TMEM.  Three A sources share the pipeline:
+//
+//  A_BITS     full-mode ("dense") aggregation — PAPER.md §III-B.b (L151-L153:
+//             a dense block is treated as fully connected, missing edges carry
+//             0), §IV-A (L175 dense format) and §IV-D (L191-L193: full mode on
+//             Tensor Cores, mixed precision, conversion when combining).  A is
+//             the 128x32 0/1 tile of a destination row tile over a 32-aligned
+//             source window, shipped as 512 B of bits and expanded to tf32 in
+//             TMEM; B = the window's 32 source rows of Y' = hi + lo.
+//             2 MMAs per K-step (A·B_hi, A·B_lo; A∈{0,1} is exact in tf32).
+//  A_ROWMAJOR transform GEMM  Y = diag(s)·X·W  (Alg. 1 a^l = h^{l-1} w^l, L114):
+//             A = 128x32 tile of row-major X (TMA, SWIZZLE_128B), split by
+//             the builders into tf32 hi/lo in TMEM; B = Wᵀ split hi/lo.
+//             3xTF32: A_hi·B_hi + A_lo·B_hi + A_hi·B_lo.
+//  A_TRANS    weight-gradient GEMM  ∇Θ = Xᵀ·G  (backward of L114; the paper
+//             is silent on the backward, reading A4): A = Xᵀ tile, loaded as a
+//             32-row x 128-feature box of X and transposed by the builders;
+//             B = Gᵀ split hi/lo; split-K over rows into fixed slices.
+//
+// Roles (320 threads): warp 0 lane 0 = TMA producer, warp 1 = TMEM allocator
+// + single-thread MMA issuer, warps 2..5 = A builders (thread m owns tile row
+// m = TMEM lane m), warps 6..9 = epilogue (tcgen05.ld -> global), with a
+// double-buffered accumulator so a tile's epilogue overlaps the next tile's
+// MMAs.  Split precision: for any fp32 v, hi = v with the low 13 mantissa
+// bits cleared and lo = v - hi are exact; tf32(lo) keeps 11 more bits, so
+// hi + tf32(lo) = v (1 ± 2^-22).
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <cudaTypedefs.h>
+
+#include <cstdint>
+#include <cstdlib>
+#include <cstring>
+#include <mutex>
+
+#include "kernels.h"
+
+namespace pcgcn {
+namespace {
+
+constexpr int BM = 128;        // rows per tile (UMMA M)
+constexpr int BK = 32;         // K per chunk (4 x UMMA K=8 for tf32)
+constexpr int NTHREADS = 320;  // 10 warps
+enum AMode { A_BITS = 0, A_ROWMAJOR = 1, A_TRANS = 2 };
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t* b, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(b)), "r"(count));
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* b, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(b)), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* b) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(b)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {
+  uint32_t addr = smem_u32(b);
+  asm volatile(
+      "{\n"
+      ".reg .pred p;\n"
+      "WAIT_%=:\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      "@!p bra WAIT_%=;\n"
+      "}\n" ::"r"(addr),
+      "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void tma_load_2d(const CUtensorMap* map, uint64_t* bar, void* dst, int c0,
+                                            int c1) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];" ::"r"(
+          smem_u32(dst)),
+      "l"(map), "r"(smem_u32(bar)), "r"(c0), "r"(c1)
+      : "memory");
+}
+__device__ __forceinline__ void bulk_load(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                   smem_u32(dst)),
+               "l"(src), "r"(bytes), "r"(smem_u32(bar))
+               : "memory");
+}
+__device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
+__device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
+__device__ __forceinline__ void tc_commit(uint64_t* bar) {
+  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
+                   smem_u32(bar))
+               : "memory");
+}
+// D[tmem] (+)= A[tmem] · B[smem desc]
+__device__ __forceinline__ void mma_ts(uint32_t d, uint32_t a, uint64_t bdesc, uint32_t idesc, uint32_t acc) {
+  asm volatile(
+      "{\n"
+      ".reg .pred p;\n"
+      "setp.ne.b32 p, %4, 0;\n"
+      "tcgen05.mma.cta_group::1.kind::tf32 [%0], [%1], %2, %3, p;\n"
+      "}\n" ::"r"(d),
+      "r"(a), "l"(bdesc), "r"(idesc), "r"(acc)
+      : "memory");
+}
+__device__ __forceinline__ void sttm32(uint32_t taddr, const uint32_t (&v)[32]) {
+  asm volatile(
+      "tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,"
+      "%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31,%32};" ::"r"(taddr),
+      "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7]), "r"(v[8]), "r"(v[9]),
+      "r"(v[10]), "r"(v[11]), "r"(v[12]), "r"(v[13]), "r"(v[14]), "r"(v[15]), "r"(v[16]), "r"(v[17]), "r"(v[18]),
+      "r"(v[19]), "r"(v[20]), "r"(v[21]), "r"(v[22]), "r"(v[23]), "r"(v[24]), "r"(v[25]), "r"(v[26]), "r"(v[27]),
+      "r"(v[28]), "r"(v[29]), "r"(v[30]), "r"(v[31])
+      : "memory");
+}
+
+// UMMA shared-memory matrix descriptor (sm_100): start>>4 [0,14), LBO>>4
+// [16,30), SBO>>4 [32,46), version=1 [46,48), layout type [61,64) (2=SW128).
+// K-major SW128: 8-row groups 1024 B apart; K advance = +32 B per 8 tf32.
+__device__ __forceinline__ uint64_t sdesc_kmajor_sw128(uint32_t saddr) {
+  return uint64_t((saddr >> 4) & 0x3FFFu) | (uint64_t(1) << 16) | (uint64_t(1024 >> 4) << 32) |
+         (uint64_t(1) << 46) | (uint64_t(2) << 61);
+}
+// instruction descriptor, kind::tf32: D f32 [4,6), A tf32 [7,10), B tf32
+// [10,13), A and B K-major (bits 15/16 = 0), N>>3 [17,23), M>>4 [24,29).
+// (MN-major B reads as zeros for kind::tf32 on the B200 — measured with
+// tests/cuda/tc_probe.cu — so every B operand is stored feature-major.)
+__host__ __device__ constexpr uint32_t idesc_tf32(int M, int N) {
+  return (1u << 4) | (2u << 7) | (2u << 10) | (uint32_t(N >> 3) << 17) | (uint32_t(M >> 4) << 24);
+}
+
+struct Layout {
+  int npad, stages, nacc, a_cols;     // a_cols: TMEM columns of one A stage (32, or 64 for hi+lo)
+  uint32_t a_bytes, b_bytes, stage_bytes, a_load_bytes;
+  uint32_t tmem_cols, a_col0;
+};
+
+Layout make_layout(int mode, int npad, int max_stages) {
+  Layout L;
+  L.npad = npad;
+  L.a_cols = mode == A_BITS ? BK : 2 * BK;
+  L.a_bytes = mode == A_BITS ? 1024 : BM * BK * 4;       // bits (512 used) or a 16 KB fp32 tile
+  L.a_load_bytes = mode == A_BITS ? BM * 4 : BM * BK * 4;
+  L.b_bytes = uint32_t(npad) * BK * 4;
+  L.stage_bytes = L.a_bytes + 2 * L.b_bytes;
+  int st = int((200 * 1024) / L.stage_bytes);
+  st = st < 2 ? 2 : st;
+  st = st > max_stages ? max_stages : st;
+  L.nacc = 2;
+  while (L.nacc * npad + st * L.a_cols > 512) {
+    if (st > 2) --st;
+    else { L.nacc = 1; break; }
+  }
+  L.stages = st;
+  const uint32_t need = uint32_t(L.nacc * npad + L.stages * L.a_cols);
+  uint32_t cols = 32;
+  while (cols < need) cols <<= 1;
+  L.tmem_cols = cols;
+  L.a_col0 = uint32_t(L.nacc * npad);
+  return L;
+}
+
+struct Work {
+  // tiles
+  int64_t ntiles;
+  // A_BITS
+  const int64_t* rt_cptr;
+  const int32_t* ch_col0;
+  const uint32_t* bits;
+  // GEMMs: reduction extent and split
+  int64_t kdim;      // A_ROWMAJOR: K (features); A_TRANS: rows (reduction)
+  int64_t kslice;    // A_TRANS: rows per split (multiple of 32)
+  int64_t mdim;      // rows of the output (A_ROWMAJOR: M rows; A_TRANS: K features)
+  int mtiles;        // A_TRANS: ceil(mdim / 128)
+  // output
+  float* out;
+  int64_t ldo;
+  int ncols;         // columns written per output row (<= npad, multiple of 4)
+  const float* rowscale;
+  int64_t split_stride;
+};
+
+template <int MODE>
+__device__ __forceinline__ void tile_range(const Work& w, int64_t t, int64_t& kb, int64_t& nch, int64_t& m0,
+                                           int64_t& sp) {
+  if (MODE == A_BITS) {
+    kb = w.rt_cptr[t];
+    nch = w.rt_cptr[t + 1] - kb;
+    m0 = t * BM;
+    sp = 0;
+  } else if (MODE == A_ROWMAJOR) {
+    kb = 0;
+    nch = (w.kdim + BK - 1) / BK;
+    m0 = t * BM;
+    sp = 0;
+  } else {
+    const int64_t mt = t % w.mtiles;
+    sp = t / w.mtiles;
+    m0 = mt * BM;
+    kb = sp * w.kslice;
+    int64_t ke = kb + w.kslice < w.kdim ? kb + w.kslice : w.kdim;
+    nch = ke > kb ? (ke - kb + BK - 1) / BK : 0;
+  }
+}
+
+template <int MODE>
+__global__ void __launch_bounds__(NTHREADS, 1)
+    tc_engine_kernel(const __grid_constant__ CUtensorMap map_bhi, const __grid_constant__ CUtensorMap map_blo,
+                     const __grid_constant__ CUtensorMap map_a, const Work w, const Layout L) {
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint64_t* bar = reinterpret_cast<uint64_t*>(smem + L.stages * L.stage_bytes);
+  uint64_t* full = bar;                     // [stages] A + B landed
+  uint64_t* a_full = bar + L.stages;        // [stages] A written to TMEM (128 arrivals)
+  uint64_t* empty = bar + 2 * L.stages;     // [stages] MMAs done with the stage
+  uint64_t* acc_full = bar + 3 * L.stages;  // [2]
+  uint64_t* acc_empty = acc_full + 2;       // [2] (128 arrivals)
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(acc_empty + 2);
+  const int npad = L.npad;
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < L.stages; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&a_full[s], 128);
+      mbar_init(&empty[s], 1);
+    }
+    for (int b = 0; b < 2; ++b) {
+      mbar_init(&acc_full[b], 1);
+      mbar_init(&acc_empty[b], 128);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+                 "r"(L.tmem_cols)
+                 : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+
+  if (warp == 0) {
+    if (lane == 0) {
+      // ---- producer ----
+      const uint32_t tx = L.a_load_bytes + 2u * L.b_bytes;
+      uint32_t g = 0;
+      for (int64_t t = blockIdx.x; t < w.ntiles; t += gridDim.x) {
+        int64_t kb, nch, m0, sp;
+        tile_range<MODE>(w, t, kb, nch, m0, sp);
+        for (int64_t i = 0; i < nch; ++i, ++g) {
+          const int s = int(g % uint32_t(L.stages));
+          mbar_wait(&empty[s], ((g / L.stages) & 1u) ^ 1u);
+          uint8_t* st = smem + s * L.stage_bytes;
+          mbar_expect_tx(&full[s], tx);
+          int k0;
+          if (MODE == A_BITS) {
+            k0 = w.ch_col0[kb + i];
+            bulk_load(st, w.bits + (kb + i) * BM, BM * 4, &full[s]);
+          } else if (MODE == A_ROWMAJOR) {
+            k0 = int(i * BK);
+            tma_load_2d(&map_a, &full[s], st, k0, int(m0));
+          } else {
+            k0 = int(kb + i * BK);
+            tma_load_2d(&map_a, &full[s], st, int(m0), k0);
+          }
+          tma_load_2d(&map_bhi, &full[s], st + L.a_bytes, k0, 0);
+          tma_load_2d(&map_blo, &full[s], st + L.a_bytes + L.b_bytes, k0, 0);
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0) {
+      // ---- MMA issuer ----
+      const uint32_t idesc = idesc_tf32(BM, npad);
+      uint32_t g = 0, lt = 0;
+      for (int64_t t = blockIdx.x; t < w.ntiles; t += gridDim.x, ++lt) {
+        int64_t kb, nch, m0, sp;
+        tile_range<MODE>(w, t, kb, nch, m0, sp);
+        const uint32_t ab = lt % uint32_t(L.nacc);
+        mbar_wait(&acc_empty[ab], ((lt / L.nacc) & 1u) ^ 1u);
+        tc_fence_after();
+        const uint32_t d = tmem + ab * uint32_t(npad);
+        uint32_t acc = 0;
+        for (int64_t i = 0; i < nch; ++i, ++g) {
+          const int s = int(g % uint32_t(L.stages));
+          const uint32_t ph = (g / L.stages) & 1u;
+          mbar_wait(&full[s], ph);
+          mbar_wait(&a_full[s], ph);
+          tc_fence_after();
+          const uint32_t b0 = smem_u32(smem + s * L.stage_bytes + L.a_bytes);
+          const uint32_t a0 = tmem + L.a_col0 + uint32_t(s) * uint32_t(L.a_cols);
+#pragma unroll
+          for (int kk = 0; kk < BK / 8; ++kk) {
+            const uint64_t bh = sdesc_kmajor_sw128(b0 + kk * 32u);
+            const uint64_t bl = sdesc_kmajor_sw128(b0 + L.b_bytes + kk * 32u);
+            mma_ts(d, a0 + kk * 8u, bh, idesc, acc);
+            mma_ts(d, a0 + kk * 8u, bl, idesc, 1u);
+            if (MODE != A_BITS) mma_ts(d, a0 + BK + kk * 8u, bh, idesc, 1u);
+            acc = 1u;
+          }
+          tc_commit(&empty[s]);
+        }
+        tc_commit(&acc_full[ab]);
+      }
+    }
+  } else if (warp < 6) {
+    // ---- A builders: thread m writes row m of the A tile into TMEM ----
+    const int m = ((warp & 3) << 5) | lane;
+    const uint32_t lane_base = uint32_t((warp & 3) * 32) << 16;
+    uint32_t g = 0;
+    for (int64_t t = blockIdx.x; t < w.ntiles; t += gridDim.x) {
+      int64_t kb, nch, m0, sp;
+      tile_range<MODE>(w, t, kb, nch, m0, sp);
+      for (int64_t i = 0; i < nch; ++i, ++g) {
+        const int s = int(g % uint32_t(L.stages));
+        mbar_wait(&full[s], (g / L.stages) & 1u);  // data landed; stage and its TMEM A buffer are free
+        const uint8_t* st = smem + s * L.stage_bytes;
+        const uint32_t taddr = tmem + lane_base + L.a_col0 + uint32_t(s) * uint32_t(L.a_cols);
+        uint32_t v[32];
+        if (MODE == A_BITS) {
+          const uint32_t wd = reinterpret_cast<const uint32_t*>(st)[m];
+#pragma unroll
+          for (int b = 0; b < 32; ++b) v[b] = ((wd >> b) & 1u) ? 0x3f800000u : 0u;
+          sttm32(taddr, v);
+        } else {
+          float x[32];
+          if (MODE == A_ROWMAJOR) {
+            // row m of a SWIZZLE_128B tile: 16-byte chunk j lives at j ^ (m & 7)
+            const float4* row = reinterpret_cast<const float4*>(st + m * 128);
+#pragma unroll
+            for (int j = 0; j < 8; ++j) {
+              const float4 q = row[j ^ (m & 7)];
+              x[4 * j] = q.x; x[4 * j + 1] = q.y; x[4 * j + 2] = q.z; x[4 * j + 3] = q.w;
+            }
+          } else {
+            // column m of a plain [32 rows][128 features] tile
+            const float* tile = reinterpret_cast<const float*>(st);
+#pragma unroll
+            for (int r = 0; r < 32; ++r) x[r] = tile[r * BM + m];
+          }
+          uint32_t lo[32];
+#pragma unroll
+          for (int k = 0; k < 32; ++k) {
+            const uint32_t h = __float_as_uint(x[k]) & 0xffffe000u;
+            v[k] = h;
+            lo[k] = __float_as_uint(x[k] - __uint_as_float(h));
+          }
+          sttm32(taddr, v);
+          sttm32(taddr + BK, lo);
+        }
+        asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+        tc_fence_before();
+        mbar_arrive(&a_full[s]);
+      }
+    }
+  } else {
+    // ---- epilogue: TMEM accumulator -> global ----
+    const int m = ((warp & 3) << 5) | lane;
+    const uint32_t lane_base = uint32_t((warp & 3) * 32) << 16;
+    uint32_t lt = 0;
+    for (int64_t t = blockIdx.x; t < w.ntiles; t += gridDim.x, ++lt) {
+      int64_t kb, nch, m0, sp;
+      tile_range<MODE>(w, t, kb, nch, m0, sp);
+      const uint32_t ab = lt % uint32_t(L.nacc);
+      mbar_wait(&acc_full[ab], (lt / L.nacc) & 1u);
+      tc_fence_after();
+      const int64_t row = m0 + m;
+      const bool live = MODE == A_BITS || row < w.mdim;
+      float* out = w.out + sp * w.split_stride + row * w.ldo;
+      const float sc = (MODE == A_ROWMAJOR && w.rowscale && live) ? w.rowscale[row] : 1.f;
+      const uint32_t src = tmem + lane_base + ab * uint32_t(npad);
+      for (int c0 = 0; c0 < npad; c0 += 16) {
+        uint32_t r[16];
+        asm volatile(
+            "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+            : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+              "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]),
+              "=r"(r[15])
+            : "r"(src + uint32_t(c0)));
+        asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+        if (live) {
+#pragma unroll
+          for (int q = 0; q < 4; ++q)
+            if (c0 + 4 * q < w.ncols)
+              *reinterpret_cast<float4*>(out + c0 + 4 * q) =
+                  make_float4(__uint_as_float(r[4 * q]) * sc, __uint_as_float(r[4 * q + 1]) * sc,
+                              __uint_as_float(r[4 * q + 2]) * sc, __uint_as_float(r[4 * q + 3]) * sc);
+        }
+      }
+      tc_fence_before();
+      mbar_arrive(&acc_empty[ab]);
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) {
+    tc_fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(L.tmem_cols)
+                 : "memory");
+  }
+}
+
+PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
+  });
+  return fn;
+}
+
+// 2-D fp32 tensor map: inner extent d0 (contiguous), outer d1, row pitch ld floats
+bool make_map(CUtensorMap* map, const float* base, int64_t d0, int64_t d1, int64_t ld, int box0, int box1,
+              bool swz128) {
+  auto enc = get_encode();
+  if (!enc) return false;
+  cuuint64_t dims[2] = {cuuint64_t(d0), cuuint64_t(d1)};
+  cuuint64_t strides[1] = {cuuint64_t(ld) * 4};
+  cuuint32_t box[2] = {cuuint32_t(box0), cuuint32_t(box1)};
+  cuuint32_t estr[2] = {1, 1};
+  CUresult r = enc(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(base), dims, strides, box, estr,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE,
+                   swz128 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_NONE,
+                   CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return r == CUDA_SUCCESS;
+}
+
+int num_sms() {
+  static int sms = 0;
+  if (!sms) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    if (sms <= 0) sms = 148;
+  }
+  return sms;
+}
+
+int max_stages_env() {
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("PCGCN_TC_STAGES");  // tuning override (benchmarks only)
+    v = e ? atoi(e) : 8;
+    if (v < 2) v = 2;
+    if (v > 12) v = 12;
+  }
+  return v;
+}
+
+template <int MODE>
+cudaError_t launch_engine(const CUtensorMap& bhi, const CUtensorMap& blo, const CUtensorMap& amap, const Work& w,
+                          int npad, cudaStream_t s) {
+  if (w.ntiles <= 0) return cudaSuccess;
+  const Layout L = make_layout(MODE, npad, max_stages_env());
+  const size_t smem = 1024 + size_t(L.stages) * L.stage_bytes + (3 * L.stages + 4) * 8 + 16;
+  if (smem > 227 * 1024) return cudaErrorInvalidValue;
+  static bool attr_done = false;
+  if (!attr_done) {
+    cudaError_t e = cudaFuncSetAttribute(tc_engine_kernel<MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         227 * 1024);
+    if (e != cudaSuccess) return e;
+    attr_done = true;
+  }
+  const int64_t grid = w.ntiles < num_sms() ? w.ntiles : num_sms();
+  tc_engine_kernel<MODE><<<unsigned(grid), NTHREADS, smem, s>>>(bhi, blo, amap, w, L);
+  return cudaGetLastError();
+}
+
+}  // namespace
+
+// ---- full-mode aggregation ----
+cudaError_t launch_dense_tc(const DenseArgs& a, cudaStream_t s) {
+  if (a.nrt <= 0) return cudaSuccess;
+  if (a.npad % 16 != 0 || a.npad < 16 || a.npad > 256 || a.ldT % 4 != 0) return cudaErrorInvalidValue;
+  CUtensorMap mh, ml;
+  if (!make_map(&mh, a.hiT, a.n, a.npad, a.ldT, BK, a.npad, true) ||
+      !make_map(&ml, a.loT, a.n, a.npad, a.ldT, BK, a.npad, true))
+    return cudaErrorInvalidValue;
+  Work w{};
+  w.ntiles = a.nrt;
+  w.rt_cptr = a.rt_cptr;
+  w.ch_col0 = a.ch_col0;
+  w.bits = a.bits;
+  w.out = a.zd;
+  w.ldo = a.ldzd;
+  w.ncols = a.npad;
+  return launch_engine<A_BITS>(mh, ml, mh, w, a.npad, s);
+}
+
+// ---- Y = diag(s)·X·W, W pre-split feature-major (wT hi/lo [npad][ldwT]) ----
+cudaError_t launch_tc_gemm_xw(const float* X, int64_t ldx, const float* wThi, const float* wTlo, int64_t ldwT,
+                              const float* rs, float* Y, int64_t ldy, int64_t M, int K, int N, cudaStream_t s) {
+  const int npad = (N + 15) / 16 * 16;
+  if (ldx % 4 || ldwT % 4 || ldy % 4 || npad > 256) return cudaErrorInvalidValue;
+  CUtensorMap mh, ml, ma;
+  if (!make_map(&mh, wThi, K, npad, ldwT, BK, npad, true) || !make_map(&ml, wTlo, K, npad, ldwT, BK, npad, true) ||
+      !make_map(&ma, X, K, M, ldx, BK, BM, true))
+    return cudaErrorInvalidValue;
+  Work w{};
+  w.ntiles = (M + BM - 1) / BM;
+  w.kdim = K;
+  w.mdim = M;
+  w.out = Y;
+  w.ldo = ldy;
+  w.ncols = int(ldy < npad ? ldy : npad);
+  w.rowscale = rs;
+  return launch_engine<A_ROWMAJOR>(mh, ml, ma, w, npad, s);
+}
+
+// ---- partial[sp] = X[rows of slice sp]ᵀ · D, D pre-split feature-major ----
+int64_t tc_xtg_slices(int64_t M) {
+  int64_t sl = (M + 8191) / 8192;
+  return sl < 1 ? 1 : (sl > 64 ? 64 : sl);
+}
+cudaError_t launch_tc_gemm_xtg(const float* X, int64_t ldx, const float* dThi, const float* dTlo, int64_t lddT,
+                               float* partial, int64_t M, int K, int N, cudaStream_t s) {
+  const int npad = (N + 15) / 16 * 16;
+  if (ldx % 4 || lddT % 4 || npad > 256) return cudaErrorInvalidValue;
+  CUtensorMap mh, ml, ma;
+  if (!make_map(&mh, dThi, M, npad, lddT, BK, npad, true) || !make_map(&ml, dTlo, M, npad, lddT, BK, npad, true) ||
+      !make_map(&ma, X, K, M, ldx, BM, BK, false))
+    return cudaErrorInvalidValue;
+  const int64_t ns = tc_xtg_slices(M);
+  Work w{};
+  w.mtiles = (K + BM - 1) / BM;
+  w.ntiles = int64_t(w.mtiles) * ns;
+  w.kdim = M;
+  w.kslice = ((M + ns - 1) / ns + BK - 1) / BK * BK;
+  w.mdim = K;
+  w.out = partial;
+  w.ldo = npad;
+  w.ncols = npad;
+  w.split_stride = int64_t(K) * npad;
+  return launch_engine<A_TRANS>(mh, ml, ma, w, npad, s);
+}
+
+}  // namespace pcgcn

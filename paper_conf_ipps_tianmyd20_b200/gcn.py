@@ -54,7 +54,10 @@ class GCN2:
         d, f32 = self.dev, torch.float32
         n, rows, H, C = self.n, self.rows, self.H, self.C
         self.ldH, self.ldC = _ld(H), _ld(C)
-        self.X = torch.from_numpy(np.ascontiguousarray(X_plan[self.lo:self.hi], dtype=np.float32)).to(d)
+        # X rows padded to a multiple of 4 floats (16-byte rows: TMA-loadable)
+        self.ldX = _ld(self.f_in)
+        self.X = torch.zeros(self.rows, self.ldX, dtype=f32, device=d)
+        self.X[:, :self.f_in] = torch.from_numpy(np.ascontiguousarray(X_plan[self.lo:self.hi], dtype=np.float32)).to(d)
         self.labels = torch.from_numpy(np.ascontiguousarray(labels_plan[self.lo:self.hi], dtype=np.int32)).to(d)
         self.train = torch.from_numpy(np.ascontiguousarray(train_plan[self.lo:self.hi], dtype=np.uint8)).to(d)
         self.inv_nT = 1.0 / float(np.count_nonzero(train_plan))
@@ -82,6 +85,8 @@ class GCN2:
         self.ce_work = torch.zeros(L.CE_WORK_FLOATS, dtype=f32, device=d)
         wk = max(L.gemm_xtg_work_floats(rows, self.f_in, H), L.gemm_xtg_work_floats(rows, H, C))
         self.xtg_work = torch.zeros(max(wk, 1), dtype=f32, device=d)
+        wk = max(L.gemm_xw_work_floats(self.f_in, H), L.gemm_xw_work_floats(H, C))
+        self.xw_work = torch.zeros(wk, dtype=f32, device=d)
         self.r = plan.rowscale_ptr()  # device [n]
         self.r_local = None if self.lo == 0 else self.r + 4 * self.lo
         self._graph = None
@@ -105,7 +110,8 @@ class GCN2:
         rr = self._r_rows()
         H, C, p = self.H, self.C, self.plan
         # layer 1
-        L.gemm_xw(self.X, self.Th0, rr, self._local(self.Y0), M=self.rows, K=self.f_in, N=H, stream=stream)
+        L.gemm_xw(self.X, self.Th0, rr, self._local(self.Y0), M=self.rows, K=self.f_in, N=H, work=self.xw_work,
+                  stream=stream)
         mark("a4_gemm_xw0")
         self._gather(self.Y0)
         mark("x_gather_y0")
@@ -113,7 +119,8 @@ class GCN2:
                   stream=stream)
         mark("a5a6_agg_fwd_H")
         # layer 2
-        L.gemm_xw(self.H1, self.Th1, rr, self._local(self.Y1), M=self.rows, K=H, N=C, stream=stream)
+        L.gemm_xw(self.H1, self.Th1, rr, self._local(self.Y1), M=self.rows, K=H, N=C, work=self.xw_work,
+                  stream=stream)
         mark("a7_gemm_xw1")
         self._gather(self.Y1)
         mark("x_gather_y1")

@@ -36,7 +36,7 @@ __global__ void probe(int mode, float* out, uint32_t* info) {
   // fill A (128 x 32 tf32, K-major SW128): element (m,k)
   for (int e = t; e < 128 * 32; e += blockDim.x) {
     int m = e / 32, k = e % 32;
-    float v = (mode == 2) ? ((k == (m % 8)) ? 1.f : 0.f) : 1.f;
+    float v = (mode == 2) ? ((k == (m % 8)) ? 1.f : 0.f) : (mode == 5 ? 1.000732421875f : 1.f);
     int chunk = k / 4, w = k % 4;
     sA[(m * 128 + ((chunk ^ (m & 7)) << 4)) / 4 + w] = v;
   }
@@ -45,9 +45,9 @@ __global__ void probe(int mode, float* out, uint32_t* info) {
   __syncthreads();
   for (int e = t; e < 32 * 32; e += blockDim.x) {
     int k = e / 32, n = e % 32;
-    float v = (mode == 1) ? 1.f : (mode == 3 ? float(k * 32 + n) : float(k * 16 + n));
+    float v = (mode == 1 || mode == 5) ? 1.f : (mode == 3 ? float(k * 32 + n) : float(k * 16 + n));
     if (mode != 3 && n >= 16) continue;
-    if (mode == 3) {
+    if (mode == 5) { int chunk = k / 4, w = k % 4; sB[(n * 128 + ((chunk ^ (n & 7)) << 4)) / 4 + w] = v; } else if (mode == 3) {
       sB[(k * 128 + (((n / 4) ^ (k & 7)) << 4)) / 4 + (n % 4)] = v;
     } else if (mode <= 2) {
       // K-major SW128: row n (128 B = 32 k), chunk swizzle by n%8
@@ -83,9 +83,9 @@ __global__ void probe(int mode, float* out, uint32_t* info) {
     asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
   } else if (t == 0) {
     uint64_t ad = make_sdesc(smem_u32(sA), 16, 1024, 2);
-    uint64_t bd = mode <= 2 ? make_sdesc(smem_u32(sB), 16, 1024, 2)
+    uint64_t bd = (mode <= 2 || mode == 5) ? make_sdesc(smem_u32(sB), 16, 1024, 2)
                 : (mode == 3 ? make_sdesc(smem_u32(sB), 4096, 1024, 2) : make_sdesc(smem_u32(sB), 2048, 512, 4));
-    uint32_t id = idesc_tf32(128, mode == 3 ? 32 : 16, mode <= 2 ? 0 : 1);
+    uint32_t id = idesc_tf32(128, mode == 3 ? 32 : 16, (mode <= 2 || mode == 5) ? 0 : 1);
     asm volatile(
         "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
         "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n}\n" ::"r"(tbase),
@@ -119,7 +119,7 @@ int main() {
   cudaMalloc(&d, 128 * 16 * 4);
   cudaMalloc(&info, 16);
   float h[128 * 16];
-  for (int mode = 0; mode < 5; ++mode) {
+  for (int mode = 0; mode < 6; ++mode) {
     cudaMemset(d, 0xff, 128 * 16 * 4);
     probe<<<1, 128>>>(mode, d, info);
     cudaError_t e = cudaDeviceSynchronize();
@@ -132,10 +132,10 @@ int main() {
       for (int c = 0; c < 16; ++c) {
         float exp = mode == 0 ? (c < 4 ? float(m + 1000 * c) : h[m * 16 + c])
                   : mode == 1 ? 8.f : mode == 2 ? float((m % 8) * 16 + c)
-                  : mode == 3 ? float(8 * c + 32 * 28) : float(8 * c + 16 * 28);
+                  : mode == 3 ? float(8 * c + 32 * 28) : mode == 5 ? 8.f : float(8 * c + 16 * 28);
         if (h[m * 16 + c] != exp) ++bad;
       }
-    printf("  mismatches %d / 2048\n", bad);
+    printf("  mismatches %d / 2048   D[0][0]=%.10f\n", bad, h[0]);
     for (int m = 0; m < 10; ++m) {
       printf("  row %3d:", m);
       for (int c = 0; c < 8; ++c) printf(" %8.1f", h[m * 16 + c]);

@@ -188,16 +188,24 @@ def _np(t):
     return t.detach().cpu().numpy().astype(np.float64)
 
 
-@pytest.mark.parametrize("M,K,N", [(1000, 602, 128), (2708, 1433, 16), (777, 128, 41), (5, 3, 7)])
-def test_gemms(M, K, N):
+@pytest.mark.parametrize("path", ["tcgen05", "simt"])
+@pytest.mark.parametrize("M,K,N", [(1000, 602, 128), (2708, 1433, 16), (777, 128, 41), (5, 3, 7),
+                                   (20000, 602, 128)])
+def test_gemms(M, K, N, path):
+    """xw / xtg / dwt vs numpy fp64.  'tcgen05' passes 16-byte aligned rows
+    and a workspace (3xTF32 engine); 'simt' passes unaligned X (fp32 cores)."""
     rng = np.random.default_rng(M + K + N)
-    X = torch.from_numpy(rng.standard_normal((M, K)).astype(np.float32)).cuda()
+    ldk = _ld(K) if path == "tcgen05" else K
+    Xfull = torch.zeros(M, ldk, device="cuda")
+    Xfull[:, :K] = torch.from_numpy(rng.standard_normal((M, K)).astype(np.float32)).cuda()
+    X = Xfull[:, :K] if path == "tcgen05" else Xfull
     W = torch.from_numpy(rng.standard_normal((K, N)).astype(np.float32)).cuda()
     s = torch.from_numpy(rng.random(M).astype(np.float32) + 0.5).cuda()
     ldn = _ld(N)
     Y = torch.full((M, ldn), float("nan"), device="cuda")
     import ctypes
-    L.gemm_xw(X, W, ctypes.c_void_p(s.data_ptr()), Y, N=N)
+    work = torch.zeros(L.gemm_xw_work_floats(K, N), device="cuda") if path == "tcgen05" else None
+    L.gemm_xw(X, W, ctypes.c_void_p(s.data_ptr()), Y, N=N, work=work)
     torch.cuda.synchronize()
     exp = _np(s)[:, None] * (_np(X) @ _np(W))
     scale = _np(s)[:, None] * (np.abs(_np(X)) @ np.abs(_np(W)))
