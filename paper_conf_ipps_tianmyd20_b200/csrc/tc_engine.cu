@@ -129,29 +129,37 @@ __host__ __device__ constexpr uint32_t idesc_tf32(int M, int N) {
   return (1u << 4) | (2u << 7) | (2u << 10) | (uint32_t(N >> 3) << 17) | (uint32_t(M >> 4) << 24);
 }
 
+// A pipeline stage holds U chunks (U > 1 only for A_BITS, where a chunk is
+// small): per-stage barrier round trips, the TMEM-store wait and the MMA
+// issue bookkeeping are paid once per U chunks.
 struct Layout {
-  int npad, stages, nacc, a_cols;     // a_cols: TMEM columns of one A stage (32, or 64 for hi+lo)
-  uint32_t a_bytes, b_bytes, stage_bytes, a_load_bytes;
+  int npad, stages, nacc, U, a_cols;  // a_cols: TMEM columns of one A stage (U*32, or 64 for hi+lo)
+  uint32_t a_bytes, b_bytes, stage_bytes, a_load_bytes;  // b_bytes: ONE chunk of ONE operand
   uint32_t tmem_cols, a_col0;
 };
 
-Layout make_layout(int mode, int npad, int max_stages) {
+Layout make_layout(int mode, int npad, int max_stages, int max_u) {
   Layout L;
   L.npad = npad;
-  L.a_cols = mode == A_BITS ? BK : 2 * BK;
-  L.a_bytes = mode == A_BITS ? 1024 : BM * BK * 4;       // bits (512 used) or a 16 KB fp32 tile
-  L.a_load_bytes = mode == A_BITS ? BM * 4 : BM * BK * 4;
   L.b_bytes = uint32_t(npad) * BK * 4;
-  L.stage_bytes = L.a_bytes + 2 * L.b_bytes;
-  int st = int((200 * 1024) / L.stage_bytes);
-  st = st < 2 ? 2 : st;
-  st = st > max_stages ? max_stages : st;
-  L.nacc = 2;
-  while (L.nacc * npad + st * L.a_cols > 512) {
-    if (st > 2) --st;
-    else { L.nacc = 1; break; }
+  for (int U = (mode == A_BITS ? max_u : 1); U >= 1; U = U > 1 ? U / 2 : 0) {
+    L.U = U;
+    L.a_cols = mode == A_BITS ? U * BK : 2 * BK;
+    L.a_bytes = mode == A_BITS ? uint32_t((U * BM * 4 + 1023) / 1024 * 1024) : BM * BK * 4;
+    L.a_load_bytes = mode == A_BITS ? BM * 4 : BM * BK * 4;  // per chunk
+    L.stage_bytes = L.a_bytes + 2 * uint32_t(U) * L.b_bytes;
+    int st = int((200 * 1024) / L.stage_bytes);
+    st = st > max_stages ? max_stages : st;
+    L.nacc = 2;
+    while (st >= 2 && L.nacc * npad + st * L.a_cols > 512) {
+      if (st > 2) --st;
+      else if (L.nacc == 2) L.nacc = 1;
+      else st = 0;
+    }
+    L.stages = st;
+    if (st >= 2 || U == 1) break;
   }
-  L.stages = st;
+  if (L.stages < 2) L.stages = 2;
   const uint32_t need = uint32_t(L.nacc * npad + L.stages * L.a_cols);
   uint32_t cols = 32;
   while (cols < need) cols <<= 1;
@@ -245,29 +253,32 @@ __global__ void __launch_bounds__(NTHREADS, 1)
   if (warp == 0) {
     if (lane == 0) {
       // ---- producer ----
-      const uint32_t tx = L.a_load_bytes + 2u * L.b_bytes;
-      uint32_t g = 0;
+      int s = 0;
+      uint32_t ph = 0;
       for (int64_t t = blockIdx.x; t < w.ntiles; t += gridDim.x) {
         int64_t kb, nch, m0, sp;
         tile_range<MODE>(w, t, kb, nch, m0, sp);
-        for (int64_t i = 0; i < nch; ++i, ++g) {
-          const int s = int(g % uint32_t(L.stages));
-          mbar_wait(&empty[s], ((g / L.stages) & 1u) ^ 1u);
+        for (int64_t i = 0; i < nch; i += L.U) {
+          const int nu = int(nch - i < L.U ? nch - i : L.U);
+          mbar_wait(&empty[s], ph ^ 1u);
           uint8_t* st = smem + s * L.stage_bytes;
-          mbar_expect_tx(&full[s], tx);
-          int k0;
-          if (MODE == A_BITS) {
-            k0 = w.ch_col0[kb + i];
-            bulk_load(st, w.bits + (kb + i) * BM, BM * 4, &full[s]);
-          } else if (MODE == A_ROWMAJOR) {
-            k0 = int(i * BK);
-            tma_load_2d(&map_a, &full[s], st, k0, int(m0));
-          } else {
-            k0 = int(kb + i * BK);
-            tma_load_2d(&map_a, &full[s], st, int(m0), k0);
+          mbar_expect_tx(&full[s], uint32_t(nu) * (L.a_load_bytes + 2u * L.b_bytes));
+          for (int u = 0; u < nu; ++u) {
+            int k0;
+            if (MODE == A_BITS) {
+              k0 = w.ch_col0[kb + i + u];
+              bulk_load(st + u * BM * 4, w.bits + (kb + i + u) * BM, BM * 4, &full[s]);
+            } else if (MODE == A_ROWMAJOR) {
+              k0 = int(i * BK);
+              tma_load_2d(&map_a, &full[s], st, k0, int(m0));
+            } else {
+              k0 = int(kb + i * BK);
+              tma_load_2d(&map_a, &full[s], st, int(m0), k0);
+            }
+            tma_load_2d(&map_bhi, &full[s], st + L.a_bytes + u * L.b_bytes, k0, 0);
+            tma_load_2d(&map_blo, &full[s], st + L.a_bytes + (L.U + u) * L.b_bytes, k0, 0);
           }
-          tma_load_2d(&map_bhi, &full[s], st + L.a_bytes, k0, 0);
-          tma_load_2d(&map_blo, &full[s], st + L.a_bytes + L.b_bytes, k0, 0);
+          if (++s == L.stages) { s = 0; ph ^= 1u; }
         }
       }
     }
@@ -275,33 +286,40 @@ __global__ void __launch_bounds__(NTHREADS, 1)
     if (lane == 0) {
       // ---- MMA issuer ----
       const uint32_t idesc = idesc_tf32(BM, npad);
-      uint32_t g = 0, lt = 0;
+      int s = 0;
+      uint32_t ph = 0, lt = 0;
       for (int64_t t = blockIdx.x; t < w.ntiles; t += gridDim.x, ++lt) {
         int64_t kb, nch, m0, sp;
         tile_range<MODE>(w, t, kb, nch, m0, sp);
-        const uint32_t ab = lt % uint32_t(L.nacc);
-        mbar_wait(&acc_empty[ab], ((lt / L.nacc) & 1u) ^ 1u);
+        const uint32_t ab = L.nacc == 2 ? (lt & 1u) : 0u;
+        const uint32_t aph = L.nacc == 2 ? ((lt >> 1) & 1u) : (lt & 1u);
+        mbar_wait(&acc_empty[ab], aph ^ 1u);
         tc_fence_after();
         const uint32_t d = tmem + ab * uint32_t(npad);
         uint32_t acc = 0;
-        for (int64_t i = 0; i < nch; ++i, ++g) {
-          const int s = int(g % uint32_t(L.stages));
-          const uint32_t ph = (g / L.stages) & 1u;
+        for (int64_t i = 0; i < nch; i += L.U) {
+          const int nu = int(nch - i < L.U ? nch - i : L.U);
           mbar_wait(&full[s], ph);
           mbar_wait(&a_full[s], ph);
           tc_fence_after();
-          const uint32_t b0 = smem_u32(smem + s * L.stage_bytes + L.a_bytes);
-          const uint32_t a0 = tmem + L.a_col0 + uint32_t(s) * uint32_t(L.a_cols);
+          const uint32_t sb = smem_u32(smem + s * L.stage_bytes + L.a_bytes);
+          const uint32_t sa = tmem + L.a_col0 + uint32_t(s) * uint32_t(L.a_cols);
+          for (int u = 0; u < nu; ++u) {
+            const uint32_t bh0 = sb + uint32_t(u) * L.b_bytes;
+            const uint32_t bl0 = sb + uint32_t(L.U + u) * L.b_bytes;
+            const uint32_t a0 = sa + uint32_t(u) * BK;
 #pragma unroll
-          for (int kk = 0; kk < BK / 8; ++kk) {
-            const uint64_t bh = sdesc_kmajor_sw128(b0 + kk * 32u);
-            const uint64_t bl = sdesc_kmajor_sw128(b0 + L.b_bytes + kk * 32u);
-            mma_ts(d, a0 + kk * 8u, bh, idesc, acc);
-            mma_ts(d, a0 + kk * 8u, bl, idesc, 1u);
-            if (MODE != A_BITS) mma_ts(d, a0 + BK + kk * 8u, bh, idesc, 1u);
-            acc = 1u;
+            for (int kk = 0; kk < BK / 8; ++kk) {
+              const uint64_t bh = sdesc_kmajor_sw128(bh0 + kk * 32u);
+              const uint64_t bl = sdesc_kmajor_sw128(bl0 + kk * 32u);
+              mma_ts(d, a0 + kk * 8u, bh, idesc, acc);
+              mma_ts(d, a0 + kk * 8u, bl, idesc, 1u);
+              if (MODE != A_BITS) mma_ts(d, a0 + BK + kk * 8u, bh, idesc, 1u);
+              acc = 1u;
+            }
           }
           tc_commit(&empty[s]);
+          if (++s == L.stages) { s = 0; ph ^= 1u; }
         }
         tc_commit(&acc_full[ab]);
       }
@@ -310,21 +328,24 @@ __global__ void __launch_bounds__(NTHREADS, 1)
     // ---- A builders: thread m writes row m of the A tile into TMEM ----
     const int m = ((warp & 3) << 5) | lane;
     const uint32_t lane_base = uint32_t((warp & 3) * 32) << 16;
-    uint32_t g = 0;
+    int s = 0;
+    uint32_t ph = 0;
     for (int64_t t = blockIdx.x; t < w.ntiles; t += gridDim.x) {
       int64_t kb, nch, m0, sp;
       tile_range<MODE>(w, t, kb, nch, m0, sp);
-      for (int64_t i = 0; i < nch; ++i, ++g) {
-        const int s = int(g % uint32_t(L.stages));
-        mbar_wait(&full[s], (g / L.stages) & 1u);  // data landed; stage and its TMEM A buffer are free
+      for (int64_t i = 0; i < nch; i += L.U) {
+        const int nu = int(nch - i < L.U ? nch - i : L.U);
+        mbar_wait(&full[s], ph);  // data landed; stage and its TMEM A buffer are free
         const uint8_t* st = smem + s * L.stage_bytes;
         const uint32_t taddr = tmem + lane_base + L.a_col0 + uint32_t(s) * uint32_t(L.a_cols);
         uint32_t v[32];
         if (MODE == A_BITS) {
-          const uint32_t wd = reinterpret_cast<const uint32_t*>(st)[m];
+          for (int u = 0; u < nu; ++u) {
+            const uint32_t wd = reinterpret_cast<const uint32_t*>(st + u * BM * 4)[m];
 #pragma unroll
-          for (int b = 0; b < 32; ++b) v[b] = ((wd >> b) & 1u) ? 0x3f800000u : 0u;
-          sttm32(taddr, v);
+            for (int b = 0; b < 32; ++b) v[b] = ((wd >> b) & 1u) ? 0x3f800000u : 0u;
+            sttm32(taddr + uint32_t(u) * BK, v);
+          }
         } else {
           float x[32];
           if (MODE == A_ROWMAJOR) {
@@ -354,6 +375,7 @@ __global__ void __launch_bounds__(NTHREADS, 1)
         asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
         tc_fence_before();
         mbar_arrive(&a_full[s]);
+        if (++s == L.stages) { s = 0; ph ^= 1u; }
       }
     }
   } else {
@@ -364,8 +386,8 @@ __global__ void __launch_bounds__(NTHREADS, 1)
     for (int64_t t = blockIdx.x; t < w.ntiles; t += gridDim.x, ++lt) {
       int64_t kb, nch, m0, sp;
       tile_range<MODE>(w, t, kb, nch, m0, sp);
-      const uint32_t ab = lt % uint32_t(L.nacc);
-      mbar_wait(&acc_full[ab], (lt / L.nacc) & 1u);
+      const uint32_t ab = L.nacc == 2 ? (lt & 1u) : 0u;
+      mbar_wait(&acc_full[ab], L.nacc == 2 ? ((lt >> 1) & 1u) : (lt & 1u));
       tc_fence_after();
       const int64_t row = m0 + m;
       const bool live = MODE == A_BITS || row < w.mdim;
@@ -454,11 +476,21 @@ int max_stages_env() {
   return v;
 }
 
+int max_u_env() {
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("PCGCN_TC_U");  // tuning override (benchmarks only)
+    v = e ? atoi(e) : 4;
+    v = v >= 4 ? 4 : (v >= 2 ? 2 : 1);
+  }
+  return v;
+}
+
 template <int MODE>
 cudaError_t launch_engine(const CUtensorMap& bhi, const CUtensorMap& blo, const CUtensorMap& amap, const Work& w,
                           int npad, cudaStream_t s) {
   if (w.ntiles <= 0) return cudaSuccess;
-  const Layout L = make_layout(MODE, npad, max_stages_env());
+  const Layout L = make_layout(MODE, npad, max_stages_env(), max_u_env());
   const size_t smem = 1024 + size_t(L.stages) * L.stage_bytes + (3 * L.stages + 4) * 8 + 16;
   if (smem > 227 * 1024) return cudaErrorInvalidValue;
   static bool attr_done = false;
