@@ -45,7 +45,14 @@ template <int G, int V, bool HAS_ZD>
 __global__ void __launch_bounds__(256) sparse_agg_kernel(AggArgs a) {
   constexpr int S = 32 / G;                 // edges in flight per warp step (slots)
   constexpr int STEPS = 32 / S;             // steps per 32-index batch
-  constexpr int UNR = (8 / V) < 1 ? 1 : (8 / V) > STEPS ? STEPS : (8 / V);  // loads in flight: UNR*V
+  // steps whose loads are all issued before any is consumed: a power of two
+  // dividing STEPS with UNR*V <= 8 float4 in flight per lane (16 measured
+  // slower on C3: the register cost lowers occupancy more than ILP gains)
+  constexpr int UCAP = 8 / V;
+  constexpr int UNR = (UCAP >= 16 && STEPS >= 16) ? 16
+                    : (UCAP >= 8 && STEPS >= 8) ? 8
+                    : (UCAP >= 4 && STEPS >= 4) ? 4
+                    : (UCAP >= 2 && STEPS >= 2) ? 2 : 1;
   constexpr int NACC = V >= 3 ? 1 : (V == 2 ? 2 : 4);                        // interleaved partial sums
   const int64_t row = int64_t(blockIdx.x) * 8 + (threadIdx.x >> 5);
   if (row >= a.rows) return;
@@ -66,9 +73,11 @@ __global__ void __launch_bounds__(256) sparse_agg_kernel(AggArgs a) {
   // Branch-free batches: every lane issues UNR*V independent 16-byte loads
   // before consuming any; edges past the row end read the zero row.
   const float* zrow = a.zrow;
+  int nextidx = (e0 + lane < e1) ? __ldg(a.col + e0 + lane) : -1;  // index batches are prefetched one ahead
   for (int64_t base = e0; base < e1; base += 32) {
     const int cnt = (e1 - base) < 32 ? int(e1 - base) : 32;
-    const int myidx = lane < cnt ? __ldg(a.col + base + lane) : -1;
+    const int myidx = nextidx;
+    nextidx = (base + 32 + lane < e1) ? __ldg(a.col + base + 32 + lane) : -1;
 #pragma unroll
     for (int k0 = 0; k0 < STEPS; k0 += UNR) {
       float4 buf[UNR][V];
