@@ -140,9 +140,10 @@ class Plan:
         self.destroy()
 
     def destroy(self):
-        if getattr(self, "_h", None):
-            lib.pcgcn_destroy(self._h)
-            self._h = None
+        h = getattr(self, "_h", None)
+        if h and lib is not None:  # lib may already be torn down at interpreter exit
+            lib.pcgcn_destroy(h)
+        self._h = None
 
     def stats(self):
         s = Stats()

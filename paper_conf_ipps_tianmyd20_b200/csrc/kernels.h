@@ -22,6 +22,8 @@ struct AggArgs {
   const float* zd;           // dense partial sums, ld ldzd
   int64_t ldzd;
   const float* zrow;         // >= 16 zero floats (load sentinel)
+  int mask_ld;               // u32 words per mask row
+  int64_t n_src;             // rows of Y (for the L2-residency decision)
   int F;
   bool relu, out_prescaled;
 };

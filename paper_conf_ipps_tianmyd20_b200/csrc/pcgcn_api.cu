@@ -166,6 +166,8 @@ pcgcn_status aggregate(pcgcn_plan_t p, const float* Y, int64_t ldy, float* Z, in
   a.zd_index = dense ? d.zd_index : nullptr;
   a.zd = d.zd; a.ldzd = npad;
   a.zrow = d.zrow;
+  a.mask_ld = (F + 31) / 32;
+  a.n_src = p->n;
   a.F = F;
   a.relu = (flags & PCGCN_RELU) != 0;
   a.out_prescaled = (flags & PCGCN_OUT_PRESCALED) != 0;

@@ -37,6 +37,31 @@ namespace {
 __device__ __forceinline__ float4 ld_f4(const float* p) {
   return __ldg(reinterpret_cast<const float4*>(p));
 }
+// L2 eviction policies: gathered source rows (re-read by many rows) stay,
+// the once-read index stream goes first (ncu on C3 showed the index stream
+// evicting Y': 4.5 GB of DRAM reads per F=128 call vs 0.75 GB algorithmic)
+__device__ __forceinline__ uint64_t policy_evict_last() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ uint64_t policy_evict_first() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ float4 ld_f4_hint(const float* p, uint64_t pol) {
+  float4 v;
+  asm volatile("ld.global.nc.L2::cache_hint.v4.f32 {%0,%1,%2,%3}, [%4], %5;"
+               : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w)
+               : "l"(p), "l"(pol));
+  return v;
+}
+__device__ __forceinline__ int ld_idx_hint(const int* p, uint64_t pol) {
+  int v;
+  asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
+  return v;
+}
 __device__ __forceinline__ void add4(float4& a, const float4& b) {
   a.x += b.x; a.y += b.y; a.z += b.z; a.w += b.w;
 }
@@ -73,11 +98,13 @@ __global__ void __launch_bounds__(256) sparse_agg_kernel(AggArgs a) {
   // Branch-free batches: every lane issues UNR*V independent 16-byte loads
   // before consuming any; edges past the row end read the zero row.
   const float* zrow = a.zrow;
-  int nextidx = (e0 + lane < e1) ? __ldg(a.col + e0 + lane) : -1;  // index batches are prefetched one ahead
+  const uint64_t keep = policy_evict_last(), stream = policy_evict_first();
+  // index batches are prefetched one ahead
+  int nextidx = (e0 + lane < e1) ? ld_idx_hint(a.col + e0 + lane, stream) : -1;
   for (int64_t base = e0; base < e1; base += 32) {
     const int cnt = (e1 - base) < 32 ? int(e1 - base) : 32;
     const int myidx = nextidx;
-    nextidx = (base + 32 + lane < e1) ? __ldg(a.col + base + 32 + lane) : -1;
+    nextidx = (base + 32 + lane < e1) ? ld_idx_hint(a.col + base + 32 + lane, stream) : -1;
 #pragma unroll
     for (int k0 = 0; k0 < STEPS; k0 += UNR) {
       float4 buf[UNR][V];
@@ -86,7 +113,7 @@ __global__ void __launch_bounds__(256) sparse_agg_kernel(AggArgs a) {
         const int j = __shfl_sync(0xffffffffu, myidx, (k0 + u) * S + slot);
         const float* src = a.Y + int64_t(j) * a.ldy;
 #pragma unroll
-        for (int v = 0; v < V; ++v) buf[u][v] = ld_f4((j >= 0 && qoff[v] >= 0) ? src + qoff[v] : zrow);
+        for (int v = 0; v < V; ++v) buf[u][v] = ld_f4_hint((j >= 0 && qoff[v] >= 0) ? src + qoff[v] : zrow, keep);
       }
 #pragma unroll
       for (int u = 0; u < UNR; ++u)
@@ -148,7 +175,7 @@ __global__ void __launch_bounds__(256) sparse_agg_kernel(AggArgs a) {
           if (v == vv) bit = (bal[v][col & 3] >> ll) & 1u;
         word |= bit << b;
       }
-      a.mask[row * mw + lane] = word;
+      a.mask[row * a.mask_ld + lane] = word;
     }
   }
 }
@@ -213,8 +240,37 @@ __global__ void __launch_bounds__(256) split_transpose_kernel(const float* __res
 
 }  // namespace
 
+cudaError_t launch_sparse_agg_pass(const AggArgs& a, cudaStream_t s);
+
+// Optional feature-split passes (64 feature columns per pass) so each pass's
+// gather set stays L2-resident.  Measured on C3 at F=128 (θ=0.04): one pass
+// reads 4.4 GB from DRAM at an 81% L2 hit rate in 4.16 ms; two passes read
+// 2 x 0.74 GB at 93.5% but take 2 x 2.37 ms — the gather is bound by the
+// per-edge work, not by the DRAM misses — so the split is OFF by default
+// (PCGCN_SPLIT_BYTES=<bytes> enables it above that Y' size).
 cudaError_t launch_sparse_agg(const AggArgs& a, cudaStream_t s) {
   if (a.rows <= 0) return cudaSuccess;
+  static int64_t split_bytes = -1;
+  if (split_bytes < 0) {
+    const char* e = getenv("PCGCN_SPLIT_BYTES");  // tuning override (benchmarks only)
+    split_bytes = e ? atoll(e) : INT64_MAX;
+  }
+  const int64_t ybytes = a.n_src * int64_t((a.F + 3) / 4 * 4) * 4;
+  if (a.F <= 64 || ybytes <= split_bytes) return launch_sparse_agg_pass(a, s);
+  for (int c0 = 0; c0 < a.F; c0 += 64) {
+    AggArgs b = a;
+    b.F = (a.F - c0) < 64 ? a.F - c0 : 64;
+    b.Y = a.Y + c0;
+    b.Z = a.Z + c0;
+    if (a.zd) b.zd = a.zd + c0;
+    if (a.mask) b.mask = a.mask + c0 / 32;
+    cudaError_t e = launch_sparse_agg_pass(b, s);
+    if (e != cudaSuccess) return e;
+  }
+  return cudaSuccess;
+}
+
+cudaError_t launch_sparse_agg_pass(const AggArgs& a, cudaStream_t s) {
   // (G lanes x V float4) per edge, minimising warp instructions per edge
   // (~G*(3+5V)/32) while keeping each v-slice of G lanes a contiguous segment
   const int nvec = (a.F + 3) / 4;

@@ -1,0 +1,83 @@
+#!/usr/bin/env python
+"""Summarise ncu output (launch list CSV + `--set full` report) into a
+markdown file under profiles/.  Runs here (no GPU needed to read reports).
+
+    python scripts/summarize_ncu.py gpurun_out/r1_launch_list.csv gpurun_out/r1_full.ncu-rep profiles/r1_ncu.md
+"""
+import csv
+import io
+import subprocess
+import sys
+from collections import OrderedDict
+
+METRICS = [
+    ("gpu__time_duration.sum", "time"),
+    ("dram__bytes_read.sum", "DRAM read"),
+    ("dram__bytes_write.sum", "DRAM write"),
+    ("lts__t_sector_hit_rate.pct", "L2 hit %"),
+    ("lts__throughput.avg.pct_of_peak_sustained_elapsed", "L2 thru %"),
+    ("dram__throughput.avg.pct_of_peak_sustained_elapsed", "DRAM thru %"),
+    ("sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_active", "tensor pipe %"),
+    ("smsp__issue_active.avg.pct_of_peak_sustained_active", "issue active %"),
+    ("sm__warps_active.avg.pct_of_peak_sustained_active", "warps active %"),
+    ("launch__registers_per_thread", "regs"),
+]
+
+
+def launch_list(path):
+    rows = list(csv.reader(open(path)))
+    hdr = None
+    out = []
+    for r in rows:
+        if "Kernel Name" in r:
+            hdr = r
+            continue
+        if hdr and len(r) == len(hdr):
+            d = dict(zip(hdr, r))
+            out.append((int(d["ID"]), d["Kernel Name"], d["Grid Size"], float(d["Metric Value"]) / 1e3))
+    return out
+
+
+def short(name):
+    name = name.replace("pcgcn::<unnamed>::", "").replace("(anonymous namespace)::", "")
+    return name.split("(")[0][:60]
+
+
+def main(csv_path, rep_path, out_path):
+    L = launch_list(csv_path)
+    total = sum(t for _, _, _, t in L)
+    agg = OrderedDict()
+    for _, nm, grid, t in L:
+        k = short(nm)
+        a = agg.setdefault(k, [0, 0.0])
+        a[0] += 1
+        a[1] += t
+    lines = ["# ncu summary (one C3 epoch, eager launches; cold-cache serialised times — compare SHARES)", "",
+             f"source: `{csv_path}` ({len(L)} launches, {total / 1e3:.3f} ms total)", "",
+             "| kernel | launches | total us | share |", "|---|---|---|---|"]
+    for k, (c, t) in sorted(agg.items(), key=lambda kv: -kv[1][1]):
+        lines.append(f"| `{k}` | {c} | {t:.1f} | {100 * t / total:.1f}% |")
+    if rep_path:
+        raw = subprocess.run(["ncu", "-i", rep_path, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+        rows = list(csv.reader(io.StringIO(raw)))
+        if rows:
+            hdr, units = rows[0], rows[1]
+            lines += ["", f"## `--set full` capture: `{rep_path}`", "",
+                      "| kernel | grid | " + " | ".join(lbl for _, lbl in METRICS) + " |",
+                      "|---|---|" + "---|" * len(METRICS)]
+            for d in rows[2:]:
+                vals = []
+                for m, _ in METRICS:
+                    if m in hdr:
+                        v, u = d[hdr.index(m)], units[hdr.index(m)]
+                        vals.append(f"{v} {u}".strip())
+                    else:
+                        vals.append("-")
+                lines.append(f"| `{short(d[hdr.index('Kernel Name')])}` | {d[hdr.index('Grid Size')]} | " +
+                             " | ".join(vals) + " |")
+    open(out_path, "w").write("\n".join(lines) + "\n")
+    print("\n".join(lines))
+
+
+if __name__ == "__main__":
+    main(sys.argv[1], sys.argv[2] if len(sys.argv) > 2 and sys.argv[2] != "-" else None, sys.argv[3])

@@ -346,3 +346,42 @@ def test_cuda_graph_replay_matches_eager():
 def test_calibrate_theta():
     th, tf, ts = L.calibrate(128, 1024, 0.05)
     assert tf > 0 and ts > 0 and 0 < th < 1
+
+
+def test_feature_split_passes_subprocess():
+    """The optional feature-split passes (64-column passes, enabled by
+    PCGCN_SPLIT_BYTES) forced on a small graph in a fresh process: same
+    result as the single pass up to summation order (the lane layout (G,V)
+    depends on the pass width, so the order of the fp32 sums differs)."""
+    import os
+    import subprocess
+    import sys
+    code = r'''
+import sys, numpy as np, torch
+sys.path.insert(0, ".")
+from paper_conf_ipps_tianmyd20_b200 import _lib as L
+from synth import configs as C
+g = C.graph(C.CORA)
+rng = np.random.default_rng(5)
+F = 200
+Y = np.zeros((g.n, 200), np.float32); Y[:] = rng.standard_normal((g.n, F))
+pl = L.Plan(g.n, g.rowptr, g.col, 8, 0.03, f_max=256)
+Yd = torch.from_numpy(Y).cuda(); Z = torch.zeros_like(Yd)
+mask = torch.zeros(g.n, 7, dtype=torch.int32, device="cuda")
+pl.forward(Yd, Z, F=F, flags=L.RELU | L.MASK_OUT, mask=mask)
+torch.cuda.synchronize()
+np.save(sys.argv[1] + "_z.npy", Z.cpu().numpy()); np.save(sys.argv[1] + "_m.npy", mask.cpu().numpy())
+'''
+    import tempfile
+    d = tempfile.mkdtemp()
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    for tag, sb in (("one", str(1 << 40)), ("split", "0")):
+        env = dict(os.environ, PCGCN_SPLIT_BYTES=sb)
+        subprocess.run([sys.executable, "-c", code, os.path.join(d, tag)], check=True, env=env, cwd=root)
+    z1, z2 = np.load(os.path.join(d, "one_z.npy")), np.load(os.path.join(d, "split_z.npy"))
+    np.testing.assert_allclose(z2, z1, rtol=1e-5, atol=1e-6)
+    m1, m2 = np.load(os.path.join(d, "one_m.npy")), np.load(os.path.join(d, "split_m.npy"))
+    differ = (m1 ^ m2).view(np.uint32)
+    # mask bits may only differ where the (ReLU-ed) value is ~0 in both runs
+    bits = ((differ[:, :, None] >> np.arange(32, dtype=np.uint32)) & 1).reshape(len(m1), -1)[:, :200]
+    assert np.all(np.abs(z1[bits.astype(bool)]) < 1e-5)
