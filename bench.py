@@ -310,26 +310,64 @@ def main():
         marks.append(e)
 
     per = {}
+    kern = {}  # per-kernel event times inside each aggregation call (PCGCN_PROFILE)
     reps = 3
     for _ in range(reps):
         names.clear(); marks.clear()
         flush.zero_()
         e0 = torch.cuda.Event(enable_timing=True)
         e0.record()
-        model.epoch(hook=hook)
+        model.epoch(hook=hook, agg_flags=L.PROFILE)
         torch.cuda.synchronize(dev)
         prev = e0
         for nm, e in zip(names, marks):
             per[nm] = per.get(nm, 0.0) + prev.elapsed_time(e) / reps
             prev = e
+    # the PROFILE events of the last call of each aggregation are re-read per call:
+    # run each aggregation once more in isolation to attribute kernel times
+    for nm, fn in (("a5a6_agg_fwd_H", lambda: pl.forward(model.Y0, model.H1, F=w.hidden,
+                                                          flags=L.IN_PRESCALED | L.RELU | L.MASK_OUT | L.PROFILE,
+                                                          mask=model.mask1)),
+                   ("a8_agg_fwd_C", lambda: pl.forward(model.Y1, model.Lg, F=w.classes,
+                                                        flags=L.IN_PRESCALED | L.PROFILE))):
+        acc = {}
+        for _ in range(reps):
+            flush.zero_()
+            fn()
+            for k, v in pl.last_timings().items():
+                acc[k] = acc.get(k, 0.0) + v / reps
+        kern[nm] = acc
     peak, peak_src = hbm_peak()
+    l2_gbs = L.probe_read_gbs(64 << 20, 50)  # L2-resident stream: the gather kernels' on-chip roofline
+    hbm_probe = L.probe_read_gbs(4 << 30, 3)
     rows = pl.row_hi - pl.row_lo
     dense_rows = int(st["row_tiles"]) * 128 if world == 1 else int(st["shard_chunks"] > 0) * rows
     bH = agg_bytes(st, g.n, rows, w.hidden, dense_rows, st["shard_chunks"])
     bC = agg_bytes(st, g.n, rows, w.classes, dense_rows, st["shard_chunks"])
     t_agg = per["a5a6_agg_fwd_H"]
-    achieved = bH / (t_agg * 1e-3) / 1e9
     agg_total = sum(per[k] for k in per if "agg" in k)
+    # dominant kernel: the selective gather of the F=H aggregations (largest share of the epoch)
+    t_sp = kern["a5a6_agg_fwd_H"]["sparse"]
+    fp4 = (w.hidden + 3) // 4 * 4
+    b_sp = (st["shard_nnz_sparse"] * 4 + (rows + 1) * 8 + rows * 4 + g.n * w.hidden * 4 + rows * w.hidden * 4
+            + dense_rows * w.hidden * 4 + rows * ((w.hidden + 31) // 32) * 4)
+    achieved = b_sp / (t_sp * 1e-3) / 1e9
+    gather = st["shard_nnz_sparse"] * fp4 * 4 / (t_sp * 1e-3) / 1e9
+    t_tc = kern["a5a6_agg_fwd_H"]["dense_tc"]
+    npad = (w.hidden + 15) // 16 * 16
+    tc_flops = st["shard_chunks"] * 2 * 128 * 32 * npad * 2  # 2 MMAs (hi, lo) per chunk
+    tc_tf = tc_flops / (t_tc * 1e-3) / 1e12 if t_tc > 0 else None
+    try:
+        tc_peak = float(json.load(open(MEASURED_PEAKS))["bf16_tflops"]) / 2
+    except Exception:
+        tc_peak = 1590.0 / 2
+    traffic = None
+    tpath = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tpath):
+        try:
+            traffic = json.load(open(tpath)).get("sparse_agg_F%d" % w.hidden)
+        except Exception:
+            traffic = None
 
     # ---- e2e: host buffers, H2D of the step's inputs and D2H of the loss inside the region ----
     e2e = None
@@ -388,11 +426,20 @@ def main():
                                             "row_tiles", "chunks", "intra_edges", "lp_sweeps", "clusters",
                                             "partition_ms", "plan_ms")},
             },
-            "roofline": {"kernel": "aggregation F=H (prescale/split + tcgen05 full tiles + selective gather), fwd layer 1",
+            "roofline": {"kernel": "sparse_agg (selective-mode gather), layer-1 forward, F=%d" % w.hidden,
                          "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak, "traffic": None, "peak_source": peak_src,
-                         "algorithmic_bytes": bH, "ms": t_agg,
-                         "gather_GBs": st["shard_nnz_sparse"] * w.hidden * 4 / (t_agg * 1e-3) / 1e9},
+                         "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
+                         "algorithmic_bytes": b_sp, "ms": t_sp,
+                         "traffic_source": "profiles/traffic.json (ncu --set full, dram read+write per launch)",
+                         "l2_view": {"gather_bytes": st["shard_nnz_sparse"] * fp4 * 4, "achieved": gather,
+                                     "peak": l2_gbs, "unit": "GB/s", "frac": gather / l2_gbs,
+                                     "peak_source": "measured: pcgcn_probe_read_gbs(64 MiB L2-resident)"},
+                         "hbm_probe_GBs": hbm_probe},
+            "tensor_view": {"kernel": "tc_engine<A_BITS> full-mode tiles, layer-1 forward",
+                            "ms": t_tc, "achieved": tc_tf, "unit": "TFLOP/s (tf32)", "peak": tc_peak,
+                            "frac": (tc_tf / tc_peak) if tc_tf else None,
+                            "peak_source": "measured bf16 dense (MEASURED_PEAKS.json) x 0.5 (tf32:bf16 nominal ratio)"},
+            "agg_kernels_ms": kern,
             "agg_GBs": {"fwd_H": bH / (per["a5a6_agg_fwd_H"] * 1e-3) / 1e9,
                         "fwd_C": bC / (per["a8_agg_fwd_C"] * 1e-3) / 1e9,
                         "bwd_C": bC / (per["a10_agg_bwd_C"] * 1e-3) / 1e9,

@@ -117,8 +117,20 @@ enum {
   PCGCN_IN_PRESCALED = 1u,  /* Y already holds diag(r)·Y (r = d̃^-½ applied by the producing GEMM) */
   PCGCN_RELU = 2u,          /* Z = max(Z, 0) */
   PCGCN_MASK_OUT = 4u,      /* write mask bit [Z_pre > 0], 1 bit per element, row stride ceil(F/32) u32 */
-  PCGCN_OUT_PRESCALED = 8u  /* Z = diag(r)·Z again (feeds the next aggregation directly) */
+  PCGCN_OUT_PRESCALED = 8u, /* Z = diag(r)·Z again (feeds the next aggregation directly) */
+  PCGCN_PROFILE = 16u       /* record CUDA events around each internal kernel (not graph-capturable);
+                               read them with pcgcn_plan_last_timings after the stream completes */
 };
+
+/* Per-kernel times (ms) of the last PCGCN_PROFILE call on this plan:
+ * ms[0] prescale, ms[1] tf32 split, ms[2] full-mode (tcgen05) tiles, ms[3] selective gather
+ * (0 for kernels that did not run).  Synchronises on the recorded events. */
+pcgcn_status pcgcn_plan_last_timings(pcgcn_plan_t p, float ms[4]);
+
+/* Measurement helper: streams `bytes` of device memory `iters` times with 16-byte
+ * loads from all SMs and returns the read bandwidth in GB/s (an L2-resident size
+ * measures the L2->SM path, a size >> 126 MB the HBM path).  Synchronises. */
+pcgcn_status pcgcn_probe_read_gbs(int64_t bytes, int32_t iters, float* gbs);
 
 /* Z = Â·Y  (Eq. 1 propagation; Alg. 1 inner loop h_k = Σ_i f(E_{k,i}, a_i), L118-L121).
  *   Y: DEVICE [n x F] (full plan order, all n rows even on a shard), ld ldy.

@@ -26,7 +26,8 @@ c_i32, c_i64, c_f32, c_u32, c_vp = ctypes.c_int32, ctypes.c_int64, ctypes.c_floa
 OK, EINVAL, ENOTSYM, ECUDA, ENOMEM, ENCCL, EUNSUP = range(7)
 NORM_SYM, NORM_NONE = 0, 1
 DENSE_TF32X2, DENSE_FP32_SIMT = 0, 1
-IN_PRESCALED, RELU, MASK_OUT, OUT_PRESCALED = 1, 2, 4, 8
+IN_PRESCALED, RELU, MASK_OUT, OUT_PRESCALED, PROFILE = 1, 2, 4, 8, 16
+TIMING_NAMES = ("prescale", "split", "dense_tc", "sparse")
 X_NAMES = ["part", "perm", "pstart", "r", "blk_k", "blk_i", "blk_nnz", "blk_dense", "sp_rowptr", "sp_col",
            "rt_row0", "rt_nrows", "rt_cptr", "ch_col0", "bits", "zd_index", "sweeps"]
 X_DTYPES = [np.int32, np.int32, np.int64, np.float32, np.int32, np.int32, np.int64, np.uint8, np.int64,
@@ -82,6 +83,8 @@ _sig("pcgcn_plan_export_bytes", c_i64, c_vp, c_i32)
 _sig("pcgcn_plan_export", c_i32, c_vp, c_i32, c_vp, c_i64)
 _sig("pcgcn_calibrate", c_i32, c_i32, c_i32, c_f32, ctypes.POINTER(c_f32), ctypes.POINTER(c_f32),
      ctypes.POINTER(c_f32))
+_sig("pcgcn_plan_last_timings", c_i32, c_vp, ctypes.POINTER(c_f32))
+_sig("pcgcn_probe_read_gbs", c_i32, c_i64, c_i32, ctypes.POINTER(c_f32))
 _sig("pcgcn_last_error", ctypes.c_char_p)
 _sig("pcgcn_abi_version", c_i32)
 
@@ -166,6 +169,12 @@ class Plan:
     def rowscale_ptr(self):
         return lib.pcgcn_plan_rowscale(self._h)
 
+    def last_timings(self):
+        """{kernel: ms} of the last PROFILE-flagged forward/backward (syncs)."""
+        ms = (c_f32 * 4)()
+        check(lib.pcgcn_plan_last_timings(self._h, ms), "pcgcn_plan_last_timings")
+        return dict(zip(TIMING_NAMES, [float(x) for x in ms]))
+
     def forward(self, Y, Z, F=None, flags=0, mask=None, stream=None):
         F = Y.shape[1] if F is None else F
         check(lib.pcgcn_forward(self._h, _ptr(Y), Y.stride(0), _ptr(Z), Z.stride(0), F, flags, _ptr(mask),
@@ -224,6 +233,12 @@ def adam(theta, grad, m, v, lr, step, b1=0.9, b2=0.999, eps=1e-8, stream=None):
 
 def sgd(theta, grad, lr, stream=None):
     check(lib.pcgcn_sgd(_ptr(theta), _ptr(grad), theta.numel(), lr, _stream(stream)), "pcgcn_sgd")
+
+
+def probe_read_gbs(nbytes, iters=20):
+    v = c_f32()
+    check(lib.pcgcn_probe_read_gbs(int(nbytes), int(iters), ctypes.byref(v)), "pcgcn_probe_read_gbs")
+    return v.value
 
 
 def calibrate(F, block_rows=2048, p_ref=0.05):

@@ -60,6 +60,8 @@ bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) ==
 void set_error(const std::string& msg) { g_err = msg; }
 
 void free_device_plan(pcgcn_plan_s* p) {
+  for (void*& ev : p->d.ev)
+    if (ev) cudaEventDestroy(static_cast<cudaEvent_t>(ev));
   for (void* q : p->d.owned) dev_free(q);
   p->d = DevicePlan();
 }
@@ -108,8 +110,8 @@ pcgcn_status upload_plan(pcgcn_plan_s* p) {
     UP(&d.ch_col0, p->ch_col0.data() + ch_lo, d.nch);
     UP(&d.bits, p->bits.data() + ch_lo * TILE_M, d.nch * TILE_M);
     UP(&d.zd, (float*)nullptr, d.nrt * TILE_M * d.fpad_max);
-    UP(&d.yhi, (float*)nullptr, d.n_pad * d.fpad_max);
-    UP(&d.ylo, (float*)nullptr, d.n_pad * d.fpad_max);
+    // hi rows then lo rows of the feature-major split (per call: lo = hi + npad*n_pad)
+    UP(&d.yhi, (float*)nullptr, 2 * d.n_pad * d.fpad_max);
   }
   UP(&d.ypre, (float*)nullptr, n * d.fpad_max);
   UP(&d.zrow, (float*)nullptr, 256);
@@ -142,18 +144,32 @@ pcgcn_status aggregate(pcgcn_plan_t p, const float* Y, int64_t ldy, float* Z, in
   const float* src = Y;
   int64_t ldsrc = ldy;
   const bool tc = p->opts.dense_prec == PCGCN_DENSE_TF32X2;
+  const bool prof = (flags & PCGCN_PROFILE) != 0;
+  auto mark = [&](int k) {
+    if (!prof) return;
+    if (!d.ev[k]) cudaEventCreate(reinterpret_cast<cudaEvent_t*>(&d.ev[k]));
+    cudaEventRecord(static_cast<cudaEvent_t>(d.ev[k]), s);
+  };
+  if (prof) for (int k = 0; k < 4; ++k) d.ev_used[k] = false;
+  mark(0);
   if (!prescaled) {
+    if (prof) d.ev_used[0] = true;
     e = launch_prescale(Y, ldy, d.r, p->n, F, d.ypre, ld4, s);
     if (e != cudaSuccess) return cuda_fail(e, "prescale");
     src = d.ypre;
     ldsrc = ld4;
   }
+  mark(1);
+  float* ylo = d.yhi ? d.yhi + int64_t(npad) * d.n_pad : nullptr;
   if (dense && tc) {
-    e = launch_split_transpose(src, ldsrc, p->n, F, npad, d.yhi, d.ylo, d.n_pad, s);
+    if (prof) d.ev_used[1] = true;
+    e = launch_split_transpose(src, ldsrc, p->n, F, npad, d.yhi, ylo, d.n_pad, s);
     if (e != cudaSuccess) return cuda_fail(e, "split_transpose");
   }
+  mark(2);
   if (dense) {
-    DenseArgs da{d.yhi, d.ylo, d.n_pad, d.n_pad, d.rt_row0, d.rt_nrows, d.rt_cptr, d.ch_col0, d.bits,
+    if (prof) d.ev_used[2] = true;
+    DenseArgs da{d.yhi, ylo, d.n_pad, d.n_pad, d.rt_row0, d.rt_nrows, d.rt_cptr, d.ch_col0, d.bits,
                  d.nrt, d.zd, npad, npad};
     e = tc ? launch_dense_tc(da, s) : launch_dense_simt_y(da, src, ldsrc, F, s);
     if (e != cudaSuccess) return cuda_fail(e, "dense-mode kernel");
@@ -171,8 +187,11 @@ pcgcn_status aggregate(pcgcn_plan_t p, const float* Y, int64_t ldy, float* Z, in
   a.F = F;
   a.relu = (flags & PCGCN_RELU) != 0;
   a.out_prescaled = (flags & PCGCN_OUT_PRESCALED) != 0;
+  mark(3);
+  if (prof) d.ev_used[3] = true;
   e = launch_sparse_agg(a, s);
   if (e != cudaSuccess) return cuda_fail(e, "selective-mode kernel");
+  mark(4);
   return PCGCN_OK;
 }
 
@@ -275,6 +294,19 @@ pcgcn_status pcgcn_plan_stats(pcgcn_plan_t p, pcgcn_stats* s) {
 }
 
 const float* pcgcn_plan_rowscale(pcgcn_plan_t p) { return p && p->d.built ? p->d.r : nullptr; }
+
+pcgcn_status pcgcn_plan_last_timings(pcgcn_plan_t p, float ms[4]) {
+  if (!p || !ms) { set_error("null argument"); return PCGCN_EINVAL; }
+  for (int k = 0; k < 4; ++k) {
+    ms[k] = 0.f;
+    if (!p->d.ev_used[k] || !p->d.ev[k] || !p->d.ev[k + 1]) continue;
+    cudaEvent_t a = static_cast<cudaEvent_t>(p->d.ev[k]), b = static_cast<cudaEvent_t>(p->d.ev[k + 1]);
+    cudaError_t e = cudaEventSynchronize(b);
+    if (e == cudaSuccess) e = cudaEventElapsedTime(&ms[k], a, b);
+    if (e != cudaSuccess) return cuda_fail(e, "plan_last_timings");
+  }
+  return PCGCN_OK;
+}
 
 int64_t pcgcn_plan_export_bytes(pcgcn_plan_t p, int32_t which) {
   if (!p) return -1;

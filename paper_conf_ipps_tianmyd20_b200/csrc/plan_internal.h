@@ -24,8 +24,8 @@ struct DevicePlan {
   int32_t* ch_col0 = nullptr;     // [nch shard]
   uint32_t* bits = nullptr;       // [nch*128]
   float* zd = nullptr;            // [nrt*128*fpad_max] dense partial sums
-  float* yhi = nullptr;           // [fpad_max x n_pad] tf32 hi part of the (prescaled) input, feature-major
-  float* ylo = nullptr;           // [fpad_max x n_pad] lo part
+  float* yhi = nullptr;           // [2*fpad_max x n_pad] tf32 split of the (prescaled) input, feature-major:
+                                  // rows [0,npad) hi, rows [npad,2npad) lo for a call of width npad
   float* ypre = nullptr;          // [n*fpad_max] prescaled copy for un-prescaled inputs
   float* zrow = nullptr;          // [256] zeros: gather sentinel
   int64_t rows = 0, nnz_s = 0, nrt = 0, nch = 0;
@@ -33,6 +33,8 @@ struct DevicePlan {
   int fpad_max = 0;
   int64_t bytes = 0;
   std::vector<void*> owned;
+  void* ev[5] = {nullptr, nullptr, nullptr, nullptr, nullptr};  // PCGCN_PROFILE events (cudaEvent_t)
+  bool ev_used[4] = {false, false, false, false};
 };
 
 }  // namespace pcgcn

@@ -186,6 +186,7 @@ struct Work {
   int ncols;         // columns written per output row (<= npad, multiple of 4)
   const float* rowscale;
   int64_t split_stride;
+  int b_fused;       // B lo rows follow the hi rows in memory: one TMA box {32, 2*npad} per chunk
 };
 
 template <int MODE>
@@ -263,11 +264,12 @@ __global__ void __launch_bounds__(NTHREADS, 1)
           mbar_wait(&empty[s], ph ^ 1u);
           uint8_t* st = smem + s * L.stage_bytes;
           mbar_expect_tx(&full[s], uint32_t(nu) * (L.a_load_bytes + 2u * L.b_bytes));
+          // the bits of a tile's chunks are contiguous: one bulk copy per stage
+          if (MODE == A_BITS) bulk_load(st, w.bits + (kb + i) * BM, uint32_t(nu) * BM * 4, &full[s]);
           for (int u = 0; u < nu; ++u) {
             int k0;
             if (MODE == A_BITS) {
               k0 = w.ch_col0[kb + i + u];
-              bulk_load(st + u * BM * 4, w.bits + (kb + i + u) * BM, BM * 4, &full[s]);
             } else if (MODE == A_ROWMAJOR) {
               k0 = int(i * BK);
               tma_load_2d(&map_a, &full[s], st, k0, int(m0));
@@ -275,8 +277,14 @@ __global__ void __launch_bounds__(NTHREADS, 1)
               k0 = int(kb + i * BK);
               tma_load_2d(&map_a, &full[s], st, int(m0), k0);
             }
-            tma_load_2d(&map_bhi, &full[s], st + L.a_bytes + u * L.b_bytes, k0, 0);
-            tma_load_2d(&map_blo, &full[s], st + L.a_bytes + (L.U + u) * L.b_bytes, k0, 0);
+            // chunk u's B tile in smem: [hi: npad rows][lo: npad rows] x 128 B
+            uint8_t* bdst = st + L.a_bytes + u * 2 * L.b_bytes;
+            if (w.b_fused) {
+              tma_load_2d(&map_bhi, &full[s], bdst, k0, 0);  // one box {32, 2*npad}: hi rows then lo rows
+            } else {
+              tma_load_2d(&map_bhi, &full[s], bdst, k0, 0);
+              tma_load_2d(&map_blo, &full[s], bdst + L.b_bytes, k0, 0);
+            }
           }
           if (++s == L.stages) { s = 0; ph ^= 1u; }
         }
@@ -305,8 +313,8 @@ __global__ void __launch_bounds__(NTHREADS, 1)
           const uint32_t sb = smem_u32(smem + s * L.stage_bytes + L.a_bytes);
           const uint32_t sa = tmem + L.a_col0 + uint32_t(s) * uint32_t(L.a_cols);
           for (int u = 0; u < nu; ++u) {
-            const uint32_t bh0 = sb + uint32_t(u) * L.b_bytes;
-            const uint32_t bl0 = sb + uint32_t(L.U + u) * L.b_bytes;
+            const uint32_t bh0 = sb + uint32_t(u) * 2u * L.b_bytes;
+            const uint32_t bl0 = bh0 + L.b_bytes;
             const uint32_t a0 = sa + uint32_t(u) * BK;
 #pragma unroll
             for (int kk = 0; kk < BK / 8; ++kk) {
@@ -476,6 +484,18 @@ int max_stages_env() {
   return v;
 }
 
+// B operand maps over a feature-major split [npad rows hi][npad rows lo]: when
+// lo directly follows hi and 2*npad fits one box, a single map/box covers both
+bool make_b_maps(const float* hi, const float* lo, int64_t d0, int64_t ld, int npad, CUtensorMap* mh,
+                 CUtensorMap* ml, int* fused) {
+  *fused = (lo == hi + int64_t(npad) * ld && 2 * npad <= 256) ? 1 : 0;
+  if (*fused) {
+    *ml = CUtensorMap{};
+    return make_map(mh, hi, d0, 2 * npad, ld, BK, 2 * npad, true);
+  }
+  return make_map(mh, hi, d0, npad, ld, BK, npad, true) && make_map(ml, lo, d0, npad, ld, BK, npad, true);
+}
+
 int max_u_env() {
   static int v = -1;
   if (v < 0) {
@@ -512,10 +532,10 @@ cudaError_t launch_dense_tc(const DenseArgs& a, cudaStream_t s) {
   if (a.nrt <= 0) return cudaSuccess;
   if (a.npad % 16 != 0 || a.npad < 16 || a.npad > 256 || a.ldT % 4 != 0) return cudaErrorInvalidValue;
   CUtensorMap mh, ml;
-  if (!make_map(&mh, a.hiT, a.n, a.npad, a.ldT, BK, a.npad, true) ||
-      !make_map(&ml, a.loT, a.n, a.npad, a.ldT, BK, a.npad, true))
-    return cudaErrorInvalidValue;
+  int fused = 0;
+  if (!make_b_maps(a.hiT, a.loT, a.n, a.ldT, a.npad, &mh, &ml, &fused)) return cudaErrorInvalidValue;
   Work w{};
+  w.b_fused = fused;
   w.ntiles = a.nrt;
   w.rt_cptr = a.rt_cptr;
   w.ch_col0 = a.ch_col0;
@@ -532,10 +552,11 @@ cudaError_t launch_tc_gemm_xw(const float* X, int64_t ldx, const float* wThi, co
   const int npad = (N + 15) / 16 * 16;
   if (ldx % 4 || ldwT % 4 || ldy % 4 || npad > 256) return cudaErrorInvalidValue;
   CUtensorMap mh, ml, ma;
-  if (!make_map(&mh, wThi, K, npad, ldwT, BK, npad, true) || !make_map(&ml, wTlo, K, npad, ldwT, BK, npad, true) ||
-      !make_map(&ma, X, K, M, ldx, BK, BM, true))
+  int fused = 0;
+  if (!make_b_maps(wThi, wTlo, K, ldwT, npad, &mh, &ml, &fused) || !make_map(&ma, X, K, M, ldx, BK, BM, true))
     return cudaErrorInvalidValue;
   Work w{};
+  w.b_fused = fused;
   w.ntiles = (M + BM - 1) / BM;
   w.kdim = K;
   w.mdim = M;
@@ -556,8 +577,8 @@ cudaError_t launch_tc_gemm_xtg(const float* X, int64_t ldx, const float* dThi, c
   const int npad = (N + 15) / 16 * 16;
   if (ldx % 4 || lddT % 4 || npad > 256) return cudaErrorInvalidValue;
   CUtensorMap mh, ml, ma;
-  if (!make_map(&mh, dThi, M, npad, lddT, BK, npad, true) || !make_map(&ml, dTlo, M, npad, lddT, BK, npad, true) ||
-      !make_map(&ma, X, K, M, ldx, BM, BK, false))
+  int fused = 0;
+  if (!make_b_maps(dThi, dTlo, M, lddT, npad, &mh, &ml, &fused) || !make_map(&ma, X, K, M, ldx, BM, BK, false))
     return cudaErrorInvalidValue;
   const int64_t ns = tc_xtg_slices(M);
   Work w{};
@@ -570,6 +591,7 @@ cudaError_t launch_tc_gemm_xtg(const float* X, int64_t ldx, const float* dThi, c
   w.ldo = npad;
   w.ncols = npad;
   w.split_stride = int64_t(K) * npad;
+  w.b_fused = fused;
   return launch_engine<A_TRANS>(mh, ml, ma, w, npad, s);
 }
 

@@ -103,7 +103,7 @@ class GCN2:
         if self.exchange is not None:
             self.exchange.gather(full, self.lo, self.hi)
 
-    def epoch(self, stream=None, hook=None):
+    def epoch(self, stream=None, hook=None, agg_flags=0):
         """One epoch; ``hook(name)`` (optional) is called after every step so a
         caller can record CUDA events between them."""
         mark = hook or (lambda name: None)
@@ -115,7 +115,7 @@ class GCN2:
         mark("a4_gemm_xw0")
         self._gather(self.Y0)
         mark("x_gather_y0")
-        p.forward(self.Y0, self.H1, F=H, flags=L.IN_PRESCALED | L.RELU | L.MASK_OUT, mask=self.mask1,
+        p.forward(self.Y0, self.H1, F=H, flags=L.IN_PRESCALED | L.RELU | L.MASK_OUT | agg_flags, mask=self.mask1,
                   stream=stream)
         mark("a5a6_agg_fwd_H")
         # layer 2
@@ -124,7 +124,7 @@ class GCN2:
         mark("a7_gemm_xw1")
         self._gather(self.Y1)
         mark("x_gather_y1")
-        p.forward(self.Y1, self.Lg, F=C, flags=L.IN_PRESCALED, stream=stream)
+        p.forward(self.Y1, self.Lg, F=C, flags=L.IN_PRESCALED | agg_flags, stream=stream)
         mark("a8_agg_fwd_C")
         # loss
         L.softmax_ce(self.Lg, self.labels, self.train, self.inv_nT, rr, self._local(self.dL), self.loss,
@@ -133,7 +133,7 @@ class GCN2:
         self._gather(self.dL)
         mark("x_gather_dl")
         # backward
-        p.backward(self.dL, self.G1, F=C, flags=L.IN_PRESCALED, stream=stream)
+        p.backward(self.dL, self.G1, F=C, flags=L.IN_PRESCALED | agg_flags, stream=stream)
         mark("a10_agg_bwd_C")
         L.gemm_xtg(self.H1, self.G1, self.gTh1, self.xtg_work, M=self.rows, K=H, N=C, stream=stream)
         L.gemm_dwt(self.G1, self.Th1, self.mask1, rr, self._local(self.dP1), M=self.rows, N=C, K=H,
@@ -141,7 +141,7 @@ class GCN2:
         mark("a11_gemm_xtg1_dwt")
         self._gather(self.dP1)
         mark("x_gather_dp1")
-        p.backward(self.dP1, self.G0, F=H, flags=L.IN_PRESCALED, stream=stream)
+        p.backward(self.dP1, self.G0, F=H, flags=L.IN_PRESCALED | agg_flags, stream=stream)
         mark("a12_agg_bwd_H")
         L.gemm_xtg(self.X, self.G0, self.gTh0, self.xtg_work, M=self.rows, K=self.f_in, N=H, stream=stream)
         mark("a13_gemm_xtg0")

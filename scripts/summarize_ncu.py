@@ -77,6 +77,23 @@ def main(csv_path, rep_path, out_path):
                              " | ".join(vals) + " |")
     open(out_path, "w").write("\n".join(lines) + "\n")
     print("\n".join(lines))
+    # per-launch DRAM traffic of the selective kernel for bench.py's roofline.traffic:
+    # the capture's first sparse_agg launch is the layer-1 forward (F=H), the second the layer-2 one (F=C)
+    if rep_path and len(sys.argv) > 5:
+        import json
+        import os
+        fH, fC = int(sys.argv[4]), int(sys.argv[5])
+        sp = [d for d in rows[2:] if "sparse_agg" in d[hdr.index("Kernel Name")]]
+        tr = {}
+        for key, d in zip(("sparse_agg_F%d" % fH, "sparse_agg_F%d" % fC), sp[:2]):
+            rd = float(d[hdr.index("dram__bytes_read.sum")])
+            wr = float(d[hdr.index("dram__bytes_write.sum")])
+            scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}
+            rd *= scale.get(units[hdr.index("dram__bytes_read.sum")], 1)
+            wr *= scale.get(units[hdr.index("dram__bytes_write.sum")], 1)
+            tr[key] = int(rd + wr)
+        tr["source"] = rep_path
+        json.dump(tr, open(os.path.join(os.path.dirname(out_path), "traffic.json"), "w"), indent=1)
 
 
 if __name__ == "__main__":
