@@ -248,20 +248,44 @@ def main():
     torch.cuda.set_device(dev)
     w, g, X, Th0, Th1, labels, T = load_workload(args.workload)
     P = args.P or w.P
+    fmax = max(w.hidden, w.classes)
+    theta_c = None
     if args.theta == "auto":
+        # 1) the paper's procedure (L161) on synthetic p-blocks -> initial θ0
         avg_part = max(64, min(8192, g.n // P))
-        theta, t_f, t_s = L.calibrate(w.hidden, avg_part, 0.05)
-        theta_src = f"calibrated (L161): T_f={t_f:.4f}ms T_s={t_s:.4f}ms at p=0.05, {avg_part}-row blocks, F={w.hidden}"
+        theta0, t_f, t_s = L.calibrate(w.hidden, avg_part, 0.05)
+        theta_src = (f"L161 synthetic: T_f={t_f:.4f}ms T_s={t_s:.4f}ms at p=0.05 ({avg_part}-row blocks, F={w.hidden})"
+                     f" -> theta0={theta0:.4g}; ")
+        # 2) in-situ refinement per width on this workload (pcgcn_refine_theta)
+        pl0 = L.Plan(g.n, g.rowptr, g.col, P, theta0, f_max=fmax, rank=rank, world=world)
+        perm = pl0.perm()
+        Xp = np.ascontiguousarray(X[perm])
+        m0 = GCN2(pl0, Xp, labels[perm], T[perm], Th0, Th1, optimizer="sgd", lr=0.0, device=dev,
+                  exchange=RowExchange(pl0.row_lo, pl0.row_hi) if world > 1 else None)
+        m0.epoch()
+        torch.cuda.synchronize(dev)
+        theta, ccH, ceH = L.refine_theta(pl0, m0.Y0, m0.H1, w.hidden)
+        theta_c, ccC, ceC = L.refine_theta(pl0, m0.Y1, m0.Lg, w.classes)
+        if world > 1:  # one θ per width for all ranks
+            t = torch.tensor([theta, theta_c], device=dev, dtype=torch.float64)
+            dist.all_reduce(t)
+            theta, theta_c = float(t[0]) / world, float(t[1]) / world
+        theta_src += (f"in-situ: F={w.hidden} {ccH:.2f} ns/chunk {ceH:.4f} ns/edge -> {theta:.4g}; "
+                      f"F={w.classes} {ccC:.2f} ns/chunk {ceC:.4f} ns/edge -> {theta_c:.4g}")
+        del m0, pl0
     else:
         theta, theta_src = float(args.theta), "fixed"
     t0 = time.time()
-    pl = L.Plan(g.n, g.rowptr, g.col, P, theta, f_max=max(w.hidden, w.classes), rank=rank, world=world)
+    pl = L.Plan(g.n, g.rowptr, g.col, P, theta, f_max=fmax, rank=rank, world=world)
+    pl_c = L.Plan(g.n, g.rowptr, g.col, P, theta_c, f_max=fmax, rank=rank, world=world) if theta_c else None
     st = pl.stats()
-    log(f"[bench] plan in {time.time() - t0:.1f}s theta={theta:.4g} ({theta_src}) stats={st}")
+    st_c = pl_c.stats() if pl_c else st
+    log(f"[bench] plans in {time.time() - t0:.1f}s theta={theta:.4g} theta_c={theta_c} ({theta_src}) stats={st}")
     perm = pl.perm()
     Xp = np.ascontiguousarray(X[perm])
     exch = RowExchange(pl.row_lo, pl.row_hi) if world > 1 else None
-    model = GCN2(pl, Xp, labels[perm], T[perm], Th0, Th1, optimizer="adam", lr=0.01, device=dev, exchange=exch)
+    model = GCN2(pl, Xp, labels[perm], T[perm], Th0, Th1, optimizer="adam", lr=0.01, device=dev, exchange=exch,
+                 plan_c=pl_c)
     use_graph = world == 1 and not args.eager
     stream = torch.cuda.current_stream(dev)
     if use_graph:
@@ -328,7 +352,7 @@ def main():
     for nm, fn in (("a5a6_agg_fwd_H", lambda: pl.forward(model.Y0, model.H1, F=w.hidden,
                                                           flags=L.IN_PRESCALED | L.RELU | L.MASK_OUT | L.PROFILE,
                                                           mask=model.mask1)),
-                   ("a8_agg_fwd_C", lambda: pl.forward(model.Y1, model.Lg, F=w.classes,
+                   ("a8_agg_fwd_C", lambda: model.plan_c.forward(model.Y1, model.Lg, F=w.classes,
                                                         flags=L.IN_PRESCALED | L.PROFILE))):
         acc = {}
         for _ in range(reps):
@@ -343,7 +367,7 @@ def main():
     rows = pl.row_hi - pl.row_lo
     dense_rows = int(st["row_tiles"]) * 128 if world == 1 else int(st["shard_chunks"] > 0) * rows
     bH = agg_bytes(st, g.n, rows, w.hidden, dense_rows, st["shard_chunks"])
-    bC = agg_bytes(st, g.n, rows, w.classes, dense_rows, st["shard_chunks"])
+    bC = agg_bytes(st_c, g.n, rows, w.classes, int(st_c["row_tiles"]) * 128 if world == 1 else rows, st_c["shard_chunks"])
     t_agg = per["a5a6_agg_fwd_H"]
     agg_total = sum(per[k] for k in per if "agg" in k)
     # dominant kernel: the selective gather of the F=H aggregations (largest share of the epoch)
@@ -418,7 +442,7 @@ def main():
             "config": {
                 "workload": f"{w.name}-shaped DC-SBM (BASELINE configs[2]) n={g.n} nnz(A+I)={st['nnz']} "
                             f"F={w.f_in}->{w.hidden}->{w.classes}",
-                "P": P, "theta": theta, "theta_source": theta_src, "optimizer": "adam",
+                "P": P, "theta": theta, "theta_c": theta_c if theta_c else theta, "theta_source": theta_src, "optimizer": "adam",
                 "parallelism": f"dp-rows{world}" if world > 1 else "single",
                 "l2": "flushed (256 MiB write) between timed steps",
                 "cuda_graph": use_graph,

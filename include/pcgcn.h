@@ -228,6 +228,17 @@ pcgcn_status pcgcn_plan_export(pcgcn_plan_t p, int32_t which, void* host_buf, in
 pcgcn_status pcgcn_calibrate(int32_t F, int32_t block_rows, float p_ref, float* theta_out,
                              float* t_full_ms, float* t_sel_ms);
 
+/* In-situ refinement of θ for one feature width F (the L161 procedure applied
+ * to the workload itself): times the plan's full-mode tiles and selective
+ * gather on the caller's (prescaled) input Y with PCGCN_PROFILE (median of 5),
+ * derives the cost of one 128x32 full-mode chunk (c_chunk) and of one
+ * selective edge (c_edge), and returns θ_F = c_chunk / (4096·c_edge): the block
+ * density at which a chunk costs as much as its edges would in selective mode.
+ * Needs a plan with both modes present (else returns the plan's θ).  Z is a
+ * DEVICE scratch output [rows x F] (ld ldz).  Synchronises its own stream. */
+pcgcn_status pcgcn_refine_theta(pcgcn_plan_t p, const float* Y, int64_t ldy, float* Z, int64_t ldz, int32_t F,
+                                float* theta_out, float* c_chunk_ns, float* c_edge_ns);
+
 const char* pcgcn_last_error(void);
 /* optional device allocator hook (e.g. PyTorch's caching allocator); NULL => cudaMalloc/cudaFree */
 void pcgcn_set_allocator(void* (*alloc)(size_t bytes, void* ctx), void (*release)(void* ptr, void* ctx),

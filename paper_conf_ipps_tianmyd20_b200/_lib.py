@@ -84,6 +84,8 @@ _sig("pcgcn_plan_export", c_i32, c_vp, c_i32, c_vp, c_i64)
 _sig("pcgcn_calibrate", c_i32, c_i32, c_i32, c_f32, ctypes.POINTER(c_f32), ctypes.POINTER(c_f32),
      ctypes.POINTER(c_f32))
 _sig("pcgcn_plan_last_timings", c_i32, c_vp, ctypes.POINTER(c_f32))
+_sig("pcgcn_refine_theta", c_i32, c_vp, c_vp, c_i64, c_vp, c_i64, c_i32, ctypes.POINTER(c_f32),
+     ctypes.POINTER(c_f32), ctypes.POINTER(c_f32))
 _sig("pcgcn_probe_read_gbs", c_i32, c_i64, c_i32, ctypes.POINTER(c_f32))
 _sig("pcgcn_last_error", ctypes.c_char_p)
 _sig("pcgcn_abi_version", c_i32)
@@ -233,6 +235,14 @@ def adam(theta, grad, m, v, lr, step, b1=0.9, b2=0.999, eps=1e-8, stream=None):
 
 def sgd(theta, grad, lr, stream=None):
     check(lib.pcgcn_sgd(_ptr(theta), _ptr(grad), theta.numel(), lr, _stream(stream)), "pcgcn_sgd")
+
+
+def refine_theta(plan, Y, Z, F, stream=None):
+    """In-situ θ for width F on the plan's own workload: (θ_F, ns/chunk, ns/edge)."""
+    th, cc, ce = c_f32(), c_f32(), c_f32()
+    check(lib.pcgcn_refine_theta(plan._h, _ptr(Y), Y.stride(0), _ptr(Z), Z.stride(0), F, ctypes.byref(th),
+                                 ctypes.byref(cc), ctypes.byref(ce)), "pcgcn_refine_theta")
+    return th.value, cc.value, ce.value
 
 
 def probe_read_gbs(nbytes, iters=20):

@@ -47,6 +47,42 @@ float time_forward(pcgcn_plan_t p, const float* Y, float* Z, int F, int64_t ld, 
 
 }  // namespace
 
+extern "C" pcgcn_status pcgcn_refine_theta(pcgcn_plan_t p, const float* Y, int64_t ldy, float* Z, int64_t ldz,
+                                           int32_t F, float* theta_out, float* c_chunk_ns, float* c_edge_ns) {
+  if (!p || !Y || !Z || !theta_out) {
+    pcgcn::set_error("refine_theta: null argument");
+    return PCGCN_EINVAL;
+  }
+  *theta_out = p->theta;
+  if (c_chunk_ns) *c_chunk_ns = 0.f;
+  if (c_edge_ns) *c_edge_ns = 0.f;
+  const int64_t chunks = p->stats.shard_chunks, edges = p->stats.shard_nnz_sparse;
+  if (chunks == 0 || edges == 0) return PCGCN_OK;  // one mode absent: nothing to compare
+  cudaStream_t s = nullptr;
+  if (cudaStreamCreate(&s) != cudaSuccess) {
+    pcgcn::set_error("refine_theta: stream");
+    return PCGCN_ECUDA;
+  }
+  std::vector<float> td, ts;
+  for (int it = 0; it < 7; ++it) {
+    pcgcn_status st = pcgcn_forward(p, Y, ldy, Z, ldz, F, PCGCN_IN_PRESCALED | PCGCN_PROFILE, nullptr, s);
+    if (st != PCGCN_OK) { cudaStreamDestroy(s); return st; }
+    float ms[4];
+    st = pcgcn_plan_last_timings(p, ms);
+    if (st != PCGCN_OK) { cudaStreamDestroy(s); return st; }
+    if (it >= 2) { td.push_back(ms[2]); ts.push_back(ms[3]); }
+  }
+  cudaStreamDestroy(s);
+  std::sort(td.begin(), td.end());
+  std::sort(ts.begin(), ts.end());
+  const double cc = double(td[td.size() / 2]) * 1e6 / double(chunks);  // ns per chunk
+  const double ce = double(ts[ts.size() / 2]) * 1e6 / double(edges);   // ns per selective edge
+  if (c_chunk_ns) *c_chunk_ns = float(cc);
+  if (c_edge_ns) *c_edge_ns = float(ce);
+  if (ce > 0) *theta_out = float(cc / (4096.0 * ce));
+  return PCGCN_OK;
+}
+
 extern "C" pcgcn_status pcgcn_calibrate(int32_t F, int32_t block_rows, float p_ref, float* theta_out,
                                         float* t_full_ms, float* t_sel_ms) {
   if (F < 1 || F > 256 || block_rows < 32 || !(p_ref > 0.f && p_ref <= 1.f) || !theta_out) {
@@ -59,7 +95,7 @@ extern "C" pcgcn_status pcgcn_calibrate(int32_t F, int32_t block_rows, float p_r
   // the 148 SMs idle and overstate T_f).
   const int64_t B = block_rows;
   const int64_t tiles_per_block = (B + 127) / 128;
-  int64_t Pc = (296 + tiles_per_block - 1) / tiles_per_block;
+  int64_t Pc = (8 * 148 + tiles_per_block - 1) / tiles_per_block;  // >= 8 row tiles per SM: balanced waves
   Pc = std::max<int64_t>(2, Pc + (Pc & 1));
   const int64_t n = Pc * B;
   const uint64_t thr = uint64_t(double(p_ref) * 18446744073709551615.0);

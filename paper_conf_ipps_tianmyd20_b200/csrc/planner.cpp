@@ -368,14 +368,13 @@ pcgcn_status build_host_plan(const pcgcn_csr* A, int32_t P, float theta, const p
   }
   part_rt[P] = int64_t(p->rt_row0.size());
 
-  // shard: contiguous partition ranges balanced by a cost model
+  // shard: contiguous partition ranges balanced by cost_k = nnz(Ã rows of V_k)
+  // + |V_k| — independent of θ, so plans of the same graph built for
+  // different feature widths (per-width θ) shard identically
   {
     std::vector<double> cost(P, 0.0);
-    for (int32_t k = 0; k < P; ++k) {
-      int64_t sp = p->sp_rowptr[p->pstart[k + 1]] - p->sp_rowptr[p->pstart[k]];
-      int64_t ch = p->rt_cptr[part_rt[k + 1]] - p->rt_cptr[part_rt[k]];
-      cost[k] = double(sp) + 16.0 * double(ch) + double(psize[k]);
-    }
+    for (int32_t k = 0; k < P; ++k)
+      cost[k] = double(tptr[p->pstart[k + 1]] - tptr[p->pstart[k]]) + double(psize[k]);
     double tot = 0;
     for (double c : cost) tot += c;
     auto bound = [&](int32_t q) -> int32_t {

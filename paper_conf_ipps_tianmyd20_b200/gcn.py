@@ -35,11 +35,15 @@ def _ld(F: int) -> int:
 class GCN2:
     def __init__(self, plan: L.Plan, X_plan: np.ndarray, labels_plan: np.ndarray, train_plan: np.ndarray,
                  Th0: np.ndarray, Th1: np.ndarray, *, optimizer: str = "adam", lr: float = 0.01,
-                 device: str | torch.device = "cuda", exchange=None):
+                 device: str | torch.device = "cuda", exchange=None, plan_c: L.Plan | None = None):
         """All row-indexed host arrays are already in plan order (X_plan = X[perm]).
         ``exchange`` (sharded runs): object with ``gather(local, full)`` and
-        ``allreduce(t)``; rows owned here are plan.row_lo:plan.row_hi."""
+        ``allreduce(t)``; rows owned here are plan.row_lo:plan.row_hi.
+        ``plan_c`` (optional): plan of the same graph and partition with its own
+        θ, used for the width-C aggregations (per-width mode choice)."""
         self.plan = plan
+        self.plan_c = plan_c if plan_c is not None else plan
+        assert (self.plan_c.row_lo, self.plan_c.row_hi) == (plan.row_lo, plan.row_hi)
         self.dev = torch.device(device)
         self.n = plan.n
         self.lo, self.hi = plan.row_lo, plan.row_hi
@@ -124,7 +128,7 @@ class GCN2:
         mark("a7_gemm_xw1")
         self._gather(self.Y1)
         mark("x_gather_y1")
-        p.forward(self.Y1, self.Lg, F=C, flags=L.IN_PRESCALED | agg_flags, stream=stream)
+        self.plan_c.forward(self.Y1, self.Lg, F=C, flags=L.IN_PRESCALED | agg_flags, stream=stream)
         mark("a8_agg_fwd_C")
         # loss
         L.softmax_ce(self.Lg, self.labels, self.train, self.inv_nT, rr, self._local(self.dL), self.loss,
@@ -133,7 +137,7 @@ class GCN2:
         self._gather(self.dL)
         mark("x_gather_dl")
         # backward
-        p.backward(self.dL, self.G1, F=C, flags=L.IN_PRESCALED | agg_flags, stream=stream)
+        self.plan_c.backward(self.dL, self.G1, F=C, flags=L.IN_PRESCALED | agg_flags, stream=stream)
         mark("a10_agg_bwd_C")
         L.gemm_xtg(self.H1, self.G1, self.gTh1, self.xtg_work, M=self.rows, K=H, N=C, stream=stream)
         L.gemm_dwt(self.G1, self.Th1, self.mask1, rr, self._local(self.dP1), M=self.rows, N=C, K=H,

@@ -1,0 +1,2 @@
+timeout 500 python -m pytest tests/test_gpu_parity.py tests/test_dist.py -q -x > gpurun_out/gpu_tests.log 2>&1
+timeout 600 python bench.py --steps 10 --warmup 3 --no-cpu-baseline > gpurun_out/i_auto.json 2> gpurun_out/i_auto.err
