@@ -74,29 +74,33 @@ def aggregate(Ahat: sp.csr_matrix, Y: np.ndarray) -> np.ndarray:
     return np.asarray(Ahat @ np.asarray(Y, dtype=np.float64))
 
 
-def aggregate_rows(n: int, rowptr, col, Y: np.ndarray, rows, norm: str = "sym") -> np.ndarray:
+def clean_degrees(n: int, rowptr, col) -> np.ndarray:
+    """deg_i = |N(i)| after dropping self-loops and duplicates (reading #3)."""
+    rowptr = np.asarray(rowptr, dtype=np.int64)
+    rows = np.repeat(np.arange(n, dtype=np.int64), np.diff(rowptr))
+    col = np.asarray(col, dtype=np.int64)
+    keep = rows != col
+    keys = np.unique(rows[keep] * n + col[keep])
+    return np.bincount(keys // n, minlength=n).astype(np.int64)
+
+
+def aggregate_rows(n: int, rowptr, col, Y: np.ndarray, rows, norm: str = "sym", deg=None) -> np.ndarray:
     """Z_i for selected rows only, straight from the edge definition
-    (pin P15 at full scale): Z_i = r_i Σ_{j∈N(i)∪{i}} r_j Y_j."""
+    (pin P15 at full scale): Z_i = r_i Σ_{j∈N(i)∪{i}} r_j Y_j, r = (1+deg)^-½.
+    ``deg`` (optional) is clean_degrees() of the same graph, to reuse it."""
     rowptr = np.asarray(rowptr, dtype=np.int64)
     col = np.asarray(col, dtype=np.int64)
-    # neighbour sets after dropping self-loops and duplicates, computed lazily
-    cache = {}
-
-    def nbrs(v):
-        if v not in cache:
-            s = col[rowptr[v]:rowptr[v + 1]]
-            cache[v] = np.unique(s[s != v])
-        return cache[v]
-
+    if deg is None and norm != "none":
+        deg = clean_degrees(n, rowptr, col)
     out = np.zeros((len(rows), Y.shape[1]), dtype=np.float64)
     for t, i in enumerate(rows):
-        nb = np.concatenate([nbrs(i), [i]])
+        s = col[rowptr[i]:rowptr[i + 1]]
+        nb = np.concatenate([np.unique(s[s != i]), [i]])
         if norm == "none":
             out[t] = np.asarray(Y[nb], dtype=np.float64).sum(axis=0)
             continue
-        dj = np.array([len(nbrs(j)) + 1 for j in nb], dtype=np.float64)
-        wj = 1.0 / np.sqrt(dj)
-        ri = 1.0 / np.sqrt(len(nbrs(i)) + 1.0)
+        wj = 1.0 / np.sqrt(deg[nb] + 1.0)
+        ri = 1.0 / np.sqrt(deg[i] + 1.0)
         out[t] = ri * (wj[:, None] * np.asarray(Y[nb], dtype=np.float64)).sum(axis=0)
     return out
 

@@ -1,0 +1,61 @@
+"""At-scale parity on the bench workload (C3, Reddit-shaped: 233K vertices,
+114.8M nnz(A+I), P=128) in the launch configuration bench.py times
+(hybrid plans at the widths H=128 and C=41).  The full fp64 oracle does not
+finish in seconds here, so:
+  * P15  sampled rows: Z_i = r_i Σ_j r_j Y_j computed one by one in fp64
+         (oracle.gcn.aggregate_rows) for seeded random rows + the
+         highest-degree rows, condition-scaled error <= 1e-5;
+  * P6   the universal eigenvector s = sqrt(d̃): Â·s = s for every row.
+"""
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+from oracle import gcn as O  # noqa: E402
+from synth import configs as C  # noqa: E402
+
+L = pytest.importorskip("paper_conf_ipps_tianmyd20_b200._lib")
+
+
+@pytest.fixture(scope="module")
+def c3():
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    w = C.REDDIT
+    g = C.graph(w)
+    return w, g, O.clean_degrees(g.n, g.rowptr, g.col)
+
+
+@pytest.mark.parametrize("F,theta", [(128, 0.02), (41, 0.04), (128, 2.0)])
+def test_c3_sampled_rows_and_eigenvector(c3, F, theta):
+    w, g, deg = c3
+    pl = L.Plan(g.n, g.rowptr, g.col, w.P, theta, f_max=128)
+    st = pl.stats()
+    if theta < 1:
+        assert st["nnz_dense"] > 0 and st["nnz_sparse"] > 0   # both modes exercised
+    perm = pl.perm()
+    inv = np.argsort(perm)
+    ld = (F + 3) // 4 * 4
+    rng = np.random.default_rng(31)
+    Y = rng.standard_normal((g.n, F)).astype(np.float32)
+    s = np.sqrt(deg + 1.0)                       # universal eigenvector s = sqrt(d̃)
+    Y[:, 0] = s.astype(np.float32)
+    Yp = np.zeros((g.n, ld), np.float32)
+    Yp[:, :F] = Y[perm]
+    Yd = torch.from_numpy(Yp).cuda()
+    Zd = torch.zeros_like(Yd)
+    pl.forward(Yd, Zd, F=F)                      # un-prescaled input: Z = Â·Y
+    torch.cuda.synchronize()
+    Z = Zd.cpu().numpy()[:, :F][inv]             # back to vertex ids
+    # P6 on every row (column 0 carries fp32(s): compare with the fp32-rounded input's image)
+    s32 = Y[:, 0].astype(np.float64)
+    rel = np.abs(Z[:, 0] - s32) / s32
+    assert rel.max() < 2e-5, rel.max()
+    # P15 sampled rows (seeded random + the 64 highest-degree vertices)
+    rows = np.unique(np.concatenate([rng.choice(g.n, 1500, replace=False), np.argsort(-deg)[:64]]))
+    ref = O.aggregate_rows(g.n, g.rowptr, g.col, Y, rows, deg=deg)
+    scale = O.aggregate_rows(g.n, g.rowptr, g.col, np.abs(Y), rows, deg=deg)
+    err = np.max(np.abs(Z[rows] - ref) / np.maximum(scale, 1e-30))
+    assert err <= 1e-5, err
