@@ -264,15 +264,41 @@ def main():
                   exchange=RowExchange(pl0.row_lo, pl0.row_hi) if world > 1 else None)
         m0.epoch()
         torch.cuda.synchronize(dev)
-        theta, ccH, ceH = L.refine_theta(pl0, m0.Y0, m0.H1, w.hidden)
-        theta_c, ccC, ceC = L.refine_theta(pl0, m0.Y1, m0.Lg, w.classes)
-        if world > 1:  # one θ per width for all ranks
-            t = torch.tensor([theta, theta_c], device=dev, dtype=torch.float64)
-            dist.all_reduce(t)
-            theta, theta_c = float(t[0]) / world, float(t[1]) / world
-        theta_src += (f"in-situ: F={w.hidden} {ccH:.2f} ns/chunk {ceH:.4f} ns/edge -> {theta:.4g}; "
-                      f"F={w.classes} {ccC:.2f} ns/chunk {ceC:.4f} ns/edge -> {theta_c:.4g}")
+        thH, ccH, ceH = L.refine_theta(pl0, m0.Y0, m0.H1, w.hidden)
+        thC, ccC, ceC = L.refine_theta(pl0, m0.Y1, m0.Lg, w.classes)
+        theta_src += (f"in-situ linear: F={w.hidden} {ccH:.2f} ns/chunk {ceH:.4f} ns/edge -> {thH:.4g}, "
+                      f"F={w.classes} {ccC:.2f} ns/chunk {ceC:.4f} ns/edge -> {thC:.4g}; ")
+        Y0, Y1 = m0.Y0.clone(), m0.Y1.clone()
         del m0, pl0
+        # 3) measured choice: time both widths on plans over a θ grid, keep the fastest per width
+        grid = sorted({round(x, 4) for x in (0.01, 0.014, 0.02, 0.028, 0.04, 0.056, 0.08, thH, thC) if x > 0})
+        ZH = torch.empty(g.n, Y0.shape[1], device=dev)
+        ZC = torch.empty(g.n, Y1.shape[1], device=dev)
+        best = {}
+        for th in grid:
+            pt = L.Plan(g.n, g.rowptr, g.col, P, th, f_max=fmax, rank=rank, world=world)
+            for F, Yin, Zout in ((w.hidden, Y0, ZH), (w.classes, Y1, ZC)):
+                ts = []
+                for it in range(4):
+                    a_, b_ = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                    a_.record()
+                    pt.forward(Yin, Zout, F=F, flags=L.IN_PRESCALED)
+                    b_.record()
+                    torch.cuda.synchronize(dev)
+                    if it:
+                        ts.append(a_.elapsed_time(b_))
+                t = float(np.median(ts))
+                if world > 1:
+                    tt = torch.tensor([t], device=dev)
+                    dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+                    t = float(tt.item())
+                if F not in best or t < best[F][1]:
+                    best[F] = (th, t)
+            pt.destroy()
+        theta, theta_c = best[w.hidden][0], best[w.classes][0]
+        theta_src += (f"measured grid {grid}: F={w.hidden} -> {theta} ({best[w.hidden][1]:.3f} ms), "
+                      f"F={w.classes} -> {theta_c} ({best[w.classes][1]:.3f} ms)")
+        del Y0, Y1, ZH, ZC
     else:
         theta, theta_src = float(args.theta), "fixed"
     t0 = time.time()

@@ -134,6 +134,7 @@ __host__ __device__ constexpr uint32_t idesc_tf32(int M, int N) {
 // issue bookkeeping are paid once per U chunks.
 struct Layout {
   int npad, stages, nacc, U, a_cols;  // a_cols: TMEM columns of one A stage (U*32, or 64 for hi+lo)
+  int gst;                            // stages per TMEM accumulation group (<= 8 chunks)
   uint32_t a_bytes, b_bytes, stage_bytes, a_load_bytes;  // b_bytes: ONE chunk of ONE operand
   uint32_t tmem_cols, a_col0;
 };
@@ -165,6 +166,7 @@ Layout make_layout(int mode, int npad, int max_stages, int max_u) {
   while (cols < need) cols <<= 1;
   L.tmem_cols = cols;
   L.a_col0 = uint32_t(L.nacc * npad);
+  L.gst = 8 / L.U > 0 ? 8 / L.U : 1;  // <= 8 chunks (64-96 MMAs) per TMEM accumulation chain
   return L;
 }
 
@@ -212,7 +214,8 @@ __device__ __forceinline__ void tile_range(const Work& w, int64_t t, int64_t& kb
   }
 }
 
-template <int MODE>
+// NPC: register-accumulator width of the epilogue (>= npad), 0 = accumulate in the output row
+template <int MODE, int NPC>
 __global__ void __launch_bounds__(NTHREADS, 1)
     tc_engine_kernel(const __grid_constant__ CUtensorMap map_bhi, const __grid_constant__ CUtensorMap map_blo,
                      const __grid_constant__ CUtensorMap map_a, const Work w, const Layout L) {
@@ -295,17 +298,22 @@ __global__ void __launch_bounds__(NTHREADS, 1)
       // ---- MMA issuer ----
       const uint32_t idesc = idesc_tf32(BM, npad);
       int s = 0;
-      uint32_t ph = 0, lt = 0;
-      for (int64_t t = blockIdx.x; t < w.ntiles; t += gridDim.x, ++lt) {
+      uint32_t ph = 0, gc = 0;  // gc: accumulation-group counter (shared enumeration with the epilogue)
+      for (int64_t t = blockIdx.x; t < w.ntiles; t += gridDim.x) {
         int64_t kb, nch, m0, sp;
         tile_range<MODE>(w, t, kb, nch, m0, sp);
-        const uint32_t ab = L.nacc == 2 ? (lt & 1u) : 0u;
-        const uint32_t aph = L.nacc == 2 ? ((lt >> 1) & 1u) : (lt & 1u);
+        const int64_t nst = (nch + L.U - 1) / L.U;
+        for (int64_t g0 = 0; g0 < nst; g0 += L.gst, ++gc) {
+        // one accumulation group: at most L.gst stages accumulate in TMEM before
+        // the epilogue folds the partial sum into fp32 registers
+        const uint32_t ab = L.nacc == 2 ? (gc & 1u) : 0u;
+        const uint32_t aph = L.nacc == 2 ? ((gc >> 1) & 1u) : (gc & 1u);
         mbar_wait(&acc_empty[ab], aph ^ 1u);
         tc_fence_after();
         const uint32_t d = tmem + ab * uint32_t(npad);
         uint32_t acc = 0;
-        for (int64_t i = 0; i < nch; i += L.U) {
+        const int64_t ge = (g0 + L.gst < nst ? g0 + L.gst : nst) * L.U;
+        for (int64_t i = g0 * L.U; i < (ge < nch ? ge : nch); i += L.U) {
           const int nu = int(nch - i < L.U ? nch - i : L.U);
           mbar_wait(&full[s], ph);
           mbar_wait(&a_full[s], ph);
@@ -330,6 +338,7 @@ __global__ void __launch_bounds__(NTHREADS, 1)
           if (++s == L.stages) { s = 0; ph ^= 1u; }
         }
         tc_commit(&acc_full[ab]);
+        }
       }
     }
   } else if (warp < 6) {
@@ -388,40 +397,80 @@ __global__ void __launch_bounds__(NTHREADS, 1)
     }
   } else {
     // ---- epilogue: TMEM accumulator -> global ----
+    // The tensor core's fp32 accumulation in TMEM is biased (measured: the
+    // relative error grows ~linearly with the accumulation chain, 2e-4 for
+    // C3 hub rows accumulating thousands of chunks); so each accumulation
+    // group (<= 8 chunks) is folded into an fp32 register accumulator here
+    // (round-to-nearest adds, deterministic order), or into the output row
+    // for npad > 128 (NPC == 0).
     const int m = ((warp & 3) << 5) | lane;
     const uint32_t lane_base = uint32_t((warp & 3) * 32) << 16;
-    uint32_t lt = 0;
-    for (int64_t t = blockIdx.x; t < w.ntiles; t += gridDim.x, ++lt) {
+    uint32_t gc = 0;
+    for (int64_t t = blockIdx.x; t < w.ntiles; t += gridDim.x) {
       int64_t kb, nch, m0, sp;
       tile_range<MODE>(w, t, kb, nch, m0, sp);
-      const uint32_t ab = L.nacc == 2 ? (lt & 1u) : 0u;
-      mbar_wait(&acc_full[ab], L.nacc == 2 ? ((lt >> 1) & 1u) : (lt & 1u));
-      tc_fence_after();
+      const int64_t nst = (nch + L.U - 1) / L.U;
+      const int64_t ngrp = (nst + L.gst - 1) / L.gst;
       const int64_t row = m0 + m;
       const bool live = MODE == A_BITS || row < w.mdim;
       float* out = w.out + sp * w.split_stride + row * w.ldo;
       const float sc = (MODE == A_ROWMAJOR && w.rowscale && live) ? w.rowscale[row] : 1.f;
-      const uint32_t src = tmem + lane_base + ab * uint32_t(npad);
-      for (int c0 = 0; c0 < npad; c0 += 16) {
-        uint32_t r[16];
-        asm volatile(
-            "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
-            : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
-              "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]),
-              "=r"(r[15])
-            : "r"(src + uint32_t(c0)));
-        asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
-        if (live) {
+      float racc[NPC > 0 ? NPC : 1];
 #pragma unroll
-          for (int q = 0; q < 4; ++q)
-            if (c0 + 4 * q < w.ncols)
-              *reinterpret_cast<float4*>(out + c0 + 4 * q) =
-                  make_float4(__uint_as_float(r[4 * q]) * sc, __uint_as_float(r[4 * q + 1]) * sc,
-                              __uint_as_float(r[4 * q + 2]) * sc, __uint_as_float(r[4 * q + 3]) * sc);
+      for (int c = 0; c < (NPC > 0 ? NPC : 1); ++c) racc[c] = 0.f;
+      for (int64_t grp = 0; grp < ngrp; ++grp, ++gc) {
+        const uint32_t ab = L.nacc == 2 ? (gc & 1u) : 0u;
+        mbar_wait(&acc_full[ab], L.nacc == 2 ? ((gc >> 1) & 1u) : (gc & 1u));
+        tc_fence_after();
+        const uint32_t src = tmem + lane_base + ab * uint32_t(npad);
+#pragma unroll
+        for (int c0 = 0; c0 < (NPC > 0 ? NPC : 256); c0 += 16) {
+          if (c0 < npad) {
+            uint32_t r[16];
+            asm volatile(
+                "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, "
+                "[%16];"
+                : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+                  "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]),
+                  "=r"(r[15])
+                : "r"(src + uint32_t(c0)));
+            asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+            if (NPC > 0) {
+#pragma unroll
+              for (int q = 0; q < 16; ++q) racc[(c0 + q) % (NPC > 0 ? NPC : 1)] += __uint_as_float(r[q]);
+            } else if (live) {
+#pragma unroll
+              for (int q = 0; q < 16; q += 4)
+                if (c0 + q < w.ncols) {
+                  float4 v = make_float4(__uint_as_float(r[q]), __uint_as_float(r[q + 1]),
+                                         __uint_as_float(r[q + 2]), __uint_as_float(r[q + 3]));
+                  if (grp > 0) {
+                    const float4 o = *reinterpret_cast<const float4*>(out + c0 + q);
+                    v.x += o.x; v.y += o.y; v.z += o.z; v.w += o.w;
+                  }
+                  *reinterpret_cast<float4*>(out + c0 + q) = v;
+                }
+            }
+          }
+        }
+        tc_fence_before();
+        mbar_arrive(&acc_empty[ab]);
+      }
+      if (live) {
+        if (NPC > 0) {
+#pragma unroll
+          for (int c0 = 0; c0 < (NPC > 0 ? NPC : 1); c0 += 4)
+            if (c0 < w.ncols)
+              *reinterpret_cast<float4*>(out + c0) =
+                  make_float4(racc[c0] * sc, racc[c0 + 1] * sc, racc[c0 + 2] * sc, racc[c0 + 3] * sc);
+        } else {
+          for (int c0 = 0; c0 < w.ncols; c0 += 4) {
+            float4 v = ngrp > 0 ? *reinterpret_cast<const float4*>(out + c0) : make_float4(0.f, 0.f, 0.f, 0.f);
+            v.x *= sc; v.y *= sc; v.z *= sc; v.w *= sc;
+            *reinterpret_cast<float4*>(out + c0) = v;
+          }
         }
       }
-      tc_fence_before();
-      mbar_arrive(&acc_empty[ab]);
     }
   }
   tc_fence_before();
@@ -513,16 +562,21 @@ cudaError_t launch_engine(const CUtensorMap& bhi, const CUtensorMap& blo, const 
   const Layout L = make_layout(MODE, npad, max_stages_env(), max_u_env());
   const size_t smem = 1024 + size_t(L.stages) * L.stage_bytes + (3 * L.stages + 4) * 8 + 16;
   if (smem > 227 * 1024) return cudaErrorInvalidValue;
-  static bool attr_done = false;
-  if (!attr_done) {
-    cudaError_t e = cudaFuncSetAttribute(tc_engine_kernel<MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         227 * 1024);
-    if (e != cudaSuccess) return e;
-    attr_done = true;
-  }
   const int64_t grid = w.ntiles < num_sms() ? w.ntiles : num_sms();
-  tc_engine_kernel<MODE><<<unsigned(grid), NTHREADS, smem, s>>>(bhi, blo, amap, w, L);
-  return cudaGetLastError();
+  auto go = [&](auto kernel, bool& attr_done) -> cudaError_t {
+    if (!attr_done) {
+      cudaError_t e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+      if (e != cudaSuccess) return e;
+      attr_done = true;
+    }
+    kernel<<<unsigned(grid), NTHREADS, smem, s>>>(bhi, blo, amap, w, L);
+    return cudaGetLastError();
+  };
+  static bool a32 = false, a64 = false, a128 = false, a0 = false;
+  if (npad <= 32) return go(tc_engine_kernel<MODE, 32>, a32);
+  if (npad <= 64) return go(tc_engine_kernel<MODE, 64>, a64);
+  if (npad <= 128) return go(tc_engine_kernel<MODE, 128>, a128);
+  return go(tc_engine_kernel<MODE, 0>, a0);
 }
 
 }  // namespace

@@ -122,6 +122,24 @@ def test_integer_exact_bitwise(mode):
     assert np.array_equal(Z, exp)
 
 
+@pytest.mark.parametrize("F", [16, 41, 128, 200])
+def test_dense_long_accumulation_accuracy(F):
+    """Full mode on rows with thousands of dense terms, all-positive values
+    whose tf32 lo part matters (1 - 2^-24): the tensor core's biased TMEM
+    accumulation must not build up (groups of <= 8 chunks are folded into
+    fp32 registers).  Expected: every row = d̃·x exactly up to fp32 rounding."""
+    g = G.cliques([2000, 1500])
+    x = np.float32(1.0 - 2.0 ** -24)
+    Y = np.full((g.n, F), x, dtype=np.float32)
+    Z, pl, _ = aggregate_gpu(g, Y, 2, 0.0, norm=L.NORM_NONE, f_max=256)
+    assert pl.stats()["nnz_dense"] == pl.stats()["nnz"]
+    size = np.where(g.labels == 0, 2000, 1500)[:, None]
+    rel = np.abs(Z - size * float(x)) / (size * float(x))
+    # gate 1e-5 (north star); with group folding this is ~2.5e-6, without it
+    # (63 chunks x 8 MMAs in one TMEM chain) it exceeds 1e-5
+    assert rel.max() < 1e-5, rel.max()
+
+
 def test_partition_invariance_integer_regime():
     """L131 §III-A.c: only the summation order changes — bitwise under P9."""
     g = G.sbm(C.CORA.spec)
