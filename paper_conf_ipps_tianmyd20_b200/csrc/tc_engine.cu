@@ -166,7 +166,13 @@ Layout make_layout(int mode, int npad, int max_stages, int max_u) {
   while (cols < need) cols <<= 1;
   L.tmem_cols = cols;
   L.a_col0 = uint32_t(L.nacc * npad);
-  L.gst = 8 / L.U > 0 ? 8 / L.U : 1;  // <= 8 chunks (64-96 MMAs) per TMEM accumulation chain
+  static int group_chunks = -1;  // chunks per TMEM accumulation chain (PCGCN_TC_GROUP: tuning override)
+  if (group_chunks < 0) {
+    const char* e = getenv("PCGCN_TC_GROUP");
+    group_chunks = e ? atoi(e) : 8;
+    if (group_chunks < 1) group_chunks = 1;
+  }
+  L.gst = group_chunks / L.U > 0 ? group_chunks / L.U : 1;  // <= 8 chunks (64-96 MMAs) per chain by default
   return L;
 }
 
