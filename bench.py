@@ -47,6 +47,7 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--eager", action="store_true", help="no CUDA graph")
+    ap.add_argument("--sweep", default="", help="comma list of θ: per-θ aggregation times (Table III replica)")
     return ap.parse_args()
 
 
@@ -271,7 +272,11 @@ def main():
         Y0, Y1 = m0.Y0.clone(), m0.Y1.clone()
         del m0, pl0
         # 3) measured choice: time both widths on plans over a θ grid, keep the fastest per width
-        grid = sorted({round(x, 4) for x in (0.01, 0.014, 0.02, 0.028, 0.04, 0.056, 0.08, thH, thC) if x > 0})
+        #    (large graphs: the in-situ estimates plus the L161 value only — each plan costs seconds)
+        if g.nnz < 200_000_000:
+            grid = sorted({round(x, 4) for x in (0.01, 0.014, 0.02, 0.028, 0.04, 0.056, 0.08, thH, thC) if x > 0})
+        else:
+            grid = sorted({round(x, 5) for x in (thH, thC, theta0) if x > 0})
         ZH = torch.empty(g.n, Y0.shape[1], device=dev)
         ZC = torch.empty(g.n, Y1.shape[1], device=dev)
         best = {}
@@ -450,6 +455,36 @@ def main():
             e2e_ms = float(t.item())
         e2e = {"value": e2e_ms, "unit": "ms", "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": 4}
 
+    sweep = None
+    if args.sweep:
+        # Table III replica (L263-L281): forward aggregation at both widths per θ
+        # (θ >= 1: PCGCN-sel; small θ: full mode for every block above it; the
+        # hybrid = the calibrated plans above).  Times: median of 3 warm calls.
+        sweep = []
+        ZH = torch.empty(model.H1.shape, device=dev)
+        ZC = torch.empty(model.Lg.shape, device=dev)
+        for th in [float(x) for x in args.sweep.split(",")]:
+            try:
+                pt = L.Plan(g.n, g.rowptr, g.col, P, th, f_max=fmax, rank=rank, world=world)
+            except Exception as e:  # e.g. a full-mode plan that does not fit (the paper's "oom", L276)
+                sweep.append({"theta": th, "error": str(e)[:120]})
+                continue
+            ent = {"theta": th, "nnz_dense": pt.stats()["nnz_dense"], "chunks": pt.stats()["chunks"]}
+            for key, F, Yin, Zout in (("agg_ms_H", w.hidden, model.Y0, ZH), ("agg_ms_C", w.classes, model.Y1, ZC)):
+                ts = []
+                for it in range(4):
+                    a_, b_ = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                    a_.record()
+                    pt.forward(Yin, Zout, F=F, flags=L.IN_PRESCALED)
+                    b_.record()
+                    torch.cuda.synchronize(dev)
+                    if it:
+                        ts.append(a_.elapsed_time(b_))
+                ent[key] = float(np.median(ts))
+            pt.destroy()
+            sweep.append(ent)
+            log(f"[bench] sweep {ent}")
+
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         try:
@@ -468,7 +503,7 @@ def main():
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": False,
             "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
             "config": {
-                "workload": f"{w.name}-shaped DC-SBM (BASELINE configs[2]) n={g.n} nnz(A+I)={st['nnz']} "
+                "workload": f"{w.name}-shaped DC-SBM (BASELINE configs[{ {'cora': 0, 'pubmed': 1, 'reddit': 2, 'sbm4m': 3}.get(w.name)}]) n={g.n} nnz(A+I)={st['nnz']} "
                             f"F={w.f_in}->{w.hidden}->{w.classes}",
                 "P": P, "theta": theta, "theta_c": theta_c if theta_c else theta, "theta_source": theta_src, "optimizer": "adam",
                 "parallelism": f"dp-rows{world}" if world > 1 else "single",
@@ -498,6 +533,7 @@ def main():
                         "bwd_H": bH / (per["a12_agg_bwd_H"] * 1e-3) / 1e9},
             "step_breakdown_ms": {k: round(v, 4) for k, v in per.items()},
             "agg_share": agg_total / max(sum(per.values()), 1e-9),
+            "theta_sweep": sweep,
             "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": model.launches_per_epoch() * args.steps,
             "clocks": clocks,
         }

@@ -54,14 +54,25 @@ REDDIT = Workload(
                       m_target=57_307_946, alpha=2.5, cap=200.0, seed=3001),
     f_in=602, hidden=128, classes=41, P=128, feat_kind="normal", feat_seed=3002, theta_seed=3003)
 
-WORKLOADS = {w.name: w for w in (CORA, PUBMED, REDDIT)}
+# C4: 256 communities of 16,384 in 4 tiers x 64 with intra degree d_in in
+# {8, 32, 128, 512} (intra block density 0.05%..3.1%) + 10% inter-community
+# edges: the dual-mode threshold sweep graph.
+_C4_TIERS = [8.0] * 64 + [32.0] * 64 + [128.0] * 64 + [512.0] * 64
+SBM4M = Workload(
+    "sbm4m", SBMSpec([16_384] * 256, sub_size=0, p_sub=0.0, p_class=0.9,
+                     m_target=int(round(64 * 16_384 * (8 + 32 + 128 + 512) / 2 / 0.9)), seed=4001,
+                     class_weight=[t / 8.0 for t in _C4_TIERS]),
+    f_in=128, hidden=128, classes=32, P=2048, feat_kind="normal", feat_seed=4002, theta_seed=4003)
+
+WORKLOADS = {w.name: w for w in (CORA, PUBMED, REDDIT, SBM4M)}
 
 
 def scaled(w: Workload, frac: float, name: str | None = None) -> Workload:
     """Same recipe at a fraction of the vertices and edges (test sizes)."""
     sizes = [max(2, int(round(c * frac))) for c in w.spec.class_sizes]
     spec = SBMSpec(sizes, w.spec.sub_size, w.spec.p_sub, w.spec.p_class,
-                   max(1, int(round(w.spec.m_target * frac))), w.spec.alpha, w.spec.cap, w.spec.seed)
+                   max(1, int(round(w.spec.m_target * frac))), w.spec.alpha, w.spec.cap, w.spec.seed,
+                   w.spec.class_weight)
     return Workload(name or f"{w.name}@{frac}", spec, w.f_in, w.hidden, w.classes,
                     max(1, int(round(w.P * frac ** 0.5))), w.feat_kind, w.feat_seed, w.theta_seed)
 

@@ -61,6 +61,7 @@ class SBMSpec:
     alpha: float = 2.5  # Pareto tail exponent of the propensities
     cap: float = 200.0  # propensity cap, as a multiple of the minimum
     seed: int = 0
+    class_weight: list | None = None  # per-class propensity (tiered SBM); replaces the Pareto draw
 
     @property
     def n(self) -> int:
@@ -85,9 +86,12 @@ def _structure(spec: SBMSpec):
     sub_start = np.concatenate([[0], np.cumsum(sub_sizes)]).astype(np.int64)
     class_of = np.repeat(np.arange(len(class_sizes), dtype=np.int32), class_sizes)
     sub_of = np.repeat(np.arange(len(sub_sizes), dtype=np.int32), sub_sizes)
-    g = np.random.default_rng([spec.seed, 1])
-    u = g.random(n)
-    x = np.minimum((1.0 - u) ** (-1.0 / (spec.alpha - 1.0)), spec.cap)
+    if spec.class_weight is not None:
+        x = np.asarray(spec.class_weight, dtype=np.float64)[class_of]
+    else:
+        g = np.random.default_rng([spec.seed, 1])
+        u = g.random(n)
+        x = np.minimum((1.0 - u) ** (-1.0 / (spec.alpha - 1.0)), spec.cap)
     w = np.maximum(1, np.rint(x * 64.0)).astype(np.int64)
     cdf = np.concatenate([[0], np.cumsum(w)]).astype(np.int64)
     id_of = np.random.default_rng([spec.seed, 2]).permutation(n).astype(np.int64)

@@ -28,9 +28,29 @@ def c3():
     return w, g, O.clean_degrees(g.n, g.rowptr, g.col)
 
 
+@pytest.fixture(scope="module")
+def c4s():
+    """C4 (tiered SBM, BASELINE configs[3]) at 1/16 scale: 262K vertices,
+    communities of 1,024 in four density tiers."""
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    w = C.scaled(C.SBM4M, 1 / 16)
+    g = C.graph(w)
+    return w, g, O.clean_degrees(g.n, g.rowptr, g.col)
+
+
+@pytest.mark.parametrize("F,theta", [(128, 0.01), (32, 0.002)])
+def test_c4_scaled_sampled_rows_and_eigenvector(c4s, F, theta):
+    _check(c4s, F, theta)
+
+
 @pytest.mark.parametrize("F,theta", [(128, 0.02), (41, 0.04), (128, 2.0)])
 def test_c3_sampled_rows_and_eigenvector(c3, F, theta):
-    w, g, deg = c3
+    _check(c3, F, theta)
+
+
+def _check(wgd, F, theta):
+    w, g, deg = wgd
     pl = L.Plan(g.n, g.rowptr, g.col, w.P, theta, f_max=128)
     st = pl.stats()
     if theta < 1:
