@@ -52,6 +52,9 @@ struct DenseArgs {
   int npad;                  // UMMA N (multiple of 16, >= F)
 };
 cudaError_t launch_dense_tc(const DenseArgs& a, cudaStream_t s);
+// CTA-pair (cta_group::2) variant of the full mode (tc_pair.cu); map_b covers [hi rows; lo rows]
+bool dense_pair_eligible(int npad);
+cudaError_t launch_dense_pair(const DenseArgs& a, const struct CUtensorMap_st& map_b, cudaStream_t s);
 // CUDA-core fp32 full mode (§IV-C) on the prescaled input y
 cudaError_t launch_dense_simt_y(const DenseArgs& a, const float* y, int64_t ldy, int F,
                                 cudaStream_t s);

@@ -37,6 +37,7 @@
 #include <mutex>
 
 #include "kernels.h"
+#include "tc_common.cuh"
 
 namespace pcgcn {
 namespace {
@@ -46,89 +47,7 @@ constexpr int BK = 32;         // K per chunk (4 x UMMA K=8 for tf32)
 constexpr int NTHREADS = 320;  // 10 warps
 enum AMode { A_BITS = 0, A_ROWMAJOR = 1, A_TRANS = 2 };
 
-__device__ __forceinline__ uint32_t smem_u32(const void* p) {
-  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
-}
-__device__ __forceinline__ void mbar_init(uint64_t* b, uint32_t count) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(b)), "r"(count));
-}
-__device__ __forceinline__ void mbar_expect_tx(uint64_t* b, uint32_t bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(b)), "r"(bytes)
-               : "memory");
-}
-__device__ __forceinline__ void mbar_arrive(uint64_t* b) {
-  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(b)) : "memory");
-}
-__device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {
-  uint32_t addr = smem_u32(b);
-  asm volatile(
-      "{\n"
-      ".reg .pred p;\n"
-      "WAIT_%=:\n"
-      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
-      "@!p bra WAIT_%=;\n"
-      "}\n" ::"r"(addr),
-      "r"(parity)
-      : "memory");
-}
-__device__ __forceinline__ void tma_load_2d(const CUtensorMap* map, uint64_t* bar, void* dst, int c0,
-                                            int c1) {
-  asm volatile(
-      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];" ::"r"(
-          smem_u32(dst)),
-      "l"(map), "r"(smem_u32(bar)), "r"(c0), "r"(c1)
-      : "memory");
-}
-__device__ __forceinline__ void bulk_load(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
-  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-                   smem_u32(dst)),
-               "l"(src), "r"(bytes), "r"(smem_u32(bar))
-               : "memory");
-}
-__device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
-__device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
-__device__ __forceinline__ void tc_commit(uint64_t* bar) {
-  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
-                   smem_u32(bar))
-               : "memory");
-}
-// D[tmem] (+)= A[tmem] · B[smem desc]
-__device__ __forceinline__ void mma_ts(uint32_t d, uint32_t a, uint64_t bdesc, uint32_t idesc, uint32_t acc) {
-  asm volatile(
-      "{\n"
-      ".reg .pred p;\n"
-      "setp.ne.b32 p, %4, 0;\n"
-      "tcgen05.mma.cta_group::1.kind::tf32 [%0], [%1], %2, %3, p;\n"
-      "}\n" ::"r"(d),
-      "r"(a), "l"(bdesc), "r"(idesc), "r"(acc)
-      : "memory");
-}
-__device__ __forceinline__ void sttm32(uint32_t taddr, const uint32_t (&v)[32]) {
-  asm volatile(
-      "tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,"
-      "%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31,%32};" ::"r"(taddr),
-      "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7]), "r"(v[8]), "r"(v[9]),
-      "r"(v[10]), "r"(v[11]), "r"(v[12]), "r"(v[13]), "r"(v[14]), "r"(v[15]), "r"(v[16]), "r"(v[17]), "r"(v[18]),
-      "r"(v[19]), "r"(v[20]), "r"(v[21]), "r"(v[22]), "r"(v[23]), "r"(v[24]), "r"(v[25]), "r"(v[26]), "r"(v[27]),
-      "r"(v[28]), "r"(v[29]), "r"(v[30]), "r"(v[31])
-      : "memory");
-}
-
-// UMMA shared-memory matrix descriptor (sm_100): start>>4 [0,14), LBO>>4
-// [16,30), SBO>>4 [32,46), version=1 [46,48), layout type [61,64) (2=SW128).
-// K-major SW128: 8-row groups 1024 B apart; K advance = +32 B per 8 tf32.
-__device__ __forceinline__ uint64_t sdesc_kmajor_sw128(uint32_t saddr) {
-  return uint64_t((saddr >> 4) & 0x3FFFu) | (uint64_t(1) << 16) | (uint64_t(1024 >> 4) << 32) |
-         (uint64_t(1) << 46) | (uint64_t(2) << 61);
-}
-// instruction descriptor, kind::tf32: D f32 [4,6), A tf32 [7,10), B tf32
-// [10,13), A and B K-major (bits 15/16 = 0), N>>3 [17,23), M>>4 [24,29).
-// (MN-major B reads as zeros for kind::tf32 on the B200 — measured with
-// tests/cuda/tc_probe.cu — so every B operand is stored feature-major.)
-__host__ __device__ constexpr uint32_t idesc_tf32(int M, int N) {
-  return (1u << 4) | (2u << 7) | (2u << 10) | (uint32_t(N >> 3) << 17) | (uint32_t(M >> 4) << 24);
-}
-
+using namespace tc;
 // A pipeline stage holds U chunks (U > 1 only for A_BITS, where a chunk is
 // small): per-stage barrier round trips, the TMEM-store wait and the MMA
 // issue bookkeeping are paid once per U chunks.
@@ -592,6 +511,11 @@ cudaError_t launch_dense_tc(const DenseArgs& a, cudaStream_t s) {
   if (a.nrt <= 0) return cudaSuccess;
   if (a.npad % 16 != 0 || a.npad < 16 || a.npad > 256 || a.ldT % 4 != 0) return cudaErrorInvalidValue;
   CUtensorMap mh, ml;
+  if (dense_pair_eligible(a.npad) && a.loT == a.hiT + int64_t(a.npad) * a.ldT) {
+    // CTA-pair kernel (tc_pair.cu): one map over [hi rows; lo rows], box = half the features
+    if (!make_map(&mh, a.hiT, a.n, 2 * a.npad, a.ldT, BK, a.npad / 2, true)) return cudaErrorInvalidValue;
+    return launch_dense_pair(a, mh, s);
+  }
   int fused = 0;
   if (!make_b_maps(a.hiT, a.loT, a.n, a.ldT, a.npad, &mh, &ml, &fused)) return cudaErrorInvalidValue;
   Work w{};

@@ -366,6 +366,45 @@ def test_calibrate_theta():
     assert tf > 0 and ts > 0 and 0 < th < 1
 
 
+def test_dense_pair_kernel_subprocess():
+    """The opt-in CTA-pair (tcgen05 cta_group::2) full-mode kernel, enabled
+    with PCGCN_DENSE_PAIR=1 in a fresh process: integer-exact regime bitwise
+    vs the oracle, and condition-scaled 1e-5 on a hybrid Cora plan, F=128."""
+    import os
+    import subprocess
+    import sys
+    code = r'''
+import sys, numpy as np, torch
+sys.path.insert(0, ".")
+from paper_conf_ipps_tianmyd20_b200 import _lib as L
+from oracle import gcn as O
+from synth import configs as C, graphs as G
+for g, P, theta, norm in ((G.cliques([300, 129, 64, 33, 2], seed=5), 5, 0.0, "none"),
+                          (C.graph(C.CORA), 8, 0.02, "sym"), (G.cliques([200] * 9), 3, 0.0, "none")):
+    rng = np.random.default_rng(3)
+    Y = (rng.integers(-1000, 1000, size=(g.n, 128)) if norm == "none" else rng.standard_normal((g.n, 128))).astype(np.float32)
+    pl = L.Plan(g.n, g.rowptr, g.col, P, theta, norm=L.NORM_NONE if norm == "none" else L.NORM_SYM)
+    perm = pl.perm()
+    Yd = torch.from_numpy(np.ascontiguousarray(Y[perm])).cuda(); Z = torch.zeros_like(Yd)
+    pl.forward(Yd, Z, F=128); torch.cuda.synchronize()
+    Zo = np.empty((g.n, 128)); Zo[perm] = Z.cpu().numpy()
+    A = O.normalized_adjacency(g.n, g.rowptr, g.col, norm)[0]
+    ref = O.aggregate(A, Y.astype(np.float64))
+    if norm == "none":
+        assert np.array_equal(Zo, ref), "pair kernel: integer regime not exact"
+    else:
+        sc = O.aggregate(abs(A), np.abs(Y.astype(np.float64)))
+        err = np.max(np.abs(Zo - ref) / np.maximum(sc, 1e-30))
+        assert err <= 1e-5, err
+print("ok")
+'''
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, PCGCN_DENSE_PAIR="1")
+    out = subprocess.run([sys.executable, "-c", code], check=True, env=env, cwd=root, capture_output=True,
+                         text=True, timeout=300)
+    assert out.stdout.strip().endswith("ok")
+
+
 def test_feature_split_passes_subprocess():
     """The optional feature-split passes (64-column passes, enabled by
     PCGCN_SPLIT_BYTES) forced on a small graph in a fresh process: same
