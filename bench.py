@@ -435,6 +435,7 @@ def main():
         tr_h = model.train.cpu().pin_memory()
         loss_h = torch.empty(1, dtype=torch.float32).pin_memory()
         h2d = Xh.numel() * 4 + lab_h.numel() * 4 + tr_h.numel()
+        # (a) serial: copy the step's inputs, run it, read the loss back — per-step events
         e2e_ev = []
         for i in range(args.steps):
             flush.zero_()
@@ -448,12 +449,65 @@ def main():
             b.record()
             e2e_ev.append((a, b))
         torch.cuda.synchronize(dev)
-        e2e_ms = float(np.mean([a.elapsed_time(b) for a, b in e2e_ev]))
+        serial_ms = float(np.mean([a.elapsed_time(b) for a, b in e2e_ev]))
+        # (b) pipelined input path (double-buffered inputs, copy stream): step k+1's
+        #     H2D overlaps step k's epoch; every step still copies its inputs from
+        #     pinned host memory and reads its loss back inside the timed region
+        bufs = [(model.X, model.labels, model.train),
+                (model.X.clone(), model.labels.clone(), model.train.clone())]
+        graphs = []
+        if use_graph:
+            for bx in bufs:
+                model.X, model.labels, model.train = bx
+                graphs.append(model.capture(warmup=1))
+        model.X, model.labels, model.train = bufs[0]
+        cs = torch.cuda.Stream(device=dev)
+        cur = torch.cuda.current_stream(dev)
+        ev_copy = [torch.cuda.Event() for _ in range(2)]
+        ev_done = [torch.cuda.Event() for _ in range(2)]
+        loss_hs = [torch.empty(1, dtype=torch.float32).pin_memory() for _ in range(args.steps)]
+
+        def copy_into(bi):
+            with torch.cuda.stream(cs):
+                for dst, src in zip(bufs[bi], (Xh, lab_h, tr_h)):
+                    dst.copy_(src, non_blocking=True)
+                ev_copy[bi].record(cs)
+
+        torch.cuda.synchronize(dev)
         if world > 1:
-            t = torch.tensor([e2e_ms], device=dev)
+            dist.barrier()
+        e_a, e_b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e_a.record(cur)
+        cs.wait_event(e_a)
+        copy_into(0)
+        for k in range(args.steps):
+            bi = k % 2
+            cur.wait_event(ev_copy[bi])
+            if use_graph:
+                graphs[bi].replay()
+            else:
+                model.X, model.labels, model.train = bufs[bi]
+                model.epoch()
+            loss_hs[k].copy_(model.loss, non_blocking=True)
+            ev_done[bi].record(cur)
+            if k + 1 < args.steps:
+                nb = (k + 1) % 2
+                if k >= 1:
+                    cs.wait_event(ev_done[nb])  # buffer nb was read by step k-1
+                copy_into(nb)
+        e_b.record(cur)
+        torch.cuda.synchronize(dev)
+        e2e_ms = e_a.elapsed_time(e_b) / args.steps
+        model.X, model.labels, model.train = bufs[0]
+        if use_graph:
+            model._graph = graphs[0]
+        if world > 1:
+            t = torch.tensor([e2e_ms, serial_ms], device=dev)
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            e2e_ms = float(t.item())
-        e2e = {"value": e2e_ms, "unit": "ms", "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": 4}
+            e2e_ms, serial_ms = float(t[0]), float(t[1])
+        e2e = {"value": e2e_ms, "unit": "ms", "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": 4,
+               "pipeline": "double-buffered inputs on a copy stream: step k+1's H2D overlaps step k",
+               "serial_value": serial_ms}
 
     sweep = None
     if args.sweep:
