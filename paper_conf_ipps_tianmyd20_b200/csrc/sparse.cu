@@ -37,9 +37,8 @@ namespace {
 __device__ __forceinline__ float4 ld_f4(const float* p) {
   return __ldg(reinterpret_cast<const float4*>(p));
 }
-// L2 eviction policies: gathered source rows (re-read by many rows) stay,
-// the once-read index stream goes first (ncu on C3 showed the index stream
-// evicting Y': 4.5 GB of DRAM reads per F=128 call vs 0.75 GB algorithmic)
+// L2 eviction policies for the gather loads; see gather_hint() for the
+// measured choice (the once-read index stream is marked evict_first)
 __device__ __forceinline__ uint64_t policy_evict_last() {
   uint64_t p;
   asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
@@ -57,6 +56,13 @@ __device__ __forceinline__ float4 ld_f4_hint(const float* p, uint64_t pol) {
                : "l"(p), "l"(pol));
   return v;
 }
+__device__ __forceinline__ float4 ld_f4_na_hint(const float* p, uint64_t pol) {
+  float4 v;
+  asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.f32 {%0,%1,%2,%3}, [%4], %5;"
+               : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w)
+               : "l"(p), "l"(pol));
+  return v;
+}
 __device__ __forceinline__ int ld_idx_hint(const int* p, uint64_t pol) {
   int v;
   asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
@@ -66,7 +72,7 @@ __device__ __forceinline__ void add4(float4& a, const float4& b) {
   a.x += b.x; a.y += b.y; a.z += b.z; a.w += b.w;
 }
 
-template <int G, int V, bool HAS_ZD>
+template <int G, int V, bool HAS_ZD, int HINT>
 __global__ void __launch_bounds__(256) sparse_agg_kernel(AggArgs a) {
   constexpr int S = 32 / G;                 // edges in flight per warp step (slots)
   constexpr int STEPS = 32 / S;             // steps per 32-index batch
@@ -99,8 +105,9 @@ __global__ void __launch_bounds__(256) sparse_agg_kernel(AggArgs a) {
   // before consuming any; edges past the row end read the zero row.
   const float* zrow = a.zrow;
   const uint64_t keep = policy_evict_last(), stream = policy_evict_first();
+  auto ld_idx = [](const int* p, uint64_t pol) { return HINT == 3 ? __ldg(p) : ld_idx_hint(p, pol); };
   // index batches are prefetched one ahead
-  int nextidx = (e0 + lane < e1) ? ld_idx_hint(a.col + e0 + lane, stream) : -1;
+  int nextidx = (e0 + lane < e1) ? ld_idx(a.col + e0 + lane, stream) : -1;
   // Loads rotate over NACC interleaved accumulators (a slot adds <= d/(S*NACC)
   // terms sequentially).  Measured on C3 hub rows (d = 25K, all-positive
   // eigenvector input): 1.2e-7 relative error, far inside the 1e-5 gate; a
@@ -108,7 +115,7 @@ __global__ void __launch_bounds__(256) sparse_agg_kernel(AggArgs a) {
   for (int64_t base = e0; base < e1; base += 32) {
     const int cnt = (e1 - base) < 32 ? int(e1 - base) : 32;
     const int myidx = nextidx;
-    nextidx = (base + 32 + lane < e1) ? ld_idx_hint(a.col + base + 32 + lane, stream) : -1;
+    nextidx = (base + 32 + lane < e1) ? ld_idx(a.col + base + 32 + lane, stream) : -1;
 #pragma unroll
     for (int k0 = 0; k0 < STEPS; k0 += UNR) {
       float4 buf[UNR][V];
@@ -117,7 +124,12 @@ __global__ void __launch_bounds__(256) sparse_agg_kernel(AggArgs a) {
         const int j = __shfl_sync(0xffffffffu, myidx, (k0 + u) * S + slot);
         const float* src = a.Y + int64_t(j) * a.ldy;
 #pragma unroll
-        for (int v = 0; v < V; ++v) buf[u][v] = ld_f4_hint((j >= 0 && qoff[v] >= 0) ? src + qoff[v] : zrow, keep);
+        for (int v = 0; v < V; ++v) {
+          const float* p = (j >= 0 && qoff[v] >= 0) ? src + qoff[v] : zrow;
+          if (HINT == 1) buf[u][v] = ld_f4_hint(p, keep);
+          else if (HINT == 2) buf[u][v] = ld_f4_na_hint(p, keep);
+          else buf[u][v] = ld_f4(p);
+        }
       }
 #pragma unroll
       for (int u = 0; u < UNR; ++u)
@@ -184,13 +196,41 @@ __global__ void __launch_bounds__(256) sparse_agg_kernel(AggArgs a) {
   }
 }
 
-template <int G, int V>
-cudaError_t launch_gv(const AggArgs& a, cudaStream_t s) {
+int gather_hint() {
+  // Gather cache policy (PCGCN_GATHER_HINT, tuning override).  Measured on C3
+  // (bench, 10 steps, two interleaved runs each), F=128 / F=41 sparse ms:
+  //   0 (default) rows plain ld.global.nc, index evict_first  3.40 / 1.41
+  //   1 rows L2::evict_last                                    3.83 / 1.50
+  //   2 rows L1::no_allocate + evict_last                      3.83 / 2.81
+  //   3 rows and index plain                                   3.43 / 1.39
+  // (evict_last pins all of Y' and starves the L1/L2 replacement of the
+  // hot hub rows; no_allocate loses the L1 hits of the narrow rows)
+  static int h = -1;
+  if (h < 0) {
+    const char* e = getenv("PCGCN_GATHER_HINT");
+    h = e ? atoi(e) : 0;
+    if (h < 0 || h > 3) h = 0;
+  }
+  return h;
+}
+
+template <int G, int V, int HINT>
+void launch_ghv(const AggArgs& a, cudaStream_t s) {
   dim3 grid(unsigned((a.rows + 7) / 8));
   if (a.zd_index)
-    sparse_agg_kernel<G, V, true><<<grid, 256, 0, s>>>(a);
+    sparse_agg_kernel<G, V, true, HINT><<<grid, 256, 0, s>>>(a);
   else
-    sparse_agg_kernel<G, V, false><<<grid, 256, 0, s>>>(a);
+    sparse_agg_kernel<G, V, false, HINT><<<grid, 256, 0, s>>>(a);
+}
+
+template <int G, int V>
+cudaError_t launch_gv(const AggArgs& a, cudaStream_t s) {
+  switch (gather_hint()) {
+    case 2: launch_ghv<G, V, 2>(a, s); break;
+    case 3: launch_ghv<G, V, 3>(a, s); break;
+    case 1: launch_ghv<G, V, 1>(a, s); break;
+    default: launch_ghv<G, V, 0>(a, s); break;
+  }
   return cudaGetLastError();
 }
 
