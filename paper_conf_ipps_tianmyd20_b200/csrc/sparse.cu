@@ -72,8 +72,8 @@ __device__ __forceinline__ void add4(float4& a, const float4& b) {
   a.x += b.x; a.y += b.y; a.z += b.z; a.w += b.w;
 }
 
-template <int G, int V, bool HAS_ZD, int HINT>
-__global__ void __launch_bounds__(256) sparse_agg_kernel(AggArgs a) {
+template <int G, int V, bool HAS_ZD, int HINT, int MINB>
+__global__ void __launch_bounds__(256, MINB) sparse_agg_kernel(AggArgs a) {
   constexpr int S = 32 / G;                 // edges in flight per warp step (slots)
   constexpr int STEPS = 32 / S;             // steps per 32-index batch
   // steps whose loads are all issued before any is consumed: a power of two
@@ -209,28 +209,37 @@ int gather_hint() {
   if (h < 0) {
     const char* e = getenv("PCGCN_GATHER_HINT");
     h = e ? atoi(e) : 0;
-    if (h < 0 || h > 3) h = 0;
+    if (h != 1) h = 0;
   }
   return h;
 }
 
 template <int G, int V, int HINT>
 void launch_ghv(const AggArgs& a, cudaStream_t s) {
+  // Occupancy target: 4 CTAs (32 warps) per SM caps registers at 64.  On C3
+  // (same box, interleaved runs) F=128 3.72 -> 3.62 ms, F=41 1.60 -> 1.42 ms
+  // against the unconstrained 76-80 registers (3 CTAs).  PCGCN_SPARSE_MINB=1
+  // restores the unconstrained build (tuning override).
+  static int minb = -1;
+  if (minb < 0) {
+    const char* e = getenv("PCGCN_SPARSE_MINB");
+    minb = (e && atoi(e) == 1) ? 1 : 4;
+  }
   dim3 grid(unsigned((a.rows + 7) / 8));
-  if (a.zd_index)
-    sparse_agg_kernel<G, V, true, HINT><<<grid, 256, 0, s>>>(a);
-  else
-    sparse_agg_kernel<G, V, false, HINT><<<grid, 256, 0, s>>>(a);
+#define LAUNCH(MB)                                                        \
+  if (a.zd_index)                                                         \
+    sparse_agg_kernel<G, V, true, HINT, MB><<<grid, 256, 0, s>>>(a);      \
+  else                                                                    \
+    sparse_agg_kernel<G, V, false, HINT, MB><<<grid, 256, 0, s>>>(a);
+  if (minb == 4) { LAUNCH(4) } else { LAUNCH(1) }
+#undef LAUNCH
 }
 
 template <int G, int V>
 cudaError_t launch_gv(const AggArgs& a, cudaStream_t s) {
-  switch (gather_hint()) {
-    case 2: launch_ghv<G, V, 2>(a, s); break;
-    case 3: launch_ghv<G, V, 3>(a, s); break;
-    case 1: launch_ghv<G, V, 1>(a, s); break;
-    default: launch_ghv<G, V, 0>(a, s); break;
-  }
+  // variants 2 and 3 of the table in gather_hint() are not instantiated
+  if (gather_hint() == 1) launch_ghv<G, V, 1>(a, s);
+  else launch_ghv<G, V, 0>(a, s);
   return cudaGetLastError();
 }
 
