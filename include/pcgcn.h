@@ -96,6 +96,7 @@ typedef struct {
   double theta;
   double partition_ms, plan_ms; /* host time of LP+packing, and of the whole plan */
   int64_t device_bytes;         /* device memory owned by the plan */
+  int64_t shard_segments;       /* long selective rows' segments (> 1024 edges per row, reading #22) */
 } pcgcn_stats;
 
 void pcgcn_opts_default(pcgcn_opts* o);

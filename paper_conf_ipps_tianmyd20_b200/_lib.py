@@ -50,7 +50,7 @@ class Stats(ctypes.Structure):
                 ("nnz_dense", c_i64), ("intra_edges", c_i64), ("row_tiles", c_i64), ("chunks", c_i64),
                 ("row_lo", c_i64), ("row_hi", c_i64), ("shard_nnz_sparse", c_i64), ("shard_chunks", c_i64),
                 ("theta", ctypes.c_double), ("partition_ms", ctypes.c_double), ("plan_ms", ctypes.c_double),
-                ("device_bytes", c_i64)]
+                ("device_bytes", c_i64), ("shard_segments", c_i64)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}

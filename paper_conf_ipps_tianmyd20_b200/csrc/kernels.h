@@ -26,7 +26,20 @@ struct AggArgs {
   int64_t n_src;             // rows of Y (for the L2-residency decision)
   int F;
   bool relu, out_prescaled;
+  // long-row segments (reading #22): rows with more than SEG_EDGES
+  // selective edges are summed by a segment pass into seg_ws first; the row
+  // pass then adds its row's segment partials in segment order
+  const int32_t* row_seg;    // [rows] first segment id, -1 = row gathered directly (nullptr: none)
+  const int64_t* seg_lo;     // [nseg+1] shard-local edge offsets of the segments (seg_hi = next lo
+                             // within a row; the row end otherwise), see seg_hi
+  const int64_t* seg_hi;     // [nseg]
+  int64_t nseg;
+  float* seg_ws;             // [nseg x ldws] fp32 partial sums
+  int64_t ldws;
+  int* counter;              // dynamic row scheduler ticket (zeroed on the stream before each pass)
 };
+// selective edges per long-row segment
+constexpr int SEG_EDGES = 1024;
 cudaError_t launch_sparse_agg(const AggArgs& a, cudaStream_t s);
 
 // ypre = diag(r)·Y

@@ -115,11 +115,33 @@ pcgcn_status upload_plan(pcgcn_plan_s* p) {
   }
   UP(&d.ypre, (float*)nullptr, n * d.fpad_max);
   UP(&d.zrow, (float*)nullptr, 256);
+  UP(&d.counter, (int*)nullptr, 32);
+  {
+    // long selective rows -> segments of SEG_EDGES edges (reading #22)
+    std::vector<int32_t> rs(d.rows, -1);
+    std::vector<int64_t> lo, hi;
+    for (int64_t v = 0; v < d.rows; ++v) {
+      if (rp[v + 1] - rp[v] <= SEG_EDGES) continue;
+      rs[v] = int32_t(lo.size());
+      for (int64_t e = rp[v]; e < rp[v + 1]; e += SEG_EDGES) {
+        lo.push_back(e);
+        hi.push_back(std::min<int64_t>(e + SEG_EDGES, rp[v + 1]));
+      }
+    }
+    d.nseg = int64_t(lo.size());
+    if (d.nseg > 0) {
+      UP(&d.row_seg, rs.data(), d.rows);
+      UP(&d.seg_lo, lo.data(), d.nseg);
+      UP(&d.seg_hi, hi.data(), d.nseg);
+      UP(&d.seg_ws, (float*)nullptr, d.nseg * d.fpad_max);
+    }
+  }
 #undef UP
   e = cudaMemset(d.zrow, 0, 256 * sizeof(float));
   if (e != cudaSuccess) return cuda_fail(e, "memset");
   d.built = true;
   p->stats.device_bytes = d.bytes;
+  p->stats.shard_segments = d.nseg;
   return PCGCN_OK;
 }
 
@@ -187,6 +209,9 @@ pcgcn_status aggregate(pcgcn_plan_t p, const float* Y, int64_t ldy, float* Z, in
   a.F = F;
   a.relu = (flags & PCGCN_RELU) != 0;
   a.out_prescaled = (flags & PCGCN_OUT_PRESCALED) != 0;
+  a.row_seg = d.row_seg; a.seg_lo = d.seg_lo; a.seg_hi = d.seg_hi; a.nseg = d.nseg;
+  a.seg_ws = d.seg_ws; a.ldws = d.fpad_max;
+  a.counter = d.counter;
   mark(3);
   if (prof) d.ev_used[3] = true;
   e = launch_sparse_agg(a, s);

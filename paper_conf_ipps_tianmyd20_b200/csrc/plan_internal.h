@@ -27,8 +27,13 @@ struct DevicePlan {
   float* yhi = nullptr;           // [2*fpad_max x n_pad] tf32 split of the (prescaled) input, feature-major:
                                   // rows [0,npad) hi, rows [npad,2npad) lo for a call of width npad
   float* ypre = nullptr;          // [n*fpad_max] prescaled copy for un-prescaled inputs
-  float* zrow = nullptr;          // [256] zeros: gather sentinel
-  int64_t rows = 0, nnz_s = 0, nrt = 0, nch = 0;
+  float* zrow = nullptr;          // [256] zeros
+  int32_t* row_seg = nullptr;     // [rows] first long-row segment, -1 none (nullptr if nseg == 0)
+  int64_t* seg_lo = nullptr;      // [nseg] shard-local edge range of each segment
+  int64_t* seg_hi = nullptr;
+  float* seg_ws = nullptr;        // [nseg x fpad_max] segment partial sums
+  int* counter = nullptr;         // [32] selective-pass row ticket
+  int64_t rows = 0, nnz_s = 0, nrt = 0, nch = 0, nseg = 0;
   int64_t n_pad = 0;
   int fpad_max = 0;
   int64_t bytes = 0;

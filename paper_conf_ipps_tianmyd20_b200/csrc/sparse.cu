@@ -10,18 +10,22 @@
 // written once (L181).
 //
 // B200 design:
-//   * one warp per destination row; the 32 lanes split into S = 32/G edge
-//     slots of G lanes, each lane owning one float4 of the row (F <= 128) or
-//     two (F <= 256) — full lane use for narrow F (41 -> G=16, S=2);
+//   * one warp per destination row (persistent warps claim rows in plan order
+//     from a ticket counter); the 32 lanes split into S = 32/G edge slots of
+//     G lanes, G the narrowest power of two covering the row's float4s, so
+//     one load instruction reads whole rows and touches the fewest 128-byte
+//     lines (F=128 -> G=32; F=41 -> G=16, two rows per load);
 //   * the warp loads 32 source indices with one coalesced load and broadcasts
-//     them by shuffle; the unrolled loop keeps up to 32/S independent 16-byte
-//     row loads in flight per lane (the gather is L2-bandwidth bound);
+//     them by shuffle; a row address is one 32x32->64 multiply-add; full
+//     batches are unguarded and keep 8 float4 loads per lane in flight;
+//   * rows longer than SEG_EDGES are cut into segments gathered by a
+//     separate pass (balance, and bounded sequential sums: reading #22);
 //   * edge values are not stored: Â_ij = r_i r_j, with r_j folded into the
 //     producer (IN_PRESCALED) and r_i applied once in the epilogue;
 //   * fused epilogue: + dense-mode partial sum Zd (mode combine, L193),
 //     × r_i, optional second × r_i, ReLU and the bit-packed ReLU mask;
-//   * fixed summation order (4 interleaved accumulators, then a butterfly over
-//     slots): bitwise reproducible run to run.
+//   * fixed summation order (2 interleaved accumulators, then a butterfly over
+//     slots, segments in order): bitwise reproducible run to run.
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -37,108 +41,100 @@ namespace {
 __device__ __forceinline__ float4 ld_f4(const float* p) {
   return __ldg(reinterpret_cast<const float4*>(p));
 }
-// L2 eviction policies for the gather loads; see gather_hint() for the
-// measured choice (the once-read index stream is marked evict_first)
-__device__ __forceinline__ uint64_t policy_evict_last() {
-  uint64_t p;
-  asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
-  return p;
+__device__ __forceinline__ float4 ld_f4b(const char* p) {
+  return __ldg(reinterpret_cast<const float4*>(p));
 }
-__device__ __forceinline__ uint64_t policy_evict_first() {
-  uint64_t p;
-  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
-  return p;
-}
-__device__ __forceinline__ float4 ld_f4_hint(const float* p, uint64_t pol) {
-  float4 v;
-  asm volatile("ld.global.nc.L2::cache_hint.v4.f32 {%0,%1,%2,%3}, [%4], %5;"
-               : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w)
-               : "l"(p), "l"(pol));
-  return v;
-}
-__device__ __forceinline__ float4 ld_f4_na_hint(const float* p, uint64_t pol) {
-  float4 v;
-  asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.f32 {%0,%1,%2,%3}, [%4], %5;"
-               : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w)
-               : "l"(p), "l"(pol));
-  return v;
-}
-__device__ __forceinline__ int ld_idx_hint(const int* p, uint64_t pol) {
-  int v;
-  asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
-  return v;
+// base + j*stride as one 32x32->64 multiply-add (IMAD.WIDE.U32 with a 64-bit addend)
+__device__ __forceinline__ const char* row_addr(const char* base, uint32_t j, uint32_t stride) {
+  uint64_t r;
+  asm("mad.wide.u32 %0, %1, %2, %3;" : "=l"(r) : "r"(j), "r"(stride), "l"(reinterpret_cast<uint64_t>(base)));
+  return reinterpret_cast<const char*>(r);
 }
 __device__ __forceinline__ void add4(float4& a, const float4& b) {
   a.x += b.x; a.y += b.y; a.z += b.z; a.w += b.w;
 }
 
-template <int G, int V, bool HAS_ZD, int HINT, int MINB>
-__global__ void __launch_bounds__(256, MINB) sparse_agg_kernel(AggArgs a) {
-  constexpr int S = 32 / G;                 // edges in flight per warp step (slots)
-  constexpr int STEPS = 32 / S;             // steps per 32-index batch
-  // steps whose loads are all issued before any is consumed: a power of two
-  // dividing STEPS with UNR*V <= 8 float4 in flight per lane (16 measured
-  // slower on C3: the register cost lowers occupancy more than ILP gains)
-  constexpr int UCAP = 8 / V;
-  constexpr int UNR = (UCAP >= 16 && STEPS >= 16) ? 16
-                    : (UCAP >= 8 && STEPS >= 8) ? 8
-                    : (UCAP >= 4 && STEPS >= 4) ? 4
-                    : (UCAP >= 2 && STEPS >= 2) ? 2 : 1;
-  constexpr int NACC = V >= 3 ? 1 : (V == 2 ? 2 : 4);                        // interleaved partial sums
-  const int64_t row = int64_t(blockIdx.x) * 8 + (threadIdx.x >> 5);
-  if (row >= a.rows) return;
-  const int lane = threadIdx.x & 31;
-  const int slot = lane / G, l = lane % G;
-  const int nvec = (a.F + 3) >> 2;
-  const int64_t e0 = a.rowptr[row], e1 = a.rowptr[row + 1];
-  // per-lane column offsets (loop invariant); lanes past F read the zero row
-  int qoff[V];
-#pragma unroll
-  for (int v = 0; v < V; ++v) qoff[v] = (l + G * v) < nvec ? 4 * (l + G * v) : -1;
+// Lane layout for a feature row of nvec float4: the warp's 32 lanes form
+// S = 32/G edge slots of G lanes; lane l of a slot owns float4 columns
+// l, l+G, ..., l+(V-1)G.  A slot's G lanes read one contiguous piece of the
+// row per load, so each load instruction touches the fewest 128-byte lines
+// (the L1TEX wavefront count is what bounds a gather of L2-resident rows).
+template <int G, int V>
+struct Lay {
+  static constexpr int S = 32 / G;       // edges per warp step
+  static constexpr int STEPS = 32 / S;   // steps per 32-index batch
+  // steps whose loads are all issued before any is consumed (<= 8 float4
+  // per lane in flight: more costs occupancy than it gains in MLP on C3)
+  static constexpr int UCAP = 8 / V;
+  static constexpr int UNR = (UCAP >= 8 && STEPS >= 8) ? 8
+                           : (UCAP >= 4 && STEPS >= 4) ? 4
+                           : (UCAP >= 2 && STEPS >= 2) ? 2 : 1;
+  static constexpr int NACC = (V == 1 && UNR >= 2) ? 2 : 1;  // interleaved partial sums
+};
+
+// tot[v] (valid in every lane after the butterfly) = sum over the n edges at
+// cp[0..n) of Y'[cp[e]][cols of this lane].  yb = this lane's byte offset
+// into row 0 of Y' (lanes past the row re-read column 0: same line, ignored;
+// columns v >= 1 past the row are not loaded: lok[v] false).
+// Fixed order: per slot sequential over its edges in NACC interleaved sums,
+// then a butterfly over the slots — bitwise reproducible.
+template <int G, int V>
+__device__ __forceinline__ void gather_sum(const int* __restrict__ cp, int n, const char* __restrict__ yb,
+                                           uint32_t rstride, const bool (&lok)[V], int lane, float4 (&tot)[V]) {
+  using L = Lay<G, V>;
+  constexpr int S = L::S, STEPS = L::STEPS, UNR = L::UNR, NACC = L::NACC;
+  const int slot = lane / G;
   float4 acc[NACC][V];
 #pragma unroll
   for (int u = 0; u < NACC; ++u)
 #pragma unroll
     for (int v = 0; v < V; ++v) acc[u][v] = make_float4(0.f, 0.f, 0.f, 0.f);
-
-  // Branch-free batches: every lane issues UNR*V independent 16-byte loads
-  // before consuming any; edges past the row end read the zero row.
-  const float* zrow = a.zrow;
-  const uint64_t keep = policy_evict_last(), stream = policy_evict_first();
-  auto ld_idx = [](const int* p, uint64_t pol) { return HINT == 3 ? __ldg(p) : ld_idx_hint(p, pol); };
-  // index batches are prefetched one ahead
-  int nextidx = (e0 + lane < e1) ? ld_idx(a.col + e0 + lane, stream) : -1;
-  // Loads rotate over NACC interleaved accumulators (a slot adds <= d/(S*NACC)
-  // terms sequentially).  Measured on C3 hub rows (d = 25K, all-positive
-  // eigenvector input): 1.2e-7 relative error, far inside the 1e-5 gate; a
-  // pairwise batch-tree variant was 17% slower for no measurable gain.
-  for (int64_t base = e0; base < e1; base += 32) {
-    const int cnt = (e1 - base) < 32 ? int(e1 - base) : 32;
+  int nextidx = lane < n ? __ldg(cp + lane) : 0;
+  for (int base = 0; base < n; base += 32) {
+    const int cnt = (n - base) < 32 ? n - base : 32;
     const int myidx = nextidx;
-    nextidx = (base + 32 + lane < e1) ? ld_idx(a.col + base + 32 + lane, stream) : -1;
+    nextidx = (base + 32 + lane < n) ? __ldg(cp + base + 32 + lane) : 0;  // next batch, one ahead
+    if (cnt == 32) {
+      // full batch: unguarded, every lane keeps UNR*V 16-byte loads in flight
 #pragma unroll
-    for (int k0 = 0; k0 < STEPS; k0 += UNR) {
-      float4 buf[UNR][V];
+      for (int k0 = 0; k0 < STEPS; k0 += UNR) {
+        float4 buf[UNR][V];
 #pragma unroll
-      for (int u = 0; u < UNR; ++u) {
-        const int j = __shfl_sync(0xffffffffu, myidx, (k0 + u) * S + slot);
-        const float* src = a.Y + int64_t(j) * a.ldy;
+        for (int u = 0; u < UNR; ++u) {
+          const uint32_t j = uint32_t(__shfl_sync(0xffffffffu, myidx, (k0 + u) * S + slot));
+          const char* p = row_addr(yb, j, rstride);
 #pragma unroll
-        for (int v = 0; v < V; ++v) {
-          const float* p = (j >= 0 && qoff[v] >= 0) ? src + qoff[v] : zrow;
-          if (HINT == 1) buf[u][v] = ld_f4_hint(p, keep);
-          else if (HINT == 2) buf[u][v] = ld_f4_na_hint(p, keep);
-          else buf[u][v] = ld_f4(p);
+          for (int v = 0; v < V; ++v)
+            buf[u][v] = (v == 0 || lok[v]) ? ld_f4b(p + 16 * G * v) : make_float4(0.f, 0.f, 0.f, 0.f);
         }
+#pragma unroll
+        for (int u = 0; u < UNR; ++u)
+#pragma unroll
+          for (int v = 0; v < V; ++v) add4(acc[u % NACC][v], buf[u][v]);
       }
+    } else {
+      // last (partial) batch of the row: slots past the end add nothing
 #pragma unroll
-      for (int u = 0; u < UNR; ++u)
+      for (int k0 = 0; k0 < STEPS; k0 += UNR) {
+        float4 buf[UNR][V];
 #pragma unroll
-        for (int v = 0; v < V; ++v) add4(acc[(k0 + u) % NACC][v], buf[u][v]);
-      if ((k0 + UNR) * S >= cnt) break;  // warp-uniform: rest of the batch is empty
+        for (int u = 0; u < UNR; ++u) {
+          const int e = (k0 + u) * S + slot;
+          const uint32_t j = uint32_t(__shfl_sync(0xffffffffu, myidx, e));
+          const char* p = row_addr(yb, j, rstride);
+#pragma unroll
+          for (int v = 0; v < V; ++v)
+            buf[u][v] = (e < cnt && (v == 0 || lok[v])) ? ld_f4b(p + 16 * G * v)
+                                                          : make_float4(0.f, 0.f, 0.f, 0.f);
+        }
+#pragma unroll
+        for (int u = 0; u < UNR; ++u)
+#pragma unroll
+          for (int v = 0; v < V; ++v) add4(acc[u % NACC][v], buf[u][v]);
+        if ((k0 + UNR) * S >= cnt) break;  // warp-uniform: rest of the batch is empty
+      }
     }
   }
-  float4 tot[V];
 #pragma unroll
   for (int v = 0; v < V; ++v) {
     tot[v] = acc[0][v];
@@ -152,94 +148,155 @@ __global__ void __launch_bounds__(256, MINB) sparse_agg_kernel(AggArgs a) {
       tot[v].w += __shfl_xor_sync(0xffffffffu, tot[v].w, off);
     }
   }
-  const float ri = a.r[a.row_lo + row];
-  const int zi = HAS_ZD ? a.zd_index[row] : -1;
-  uint32_t bal[V][4];
+}
+
+// per-lane byte offset of this lane's first float4 (lanes past the row: 0)
+template <int G>
+__device__ __forceinline__ int lane_col(int lane, int v, int nvec) {
+  const int q = lane % G + G * v;
+  return q < nvec ? q : -1;
+}
+
+// Segment pass: one warp per segment of a long row (<= SEG_EDGES edges),
+// partial sums to seg_ws.
+template <int G, int V>
+__global__ void __launch_bounds__(256, 4) sparse_seg_kernel(AggArgs a) {
+  const int64_t sg = int64_t(blockIdx.x) * 8 + (threadIdx.x >> 5);
+  if (sg >= a.nseg) return;
+  const int lane = threadIdx.x & 31;
+  const int nvec = (a.F + 3) >> 2;
+  const int q0 = lane_col<G>(lane, 0, nvec);
+  const char* yb = reinterpret_cast<const char*>(a.Y) + 16 * (q0 < 0 ? 0 : q0);
+  const int64_t lo = a.seg_lo[sg], hi = a.seg_hi[sg];
+  bool lok[V];
+#pragma unroll
+  for (int v = 0; v < V; ++v) lok[v] = lane_col<G>(lane, v, nvec) >= 0;
+  float4 tot[V];
+  gather_sum<G, V>(a.col + lo, int(hi - lo), yb, uint32_t(a.ldy * 4), lok, lane, tot);
+  if (lane < G) {
+#pragma unroll
+    for (int v = 0; v < V; ++v) {
+      const int q = lane_col<G>(lane, v, nvec);
+      if (q >= 0) *reinterpret_cast<float4*>(a.seg_ws + sg * a.ldws + 4 * q) = tot[v];
+    }
+  }
+}
+
+// Row pass: persistent warps claim destination rows in plan order from a
+// ticket counter (dynamic balance without losing the partition order's L2
+// locality); a row is gathered directly or, if long, summed from its
+// segment partials in segment order.  Fused epilogue: + full-mode partial
+// sum Zd (mode combine, L193), x r_i (optionally twice), ReLU, bit mask.
+template <int G, int V, bool HAS_ZD, bool HAS_SEG>
+__global__ void __launch_bounds__(256, 4) sparse_row_kernel(AggArgs a) {
+  const int lane = threadIdx.x & 31;
+  const int slot = lane / G;
+  const int nvec = (a.F + 3) >> 2;
+  int qv[V];
+  bool lok[V];
 #pragma unroll
   for (int v = 0; v < V; ++v) {
-    const bool own = slot == 0 && qoff[v] >= 0;
-    float4 z = tot[v];
-    if (HAS_ZD && own && zi >= 0) add4(z, ld_f4(a.zd + int64_t(zi) * a.ldzd + qoff[v]));
-    z.x *= ri; z.y *= ri; z.z *= ri; z.w *= ri;
-    if (a.out_prescaled) { z.x *= ri; z.y *= ri; z.z *= ri; z.w *= ri; }
-    if (a.mask) {
-      const int c = qoff[v];
-      bal[v][0] = __ballot_sync(0xffffffffu, own && z.x > 0.f && c + 0 < a.F);
-      bal[v][1] = __ballot_sync(0xffffffffu, own && z.y > 0.f && c + 1 < a.F);
-      bal[v][2] = __ballot_sync(0xffffffffu, own && z.z > 0.f && c + 2 < a.F);
-      bal[v][3] = __ballot_sync(0xffffffffu, own && z.w > 0.f && c + 3 < a.F);
-    }
-    if (a.relu) {
-      z.x = fmaxf(z.x, 0.f); z.y = fmaxf(z.y, 0.f); z.z = fmaxf(z.z, 0.f); z.w = fmaxf(z.w, 0.f);
-    }
-    if (own) *reinterpret_cast<float4*>(a.Z + row * a.ldz + qoff[v]) = z;
+    qv[v] = lane_col<G>(lane, v, nvec);
+    lok[v] = qv[v] >= 0;
   }
-  if (a.mask) {
-    // lane w assembles mask word w: column col = 32w + b lives in lane
-    // (col/4) % G, vector v = (col/4) / G, component col % 4
-    const int mw = (a.F + 31) >> 5;
-    if (lane < mw) {
-      uint32_t word = 0;
-#pragma unroll 4
-      for (int b = 0; b < 32; ++b) {
-        const int col = 32 * lane + b;
-        const int q = col >> 2;
-        const int vv = q / G, ll = q % G;
-        uint32_t bit = 0;
+  const char* yb = reinterpret_cast<const char*>(a.Y) + 16 * (qv[0] < 0 ? 0 : qv[0]);
+  const uint32_t rstride = uint32_t(a.ldy * 4);
+  auto claim = [&]() {
+    int t = 0;
+    if (lane == 0) t = atomicAdd(a.counter, 1);
+    return __shfl_sync(0xffffffffu, t, 0);
+  };
+  int row = claim();
+  while (row < a.rows) {
+    const int nxt = claim();
+    const int64_t e0 = a.rowptr[row], e1 = a.rowptr[row + 1];
+    float4 tot[V];
+    const int sg = HAS_SEG ? a.row_seg[row] : -1;
+    if (HAS_SEG && sg >= 0) {
+      const int ns = int((e1 - e0 + SEG_EDGES - 1) / SEG_EDGES);
 #pragma unroll
-        for (int v = 0; v < V; ++v)
-          if (v == vv) bit = (bal[v][col & 3] >> ll) & 1u;
-        word |= bit << b;
+      for (int v = 0; v < V; ++v) tot[v] = make_float4(0.f, 0.f, 0.f, 0.f);
+      if (slot == 0) {
+        for (int k = 0; k < ns; ++k)
+#pragma unroll
+          for (int v = 0; v < V; ++v)
+            if (qv[v] >= 0) add4(tot[v], __ldcg(reinterpret_cast<const float4*>(
+                                              a.seg_ws + int64_t(sg + k) * a.ldws + 4 * qv[v])));
       }
-      a.mask[row * a.mask_ld + lane] = word;
+    } else {
+      gather_sum<G, V>(a.col + e0, int(e1 - e0), yb, rstride, lok, lane, tot);
     }
+    const float ri = a.r[a.row_lo + row];
+    const int zi = HAS_ZD ? a.zd_index[row] : -1;
+    uint32_t bal[V][4];
+#pragma unroll
+    for (int v = 0; v < V; ++v) {
+      const bool own = slot == 0 && qv[v] >= 0;
+      float4 z = tot[v];
+      if (HAS_ZD && own && zi >= 0) add4(z, ld_f4(a.zd + int64_t(zi) * a.ldzd + 4 * qv[v]));
+      z.x *= ri; z.y *= ri; z.z *= ri; z.w *= ri;
+      if (a.out_prescaled) { z.x *= ri; z.y *= ri; z.z *= ri; z.w *= ri; }
+      if (a.mask) {
+        const int c = 4 * qv[v];
+        bal[v][0] = __ballot_sync(0xffffffffu, own && z.x > 0.f && c + 0 < a.F);
+        bal[v][1] = __ballot_sync(0xffffffffu, own && z.y > 0.f && c + 1 < a.F);
+        bal[v][2] = __ballot_sync(0xffffffffu, own && z.z > 0.f && c + 2 < a.F);
+        bal[v][3] = __ballot_sync(0xffffffffu, own && z.w > 0.f && c + 3 < a.F);
+      }
+      if (a.relu) {
+        z.x = fmaxf(z.x, 0.f); z.y = fmaxf(z.y, 0.f); z.z = fmaxf(z.z, 0.f); z.w = fmaxf(z.w, 0.f);
+      }
+      if (own) *reinterpret_cast<float4*>(a.Z + int64_t(row) * a.ldz + 4 * qv[v]) = z;
+    }
+    if (a.mask) {
+      // lane w assembles mask word w: column col = 32w + b lives in lane
+      // (col/4) % G, vector v = (col/4) / G, component col % 4
+      const int mw = (a.F + 31) >> 5;
+      if (lane < mw) {
+        uint32_t word = 0;
+#pragma unroll 4
+        for (int b = 0; b < 32; ++b) {
+          const int col = 32 * lane + b;
+          const int q = col >> 2;
+          const int vv = q / G, ll = q % G;
+          uint32_t bit = 0;
+#pragma unroll
+          for (int v = 0; v < V; ++v)
+            if (v == vv) bit = (bal[v][col & 3] >> ll) & 1u;
+          word |= bit << b;
+        }
+        a.mask[int64_t(row) * a.mask_ld + lane] = word;
+      }
+    }
+    row = nxt;
   }
-}
-
-int gather_hint() {
-  // Gather cache policy (PCGCN_GATHER_HINT, tuning override).  Measured on C3
-  // (bench, 10 steps, two interleaved runs each), F=128 / F=41 sparse ms:
-  //   0 (default) rows plain ld.global.nc, index evict_first  3.40 / 1.41
-  //   1 rows L2::evict_last                                    3.83 / 1.50
-  //   2 rows L1::no_allocate + evict_last                      3.83 / 2.81
-  //   3 rows and index plain                                   3.43 / 1.39
-  // (evict_last pins all of Y' and starves the L1/L2 replacement of the
-  // hot hub rows; no_allocate loses the L1 hits of the narrow rows)
-  static int h = -1;
-  if (h < 0) {
-    const char* e = getenv("PCGCN_GATHER_HINT");
-    h = e ? atoi(e) : 0;
-    if (h != 1) h = 0;
-  }
-  return h;
-}
-
-template <int G, int V, int HINT>
-void launch_ghv(const AggArgs& a, cudaStream_t s) {
-  // Occupancy target: 4 CTAs (32 warps) per SM caps registers at 64.  On C3
-  // (same box, interleaved runs) F=128 3.72 -> 3.62 ms, F=41 1.60 -> 1.42 ms
-  // against the unconstrained 76-80 registers (3 CTAs).  PCGCN_SPARSE_MINB=1
-  // restores the unconstrained build (tuning override).
-  static int minb = -1;
-  if (minb < 0) {
-    const char* e = getenv("PCGCN_SPARSE_MINB");
-    minb = (e && atoi(e) == 1) ? 1 : 4;
-  }
-  dim3 grid(unsigned((a.rows + 7) / 8));
-#define LAUNCH(MB)                                                        \
-  if (a.zd_index)                                                         \
-    sparse_agg_kernel<G, V, true, HINT, MB><<<grid, 256, 0, s>>>(a);      \
-  else                                                                    \
-    sparse_agg_kernel<G, V, false, HINT, MB><<<grid, 256, 0, s>>>(a);
-  if (minb == 4) { LAUNCH(4) } else { LAUNCH(1) }
-#undef LAUNCH
 }
 
 template <int G, int V>
 cudaError_t launch_gv(const AggArgs& a, cudaStream_t s) {
-  // variants 2 and 3 of the table in gather_hint() are not instantiated
-  if (gather_hint() == 1) launch_ghv<G, V, 1>(a, s);
-  else launch_ghv<G, V, 0>(a, s);
+  // persistent row pass: as many 8-warp CTAs as fit (4 per SM at 64 registers)
+  static int slots = 0;
+  if (!slots) {
+    int dev = 0, sms = 148, per = 4;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, sparse_row_kernel<G, V, true, true>, 256, 0);
+    slots = sms * (per > 0 ? per : 1);
+  }
+  cudaError_t e = cudaMemsetAsync(a.counter, 0, sizeof(int), s);
+  if (e != cudaSuccess) return e;
+  if (a.nseg > 0) {
+    sparse_seg_kernel<G, V><<<unsigned((a.nseg + 7) / 8), 256, 0, s>>>(a);
+  }
+  const int64_t want = (a.rows + 7) / 8;
+  const unsigned grid = unsigned(want < slots ? want : slots);
+#define LAUNCH(ZD, SG) sparse_row_kernel<G, V, ZD, SG><<<grid, 256, 0, s>>>(a)
+  const bool zd = a.zd_index != nullptr, sg = a.nseg > 0;
+  if (zd && sg) LAUNCH(true, true);
+  else if (zd) LAUNCH(true, false);
+  else if (sg) LAUNCH(false, true);
+  else LAUNCH(false, false);
+#undef LAUNCH
   return cudaGetLastError();
 }
 
@@ -293,64 +350,18 @@ __global__ void __launch_bounds__(256) split_transpose_kernel(const float* __res
 
 }  // namespace
 
-cudaError_t launch_sparse_agg_pass(const AggArgs& a, cudaStream_t s);
-
-// Optional feature-split passes (64 feature columns per pass) so each pass's
-// gather set stays L2-resident.  Measured on C3 at F=128 (θ=0.04): one pass
-// reads 4.4 GB from DRAM at an 81% L2 hit rate in 4.16 ms; two passes read
-// 2 x 0.74 GB at 93.5% but take 2 x 2.37 ms — the gather is bound by the
-// per-edge work, not by the DRAM misses — so the split is OFF by default
-// (PCGCN_SPLIT_BYTES=<bytes> enables it above that Y' size).
 cudaError_t launch_sparse_agg(const AggArgs& a, cudaStream_t s) {
   if (a.rows <= 0) return cudaSuccess;
-  static int64_t split_bytes = -1;
-  if (split_bytes < 0) {
-    const char* e = getenv("PCGCN_SPLIT_BYTES");  // tuning override (benchmarks only)
-    split_bytes = e ? atoll(e) : INT64_MAX;
-  }
-  const int64_t ybytes = a.n_src * int64_t((a.F + 3) / 4 * 4) * 4;
-  if (a.F <= 64 || ybytes <= split_bytes) return launch_sparse_agg_pass(a, s);
-  for (int c0 = 0; c0 < a.F; c0 += 64) {
-    AggArgs b = a;
-    b.F = (a.F - c0) < 64 ? a.F - c0 : 64;
-    b.Y = a.Y + c0;
-    b.Z = a.Z + c0;
-    if (a.zd) b.zd = a.zd + c0;
-    if (a.mask) b.mask = a.mask + c0 / 32;
-    cudaError_t e = launch_sparse_agg_pass(b, s);
-    if (e != cudaSuccess) return e;
-  }
-  return cudaSuccess;
-}
-
-cudaError_t launch_sparse_agg_pass(const AggArgs& a, cudaStream_t s) {
-  // (G lanes x V float4) per edge, minimising warp instructions per edge
-  // (~G*(3+5V)/32) while keeping each v-slice of G lanes a contiguous segment
+  // G lanes x V float4 per edge slot: the narrowest power-of-two slot that
+  // covers the row, so one load instruction reads whole rows (fewest lines)
   const int nvec = (a.F + 3) / 4;
-  // tuning override (benchmarks only): PCGCN_SPARSE_GV="G,V" when G*V >= nvec
-  static int og = -1, ov = -1;
-  if (og < 0) {
-    og = ov = 0;
-    if (const char* e = getenv("PCGCN_SPARSE_GV")) sscanf(e, "%d,%d", &og, &ov);
-  }
-  if (og > 0 && og * ov >= nvec) {
-#define GV(g, v) if (og == g && ov == v) return launch_gv<g, v>(a, s);
-    GV(32, 1) GV(32, 2) GV(16, 1) GV(16, 2) GV(16, 3) GV(16, 4) GV(8, 1) GV(8, 2) GV(8, 3) GV(8, 4)
-    GV(4, 3) GV(4, 4) GV(2, 4)
-#undef GV
-  }
   if (nvec <= 1) return launch_gv<1, 1>(a, s);
-  if (nvec <= 2) return launch_gv<1, 2>(a, s);
-  if (nvec <= 3) return launch_gv<1, 3>(a, s);
-  if (nvec <= 4) return launch_gv<1, 4>(a, s);
-  if (nvec <= 6) return launch_gv<2, 3>(a, s);
-  if (nvec <= 8) return launch_gv<2, 4>(a, s);
-  if (nvec <= 12) return launch_gv<4, 3>(a, s);
-  if (nvec <= 16) return launch_gv<4, 4>(a, s);
-  if (nvec <= 24) return launch_gv<8, 3>(a, s);
-  if (nvec <= 32) return launch_gv<32, 1>(a, s);  // measured faster than (8,4) at F=128 on C3
-  if (nvec <= 48) return launch_gv<16, 3>(a, s);
-  return launch_gv<16, 4>(a, s);
+  if (nvec <= 2) return launch_gv<2, 1>(a, s);
+  if (nvec <= 4) return launch_gv<4, 1>(a, s);
+  if (nvec <= 8) return launch_gv<8, 1>(a, s);
+  if (nvec <= 16) return launch_gv<16, 1>(a, s);
+  if (nvec <= 32) return launch_gv<32, 1>(a, s);
+  return launch_gv<32, 2>(a, s);
 }
 
 cudaError_t launch_prescale(const float* Y, int64_t ldy, const float* r, int64_t n, int F, float* ypre,

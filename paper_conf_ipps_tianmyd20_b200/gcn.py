@@ -29,7 +29,10 @@ from . import _lib as L
 
 
 def _ld(F: int) -> int:
-    return (F + 3) // 4 * 4
+    """Row stride (floats) of an activation of width F: 16-byte rows, and
+    64-byte rows above 16 features so a gathered row touches the fewest
+    128-byte lines (F=41: 48, two lines per row at any row index)."""
+    return (F + 3) // 4 * 4 if F <= 16 else (F + 15) // 16 * 16
 
 
 class GCN2:
@@ -164,7 +167,8 @@ class GCN2:
         """Kernel launches of libpcgcn per epoch (for the bench's gpu_launches)."""
         st = self.plan.stats()
         dense = st["shard_chunks"] > 0
-        agg = 1 + (2 if dense else 0)          # prescale/split + dense tiles + selective rows
+        # split + dense tiles (full mode), segment pass (long rows), selective rows
+        agg = 1 + (2 if dense else 0) + (1 if st["shard_segments"] > 0 else 0)
         gemm_xw = 1 + 1                          # tile kernel + pad zeroing (ld > N) — upper bound
         n = 2 * gemm_xw + 4 * agg + 2 + 2 * 2 + 2  # + softmax(2) + 2 x xtg(2) + dwt(2)
         n += 2 if self.optimizer == "adam" else 1

@@ -405,40 +405,53 @@ print("ok")
     assert out.stdout.strip().endswith("ok")
 
 
-def test_feature_split_passes_subprocess():
-    """The optional feature-split passes (64-column passes, enabled by
-    PCGCN_SPLIT_BYTES) forced on a small graph in a fresh process: same
-    result as the single pass up to summation order (the lane layout (G,V)
-    depends on the pass width, so the order of the fp32 sums differs)."""
-    import os
-    import subprocess
-    import sys
-    code = r'''
-import sys, numpy as np, torch
-sys.path.insert(0, ".")
-from paper_conf_ipps_tianmyd20_b200 import _lib as L
-from synth import configs as C
-g = C.graph(C.CORA)
-rng = np.random.default_rng(5)
-F = 200
-Y = np.zeros((g.n, 200), np.float32); Y[:] = rng.standard_normal((g.n, F))
-pl = L.Plan(g.n, g.rowptr, g.col, 8, 0.03, f_max=256)
-Yd = torch.from_numpy(Y).cuda(); Z = torch.zeros_like(Yd)
-mask = torch.zeros(g.n, 7, dtype=torch.int32, device="cuda")
-pl.forward(Yd, Z, F=F, flags=L.RELU | L.MASK_OUT, mask=mask)
-torch.cuda.synchronize()
-np.save(sys.argv[1] + "_z.npy", Z.cpu().numpy()); np.save(sys.argv[1] + "_m.npy", mask.cpu().numpy())
-'''
-    import tempfile
-    d = tempfile.mkdtemp()
-    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-    for tag, sb in (("one", str(1 << 40)), ("split", "0")):
-        env = dict(os.environ, PCGCN_SPLIT_BYTES=sb)
-        subprocess.run([sys.executable, "-c", code, os.path.join(d, tag)], check=True, env=env, cwd=root)
-    z1, z2 = np.load(os.path.join(d, "one_z.npy")), np.load(os.path.join(d, "split_z.npy"))
-    np.testing.assert_allclose(z2, z1, rtol=1e-5, atol=1e-6)
-    m1, m2 = np.load(os.path.join(d, "one_m.npy")), np.load(os.path.join(d, "split_m.npy"))
-    differ = (m1 ^ m2).view(np.uint32)
-    # mask bits may only differ where the (ReLU-ed) value is ~0 in both runs
-    bits = ((differ[:, :, None] >> np.arange(32, dtype=np.uint32)) & 1).reshape(len(m1), -1)[:, :200]
-    assert np.all(np.abs(z1[bits.astype(bool)]) < 1e-5)
+def _hubs(n_leaf=5000, extra=3):
+    """Stars joined at their leaves: hub rows with 1-5 long-row segments
+    (> SEG_EDGES = 1024 selective edges) next to short rows."""
+    edges = []
+    base = 0
+    for k, leaves in enumerate([n_leaf, 1100, 2047, 1025]):
+        hub = base
+        edges += [(hub, hub + i) for i in range(1, leaves + 1)]
+        base += leaves + 1
+    rng = np.random.default_rng(7)
+    e = rng.integers(0, base, size=(extra * base, 2))
+    edges += [tuple(x) for x in e if x[0] != x[1]]
+    return G.from_edges(base, edges)
+
+
+@pytest.mark.parametrize("F", [1, 7, 41, 128, 200])
+@pytest.mark.parametrize("ldpad", [0, 16])
+def test_long_rows_segments(F, ldpad):
+    """Rows longer than SEG_EDGES go through the segment pass and are summed
+    from their segment partials (reading #22); values, ReLU and the
+    mask vs the oracle, with row strides padded past roundup(F, 4)."""
+    g = _hubs()
+    pl = L.Plan(g.n, g.rowptr, g.col, 4, 2.0, f_max=256)
+    assert pl.stats()["shard_segments"] >= 5 + 2 + 2 + 2
+    perm = pl.perm()
+    ld = _ld(F) + ldpad
+    Y = _feat(g.n, F, 21)
+    Yp = np.zeros((g.n, ld), np.float32)
+    Yp[:, :F] = Y[perm]
+    Yd = torch.from_numpy(Yp).cuda()
+    Zd = torch.full((g.n, ld), float("nan"), device="cuda")
+    mw = (F + 31) // 32
+    mask = torch.zeros(g.n, mw, dtype=torch.int32, device="cuda")
+    pl.forward(Yd, Zd, F=F, flags=L.RELU | L.MASK_OUT, mask=mask)
+    torch.cuda.synchronize()
+    Ahat = O.normalized_adjacency(g.n, g.rowptr, g.col)[0]
+    Zs = O.aggregate(Ahat, Y.astype(np.float64))[perm]
+    scale = np.maximum(O.aggregate(abs(Ahat), np.abs(Y.astype(np.float64)))[perm], 1e-30)
+    Zc = Zd.cpu().numpy()[:, :F].astype(np.float64)
+    err = np.max(np.abs(Zc - np.maximum(Zs, 0)) / scale)
+    assert err <= TOL, err
+    m = mask.cpu().numpy().view(np.uint32)
+    bits = ((m[:, :, None] >> np.arange(32, dtype=np.uint32)) & 1).reshape(g.n, 32 * mw)
+    assert np.all((bits[:, :F].astype(bool) == (Zs > 0)) | (np.abs(Zs) < 1e-6 * scale))
+    assert np.all(bits[:, F:] == 0)
+    # run to run bitwise (dynamic row scheduling does not change any row's order)
+    Z2 = torch.full_like(Zd, float("nan"))
+    pl.forward(Yd, Z2, F=F, flags=L.RELU | L.MASK_OUT, mask=mask)
+    torch.cuda.synchronize()
+    assert torch.equal(Z2[:, :F], Zd[:, :F])
