@@ -169,10 +169,15 @@ pcgcn_status pcgcn_gemm_xtg(const float* X, int64_t ldx, const float* D, int64_t
 
 /* O = diag(s)·((D·Wᵀ) ⊙ mask):  D DEVICE [M x N] ld ldd, W DEVICE [K x N] (ld N),
  * mask DEVICE u32 bits [M x ceil(K/32)] (PCGCN_MASK_OUT layout) or NULL, s DEVICE [M] or NULL,
- * O DEVICE [M x K] ld ldo. */
+ * O DEVICE [M x K] ld ldo (pad columns [K, ldo) written as 0).  The backward of the layer-2
+ * transform through the ReLU (a11; the paper is silent on the backward).  With ldd, ldo
+ * multiples of 4, K <= 256 and `work` (DEVICE, pcgcn_gemm_dwt_work_floats(K,N) floats) it
+ * runs on the tcgen05 engine in 3xTF32 with the mask and scale in the epilogue; else (work
+ * NULL / unaligned) on fp32 CUDA cores. */
+int64_t pcgcn_gemm_dwt_work_floats(int32_t K, int32_t N);
 pcgcn_status pcgcn_gemm_dwt(const float* D, int64_t ldd, const float* W, const uint32_t* mask,
                             const float* s, float* O, int64_t ldo, int64_t M, int32_t N, int32_t K,
-                            void* stream);
+                            float* work, void* stream);
 
 /* Softmax cross-entropy over the train mask (reading #14):
  *   loss = (1/nT) Σ_{i: train_i} [logsumexp(L_i) - L_{i,y_i}]

@@ -72,7 +72,8 @@ _sig("pcgcn_gemm_xw_work_floats", c_i64, c_i32, c_i32)
 _sig("pcgcn_gemm_xw", c_i32, c_vp, c_i64, c_vp, c_i64, c_vp, c_vp, c_i64, c_i64, c_i32, c_i32, c_vp, c_vp)
 _sig("pcgcn_gemm_xtg_work_floats", c_i64, c_i64, c_i32, c_i32)
 _sig("pcgcn_gemm_xtg", c_i32, c_vp, c_i64, c_vp, c_i64, c_vp, c_i64, c_i32, c_i32, c_vp, c_vp)
-_sig("pcgcn_gemm_dwt", c_i32, c_vp, c_i64, c_vp, c_vp, c_vp, c_vp, c_i64, c_i64, c_i32, c_i32, c_vp)
+_sig("pcgcn_gemm_dwt", c_i32, c_vp, c_i64, c_vp, c_vp, c_vp, c_vp, c_i64, c_i64, c_i32, c_i32, c_vp, c_vp)
+_sig("pcgcn_gemm_dwt_work_floats", c_i64, c_i32, c_i32)
 _sig("pcgcn_softmax_ce", c_i32, c_vp, c_i64, c_vp, c_vp, c_i64, c_i32, c_f32, c_vp, c_vp, c_vp, c_vp, c_vp)
 _sig("pcgcn_adam", c_i32, c_vp, c_vp, c_vp, c_vp, c_i64, c_f32, c_f32, c_f32, c_f32, c_vp, c_vp)
 _sig("pcgcn_sgd", c_i32, c_vp, c_vp, c_i64, c_f32, c_vp)
@@ -212,12 +213,16 @@ def gemm_xtg(X, D, G, work, M=None, K=None, N=None, stream=None):
                              _stream(stream)), "pcgcn_gemm_xtg")
 
 
-def gemm_dwt(D, W, mask, s, O, M=None, N=None, K=None, stream=None):
+def gemm_dwt_work_floats(K, N):
+    return int(lib.pcgcn_gemm_dwt_work_floats(K, N))
+
+
+def gemm_dwt(D, W, mask, s, O, M=None, N=None, K=None, work=None, stream=None):
     M = D.shape[0] if M is None else M
     K = W.shape[0] if K is None else K
     N = W.shape[1] if N is None else N
     check(lib.pcgcn_gemm_dwt(_ptr(D), D.stride(0), _ptr(W), _ptr(mask), s, _ptr(O), O.stride(0), M, N, K,
-                             _stream(stream)), "pcgcn_gemm_dwt")
+                             _ptr(work), _stream(stream)), "pcgcn_gemm_dwt")
 
 
 def softmax_ce(L, labels, train, inv_nT, s, dL, loss, work, M=None, C=None, stream=None):

@@ -148,7 +148,7 @@ cudaError_t launch_gemm_xw(const float* X, int64_t ldx, const float* W, int64_t 
 
 int64_t gemm_xtg_work_floats(int64_t M, int K, int N) {
   const int64_t simt = int64_t(xtg_slices(M)) * K * N;
-  const int64_t tc = 2 * int64_t(npad16(N)) * r32(M) + tc_xtg_slices(M) * int64_t(K) * npad16(N);
+  const int64_t tc = 2 * int64_t(npad16(N)) * r32(M) + tc_xtg_slices(M, K) * int64_t(K) * npad16(N);
   return simt > tc ? simt : tc;
 }
 
@@ -181,7 +181,7 @@ cudaError_t launch_gemm_xtg(const float* X, int64_t ldx, const float* D, int64_t
     if (e != cudaSuccess) return e;
     const int64_t cnt = int64_t(K) * N;
     reduce_slices_ld_kernel<<<unsigned(std::max<int64_t>(1, std::min<int64_t>(1024, (cnt + 255) / 256))), 256, 0, st>>>(
-        part, int(tc_xtg_slices(M)), K, N, np, G);
+        part, int(tc_xtg_slices(M, K)), K, N, np, G);
     return cudaGetLastError();
   }
   // G[K x N] = Xᵀ D : output rows = K (A = X transposed), reduction over M
@@ -195,9 +195,41 @@ cudaError_t launch_gemm_xtg(const float* X, int64_t ldx, const float* D, int64_t
   return cudaGetLastError();
 }
 
+// tf32 hi/lo split of W [K x N] (ld ldw) kept row-major = feature-major for
+// the engine's B operand of O = D·Wᵀ: hi/lo [np x ldT], rows >= K and
+// columns >= N zero
+__global__ void split_rows_kernel(const float* __restrict__ W, int64_t ldw, int K, int N, int np, int64_t ldT,
+                                  float* __restrict__ hi, float* __restrict__ lo) {
+  const int64_t total = int64_t(np) * ldT;
+  for (int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < total;
+       i += int64_t(gridDim.x) * blockDim.x) {
+    const int64_t r = i / ldT, c = i - r * ldT;
+    const float v = (r < K && c < N) ? W[r * ldw + c] : 0.f;
+    const float h = __uint_as_float(__float_as_uint(v) & 0xffffe000u);
+    hi[i] = h;
+    lo[i] = v - h;
+  }
+}
+
+int64_t gemm_dwt_work_floats(int K, int N) { return 2 * int64_t(npad16(K)) * r32(N); }
+
 cudaError_t launch_gemm_dwt(const float* D, int64_t ldd, const float* W, const uint32_t* mask,
                             const float* s, float* O, int64_t ldo, int64_t M, int N, int K,
-                            cudaStream_t st) {
+                            float* work, cudaStream_t st) {
+  if (work && ldd % 4 == 0 && ldo % 4 == 0 && K <= 256 && M > 0) {
+    // tcgen05 3xTF32 (the xw engine with D as A, W rows as the feature-major
+    // B, and the ReLU' bit mask + row scale in the epilogue)
+    const int np = npad16(K);
+    const int64_t ldT = r32(N);
+    float* hi = work;
+    float* lo = work + int64_t(np) * ldT;
+    split_rows_kernel<<<unsigned(std::min<int64_t>(256, (np * ldT + 255) / 256)), 256, 0, st>>>(
+        W, N, K, N, np, ldT, hi, lo);
+    cudaError_t e = launch_tc_gemm_xw(D, ldd, hi, lo, ldT, s, O, ldo, M, N, K, st, mask, (K + 31) / 32);
+    if (e != cudaSuccess) return e;
+    if (ldo > np) zero_pad_kernel<<<256, 256, 0, st>>>(O, ldo, M, np);
+    return cudaGetLastError();
+  }
   // O[M x K] = D[M x N] · Wᵀ  with W [K x N] row-major: opB(n, k) = W[k*N + n]
   dim3 grid(unsigned((M + BM - 1) / BM), unsigned((K + BN - 1) / BN), 1);
   gemm_simt_kernel<false, true><<<grid, 256, 0, st>>>(D, ldd, W, N, O, ldo, M, K, N, N, s, mask,

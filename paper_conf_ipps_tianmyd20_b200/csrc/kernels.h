@@ -30,13 +30,13 @@ struct AggArgs {
   // selective edges are summed by a segment pass into seg_ws first; the row
   // pass then adds its row's segment partials in segment order
   const int32_t* row_seg;    // [rows] first segment id, -1 = row gathered directly (nullptr: none)
-  const int64_t* seg_lo;     // [nseg+1] shard-local edge offsets of the segments (seg_hi = next lo
-                             // within a row; the row end otherwise), see seg_hi
+  const int64_t* seg_lo;     // [nseg] shard-local edge range [seg_lo, seg_hi) of each segment
   const int64_t* seg_hi;     // [nseg]
   int64_t nseg;
   float* seg_ws;             // [nseg x ldws] fp32 partial sums
   int64_t ldws;
   int* counter;              // dynamic row scheduler ticket (zeroed on the stream before each pass)
+  bool idx_evict_first;      // L2 evict_first hint on the index stream (set by the launcher)
 };
 // selective edges per long-row segment
 constexpr int SEG_EDGES = 1024;
@@ -78,16 +78,18 @@ cudaError_t launch_gemm_xw(const float* X, int64_t ldx, const float* W, int64_t 
                            float* Y, int64_t ldy, int64_t M, int K, int N, float* work, cudaStream_t st);
 // tcgen05 engine GEMMs (tc_engine.cu)
 cudaError_t launch_tc_gemm_xw(const float* X, int64_t ldx, const float* wThi, const float* wTlo, int64_t ldwT,
-                              const float* rs, float* Y, int64_t ldy, int64_t M, int K, int N, cudaStream_t s);
-int64_t tc_xtg_slices(int64_t M);
+                              const float* rs, float* Y, int64_t ldy, int64_t M, int K, int N, cudaStream_t s,
+                              const uint32_t* mask = nullptr, int64_t mask_ld = 0);
+int64_t tc_xtg_slices(int64_t M, int K);
 cudaError_t launch_tc_gemm_xtg(const float* X, int64_t ldx, const float* dThi, const float* dTlo, int64_t lddT,
                                float* partial, int64_t M, int K, int N, cudaStream_t s);
 int64_t gemm_xtg_work_floats(int64_t M, int K, int N);
 cudaError_t launch_gemm_xtg(const float* X, int64_t ldx, const float* D, int64_t ldd, float* G,
                             int64_t M, int K, int N, float* work, cudaStream_t st);
+int64_t gemm_dwt_work_floats(int K, int N);
 cudaError_t launch_gemm_dwt(const float* D, int64_t ldd, const float* W, const uint32_t* mask,
                             const float* s, float* O, int64_t ldo, int64_t M, int N, int K,
-                            cudaStream_t st);
+                            float* work, cudaStream_t st);
 
 // ---- loss / optimiser (loss_opt.cu) ----
 cudaError_t launch_softmax_ce(const float* L, int64_t ld, const int32_t* labels,

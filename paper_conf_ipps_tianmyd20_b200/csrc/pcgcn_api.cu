@@ -408,14 +408,16 @@ pcgcn_status pcgcn_gemm_xtg(const float* X, int64_t ldx, const float* D, int64_t
   return e == cudaSuccess ? PCGCN_OK : cuda_fail(e, "gemm_xtg");
 }
 
+int64_t pcgcn_gemm_dwt_work_floats(int32_t K, int32_t N) { return gemm_dwt_work_floats(K, N); }
+
 pcgcn_status pcgcn_gemm_dwt(const float* D, int64_t ldd, const float* W, const uint32_t* mask,
                             const float* s, float* O, int64_t ldo, int64_t M, int32_t N, int32_t K,
-                            void* stream) {
+                            float* work, void* stream) {
   if (!D || !W || !O || M < 0 || K < 1 || N < 1 || ldd < N || ldo < K) {
     set_error("gemm_dwt: bad arguments");
     return PCGCN_EINVAL;
   }
-  cudaError_t e = launch_gemm_dwt(D, ldd, W, mask, s, O, ldo, M, N, K, static_cast<cudaStream_t>(stream));
+  cudaError_t e = launch_gemm_dwt(D, ldd, W, mask, s, O, ldo, M, N, K, work, static_cast<cudaStream_t>(stream));
   return e == cudaSuccess ? PCGCN_OK : cuda_fail(e, "gemm_dwt");
 }
 

@@ -50,6 +50,19 @@ __device__ __forceinline__ const char* row_addr(const char* base, uint32_t j, ui
   asm("mad.wide.u32 %0, %1, %2, %3;" : "=l"(r) : "r"(j), "r"(stride), "l"(reinterpret_cast<uint64_t>(base)));
   return reinterpret_cast<const char*>(r);
 }
+// index stream: read once per pass -> L2 evict_first so it does not push
+// Y' rows out of the L2 (tuning flag AggArgs::idx_evict_first)
+__device__ __forceinline__ int ld_idx(const int* p, bool ef, uint64_t pol) {
+  if (!ef) return __ldg(p);
+  int v;
+  asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
+  return v;
+}
+__device__ __forceinline__ uint64_t policy_evict_first() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
 __device__ __forceinline__ void add4(float4& a, const float4& b) {
   a.x += b.x; a.y += b.y; a.z += b.z; a.w += b.w;
 }
@@ -80,7 +93,8 @@ struct Lay {
 // then a butterfly over the slots — bitwise reproducible.
 template <int G, int V>
 __device__ __forceinline__ void gather_sum(const int* __restrict__ cp, int n, const char* __restrict__ yb,
-                                           uint32_t rstride, const bool (&lok)[V], int lane, float4 (&tot)[V]) {
+                                           uint32_t rstride, const bool (&lok)[V], int lane, float4 (&tot)[V],
+                                           bool ef, uint64_t pol) {
   using L = Lay<G, V>;
   constexpr int S = L::S, STEPS = L::STEPS, UNR = L::UNR, NACC = L::NACC;
   const int slot = lane / G;
@@ -89,11 +103,11 @@ __device__ __forceinline__ void gather_sum(const int* __restrict__ cp, int n, co
   for (int u = 0; u < NACC; ++u)
 #pragma unroll
     for (int v = 0; v < V; ++v) acc[u][v] = make_float4(0.f, 0.f, 0.f, 0.f);
-  int nextidx = lane < n ? __ldg(cp + lane) : 0;
+  int nextidx = lane < n ? ld_idx(cp + lane, ef, pol) : 0;
   for (int base = 0; base < n; base += 32) {
     const int cnt = (n - base) < 32 ? n - base : 32;
     const int myidx = nextidx;
-    nextidx = (base + 32 + lane < n) ? __ldg(cp + base + 32 + lane) : 0;  // next batch, one ahead
+    nextidx = (base + 32 + lane < n) ? ld_idx(cp + base + 32 + lane, ef, pol) : 0;  // next batch, one ahead
     if (cnt == 32) {
       // full batch: unguarded, every lane keeps UNR*V 16-byte loads in flight
 #pragma unroll
@@ -172,7 +186,8 @@ __global__ void __launch_bounds__(256, 4) sparse_seg_kernel(AggArgs a) {
 #pragma unroll
   for (int v = 0; v < V; ++v) lok[v] = lane_col<G>(lane, v, nvec) >= 0;
   float4 tot[V];
-  gather_sum<G, V>(a.col + lo, int(hi - lo), yb, uint32_t(a.ldy * 4), lok, lane, tot);
+  gather_sum<G, V>(a.col + lo, int(hi - lo), yb, uint32_t(a.ldy * 4), lok, lane, tot, a.idx_evict_first,
+                   policy_evict_first());
   if (lane < G) {
 #pragma unroll
     for (int v = 0; v < V; ++v) {
@@ -201,6 +216,7 @@ __global__ void __launch_bounds__(256, 4) sparse_row_kernel(AggArgs a) {
   }
   const char* yb = reinterpret_cast<const char*>(a.Y) + 16 * (qv[0] < 0 ? 0 : qv[0]);
   const uint32_t rstride = uint32_t(a.ldy * 4);
+  const uint64_t pol = policy_evict_first();
   auto claim = [&]() {
     int t = 0;
     if (lane == 0) t = atomicAdd(a.counter, 1);
@@ -224,7 +240,7 @@ __global__ void __launch_bounds__(256, 4) sparse_row_kernel(AggArgs a) {
                                               a.seg_ws + int64_t(sg + k) * a.ldws + 4 * qv[v])));
       }
     } else {
-      gather_sum<G, V>(a.col + e0, int(e1 - e0), yb, rstride, lok, lane, tot);
+      gather_sum<G, V>(a.col + e0, int(e1 - e0), yb, rstride, lok, lane, tot, a.idx_evict_first, pol);
     }
     const float ri = a.r[a.row_lo + row];
     const int zi = HAS_ZD ? a.zd_index[row] : -1;
@@ -350,8 +366,41 @@ __global__ void __launch_bounds__(256) split_transpose_kernel(const float* __res
 
 }  // namespace
 
-cudaError_t launch_sparse_agg(const AggArgs& a, cudaStream_t s) {
-  if (a.rows <= 0) return cudaSuccess;
+cudaError_t launch_sparse_pass(const AggArgs& a, cudaStream_t s);
+
+// Tuning knobs read once (benchmarks only): PCGCN_SPARSE_FSPLIT=<cols> runs
+// the gather in column slices of that width (each slice of Y' is a smaller
+// L2 working set; the index stream is re-read per slice), and
+// PCGCN_IDX_EF=0/1 the L2 evict_first hint on the index stream.
+struct SparseKnobs {
+  int fsplit = 0;
+  bool idx_ef = false;
+  SparseKnobs() {
+    if (const char* e = getenv("PCGCN_SPARSE_FSPLIT")) fsplit = atoi(e) / 32 * 32;
+    if (const char* e = getenv("PCGCN_IDX_EF")) idx_ef = atoi(e) != 0;
+  }
+};
+
+cudaError_t launch_sparse_agg(const AggArgs& a0, cudaStream_t s) {
+  if (a0.rows <= 0) return cudaSuccess;
+  static SparseKnobs knobs;
+  AggArgs a = a0;
+  a.idx_evict_first = knobs.idx_ef;
+  if (knobs.fsplit <= 0 || a.F <= knobs.fsplit) return launch_sparse_pass(a, s);
+  for (int c0 = 0; c0 < a.F; c0 += knobs.fsplit) {
+    AggArgs b = a;
+    b.F = (a.F - c0) < knobs.fsplit ? a.F - c0 : knobs.fsplit;
+    b.Y = a.Y + c0;
+    b.Z = a.Z + c0;
+    if (a.zd) b.zd = a.zd + c0;
+    if (a.mask) b.mask = a.mask + c0 / 32;
+    cudaError_t e = launch_sparse_pass(b, s);
+    if (e != cudaSuccess) return e;
+  }
+  return cudaSuccess;
+}
+
+cudaError_t launch_sparse_pass(const AggArgs& a, cudaStream_t s) {
   // G lanes x V float4 per edge slot: the narrowest power-of-two slot that
   // covers the row, so one load instruction reads whole rows (fewest lines)
   const int nvec = (a.F + 3) / 4;

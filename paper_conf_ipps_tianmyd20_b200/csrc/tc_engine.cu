@@ -112,6 +112,8 @@ struct Work {
   int64_t ldo;
   int ncols;         // columns written per output row (<= npad, multiple of 4)
   const float* rowscale;
+  const uint32_t* mask;  // A_ROWMAJOR: output column c of row r kept iff bit c of mask[r*mask_ld + c/32]
+  int64_t mask_ld;
   int64_t split_stride;
   int b_fused;       // B lo rows follow the hi rows in memory: one TMA box {32, 2*npad} per chunk
 };
@@ -382,16 +384,19 @@ __global__ void __launch_bounds__(NTHREADS, 1)
         mbar_arrive(&acc_empty[ab]);
       }
       if (live) {
+        const uint32_t* mrow = (MODE == A_ROWMAJOR && w.mask) ? w.mask + row * w.mask_ld : nullptr;
+        auto mk = [&](int c) { return mrow ? ((mrow[c >> 5] >> (c & 31)) & 1u ? sc : 0.f) : sc; };
         if (NPC > 0) {
 #pragma unroll
           for (int c0 = 0; c0 < (NPC > 0 ? NPC : 1); c0 += 4)
             if (c0 < w.ncols)
               *reinterpret_cast<float4*>(out + c0) =
-                  make_float4(racc[c0] * sc, racc[c0 + 1] * sc, racc[c0 + 2] * sc, racc[c0 + 3] * sc);
+                  make_float4(racc[c0] * mk(c0), racc[c0 + 1] * mk(c0 + 1), racc[c0 + 2] * mk(c0 + 2),
+                              racc[c0 + 3] * mk(c0 + 3));
         } else {
           for (int c0 = 0; c0 < w.ncols; c0 += 4) {
             float4 v = ngrp > 0 ? *reinterpret_cast<const float4*>(out + c0) : make_float4(0.f, 0.f, 0.f, 0.f);
-            v.x *= sc; v.y *= sc; v.z *= sc; v.w *= sc;
+            v.x *= mk(c0); v.y *= mk(c0 + 1); v.z *= mk(c0 + 2); v.w *= mk(c0 + 3);
             *reinterpret_cast<float4*>(out + c0) = v;
           }
         }
@@ -532,7 +537,8 @@ cudaError_t launch_dense_tc(const DenseArgs& a, cudaStream_t s) {
 
 // ---- Y = diag(s)·X·W, W pre-split feature-major (wT hi/lo [npad][ldwT]) ----
 cudaError_t launch_tc_gemm_xw(const float* X, int64_t ldx, const float* wThi, const float* wTlo, int64_t ldwT,
-                              const float* rs, float* Y, int64_t ldy, int64_t M, int K, int N, cudaStream_t s) {
+                              const float* rs, float* Y, int64_t ldy, int64_t M, int K, int N, cudaStream_t s,
+                              const uint32_t* mask, int64_t mask_ld) {
   const int npad = (N + 15) / 16 * 16;
   if (ldx % 4 || ldwT % 4 || ldy % 4 || npad > 256) return cudaErrorInvalidValue;
   CUtensorMap mh, ml, ma;
@@ -548,13 +554,22 @@ cudaError_t launch_tc_gemm_xw(const float* X, int64_t ldx, const float* wThi, co
   w.ldo = ldy;
   w.ncols = int(ldy < npad ? ldy : npad);
   w.rowscale = rs;
+  w.mask = mask;
+  w.mask_ld = mask_ld;
   return launch_engine<A_ROWMAJOR>(mh, ml, ma, w, npad, s);
 }
 
 // ---- partial[sp] = X[rows of slice sp]ᵀ · D, D pre-split feature-major ----
-int64_t tc_xtg_slices(int64_t M) {
-  int64_t sl = (M + 8191) / 8192;
-  return sl < 1 ? 1 : (sl > 64 ? 64 : sl);
+int64_t tc_xtg_slices(int64_t M, int K) {
+  // split-K over rows so that (output row tiles) x (slices) fills the 148
+  // SMs of a B200 once (a constant, not the queried SM count: the slicing
+  // fixes the summation order, which must not depend on the device), with
+  // >= 1024 rows per slice
+  const int64_t mt = (K + BM - 1) / BM;
+  int64_t sl = (148 + mt - 1) / mt;
+  const int64_t cap = (M + 1023) / 1024;
+  sl = sl < cap ? sl : cap;
+  return sl < 1 ? 1 : (sl > 148 ? 148 : sl);
 }
 cudaError_t launch_tc_gemm_xtg(const float* X, int64_t ldx, const float* dThi, const float* dTlo, int64_t lddT,
                                float* partial, int64_t M, int K, int N, cudaStream_t s) {
@@ -564,7 +579,7 @@ cudaError_t launch_tc_gemm_xtg(const float* X, int64_t ldx, const float* dThi, c
   int fused = 0;
   if (!make_b_maps(dThi, dTlo, M, lddT, npad, &mh, &ml, &fused) || !make_map(&ma, X, K, M, ldx, BM, BK, false))
     return cudaErrorInvalidValue;
-  const int64_t ns = tc_xtg_slices(M);
+  const int64_t ns = tc_xtg_slices(M, K);
   Work w{};
   w.mtiles = (K + BM - 1) / BM;
   w.ntiles = int64_t(w.mtiles) * ns;

@@ -92,7 +92,7 @@ class GCN2:
         self.ce_work = torch.zeros(L.CE_WORK_FLOATS, dtype=f32, device=d)
         wk = max(L.gemm_xtg_work_floats(rows, self.f_in, H), L.gemm_xtg_work_floats(rows, H, C))
         self.xtg_work = torch.zeros(max(wk, 1), dtype=f32, device=d)
-        wk = max(L.gemm_xw_work_floats(self.f_in, H), L.gemm_xw_work_floats(H, C))
+        wk = max(L.gemm_xw_work_floats(self.f_in, H), L.gemm_xw_work_floats(H, C), L.gemm_dwt_work_floats(H, C))
         self.xw_work = torch.zeros(wk, dtype=f32, device=d)
         self.r = plan.rowscale_ptr()  # device [n]
         self.r_local = None if self.lo == 0 else self.r + 4 * self.lo
@@ -144,7 +144,7 @@ class GCN2:
         mark("a10_agg_bwd_C")
         L.gemm_xtg(self.H1, self.G1, self.gTh1, self.xtg_work, M=self.rows, K=H, N=C, stream=stream)
         L.gemm_dwt(self.G1, self.Th1, self.mask1, rr, self._local(self.dP1), M=self.rows, N=C, K=H,
-                   stream=stream)
+                   work=self.xw_work, stream=stream)
         mark("a11_gemm_xtg1_dwt")
         self._gather(self.dP1)
         mark("x_gather_dp1")
@@ -170,7 +170,7 @@ class GCN2:
         # split + dense tiles (full mode), segment pass (long rows), selective rows
         agg = 1 + (2 if dense else 0) + (1 if st["shard_segments"] > 0 else 0)
         gemm_xw = 1 + 1                          # tile kernel + pad zeroing (ld > N) — upper bound
-        n = 2 * gemm_xw + 4 * agg + 2 + 2 * 2 + 2  # + softmax(2) + 2 x xtg(2) + dwt(2)
+        n = 2 * gemm_xw + 4 * agg + 2 + 2 * 3 + 3  # + softmax(2) + 2 x xtg(split, engine, reduce) + dwt(split, engine, pad)
         n += 2 if self.optimizer == "adam" else 1
         return n
 

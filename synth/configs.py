@@ -5,6 +5,8 @@ Input infrastructure only.  Sizes follow the paper's counting convention
   C1 Cora-shaped   n=2,708   m=5,278       1433 -> 16 -> 7    P=8
   C2 Pubmed-shaped n=19,717  m=44,324      500  -> 16 -> 3    P=32  (nnz 108,365 = Table I)
   C3 Reddit-shaped n=232,965 m=57,307,946  602  -> 128 -> 41  P=128
+  C4 SBM-4M        n=4,194,304 m=~398M     128  -> 128 -> 32  P=2048
+  C5 PL-32M        n=33,554,432 m=500M     128  -> 128 -> 32  P=16384
 """
 from __future__ import annotations
 
@@ -13,7 +15,7 @@ from dataclasses import dataclass
 import numpy as np
 
 from . import rng as R
-from .graphs import Graph, SBMSpec, sbm
+from .graphs import Graph, RMATSpec, SBMSpec, rmat, sbm
 
 
 @dataclass
@@ -64,7 +66,33 @@ SBM4M = Workload(
                      class_weight=[t / 8.0 for t in _C4_TIERS]),
     f_in=128, hidden=128, classes=32, P=2048, feat_kind="normal", feat_seed=4002, theta_seed=4003)
 
-WORKLOADS = {w.name: w for w in (CORA, PUBMED, REDDIT, SBM4M)}
+# C5: clustered power-law graph (BASELINE configs[4]): a degree-corrected SBM
+# with 4,096 communities of 8,192 vertices, 90% of edge draws inside the
+# community, Pareto(2.2) propensities (degree tail exponent ~2.2) capped at
+# 16,000x the minimum, 500M undirected edges -> nnz(A+I) = 1.034 B, average
+# degree ~30.  Hubs saturate their community (duplicate
+# draws collapse), so the largest degrees are ~10^4, not the 10^5 cap.
+PL32M = Workload(
+    "pl32m", SBMSpec([8_192] * 4_096, sub_size=0, p_sub=0.0, p_class=0.9, m_target=500_000_000,
+                     alpha=2.2, cap=16_000.0, seed=5001),
+    f_in=128, hidden=128, classes=32, P=16384, feat_kind="normal", feat_seed=5002, theta_seed=5003)
+
+# RMAT-{0.1,0.5,1,5,10}: the paper's synthetic density series (L251, Table I
+# L223-L227: 10,240 vertices, density = m / n^2, 128 features, 32 labels),
+# regenerated for the Table III (L263-L281) sel / full / hybrid replica.  The
+# model is this repo's 2-layer GCN with the paper's hid = 64 (L255).
+RMAT = {d: Workload(f"rmat-{d:g}", RMATSpec(10_240, int(round(d / 100 * 10_240 ** 2)), seed=6001 + i),
+                    f_in=128, hidden=64, classes=32, P=16, feat_kind="normal", feat_seed=6101 + i,
+                    theta_seed=6201 + i)
+        for i, d in enumerate((0.1, 0.5, 1.0, 5.0, 10.0))}
+
+WORKLOADS = {w.name: w for w in (CORA, PUBMED, REDDIT, SBM4M, PL32M, *RMAT.values())}
+
+
+def labels(w: Workload, g: Graph) -> np.ndarray:
+    """Vertex labels in [0, classes): the planted community modulo the class
+    count (C4 / C5 have more communities than classes)."""
+    return (g.labels % w.classes).astype(np.int32)
 
 
 def scaled(w: Workload, frac: float, name: str | None = None) -> Workload:
@@ -78,6 +106,8 @@ def scaled(w: Workload, frac: float, name: str | None = None) -> Workload:
 
 
 def graph(w: Workload, impl: str = "auto") -> Graph:
+    if isinstance(w.spec, RMATSpec):
+        return rmat(w.spec)
     return sbm(w.spec, impl=impl)
 
 

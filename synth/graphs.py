@@ -209,6 +209,69 @@ def _sbm_c(st, spec: SBMSpec):
     return rowptr, col
 
 
+@dataclass
+class RMATSpec:
+    """R-MAT graph (Chakrabarti et al. 2004; the paper's synthetic family,
+    PAPER.md L251, Table I): n vertices, ``m_target`` distinct
+    undirected edges (density = m_target / n^2), quadrant probabilities
+    (a, b, c, d = 1-a-b-c) over ceil(log2 n) levels; pairs with an endpoint
+    >= n and self-pairs are redrawn, duplicates collapse; ids shuffled."""
+
+    n: int
+    m_target: int
+    a: float = 0.45
+    b: float = 0.22
+    c: float = 0.22
+    seed: int = 0
+
+
+def _rmat_keys(spec: RMATSpec, c0: int, c1: int) -> np.ndarray:
+    n = spec.n
+    levels = max(1, int(np.ceil(np.log2(n))))
+    key = R.stream_key(spec.seed, 17)
+    ctr = np.arange(c0, c1, dtype=np.uint64)
+    u = np.zeros(len(ctr), dtype=np.int64)
+    v = np.zeros(len(ctr), dtype=np.int64)
+    ab, abc = spec.a + spec.b, spec.a + spec.b + spec.c
+    for lvl in range(levels):
+        x = R.to_unit(R.draws(key, ctr * np.uint64(levels) + np.uint64(lvl)))
+        ubit = (x >= ab).astype(np.int64)                       # quadrants c, d: lower half
+        vbit = (((x >= spec.a) & (x < ab)) | (x >= abc)).astype(np.int64)  # quadrants b, d: right half
+        u = (u << 1) | ubit
+        v = (v << 1) | vbit
+    ok = (u < n) & (v < n) & (u != v)
+    perm = np.random.default_rng([spec.seed, 2]).permutation(n).astype(np.int64)
+    a_, b_ = perm[u[ok]], perm[v[ok]]
+    return (np.minimum(a_, b_).astype(np.uint64) * np.uint64(n) + np.maximum(a_, b_).astype(np.uint64))
+
+
+def rmat(spec: RMATSpec) -> Graph:
+    """R-MAT graph with exactly m_target undirected edges (seeded subset of
+    the surplus dropped, as in sbm()).  Labels: 32 classes by the vertex's
+    position in generation order (its leading quadrant path, R-MAT's
+    recursive communities)."""
+    n = spec.n
+    if spec.m_target > n * (n - 1) // 2:
+        raise ValueError("m_target exceeds the number of vertex pairs")
+    # counters are consumed in order, batch after batch: the edge set after c
+    # counters does not depend on the batch sizes
+    seen = np.zeros(n * n, dtype=bool)  # pair bitmap (n = 10,240: 105 MB)
+    have, c = 0, 0
+    while have < spec.m_target:
+        step = max(1 << 20, min(1 << 24, 2 * (spec.m_target - have)))
+        seen[_rmat_keys(spec, c, c + step)] = True
+        have = int(np.count_nonzero(seen))
+        c += step
+    keys = _drop_surplus(np.flatnonzero(seen).astype(np.uint64), spec.m_target, spec.seed)
+    rowptr, col = _keys_to_csr(n, keys)
+    perm = np.random.default_rng([spec.seed, 2]).permutation(n).astype(np.int64)
+    levels = max(1, int(np.ceil(np.log2(n))))
+    labels = np.empty(n, dtype=np.int32)
+    labels[perm] = (np.arange(n, dtype=np.int64) * 32 // n).astype(np.int32)
+    return Graph(n=n, rowptr=rowptr, col=col, labels=labels,
+                 meta=dict(kind="rmat", m_undirected=spec.m_target, seed=spec.seed))
+
+
 # ---------------------------------------------------------------------------
 # Tiny hand-made graphs (test fixtures; closed forms live in the tests)
 # ---------------------------------------------------------------------------

@@ -245,12 +245,19 @@ def test_gemms(M, K, N, path):
     mbits = rng.integers(0, 2**32, size=(M, mw), dtype=np.uint64).astype(np.uint32)
     mask = torch.from_numpy(mbits.view(np.int32)).cuda()
     O_ = torch.full((M, _ld(K2)), float("nan"), device="cuda")
-    L.gemm_dwt(D, W2, mask, ctypes.c_void_p(s.data_ptr()), O_)
+    if path == "tcgen05":   # 16-byte rows + workspace: the engine path (K2 <= 256), else fp32 cores
+        Dp = torch.zeros(M, _ld(N), device="cuda")
+        Dp[:, :N] = D
+        L.gemm_dwt(Dp, W2, mask, ctypes.c_void_p(s.data_ptr()), O_, M=M, N=N, K=K2,
+                   work=torch.zeros(L.gemm_dwt_work_floats(K2, N), device="cuda"))
+    else:
+        L.gemm_dwt(D, W2, mask, ctypes.c_void_p(s.data_ptr()), O_)
     torch.cuda.synchronize()
     mk = ((mbits[:, :, None] >> np.arange(32, dtype=np.uint32)) & 1).reshape(M, mw * 32)[:, :K2]
     exp = _np(s)[:, None] * ((_np(D) @ _np(W2).T) * mk)
     scale = _np(s)[:, None] * (np.abs(_np(D)) @ np.abs(_np(W2)).T) + 1e-30
     assert np.max(np.abs(_np(O_)[:, :K2] - exp) / scale) < TOL
+    assert np.all(_np(O_)[:, K2:] == 0)
 
 
 def test_softmax_ce_and_adam():

@@ -139,6 +139,25 @@ def test_aggregate_rows_matches_full():
                                O.aggregate(_ahat(g, "none"), Y)[rows], rtol=1e-13)
 
 
+@pytest.mark.parametrize("seed", [1, 2, 3])
+def test_clean_degrees_matches_binary_adjacency(seed):
+    """clean_degrees (row-chunked, with the clean-row shortcut) equals the row
+    sums of the binary A built by scipy's duplicate collapsing, on messy input
+    (duplicates, self-loops, unsorted rows) with trailing empty rows, and on a
+    clean sorted CSR."""
+    g = G.messy_random(60, 200, seed)
+    n = g.n + 5                                       # 5 isolated trailing vertices
+    rowptr = np.concatenate([g.rowptr, np.full(5, g.rowptr[-1])])
+    rng = np.random.default_rng(seed)
+    col = g.col.copy()
+    for i in range(g.n):                              # shuffle inside rows
+        rng.shuffle(col[rowptr[i]:rowptr[i + 1]])
+    A = O.binary_adjacency(n, rowptr, col)
+    np.testing.assert_array_equal(O.clean_degrees(n, rowptr, col), np.asarray(A.sum(axis=1)).ravel())
+    c = G.cycle(40)
+    np.testing.assert_array_equal(O.clean_degrees(c.n, c.rowptr, c.col), np.full(40, 2))
+
+
 def _tiny_problem(seed=13, n=30, f=7, h=5, c=4):
     g = G.random_graph(n, 0.15, seed)
     rng = np.random.default_rng(seed)
