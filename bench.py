@@ -48,6 +48,10 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--eager", action="store_true", help="no CUDA graph")
     ap.add_argument("--sweep", default="", help="comma list of θ: per-θ aggregation times (Table III replica)")
+    ap.add_argument("--f2", default="",
+                    help="F2 sensitivity: 'L1,L2,..:H1,H2,..' epoch ms of the l-layer GCN over layers x hidden")
+    ap.add_argument("--f3", type=int, default=0,
+                    help="F3 convergence study (§V-E): epochs of Adam training, fp32 vs bf16 full mode")
     ap.add_argument("--table3", action="store_true",
                     help="Table III replica on RMAT-{0.1..10}: epoch ms of PCGCN-sel / -full / hybrid")
     return ap.parse_args()
@@ -308,6 +312,103 @@ def run_table3(args):
                       "paper": "Table III L263-L281 (l=4, hid=64, 1080Ti/2080Ti) — context"}), flush=True)
 
 
+def run_f3(args):
+    """SURVEY F3 / PAPER.md §V-E (L330-L334, Fig. 9): per-epoch test accuracy
+    of the same 2-layer GCN trained with the exact fp32 selective mode
+    (θ = 2), the fp32-accurate hybrid (tf32 hi/lo full mode) and the bf16
+    full mode (PCGCN_DENSE_BF16X1, hybrid θ and every block full), on the
+    workload's graph with an 80/20 train/test split.  The synthetic features
+    carry a weak class signal here (class mean vectors, 0.5 x N(0,1)) so
+    that the task is learnable; same seed and init for every variant."""
+    import torch
+    from paper_conf_ipps_tianmyd20_b200 import _lib as L
+    from paper_conf_ipps_tianmyd20_b200.gcn import GCN2
+    dev = torch.device("cuda", 0)
+    torch.cuda.set_device(dev)
+    w, g, X, Th0, Th1, labels, T = load_workload(args.workload)
+    mu = np.random.default_rng([w.feat_seed, 99]).standard_normal((w.classes, w.f_in)).astype(np.float32) * 0.5
+    X = (X + mu[labels]).astype(np.float32)
+    theta_h = float(args.theta) if args.theta != "auto" else 0.05
+    variants = [("fp32_selective", 2.0, L.DENSE_TF32X2), ("tf32x2_hybrid", theta_h, L.DENSE_TF32X2),
+                ("bf16_hybrid", theta_h, L.DENSE_BF16X1), ("bf16_full", 0.0, L.DENSE_BF16X1)]
+    curves = {}
+    for name, th, prec in variants:
+        pl = L.Plan(g.n, g.rowptr, g.col, args.P or w.P, th, dense_prec=prec, f_max=max(w.hidden, w.classes))
+        perm = pl.perm()
+        lab = labels[perm]
+        test = torch.from_numpy(~T[perm]).to(dev)
+        labd = torch.from_numpy(lab.astype(np.int64)).to(dev)
+        m = GCN2(pl, np.ascontiguousarray(X[perm]), lab, T[perm], Th0, Th1, optimizer="adam", lr=0.01, device=dev)
+        acc, losses = [], []
+        for ep in range(args.f3):
+            m.epoch()
+            if ep % 10 == 9 or ep == args.f3 - 1:
+                pred = m.Lg[:, :w.classes].argmax(dim=1)   # logits of the forward just run
+                acc.append(float((pred[test] == labd[test]).float().mean().item()))
+                losses.append(float(m.loss.item()))
+        st = pl.stats()
+        curves[name] = {"theta": th, "dense_edge_frac": st["nnz_dense"] / st["nnz"], "test_acc_every10": acc,
+                        "loss_every10": losses, "final_test_acc": acc[-1]}
+        log(f"[f3] {name}: {curves[name]['final_test_acc']:.4f} dense={curves[name]['dense_edge_frac']:.3f}")
+        del m
+        pl.destroy()
+    base = curves["fp32_selective"]["final_test_acc"]
+    for k in curves:
+        curves[k]["acc_delta_vs_fp32"] = curves[k]["final_test_acc"] - base
+    print(json.dumps({"f3": curves, "workload": w.name, "epochs": args.f3, "optimizer": "adam lr 0.01",
+                      "paper": "§V-E: PCGCN-TC accuracy drop 0.08% (pubmed), 0.19% (reddit-s) — context"}), flush=True)
+
+
+def run_f2(args):
+    """the paper-shaped l-layer model (Table II: l = 4, hid = 64,
+    L255) and its sensitivity to the hidden size and depth (L314, L326: the
+    runtime grows ~linearly in both) on one workload; one plan (θ fixed or
+    the L161 calibration at the first hidden size), CUDA-graph replays."""
+    import torch
+    from paper_conf_ipps_tianmyd20_b200 import _lib as L
+    from paper_conf_ipps_tianmyd20_b200.gcn import GCNL
+    from synth import configs as C
+    dev = torch.device("cuda", 0)
+    torch.cuda.set_device(dev)
+    w, g, X, Th0, Th1, labels, T = load_workload(args.workload)
+    layers_s, hid_s = args.f2.split(":")
+    layers = [int(x) for x in layers_s.split(",")]
+    hids = [int(x) for x in hid_s.split(",")]
+    P = args.P or w.P
+    if args.theta == "auto":
+        theta, _, _ = L.calibrate(hids[0], max(64, min(8192, g.n // P)), 0.05)
+    else:
+        theta = float(args.theta)
+    pl = L.Plan(g.n, g.rowptr, g.col, P, theta, f_max=max(max(hids), w.classes))
+    perm = pl.perm()
+    Xp = np.ascontiguousarray(X[perm])
+    out = []
+    for nl in layers:
+        for h in hids:
+            dims = [w.f_in] + [h] * (nl - 1) + [w.classes]
+            ths = [C.glorot(dims[i], dims[i + 1], w.theta_seed, 20 + i) for i in range(nl)]
+            m = GCNL(pl, Xp, labels[perm], T[perm], ths, optimizer="adam", lr=0.01, device=dev)
+            m.capture(warmup=1)
+            for _ in range(max(3, args.warmup)):
+                m.replay()
+            ts = []
+            for _ in range(args.steps):
+                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                a.record()
+                m.replay()
+                b.record()
+                torch.cuda.synchronize(dev)
+                ts.append(a.elapsed_time(b))
+            ent = {"layers": nl, "hidden": h, "epoch_ms": float(np.median(ts))}
+            log(f"[f2] {ent}")
+            out.append(ent)
+            del m
+            torch.cuda.empty_cache()
+    print(json.dumps({"f2": out, "workload": w.name, "n": g.n, "nnz": int(g.nnz + g.n), "P": P, "theta": theta,
+                      "metric": "l-layer GCN epoch ms", "unit": "ms", "steps": args.steps,
+                      "paper": "Table II model l=4 hid=64 (L255); sensitivity L314/L326 — context"}), flush=True)
+
+
 # ---------------------------------------------------------------------------
 # our arm
 # ---------------------------------------------------------------------------
@@ -328,6 +429,12 @@ def main():
         return
     if args.table3:
         run_table3(args)
+        return
+    if args.f2:
+        run_f2(args)
+        return
+    if args.f3:
+        run_f3(args)
         return
 
     from paper_conf_ipps_tianmyd20_b200 import _lib as L

@@ -69,7 +69,10 @@ typedef struct {
 enum { PCGCN_NORM_SYM = 0, PCGCN_NORM_NONE = 1 };     /* Â = D̃^-½ÃD̃^-½  |  Â = Ã (integer pin) */
 enum {
   PCGCN_DENSE_TF32X2 = 0,    /* full mode on tcgen05 (kind::tf32): A∈{0,1} exact, Y = hi + lo, 2 MMAs */
-  PCGCN_DENSE_FP32_SIMT = 1  /* full mode on CUDA cores in fp32 (the paper's §IV-C kernel, L183-L187) */
+  PCGCN_DENSE_FP32_SIMT = 1, /* full mode on CUDA cores in fp32 (the paper's §IV-C kernel, L183-L187) */
+  PCGCN_DENSE_BF16X1 = 2     /* full mode on tcgen05 with the input rounded to bf16 (RN-even), one MMA per
+                                K-step, fp32 accumulation: the paper's 16-bit tensor-core policy (L191-L193,
+                                §V-E); error <= 2^-9 per term, gate 2e-2 (BASELINE.json north_star) */
 };
 
 typedef struct {

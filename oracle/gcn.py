@@ -176,6 +176,51 @@ def epoch(Ahat, X, Th0, Th1, labels, train):
     return dict(P1=P1, H1=H1, L=L, loss=loss, dL=dL, **g)
 
 
+# ---------------------------------------------------------------------------
+# ℓ-layer GCN (Alg. 1 with general ℓ; the paper's Table II model has ℓ = 4,
+# hid = 64, L255) — SURVEY.md §8(f) F2
+# ---------------------------------------------------------------------------
+
+def forward_l(Ahat, X, Ths):
+    """Alg. 1 (L101-L125) for ℓ = len(Ths) layers: a^l = h^{l-1} Θ_l (L114),
+    P_l = Â a^l (L118-L121), h^l = ReLU(P_l) between layers (reading #14),
+    logits = P_ℓ.  Returns (Ps, Hs) with Hs[l] the INPUT of layer l (Hs[0] = X)."""
+    H = np.asarray(X, dtype=np.float64)
+    Ps, Hs = [], [H]
+    for l, Th in enumerate(Ths):
+        P = aggregate(Ahat, H @ np.asarray(Th, dtype=np.float64))
+        Ps.append(P)
+        if l < len(Ths) - 1:
+            H = np.maximum(P, 0.0)
+            Hs.append(H)
+    return Ps, Hs
+
+
+def backward_l(Ahat, Ths, Ps, Hs, dL):
+    """Chain rule through forward_l: G_ℓ = Â dL; for l = ℓ..1:
+    ∇Θ_l = h^{l-1}ᵀ G_l, and (l > 1) dP_{l-1} = (G_l Θ_lᵀ) ⊙ [P_{l-1} > 0],
+    G_{l-1} = Â dP_{l-1}  (Âᵀ = Â, reading #2)."""
+    AT = Ahat.T.tocsr()
+    G = aggregate(AT, dL)
+    grads = [None] * len(Ths)
+    Gs = [None] * len(Ths)
+    for l in range(len(Ths) - 1, -1, -1):
+        Gs[l] = G
+        grads[l] = Hs[l].T @ G
+        if l > 0:
+            dP = (G @ np.asarray(Ths[l], dtype=np.float64).T) * (Ps[l - 1] > 0)
+            G = aggregate(AT, dP)
+    return grads, Gs
+
+
+def epoch_l(Ahat, X, Ths, labels, train):
+    """One full-batch epoch of the ℓ-layer model."""
+    Ps, Hs = forward_l(Ahat, X, Ths)
+    loss, dL = softmax_ce(Ps[-1], labels, train)
+    grads, Gs = backward_l(Ahat, Ths, Ps, Hs, dL)
+    return dict(Ps=Ps, Hs=Hs, loss=loss, dL=dL, grads=grads, Gs=Gs)
+
+
 def sgd(Th, g, lr):
     return np.asarray(Th, dtype=np.float64) - lr * g
 

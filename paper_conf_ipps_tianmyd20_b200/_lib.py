@@ -25,7 +25,7 @@ c_i32, c_i64, c_f32, c_u32, c_vp = ctypes.c_int32, ctypes.c_int64, ctypes.c_floa
 # status codes
 OK, EINVAL, ENOTSYM, ECUDA, ENOMEM, ENCCL, EUNSUP = range(7)
 NORM_SYM, NORM_NONE = 0, 1
-DENSE_TF32X2, DENSE_FP32_SIMT = 0, 1
+DENSE_TF32X2, DENSE_FP32_SIMT, DENSE_BF16X1 = 0, 1, 2
 IN_PRESCALED, RELU, MASK_OUT, OUT_PRESCALED, PROFILE = 1, 2, 4, 8, 16
 TIMING_NAMES = ("prescale", "split", "dense_tc", "sparse")
 X_NAMES = ["part", "perm", "pstart", "r", "blk_k", "blk_i", "blk_nnz", "blk_dense", "sp_rowptr", "sp_col",

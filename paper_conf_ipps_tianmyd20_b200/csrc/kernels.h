@@ -45,14 +45,14 @@ cudaError_t launch_sparse_agg(const AggArgs& a, cudaStream_t s);
 // ypre = diag(r)·Y
 cudaError_t launch_prescale(const float* Y, int64_t ldy, const float* r, int64_t n, int F, float* ypre,
                             int64_t ldpre, cudaStream_t s);
-// tf32 hi/lo split of Y written feature-major: hiT/loT [npad x ldT]
+// tf32 hi/lo split of Y written feature-major: hiT/loT [npad x ldT]; loT == nullptr: hiT = bf16 RN-even of Y
 cudaError_t launch_split_transpose(const float* Y, int64_t ldy, int64_t n, int F, int npad, float* hiT,
                                    float* loT, int64_t ldT, cudaStream_t s);
 
 // ---- dense-mode tcgen05 tile contraction (dense_tc.cu) ----
 struct DenseArgs {
   const float* hiT;          // [npad x ldT] tf32 hi part of the prescaled input, feature-major
-  const float* loT;          // [npad x ldT] lo part
+  const float* loT;          // [npad x ldT] lo part; nullptr: single product on bf16-rounded hiT (BF16X1)
   int64_t n, ldT;
   const int32_t* rt_row0;    // shard row tiles
   const int32_t* rt_nrows;

@@ -165,7 +165,8 @@ pcgcn_status aggregate(pcgcn_plan_t p, const float* Y, int64_t ldy, float* Z, in
   const int64_t ld4 = round_up(F, 4);
   const float* src = Y;
   int64_t ldsrc = ldy;
-  const bool tc = p->opts.dense_prec == PCGCN_DENSE_TF32X2;
+  const bool bf16 = p->opts.dense_prec == PCGCN_DENSE_BF16X1;
+  const bool tc = p->opts.dense_prec == PCGCN_DENSE_TF32X2 || bf16;
   const bool prof = (flags & PCGCN_PROFILE) != 0;
   auto mark = [&](int k) {
     if (!prof) return;
@@ -185,14 +186,14 @@ pcgcn_status aggregate(pcgcn_plan_t p, const float* Y, int64_t ldy, float* Z, in
   float* ylo = d.yhi ? d.yhi + int64_t(npad) * d.n_pad : nullptr;
   if (dense && tc) {
     if (prof) d.ev_used[1] = true;
-    e = launch_split_transpose(src, ldsrc, p->n, F, npad, d.yhi, ylo, d.n_pad, s);
+    e = launch_split_transpose(src, ldsrc, p->n, F, npad, d.yhi, bf16 ? nullptr : ylo, d.n_pad, s);
     if (e != cudaSuccess) return cuda_fail(e, "split_transpose");
   }
   mark(2);
   if (dense) {
     if (prof) d.ev_used[2] = true;
-    DenseArgs da{d.yhi, ylo, d.n_pad, d.n_pad, d.rt_row0, d.rt_nrows, d.rt_cptr, d.ch_col0, d.bits,
-                 d.nrt, d.zd, npad, npad};
+    DenseArgs da{d.yhi, bf16 ? nullptr : ylo, d.n_pad, d.n_pad, d.rt_row0, d.rt_nrows, d.rt_cptr, d.ch_col0,
+                 d.bits, d.nrt, d.zd, npad, npad};
     e = tc ? launch_dense_tc(da, s) : launch_dense_simt_y(da, src, ldsrc, F, s);
     if (e != cudaSuccess) return cuda_fail(e, "dense-mode kernel");
   }
@@ -258,7 +259,8 @@ pcgcn_status pcgcn_plan(const pcgcn_csr* A, int32_t P, float theta, const pcgcn_
   pcgcn_opts_default(&def);
   if (!o) o = &def;
   if (o->f_max < 1 || o->f_max > 256) { set_error("f_max must be in [1, 256]"); return PCGCN_EINVAL; }
-  if (o->dense_prec != PCGCN_DENSE_TF32X2 && o->dense_prec != PCGCN_DENSE_FP32_SIMT) {
+  if (o->dense_prec != PCGCN_DENSE_TF32X2 && o->dense_prec != PCGCN_DENSE_FP32_SIMT &&
+      o->dense_prec != PCGCN_DENSE_BF16X1) {
     set_error("unknown dense_prec");
     return PCGCN_EUNSUP;
   }

@@ -91,10 +91,15 @@ struct Lay {
 // columns v >= 1 past the row are not loaded: lok[v] false).
 // Fixed order: per slot sequential over its edges in NACC interleaved sums,
 // then a butterfly over the slots — bitwise reproducible.
+// Index batches are loaded one ahead: `first` is this range's first batch
+// (lane l: cp[l] if l < n), and the prefetch slot of the last batch loads the
+// first batch of the NEXT range (cpn, nn), which is returned — so a warp
+// walking rows never waits on a row's first index load.
 template <int G, int V>
-__device__ __forceinline__ void gather_sum(const int* __restrict__ cp, int n, const char* __restrict__ yb,
-                                           uint32_t rstride, const bool (&lok)[V], int lane, float4 (&tot)[V],
-                                           bool ef, uint64_t pol) {
+__device__ __forceinline__ int gather_sum(const int* __restrict__ cp, int n, int first,
+                                          const int* __restrict__ cpn, int nn, const char* __restrict__ yb,
+                                          uint32_t rstride, const bool (&lok)[V], int lane, float4 (&tot)[V],
+                                          bool ef, uint64_t pol) {
   using L = Lay<G, V>;
   constexpr int S = L::S, STEPS = L::STEPS, UNR = L::UNR, NACC = L::NACC;
   const int slot = lane / G;
@@ -103,11 +108,14 @@ __device__ __forceinline__ void gather_sum(const int* __restrict__ cp, int n, co
   for (int u = 0; u < NACC; ++u)
 #pragma unroll
     for (int v = 0; v < V; ++v) acc[u][v] = make_float4(0.f, 0.f, 0.f, 0.f);
-  int nextidx = lane < n ? ld_idx(cp + lane, ef, pol) : 0;
+  int nextidx = first;
+  if (n == 0) nextidx = lane < nn ? ld_idx(cpn + lane, ef, pol) : 0;
   for (int base = 0; base < n; base += 32) {
     const int cnt = (n - base) < 32 ? n - base : 32;
     const int myidx = nextidx;
-    nextidx = (base + 32 + lane < n) ? ld_idx(cp + base + 32 + lane, ef, pol) : 0;  // next batch, one ahead
+    // next batch, one ahead (past the end: the next range's first batch)
+    nextidx = (base + 32 + lane < n) ? ld_idx(cp + base + 32 + lane, ef, pol)
+            : (lane < nn ? ld_idx(cpn + lane, ef, pol) : 0);
     if (cnt == 32) {
       // full batch: unguarded, every lane keeps UNR*V 16-byte loads in flight
 #pragma unroll
@@ -162,6 +170,7 @@ __device__ __forceinline__ void gather_sum(const int* __restrict__ cp, int n, co
       tot[v].w += __shfl_xor_sync(0xffffffffu, tot[v].w, off);
     }
   }
+  return nextidx;
 }
 
 // per-lane byte offset of this lane's first float4 (lanes past the row: 0)
@@ -186,8 +195,11 @@ __global__ void __launch_bounds__(256, 4) sparse_seg_kernel(AggArgs a) {
 #pragma unroll
   for (int v = 0; v < V; ++v) lok[v] = lane_col<G>(lane, v, nvec) >= 0;
   float4 tot[V];
-  gather_sum<G, V>(a.col + lo, int(hi - lo), yb, uint32_t(a.ldy * 4), lok, lane, tot, a.idx_evict_first,
-                   policy_evict_first());
+  const uint64_t pol = policy_evict_first();
+  const int n = int(hi - lo);
+  const int first = lane < n ? ld_idx(a.col + lo + lane, a.idx_evict_first, pol) : 0;
+  gather_sum<G, V>(a.col + lo, n, first, nullptr, 0, yb, uint32_t(a.ldy * 4), lok, lane, tot,
+                   a.idx_evict_first, pol);
   if (lane < G) {
 #pragma unroll
     for (int v = 0; v < V; ++v) {
@@ -222,13 +234,22 @@ __global__ void __launch_bounds__(256, 4) sparse_row_kernel(AggArgs a) {
     if (lane == 0) t = atomicAdd(a.counter, 1);
     return __shfl_sync(0xffffffffu, t, 0);
   };
+  // software pipeline over rows: the next row's ticket, row pointers and
+  // first index batch are in flight while this row gathers
+  const bool ef = a.idx_evict_first;
   int row = claim();
+  int64_t e0 = 0, e1 = 0;
+  if (row < a.rows) { e0 = a.rowptr[row]; e1 = a.rowptr[row + 1]; }
+  int pre = (e0 + lane < e1) ? ld_idx(a.col + e0 + lane, ef, pol) : 0;
   while (row < a.rows) {
     const int nxt = claim();
-    const int64_t e0 = a.rowptr[row], e1 = a.rowptr[row + 1];
+    int64_t n0 = 0, n1 = 0;
+    if (nxt < a.rows) { n0 = a.rowptr[nxt]; n1 = a.rowptr[nxt + 1]; }
     float4 tot[V];
+    int pre_next;
     const int sg = HAS_SEG ? a.row_seg[row] : -1;
     if (HAS_SEG && sg >= 0) {
+      pre_next = (n0 + lane < n1) ? ld_idx(a.col + n0 + lane, ef, pol) : 0;
       const int ns = int((e1 - e0 + SEG_EDGES - 1) / SEG_EDGES);
 #pragma unroll
       for (int v = 0; v < V; ++v) tot[v] = make_float4(0.f, 0.f, 0.f, 0.f);
@@ -240,7 +261,8 @@ __global__ void __launch_bounds__(256, 4) sparse_row_kernel(AggArgs a) {
                                               a.seg_ws + int64_t(sg + k) * a.ldws + 4 * qv[v])));
       }
     } else {
-      gather_sum<G, V>(a.col + e0, int(e1 - e0), yb, rstride, lok, lane, tot, a.idx_evict_first, pol);
+      pre_next = gather_sum<G, V>(a.col + e0, int(e1 - e0), pre, a.col + n0, int(n1 - n0), yb, rstride, lok,
+                                  lane, tot, ef, pol);
     }
     const float ri = a.r[a.row_lo + row];
     const int zi = HAS_ZD ? a.zd_index[row] : -1;
@@ -285,6 +307,9 @@ __global__ void __launch_bounds__(256, 4) sparse_row_kernel(AggArgs a) {
       }
     }
     row = nxt;
+    e0 = n0;
+    e1 = n1;
+    pre = pre_next;
   }
 }
 
@@ -357,9 +382,15 @@ __global__ void __launch_bounds__(256) split_transpose_kernel(const float* __res
     const int64_t j = j0 + tx;
     if (f < npad && j < ldT) {
       const float v = tile[tx][rr];
-      const float h = __uint_as_float(__float_as_uint(v) & 0xffffe000u);
-      hiT[int64_t(f) * ldT + j] = h;
-      loT[int64_t(f) * ldT + j] = v - h;
+      if (loT) {
+        const float h = __uint_as_float(__float_as_uint(v) & 0xffffe000u);
+        hiT[int64_t(f) * ldT + j] = h;
+        loT[int64_t(f) * ldT + j] = v - h;
+      } else {  // bf16 round-to-nearest-even (BF16X1 full mode); exact in tf32
+        uint32_t u = __float_as_uint(v);
+        u = (u + 0x7fffu + ((u >> 16) & 1u)) & 0xffff0000u;
+        hiT[int64_t(f) * ldT + j] = __uint_as_float(u);
+      }
     }
   }
 }

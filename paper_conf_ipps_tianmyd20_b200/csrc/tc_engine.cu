@@ -116,6 +116,7 @@ struct Work {
   int64_t mask_ld;
   int64_t split_stride;
   int b_fused;       // B lo rows follow the hi rows in memory: one TMA box {32, 2*npad} per chunk
+  int single;        // A_BITS: B hi only (bf16-rounded input), one MMA per K-step (PCGCN_DENSE_BF16X1)
 };
 
 template <int MODE>
@@ -193,7 +194,7 @@ __global__ void __launch_bounds__(NTHREADS, 1)
           const int nu = int(nch - i < L.U ? nch - i : L.U);
           mbar_wait(&empty[s], ph ^ 1u);
           uint8_t* st = smem + s * L.stage_bytes;
-          mbar_expect_tx(&full[s], uint32_t(nu) * (L.a_load_bytes + 2u * L.b_bytes));
+          mbar_expect_tx(&full[s], uint32_t(nu) * (L.a_load_bytes + (w.single ? 1u : 2u) * L.b_bytes));
           // the bits of a tile's chunks are contiguous: one bulk copy per stage
           if (MODE == A_BITS) bulk_load(st, w.bits + (kb + i) * BM, uint32_t(nu) * BM * 4, &full[s]);
           for (int u = 0; u < nu; ++u) {
@@ -209,7 +210,7 @@ __global__ void __launch_bounds__(NTHREADS, 1)
             }
             // chunk u's B tile in smem: [hi: npad rows][lo: npad rows] x 128 B
             uint8_t* bdst = st + L.a_bytes + u * 2 * L.b_bytes;
-            if (w.b_fused) {
+            if (w.b_fused || w.single) {
               tma_load_2d(&map_bhi, &full[s], bdst, k0, 0);  // one box {32, 2*npad}: hi rows then lo rows
             } else {
               tma_load_2d(&map_bhi, &full[s], bdst, k0, 0);
@@ -256,7 +257,7 @@ __global__ void __launch_bounds__(NTHREADS, 1)
               const uint64_t bh = sdesc_kmajor_sw128(bh0 + kk * 32u);
               const uint64_t bl = sdesc_kmajor_sw128(bl0 + kk * 32u);
               mma_ts(d, a0 + kk * 8u, bh, idesc, acc);
-              mma_ts(d, a0 + kk * 8u, bl, idesc, 1u);
+              if (!w.single) mma_ts(d, a0 + kk * 8u, bl, idesc, 1u);
               if (MODE != A_BITS) mma_ts(d, a0 + BK + kk * 8u, bh, idesc, 1u);
               acc = 1u;
             }
@@ -522,8 +523,14 @@ cudaError_t launch_dense_tc(const DenseArgs& a, cudaStream_t s) {
     return launch_dense_pair(a, mh, s);
   }
   int fused = 0;
-  if (!make_b_maps(a.hiT, a.loT, a.n, a.ldT, a.npad, &mh, &ml, &fused)) return cudaErrorInvalidValue;
   Work w{};
+  if (a.loT) {
+    if (!make_b_maps(a.hiT, a.loT, a.n, a.ldT, a.npad, &mh, &ml, &fused)) return cudaErrorInvalidValue;
+  } else {  // BF16X1: hi rows only
+    if (!make_map(&mh, a.hiT, a.n, a.npad, a.ldT, BK, a.npad, true)) return cudaErrorInvalidValue;
+    ml = mh;
+    w.single = 1;
+  }
   w.b_fused = fused;
   w.ntiles = a.nrt;
   w.rt_cptr = a.rt_cptr;
@@ -562,11 +569,11 @@ cudaError_t launch_tc_gemm_xw(const float* X, int64_t ldx, const float* wThi, co
 // ---- partial[sp] = X[rows of slice sp]ᵀ · D, D pre-split feature-major ----
 int64_t tc_xtg_slices(int64_t M, int K) {
   // split-K over rows so that (output row tiles) x (slices) fills the 148
-  // SMs of a B200 once (a constant, not the queried SM count: the slicing
-  // fixes the summation order, which must not depend on the device), with
-  // >= 1024 rows per slice
+  // SMs of a B200 in one wave (a constant, not the queried SM count: the
+  // slicing fixes the summation order, which must not depend on the device),
+  // with >= 1024 rows per slice
   const int64_t mt = (K + BM - 1) / BM;
-  int64_t sl = (148 + mt - 1) / mt;
+  int64_t sl = 148 / mt;
   const int64_t cap = (M + 1023) / 1024;
   sl = sl < cap ? sl : cap;
   return sl < 1 ? 1 : (sl > 148 ? 148 : sl);

@@ -190,3 +190,120 @@ class GCN2:
 
     def replay(self):
         self._graph.replay()
+
+
+class GCNL:
+    """ℓ-layer GCN (Alg. 1 with general ℓ, L101-L125; the paper's Table II
+    model is ℓ = 4, hid = 64, L255 — SURVEY.md §8(f) F2) as a sequence of ABI
+    calls, single GPU.  dims = [F_in, hid, ..., hid, C]; layer l: Y_l' =
+    diag(r)·H_{l-1}·Θ_l (gemm_xw), H_l = ReLU(Â Y_l) with its bit mask (hidden
+    layers) or the logits (last layer); backward: G_l = Â dY_l, ∇Θ_l =
+    H_{l-1}ᵀ G_l (gemm_xtg), dY_{l-1}' = diag(r)((G_l Θ_lᵀ) ⊙ mask_{l-1})
+    (gemm_dwt).  ``plan`` serves the hidden widths, ``plan_c`` the class
+    width (per-width modes)."""
+
+    def __init__(self, plan: L.Plan, X_plan: np.ndarray, labels_plan: np.ndarray, train_plan: np.ndarray,
+                 thetas, *, optimizer: str = "adam", lr: float = 0.01, device="cuda", plan_c: L.Plan | None = None):
+        self.plan = plan
+        self.plan_c = plan_c if plan_c is not None else plan
+        assert plan.row_lo == 0 and plan.row_hi == plan.n, "GCNL is single-GPU"
+        self.dev = torch.device(device)
+        d, f32 = self.dev, torch.float32
+        self.n = n = plan.n
+        self.dims = [X_plan.shape[1]] + [t.shape[1] for t in thetas]
+        for l, t in enumerate(thetas):
+            assert t.shape[0] == self.dims[l]
+        self.nl = len(thetas)
+        self.optimizer, self.lr = optimizer, lr
+        assert max(self.dims[1:]) <= plan.f_max
+        ld = [_ld(f) for f in self.dims]
+        self.ld = ld
+        self.X = torch.zeros(n, ld[0], dtype=f32, device=d)
+        self.X[:, :self.dims[0]] = torch.from_numpy(np.ascontiguousarray(X_plan, dtype=np.float32)).to(d)
+        self.labels = torch.from_numpy(np.ascontiguousarray(labels_plan, dtype=np.int32)).to(d)
+        self.train = torch.from_numpy(np.ascontiguousarray(train_plan, dtype=np.uint8)).to(d)
+        self.inv_nT = 1.0 / float(np.count_nonzero(train_plan))
+        flat = np.concatenate([np.asarray(t, np.float32).ravel() for t in thetas])
+        self.theta = torch.from_numpy(flat).to(d)
+        self.grad = torch.zeros_like(self.theta)
+        self.Th, self.gTh, o = [], [], 0
+        for l in range(self.nl):
+            k = self.dims[l] * self.dims[l + 1]
+            self.Th.append(self.theta[o:o + k].view(self.dims[l], self.dims[l + 1]))
+            self.gTh.append(self.grad[o:o + k].view(self.dims[l], self.dims[l + 1]))
+            o += k
+        self.m = torch.zeros_like(self.theta)
+        self.v = torch.zeros_like(self.theta)
+        self.step_ctr = torch.zeros(1, dtype=torch.int32, device=d)
+        z = lambda w: torch.zeros(n, w, dtype=f32, device=d)  # noqa: E731
+        self.Y = [z(ld[l + 1]) for l in range(self.nl)]          # prescaled transform outputs
+        self.H = [z(ld[l + 1]) for l in range(self.nl - 1)]      # hidden activations
+        self.mask = [torch.zeros(n, (self.dims[l + 1] + 31) // 32, dtype=torch.int32, device=d)
+                     for l in range(self.nl - 1)]
+        self.Lg = z(ld[-1])
+        self.dY = [z(ld[l + 1]) for l in range(self.nl)]         # backward aggregation inputs (prescaled)
+        self.G = [z(ld[l + 1]) for l in range(self.nl)]
+        self.loss = torch.zeros(1, dtype=f32, device=d)
+        self.ce_work = torch.zeros(L.CE_WORK_FLOATS, dtype=f32, device=d)
+        wk = max(max(L.gemm_xtg_work_floats(n, self.dims[l], self.dims[l + 1]) for l in range(self.nl)), 1)
+        self.xtg_work = torch.zeros(wk, dtype=f32, device=d)
+        wk = max(max(L.gemm_xw_work_floats(self.dims[l], self.dims[l + 1]) for l in range(self.nl)),
+                 max(L.gemm_dwt_work_floats(self.dims[l], self.dims[l + 1]) for l in range(self.nl)))
+        self.xw_work = torch.zeros(wk, dtype=f32, device=d)
+        import ctypes
+        self.rr = ctypes.c_void_p(plan.rowscale_ptr())
+        self._graph = None
+
+    def _plan(self, l):
+        return self.plan_c if l == self.nl - 1 else self.plan
+
+    def epoch(self, stream=None, hook=None, agg_flags=0):
+        mark = hook or (lambda name: None)
+        n, dims, rr = self.n, self.dims, self.rr
+        Hin = self.X
+        for l in range(self.nl):
+            L.gemm_xw(Hin, self.Th[l], rr, self.Y[l], M=n, K=dims[l], N=dims[l + 1], work=self.xw_work, stream=stream)
+            mark(f"xw{l}")
+            if l < self.nl - 1:
+                self._plan(l).forward(self.Y[l], self.H[l], F=dims[l + 1],
+                                      flags=L.IN_PRESCALED | L.RELU | L.MASK_OUT | agg_flags, mask=self.mask[l],
+                                      stream=stream)
+                Hin = self.H[l]
+            else:
+                self._plan(l).forward(self.Y[l], self.Lg, F=dims[l + 1], flags=L.IN_PRESCALED | agg_flags,
+                                      stream=stream)
+            mark(f"agg_fwd{l}")
+        L.softmax_ce(self.Lg, self.labels, self.train, self.inv_nT, rr, self.dY[-1], self.loss, self.ce_work,
+                     M=n, C=dims[-1], stream=stream)
+        mark("softmax_ce")
+        for l in range(self.nl - 1, -1, -1):
+            self._plan(l).backward(self.dY[l], self.G[l], F=dims[l + 1], flags=L.IN_PRESCALED | agg_flags,
+                                   stream=stream)
+            mark(f"agg_bwd{l}")
+            Hl = self.X if l == 0 else self.H[l - 1]
+            L.gemm_xtg(Hl, self.G[l], self.gTh[l], self.xtg_work, M=n, K=dims[l], N=dims[l + 1], stream=stream)
+            if l > 0:
+                L.gemm_dwt(self.G[l], self.Th[l], self.mask[l - 1], rr, self.dY[l - 1], M=n, N=dims[l + 1],
+                           K=dims[l], work=self.xw_work, stream=stream)
+            mark(f"grad{l}")
+        if self.optimizer == "adam":
+            L.adam(self.theta, self.grad, self.m, self.v, self.lr, self.step_ctr, stream=stream)
+        elif self.optimizer == "sgd":
+            L.sgd(self.theta, self.grad, self.lr, stream=stream)
+        mark("update")
+
+    def capture(self, warmup: int = 2):
+        s = torch.cuda.Stream(device=self.dev)
+        s.wait_stream(torch.cuda.current_stream(self.dev))
+        with torch.cuda.stream(s):
+            for _ in range(warmup):
+                self.epoch(stream=s)
+        torch.cuda.current_stream(self.dev).wait_stream(s)
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=s):
+            self.epoch(stream=s)
+        self._graph = g
+        return g
+
+    def replay(self):
+        self._graph.replay()

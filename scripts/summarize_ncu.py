@@ -52,7 +52,7 @@ def main(csv_path, rep_path, out_path):
         a = agg.setdefault(k, [0, 0.0])
         a[0] += 1
         a[1] += t
-    lines = ["# ncu summary (one C3 epoch, eager launches; cold-cache serialised times — compare SHARES)", "",
+    lines = ["# ncu summary (one epoch, eager launches; cold-cache serialised times — compare SHARES)", "",
              f"source: `{csv_path}` ({len(L)} launches, {total / 1e3:.3f} ms total)", "",
              "| kernel | launches | total us | share |", "|---|---|---|---|"]
     for k, (c, t) in sorted(agg.items(), key=lambda kv: -kv[1][1]):
@@ -83,15 +83,27 @@ def main(csv_path, rep_path, out_path):
         import json
         import os
         fH, fC = int(sys.argv[4]), int(sys.argv[5])
-        sp = [d for d in rows[2:] if "sparse_agg" in d[hdr.index("Kernel Name")]]
+        # the selective pass = segment kernel + row kernel; the capture holds the
+        # layer-1 forward (F=H) launches first, then the layer-2 ones (F=C):
+        # group by the lane-slot template argument G of the kernel name
+        sp = [d for d in rows[2:] if "sparse_" in d[hdr.index("Kernel Name")]]
+        scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}
+        def g_of(d):
+            nm = d[hdr.index("Kernel Name")]
+            return nm.split("<", 1)[1].split(",", 1)[0]
         tr = {}
-        for key, d in zip(("sparse_agg_F%d" % fH, "sparse_agg_F%d" % fC), sp[:2]):
-            rd = float(d[hdr.index("dram__bytes_read.sum")])
-            wr = float(d[hdr.index("dram__bytes_write.sum")])
-            scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}
-            rd *= scale.get(units[hdr.index("dram__bytes_read.sum")], 1)
-            wr *= scale.get(units[hdr.index("dram__bytes_write.sum")], 1)
-            tr[key] = int(rd + wr)
+        groups = []
+        for d in sp:
+            if not groups or g_of(d) != g_of(groups[-1][0]):
+                groups.append([])
+            groups[-1].append(d)
+        for key, grp in zip(("sparse_agg_F%d" % fH, "sparse_agg_F%d" % fC), groups[:2]):
+            tot = 0.0
+            for d in grp:
+                for m in ("dram__bytes_read.sum", "dram__bytes_write.sum"):
+                    tot += float(d[hdr.index(m)]) * scale.get(units[hdr.index(m)], 1)
+            tr[key] = int(tot)
+            tr[key + "_kernels"] = [short(d[hdr.index("Kernel Name")]) for d in grp]
         tr["source"] = rep_path
         json.dump(tr, open(os.path.join(os.path.dirname(out_path), "traffic.json"), "w"), indent=1)
 

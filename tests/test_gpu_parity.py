@@ -81,17 +81,21 @@ SMALL = {
 
 
 @pytest.mark.parametrize("name", list(SMALL))
-@pytest.mark.parametrize("mode", ["sparse", "dense_tc", "dense_simt", "hybrid"])
+@pytest.mark.parametrize("mode", ["sparse", "dense_tc", "dense_simt", "hybrid", "dense_bf16"])
 @pytest.mark.parametrize("F", [1, 7, 16, 41, 128])
 def test_aggregation_parity(name, mode, F):
     g = SMALL[name]()
     P = max(1, min(8, g.n // 40))
-    theta = {"sparse": 2.0, "dense_tc": 0.0, "dense_simt": 0.0, "hybrid": 0.05}[mode]
-    dense = L.DENSE_FP32_SIMT if mode == "dense_simt" else L.DENSE_TF32X2
+    theta = {"sparse": 2.0, "dense_tc": 0.0, "dense_simt": 0.0, "hybrid": 0.05, "dense_bf16": 0.0}[mode]
+    dense = {"dense_simt": L.DENSE_FP32_SIMT, "dense_bf16": L.DENSE_BF16X1}.get(mode, L.DENSE_TF32X2)
     Y = _feat(g.n, F, 11)
     Z, pl, _ = aggregate_gpu(g, Y, P, theta, dense=dense)
     err, _ = cond_err(g, Y, Z)
-    assert err <= TOL, (name, mode, F, err, pl.stats())
+    # bf16 inputs (PCGCN_DENSE_BF16X1): |rounding| <= 2^-9 per term; gate 2e-2 (north star)
+    tol = 2e-2 if mode == "dense_bf16" else TOL
+    assert err <= tol, (name, mode, F, err, pl.stats())
+    if mode == "dense_bf16":
+        assert err <= 2.0 ** -8, err   # what the rounding bound predicts
 
 
 def test_closed_forms_complete_and_cycle_dense():
@@ -462,3 +466,54 @@ def test_long_rows_segments(F, ldpad):
     pl.forward(Yd, Z2, F=F, flags=L.RELU | L.MASK_OUT, mask=mask)
     torch.cuda.synchronize()
     assert torch.equal(Z2[:, :F], Zd[:, :F])
+
+
+@pytest.mark.parametrize("wname,theta,nl", [("cora", 0.05, 4), ("pubmed", 0.0, 4), ("cora", 2.0, 3)])
+def test_epoch_parity_deep(wname, theta, nl):
+    """The ℓ-layer model (the paper's Table II shape ℓ = 4, L255)
+    vs the oracle's forward_l/backward_l + one SGD step.  ReLU decisions with
+    |P| within 1e-6 of their condition scale may go either way in fp32: the
+    oracle takes the GPU's decision there (read back from the bit masks) and
+    must agree everywhere else."""
+    from paper_conf_ipps_tianmyd20_b200.gcn import GCNL
+    w = C.WORKLOADS[wname]
+    g = C.graph(w)
+    X = C.features(w, g.n)
+    rng = np.random.default_rng(nl)
+    dims = [w.f_in] + [w.hidden] * (nl - 1) + [w.classes]
+    Ths = [C.glorot(dims[i], dims[i + 1], w.theta_seed, 10 + i) for i in range(nl)]
+    y = C.labels(w, g)
+    T = C.train_mask(g.n, w.theta_seed)
+    pl = L.Plan(g.n, g.rowptr, g.col, w.P, theta)
+    perm = pl.perm()
+    inv = np.argsort(perm)
+    model = GCNL(pl, X[perm], y[perm], T[perm], Ths, optimizer="sgd", lr=0.1)
+    model.epoch()
+    torch.cuda.synchronize()
+    Ahat = O.normalized_adjacency(g.n, g.rowptr, g.col)[0]
+    Ps, Hs = O.forward_l(Ahat, X, Ths)
+    # condition scales of the pre-activations, layer by layer
+    absH = np.abs(X.astype(np.float64))
+    for l in range(nl - 1):
+        scale = O.aggregate(abs(Ahat), absH @ np.abs(Ths[l].astype(np.float64)))
+        mw = (dims[l + 1] + 31) // 32
+        m = model.mask[l].cpu().numpy().view(np.uint32)
+        bits = ((m[:, :, None] >> np.arange(32, dtype=np.uint32)) & 1).reshape(g.n, 32 * mw)[:, :dims[l + 1]][inv]
+        amb = np.abs(Ps[l]) <= 1e-6 * scale
+        assert np.all((bits.astype(bool) == (Ps[l] > 0)) | amb), l
+        assert amb.sum() <= 16
+        Ps[l] = np.where(amb, np.where(bits.astype(bool), 1e-300, -1e-300), Ps[l])
+        absH = np.maximum(scale, 0)
+    loss, dL = O.softmax_ce(Ps[-1], y, T)
+    grads, Gs = O.backward_l(Ahat, Ths, Ps, Hs, dL)
+
+    def rel(a, b):
+        return np.max(np.abs(a - b)) / max(np.max(np.abs(b)), 1e-30)
+
+    assert abs(model.loss.item() - loss) <= 1e-5 * abs(loss)
+    assert rel(_np(model.Lg)[:, :dims[-1]][inv], Ps[-1]) < 1e-5
+    for l in range(nl):
+        assert rel(_np(model.G[l])[:, :dims[l + 1]][inv], Gs[l]) < 1e-4, l
+        assert rel(_np(model.gTh[l]).ravel(), grads[l].ravel()) < 1e-4, l
+        step = (Ths[l].astype(np.float64) - _np(model.Th[l])) / 0.1          # the SGD update applied
+        assert rel(step.ravel(), grads[l].ravel()) < 1e-3, l

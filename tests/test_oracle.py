@@ -212,6 +212,67 @@ def test_p13_torch_autograd():
     np.testing.assert_allclose(L.detach().numpy(), out["L"], rtol=1e-12, atol=1e-14)
 
 
+# P12/P13 for the ℓ-layer model: finite differences and torch
+# fp64 autograd of the same ℓ = 4 network
+def _deep_problem(seed=15, n=28, dims=(6, 5, 4, 5, 3)):
+    g = G.random_graph(n, 0.2, seed)
+    rng = np.random.default_rng(seed)
+    X = rng.standard_normal((n, dims[0]))
+    Ths = [rng.standard_normal((dims[i], dims[i + 1])) * 0.6 for i in range(len(dims) - 1)]
+    y = rng.integers(0, dims[-1], n)
+    T = rng.random(n) < 0.7
+    return g, X, Ths, y, T
+
+
+def test_deep_finite_differences():
+    g, X, Ths, y, T = _deep_problem()
+    Ahat = _ahat(g)
+    out = O.epoch_l(Ahat, X, Ths, y, T)
+
+    def loss(ths):
+        return O.softmax_ce(O.forward_l(Ahat, X, ths)[0][-1], y, T)[0]
+
+    h = 1e-6
+    rng = np.random.default_rng(1)
+    for l in range(len(Ths)):
+        for _ in range(4):
+            i, j = rng.integers(0, Ths[l].shape[0]), rng.integers(0, Ths[l].shape[1])
+            P = [t.copy() for t in Ths]
+            M = [t.copy() for t in Ths]
+            P[l][i, j] += h
+            M[l][i, j] -= h
+            fd = (loss(P) - loss(M)) / (2 * h)
+            an = out["grads"][l][i, j]
+            assert abs(fd - an) <= 1e-7 * max(1.0, abs(an)) + 1e-9, (l, fd, an)
+
+
+def test_deep_torch_autograd_and_two_layer_special_case():
+    torch = pytest.importorskip("torch")
+    g, X, Ths, y, T = _deep_problem(seed=16)
+    Ahat = _ahat(g)
+    out = O.epoch_l(Ahat, X, Ths, y, T)
+    A = torch.tensor(Ahat.toarray(), dtype=torch.float64)
+    ts = [torch.tensor(t, requires_grad=True) for t in Ths]
+    H = torch.tensor(X)
+    for l, t in enumerate(ts):
+        H = A @ H @ t
+        if l < len(ts) - 1:
+            H = torch.relu(H)
+    Tm = torch.tensor(T)
+    ce = torch.nn.functional.cross_entropy(H[Tm], torch.tensor(y)[Tm])
+    ce.backward()
+    assert abs(ce.item() - out["loss"]) < 1e-13
+    for t, gr in zip(ts, out["grads"]):
+        np.testing.assert_allclose(t.grad.numpy(), gr, rtol=1e-11, atol=1e-14)
+    # ℓ = 2 is the 2-layer model of forward()/backward()
+    g2, X2, Th0, Th1, y2, T2 = _tiny_problem(seed=17)
+    A2 = _ahat(g2)
+    o2 = O.epoch(A2, X2, Th0, Th1, y2, T2)
+    ol = O.epoch_l(A2, X2, [Th0, Th1], y2, T2)
+    np.testing.assert_allclose(ol["grads"][0], o2["gTh0"], rtol=1e-12, atol=1e-15)
+    np.testing.assert_allclose(ol["grads"][1], o2["gTh1"], rtol=1e-12, atol=1e-15)
+
+
 # P14: uniform logits
 def test_p14_softmax_ce_uniform():
     n, c = 12, 5
