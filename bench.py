@@ -129,6 +129,11 @@ def load_workload(name):
 HUGE_NNZ = 500_000_000  # C5-sized graphs: single calibrated plan, row-wise oracle sample, serial e2e
 
 
+def _ld_bytes(F):
+    """Row stride in bytes of an activation of width F (gcn._ld)."""
+    return 4 * ((F + 3) // 4 * 4 if F <= 16 else (F + 15) // 16 * 16)
+
+
 def hbm_peak():
     try:
         j = json.load(open(MEASURED_PEAKS))
@@ -602,6 +607,11 @@ def main():
     # 3 repetitions at each of several L2-resident sizes.
     l2_gbs = max(L.probe_read_gbs(mb << 20, 50) for mb in (16, 32, 48, 64) for _ in range(3))
     hbm_probe = L.probe_read_gbs(4 << 30, 3)
+    # random-row gather ceilings at the kernel's row size (pcgcn_probe_gather_gbs):
+    # rows served by L1 (64 KB buffer), by L2 (64 MB) and by HBM (4 GB)
+    rb = _ld_bytes(w.hidden)
+    gprobe = {lvl: max(L.probe_gather_gbs(nb, rb, 256) for _ in range(3))
+              for lvl, nb in (("l1", 64 << 10), ("l2", 64 << 20), ("hbm", 4 << 30))}
     rows = pl.row_hi - pl.row_lo
     dense_rows = int(st["row_tiles"]) * 128 if world == 1 else int(st["shard_chunks"] > 0) * rows
     bH = agg_bytes(st, g.n, rows, w.hidden, dense_rows, st["shard_chunks"])
@@ -623,11 +633,13 @@ def main():
         tc_peak = float(json.load(open(MEASURED_PEAKS))["bf16_tflops"]) / 2
     except Exception:
         tc_peak = 1590.0 / 2
-    traffic = None
+    traffic = l2_read = None
     tpath = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tpath):
         try:
-            traffic = json.load(open(tpath)).get("sparse_agg_F%d" % w.hidden)
+            tj = json.load(open(tpath)).get(w.name, {})
+            traffic = tj.get("sparse_agg_F%d" % w.hidden)
+            l2_read = tj.get("sparse_agg_F%d_l2_read_bytes" % w.hidden)
         except Exception:
             traffic = None
 
@@ -787,10 +799,25 @@ def main():
                          "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
                          "algorithmic_bytes": b_sp, "ms": t_sp,
                          "traffic_source": "profiles/traffic.json (ncu --set full, dram read+write per launch)",
-                         "l2_view": {"gather_bytes": st["shard_nnz_sparse"] * fp4 * 4, "achieved": gather,
-                                     "peak": l2_gbs, "unit": "GB/s", "frac": gather / l2_gbs,
+                         "l2_view": {"l2_read_bytes": l2_read,
+                                     "achieved": (l2_read / (t_sp * 1e-3) / 1e9) if l2_read else None,
+                                     "peak": l2_gbs, "unit": "GB/s",
+                                     "frac": (l2_read / (t_sp * 1e-3) / 1e9 / l2_gbs) if l2_read else None,
+                                     "bytes_source": "ncu lts__t_sectors_srcunit_tex_op_read x 32 per launch "
+                                                     "(profiles/traffic.json); the L1 serves the rest of the gather",
+                                     "gather_bytes": st["shard_nnz_sparse"] * fp4 * 4,
+                                     "gather_GBs": gather,
                                      "peak_source": "measured: max of pcgcn_probe_read_gbs over 16-64 MiB L2-resident buffers, 3 reps each"},
-                         "hbm_probe_GBs": hbm_probe},
+                         "hbm_probe_GBs": hbm_probe,
+                         "gather_view": {"row_bytes": rb, "rows": st["shard_nnz_sparse"],
+                                         "achieved": st["shard_nnz_sparse"] * rb / (t_sp * 1e-3) / 1e9,
+                                         "unit": "GB/s",
+                                         "ceilings": gprobe,
+                                         "frac_of_l2_ceiling": st["shard_nnz_sparse"] * rb / (t_sp * 1e-3) / 1e9 / gprobe["l2"],
+                                         "frac_of_hbm_ceiling": st["shard_nnz_sparse"] * rb / (t_sp * 1e-3) / 1e9 / gprobe["hbm"],
+                                         "source": "pcgcn_probe_gather_gbs: the kernel's access pattern (random "
+                                                   "rows of row_bytes, 8 in flight per lane, 32 warps/SM) from "
+                                                   "64 KB / 64 MB / 4 GB buffers, best of 3"}},
             "tensor_view": {"kernel": "tc_engine<A_BITS> full-mode tiles, layer-1 forward",
                             "ms": t_tc, "achieved": tc_tf, "unit": "TFLOP/s (tf32)", "peak": tc_peak,
                             "frac": (tc_tf / tc_peak) if tc_tf else None,

@@ -136,6 +136,16 @@ pcgcn_status pcgcn_plan_last_timings(pcgcn_plan_t p, float ms[4]);
  * measures the L2->SM path, a size >> 126 MB the HBM path).  Synchronises. */
 pcgcn_status pcgcn_probe_read_gbs(int64_t bytes, int32_t iters, float* gbs);
 
+/* Measurement helper: the selective kernel's access pattern (L149, L181: one source
+ * feature row per edge) without its index stream — every warp slot of G = row_bytes/16
+ * lanes (G the narrowest power of two covering the row, as in the kernel) reads
+ * pseudo-random rows of `row_bytes` (multiple of 16, 16..512; row stride = row_bytes) from a buffer
+ * of `bytes`, 8 rows in flight per lane, `steps` (>= 8) rows per slot; returns the
+ * gathered GB/s.  The buffer size selects the level serving the rows (L1 ~<= 128 KB,
+ * L2 << 126 MB, HBM >> 126 MB): the measured ceilings of the gather roofline
+ * (DESIGN.md §6).  Allocates and frees a device buffer; synchronises. */
+pcgcn_status pcgcn_probe_gather_gbs(int64_t bytes, int32_t row_bytes, int32_t steps, float* gbs);
+
 /* Z = Â·Y  (Eq. 1 propagation; Alg. 1 inner loop h_k = Σ_i f(E_{k,i}, a_i), L118-L121).
  *   Y: DEVICE [n x F] (full plan order, all n rows even on a shard), ld ldy.
  *   Z: DEVICE [rows x F] with rows = row_hi - row_lo of this shard (n unsharded), ld ldz.

@@ -88,6 +88,7 @@ _sig("pcgcn_plan_last_timings", c_i32, c_vp, ctypes.POINTER(c_f32))
 _sig("pcgcn_refine_theta", c_i32, c_vp, c_vp, c_i64, c_vp, c_i64, c_i32, ctypes.POINTER(c_f32),
      ctypes.POINTER(c_f32), ctypes.POINTER(c_f32))
 _sig("pcgcn_probe_read_gbs", c_i32, c_i64, c_i32, ctypes.POINTER(c_f32))
+_sig("pcgcn_probe_gather_gbs", c_i32, c_i64, c_i32, c_i32, ctypes.POINTER(c_f32))
 _sig("pcgcn_last_error", ctypes.c_char_p)
 _sig("pcgcn_abi_version", c_i32)
 
@@ -261,3 +262,11 @@ def calibrate(F, block_rows=2048, p_ref=0.05):
     check(lib.pcgcn_calibrate(F, block_rows, p_ref, ctypes.byref(th), ctypes.byref(tf), ctypes.byref(ts)),
           "pcgcn_calibrate")
     return th.value, tf.value, ts.value
+
+
+def probe_gather_gbs(nbytes, row_bytes=512, steps=256):
+    """Random-row gather bandwidth (GB/s) from a buffer of nbytes (pcgcn_probe_gather_gbs)."""
+    v = c_f32()
+    check(lib.pcgcn_probe_gather_gbs(int(nbytes), int(row_bytes), int(steps), ctypes.byref(v)),
+          "pcgcn_probe_gather_gbs")
+    return float(v.value)

@@ -37,9 +37,11 @@ struct AggArgs {
   int64_t ldws;
   int* counter;              // dynamic row scheduler ticket (zeroed on the stream before each pass)
   bool idx_evict_first;      // L2 evict_first hint on the index stream (set by the launcher)
+  int phase = 0;             // 0: segment pass + row pass; 1: segment pass only; 2: row pass only
 };
 // selective edges per long-row segment
 constexpr int SEG_EDGES = 1024;
+bool sparse_fsplit_active(int F);  // benchmark knob PCGCN_SPARSE_FSPLIT splits this width
 cudaError_t launch_sparse_agg(const AggArgs& a, cudaStream_t s);
 
 // ypre = diag(r)·Y

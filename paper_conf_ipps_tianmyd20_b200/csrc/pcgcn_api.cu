@@ -6,6 +6,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 #include <new>
 #include <string>
@@ -62,6 +63,9 @@ void set_error(const std::string& msg) { g_err = msg; }
 void free_device_plan(pcgcn_plan_s* p) {
   for (void*& ev : p->d.ev)
     if (ev) cudaEventDestroy(static_cast<cudaEvent_t>(ev));
+  if (p->d.ev_fork) cudaEventDestroy(static_cast<cudaEvent_t>(p->d.ev_fork));
+  if (p->d.ev_join) cudaEventDestroy(static_cast<cudaEvent_t>(p->d.ev_join));
+  if (p->d.side) cudaStreamDestroy(static_cast<cudaStream_t>(p->d.side));
   for (void* q : p->d.owned) dev_free(q);
   p->d = DevicePlan();
 }
@@ -139,6 +143,23 @@ pcgcn_status upload_plan(pcgcn_plan_s* p) {
 #undef UP
   e = cudaMemset(d.zrow, 0, 256 * sizeof(float));
   if (e != cudaSuccess) return cuda_fail(e, "memset");
+  if (d.nseg > 0 && d.nch > 0) {
+    // high-priority side stream for the split + full-mode tiles, which run
+    // concurrently with the long-row segment pass on the caller's stream (the
+    // two are independent; fork/join by events, CUDA-graph capturable); the
+    // priority lets the engine's CTAs claim SMs first, segment CTAs fill in
+    cudaStream_t side;
+    cudaEvent_t f, j;
+    int lo_pri = 0, hi_pri = 0;
+    cudaDeviceGetStreamPriorityRange(&lo_pri, &hi_pri);
+    if ((e = cudaStreamCreateWithPriority(&side, cudaStreamNonBlocking, hi_pri)) != cudaSuccess)
+      return cuda_fail(e, "side stream");
+    d.side = side;
+    if ((e = cudaEventCreateWithFlags(&f, cudaEventDisableTiming)) != cudaSuccess) return cuda_fail(e, "event");
+    d.ev_fork = f;
+    if ((e = cudaEventCreateWithFlags(&j, cudaEventDisableTiming)) != cudaSuccess) return cuda_fail(e, "event");
+    d.ev_join = j;
+  }
   d.built = true;
   p->stats.device_bytes = d.bytes;
   p->stats.shard_segments = d.nseg;
@@ -146,6 +167,16 @@ pcgcn_status upload_plan(pcgcn_plan_s* p) {
 }
 
 namespace {
+
+// PCGCN_OVERLAP=0 serialises the segment pass behind the full-mode tiles (A/B knob)
+bool overlap_enabled() {
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("PCGCN_OVERLAP");
+    v = e ? (atoi(e) != 0) : 1;
+  }
+  return v != 0;
+}
 
 pcgcn_status aggregate(pcgcn_plan_t p, const float* Y, int64_t ldy, float* Z, int64_t ldz, int32_t F,
                        uint32_t flags, uint32_t* mask, void* stream) {
@@ -183,20 +214,6 @@ pcgcn_status aggregate(pcgcn_plan_t p, const float* Y, int64_t ldy, float* Z, in
     ldsrc = ld4;
   }
   mark(1);
-  float* ylo = d.yhi ? d.yhi + int64_t(npad) * d.n_pad : nullptr;
-  if (dense && tc) {
-    if (prof) d.ev_used[1] = true;
-    e = launch_split_transpose(src, ldsrc, p->n, F, npad, d.yhi, bf16 ? nullptr : ylo, d.n_pad, s);
-    if (e != cudaSuccess) return cuda_fail(e, "split_transpose");
-  }
-  mark(2);
-  if (dense) {
-    if (prof) d.ev_used[2] = true;
-    DenseArgs da{d.yhi, bf16 ? nullptr : ylo, d.n_pad, d.n_pad, d.rt_row0, d.rt_nrows, d.rt_cptr, d.ch_col0,
-                 d.bits, d.nrt, d.zd, npad, npad};
-    e = tc ? launch_dense_tc(da, s) : launch_dense_simt_y(da, src, ldsrc, F, s);
-    if (e != cudaSuccess) return cuda_fail(e, "dense-mode kernel");
-  }
   AggArgs a;
   a.Y = src; a.ldy = ldsrc; a.Z = Z; a.ldz = ldz;
   a.mask = (flags & PCGCN_MASK_OUT) ? mask : nullptr;
@@ -213,8 +230,46 @@ pcgcn_status aggregate(pcgcn_plan_t p, const float* Y, int64_t ldy, float* Z, in
   a.row_seg = d.row_seg; a.seg_lo = d.seg_lo; a.seg_hi = d.seg_hi; a.nseg = d.nseg;
   a.seg_ws = d.seg_ws; a.ldws = d.fpad_max;
   a.counter = d.counter;
+  // the split + full-mode tiles run on the plan's high-priority side stream,
+  // concurrently with the long-row segment pass on the caller's stream;
+  // PROFILE calls stay serial so per-kernel times add up
+  const bool overlap = overlap_enabled() && !prof && dense && d.nseg > 0 && d.side && d.rows > 0 &&
+                       !sparse_fsplit_active(F);
+  cudaStream_t ms = s;  // stream of the full-mode work
+  if (overlap) {
+    cudaStream_t side = static_cast<cudaStream_t>(d.side);
+    cudaEvent_t ef = static_cast<cudaEvent_t>(d.ev_fork);
+    if ((e = cudaEventRecord(ef, s)) != cudaSuccess) return cuda_fail(e, "fork");
+    if ((e = cudaStreamWaitEvent(side, ef, 0)) != cudaSuccess) return cuda_fail(e, "fork");
+    ms = side;
+  }
+  float* ylo = d.yhi ? d.yhi + int64_t(npad) * d.n_pad : nullptr;
+  if (dense && tc) {
+    if (prof) d.ev_used[1] = true;
+    e = launch_split_transpose(src, ldsrc, p->n, F, npad, d.yhi, bf16 ? nullptr : ylo, d.n_pad, ms);
+    if (e != cudaSuccess) return cuda_fail(e, "split_transpose");
+  }
+  mark(2);
+  if (dense) {
+    if (prof) d.ev_used[2] = true;
+    DenseArgs da{d.yhi, bf16 ? nullptr : ylo, d.n_pad, d.n_pad, d.rt_row0, d.rt_nrows, d.rt_cptr, d.ch_col0,
+                 d.bits, d.nrt, d.zd, npad, npad};
+    e = tc ? launch_dense_tc(da, ms) : launch_dense_simt_y(da, src, ldsrc, F, ms);
+    if (e != cudaSuccess) return cuda_fail(e, "dense-mode kernel");
+  }
+  if (overlap) {
+    if ((e = cudaEventRecord(static_cast<cudaEvent_t>(d.ev_join), ms)) != cudaSuccess) return cuda_fail(e, "join");
+    AggArgs sa = a;
+    sa.phase = 1;
+    if ((e = launch_sparse_agg(sa, s)) != cudaSuccess) return cuda_fail(e, "segment pass");
+  }
   mark(3);
   if (prof) d.ev_used[3] = true;
+  if (overlap) {
+    if ((e = cudaStreamWaitEvent(s, static_cast<cudaEvent_t>(d.ev_join), 0)) != cudaSuccess)
+      return cuda_fail(e, "join");
+    a.phase = 2;
+  }
   e = launch_sparse_agg(a, s);
   if (e != cudaSuccess) return cuda_fail(e, "selective-mode kernel");
   mark(4);

@@ -40,6 +40,9 @@ struct DevicePlan {
   std::vector<void*> owned;
   void* ev[5] = {nullptr, nullptr, nullptr, nullptr, nullptr};  // PCGCN_PROFILE events (cudaEvent_t)
   bool ev_used[4] = {false, false, false, false};
+  void* side = nullptr;                    // cudaStream_t: segment pass overlapped with the full mode
+  void* ev_fork = nullptr;                 // cudaEvent_t (timing disabled)
+  void* ev_join = nullptr;
 };
 
 }  // namespace pcgcn

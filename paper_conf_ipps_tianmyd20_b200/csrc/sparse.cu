@@ -182,9 +182,11 @@ __device__ __forceinline__ int lane_col(int lane, int v, int nvec) {
 
 // Segment pass: one warp per segment of a long row (<= SEG_EDGES edges),
 // partial sums to seg_ws.
+// 4-warp CTAs (8K registers): small enough to co-reside with a full-mode
+// engine CTA (tc_engine, 320 threads) when the two run concurrently
 template <int G, int V>
-__global__ void __launch_bounds__(256, 4) sparse_seg_kernel(AggArgs a) {
-  const int64_t sg = int64_t(blockIdx.x) * 8 + (threadIdx.x >> 5);
+__global__ void __launch_bounds__(128, 8) sparse_seg_kernel(AggArgs a) {
+  const int64_t sg = int64_t(blockIdx.x) * 4 + (threadIdx.x >> 5);
   if (sg >= a.nseg) return;
   const int lane = threadIdx.x & 31;
   const int nvec = (a.F + 3) >> 2;
@@ -324,11 +326,12 @@ cudaError_t launch_gv(const AggArgs& a, cudaStream_t s) {
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, sparse_row_kernel<G, V, true, true>, 256, 0);
     slots = sms * (per > 0 ? per : 1);
   }
+  if (a.nseg > 0 && a.phase != 2) {
+    sparse_seg_kernel<G, V><<<unsigned((a.nseg + 3) / 4), 128, 0, s>>>(a);
+    if (a.phase == 1) return cudaGetLastError();
+  }
   cudaError_t e = cudaMemsetAsync(a.counter, 0, sizeof(int), s);
   if (e != cudaSuccess) return e;
-  if (a.nseg > 0) {
-    sparse_seg_kernel<G, V><<<unsigned((a.nseg + 7) / 8), 256, 0, s>>>(a);
-  }
   const int64_t want = (a.rows + 7) / 8;
   const unsigned grid = unsigned(want < slots ? want : slots);
 #define LAUNCH(ZD, SG) sparse_row_kernel<G, V, ZD, SG><<<grid, 256, 0, s>>>(a)
@@ -412,15 +415,22 @@ struct SparseKnobs {
   }
 };
 
+static SparseKnobs& knobs() {
+  static SparseKnobs k;
+  return k;
+}
+
+bool sparse_fsplit_active(int F) { return knobs().fsplit > 0 && F > knobs().fsplit; }
+
 cudaError_t launch_sparse_agg(const AggArgs& a0, cudaStream_t s) {
   if (a0.rows <= 0) return cudaSuccess;
-  static SparseKnobs knobs;
+  const SparseKnobs& kn = knobs();
   AggArgs a = a0;
-  a.idx_evict_first = knobs.idx_ef;
-  if (knobs.fsplit <= 0 || a.F <= knobs.fsplit) return launch_sparse_pass(a, s);
-  for (int c0 = 0; c0 < a.F; c0 += knobs.fsplit) {
+  a.idx_evict_first = kn.idx_ef;
+  if (kn.fsplit <= 0 || a.F <= kn.fsplit) return launch_sparse_pass(a, s);
+  for (int c0 = 0; c0 < a.F; c0 += kn.fsplit) {
     AggArgs b = a;
-    b.F = (a.F - c0) < knobs.fsplit ? a.F - c0 : knobs.fsplit;
+    b.F = (a.F - c0) < kn.fsplit ? a.F - c0 : kn.fsplit;
     b.Y = a.Y + c0;
     b.Z = a.Z + c0;
     if (a.zd) b.zd = a.zd + c0;

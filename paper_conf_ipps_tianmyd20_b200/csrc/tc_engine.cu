@@ -493,7 +493,13 @@ cudaError_t launch_engine(const CUtensorMap& bhi, const CUtensorMap& blo, const 
   const Layout L = make_layout(MODE, npad, max_stages_env(), max_u_env());
   const size_t smem = 1024 + size_t(L.stages) * L.stage_bytes + (3 * L.stages + 4) * 8 + 16;
   if (smem > 227 * 1024) return cudaErrorInvalidValue;
-  const int64_t grid = w.ntiles < num_sms() ? w.ntiles : num_sms();
+  static int grid_cap = -1;  // PCGCN_TC_GRID: full-mode CTAs (tuning override, benchmarks only)
+  if (grid_cap < 0) {
+    const char* e = getenv("PCGCN_TC_GRID");
+    grid_cap = e ? atoi(e) : 0;
+  }
+  int64_t grid = w.ntiles < num_sms() ? w.ntiles : num_sms();
+  if (MODE == A_BITS && grid_cap > 0 && grid > grid_cap) grid = grid_cap;
   auto go = [&](auto kernel, bool& attr_done) -> cudaError_t {
     if (!attr_done) {
       cudaError_t e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);

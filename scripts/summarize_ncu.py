@@ -2,7 +2,12 @@
 """Summarise ncu output (launch list CSV + `--set full` report) into a
 markdown file under profiles/.  Runs here (no GPU needed to read reports).
 
-    python scripts/summarize_ncu.py gpurun_out/r1_launch_list.csv gpurun_out/r1_full.ncu-rep profiles/r1_ncu.md
+    python scripts/summarize_ncu.py gpurun_out/r1_launch_list.csv gpurun_out/r1_full.ncu-rep profiles/r1_ncu.md \
+        [F_H F_C [workload]]
+
+With F_H F_C it also merges the selective kernel's per-launch DRAM traffic and
+L2->L1 read bytes into profiles/traffic.json under the workload's name (bench.py's
+roofline.traffic and l2_view).
 """
 import csv
 import io
@@ -15,6 +20,7 @@ METRICS = [
     ("dram__bytes_read.sum", "DRAM read"),
     ("dram__bytes_write.sum", "DRAM write"),
     ("lts__t_sector_hit_rate.pct", "L2 hit %"),
+    ("lts__t_sectors_srcunit_tex_op_read.sum", "L2->L1 read sectors"),
     ("lts__throughput.avg.pct_of_peak_sustained_elapsed", "L2 thru %"),
     ("dram__throughput.avg.pct_of_peak_sustained_elapsed", "DRAM thru %"),
     ("sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_active", "tensor pipe %"),
@@ -83,11 +89,13 @@ def main(csv_path, rep_path, out_path):
         import json
         import os
         fH, fC = int(sys.argv[4]), int(sys.argv[5])
+        wl = sys.argv[6] if len(sys.argv) > 6 else "reddit"
         # the selective pass = segment kernel + row kernel; the capture holds the
         # layer-1 forward (F=H) launches first, then the layer-2 ones (F=C):
         # group by the lane-slot template argument G of the kernel name
         sp = [d for d in rows[2:] if "sparse_" in d[hdr.index("Kernel Name")]]
-        scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}
+        scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9,
+                 "sector": 1, "Ksector": 1e3, "Msector": 1e6, "Gsector": 1e9}
         def g_of(d):
             nm = d[hdr.index("Kernel Name")]
             return nm.split("<", 1)[1].split(",", 1)[0]
@@ -98,14 +106,21 @@ def main(csv_path, rep_path, out_path):
                 groups.append([])
             groups[-1].append(d)
         for key, grp in zip(("sparse_agg_F%d" % fH, "sparse_agg_F%d" % fC), groups[:2]):
-            tot = 0.0
+            tot, l2 = 0.0, 0.0
             for d in grp:
                 for m in ("dram__bytes_read.sum", "dram__bytes_write.sum"):
-                    tot += float(d[hdr.index(m)]) * scale.get(units[hdr.index(m)], 1)
+                    tot += float(d[hdr.index(m)].replace(",", "")) * scale.get(units[hdr.index(m)], 1)
+                m = "lts__t_sectors_srcunit_tex_op_read.sum"
+                if m in hdr:
+                    l2 += 32.0 * float(d[hdr.index(m)].replace(",", "")) * scale.get(units[hdr.index(m)], 1)
             tr[key] = int(tot)
+            tr[key + "_l2_read_bytes"] = int(l2) if l2 else None
             tr[key + "_kernels"] = [short(d[hdr.index("Kernel Name")]) for d in grp]
         tr["source"] = rep_path
-        json.dump(tr, open(os.path.join(os.path.dirname(out_path), "traffic.json"), "w"), indent=1)
+        tp = os.path.join(os.path.dirname(out_path), "traffic.json")
+        allt = json.load(open(tp)) if os.path.exists(tp) else {}
+        allt[wl] = tr
+        json.dump(allt, open(tp, "w"), indent=1)
 
 
 if __name__ == "__main__":

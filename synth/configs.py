@@ -105,10 +105,41 @@ def scaled(w: Workload, frac: float, name: str | None = None) -> Workload:
                     max(1, int(round(w.P * frac ** 0.5))), w.feat_kind, w.feat_seed, w.theta_seed)
 
 
+def _cache_key(w: Workload) -> str:
+    """Workload recipe + generator source digest: a cache entry written by
+    another generator version is never read back."""
+    import hashlib
+    import os
+    h = hashlib.sha1(repr(w.spec).encode())
+    d = os.path.dirname(os.path.abspath(__file__))
+    for f in ("graphs.py", "rng.py", os.path.join("csrc", "synth_gen.cpp")):
+        p = os.path.join(d, f)
+        if os.path.exists(p):
+            h.update(open(p, "rb").read())
+    return f"{w.name}-{h.hexdigest()[:16]}"
+
+
 def graph(w: Workload, impl: str = "auto") -> Graph:
-    if isinstance(w.spec, RMATSpec):
-        return rmat(w.spec)
-    return sbm(w.spec, impl=impl)
+    """The workload's graph.  PCGCN_GRAPH_CACHE=<dir> (benchmark scripts only)
+    keeps generated graphs as .npy files so one GPU job can reuse a C5-sized
+    graph across several processes instead of regenerating it (minutes)."""
+    import os
+    cdir = os.environ.get("PCGCN_GRAPH_CACHE")
+    if cdir:
+        base = os.path.join(cdir, _cache_key(w))
+        if os.path.exists(base + ".done"):
+            lab = np.load(base + ".labels.npy") if os.path.exists(base + ".labels.npy") else None
+            return Graph(int(np.load(base + ".rowptr.npy", mmap_mode="r").shape[0] - 1),
+                         np.load(base + ".rowptr.npy"), np.load(base + ".col.npy"), lab, {"cached": base})
+    g = rmat(w.spec) if isinstance(w.spec, RMATSpec) else sbm(w.spec, impl=impl)
+    if cdir:
+        os.makedirs(cdir, exist_ok=True)
+        np.save(base + ".rowptr.npy", g.rowptr)
+        np.save(base + ".col.npy", g.col)
+        if g.labels is not None:
+            np.save(base + ".labels.npy", g.labels)
+        open(base + ".done", "w").close()
+    return g
 
 
 def features(w: Workload, n: int) -> np.ndarray:
