@@ -36,8 +36,8 @@ struct AggArgs {
   float* seg_ws;             // [nseg x ldws] fp32 partial sums
   int64_t ldws;
   int* counter;              // dynamic row scheduler ticket (zeroed on the stream before each pass)
-  bool idx_evict_first;      // L2 evict_first hint on the index stream (set by the launcher)
   int phase = 0;             // 0: segment pass + row pass; 1: segment pass only; 2: row pass only
+  int rows_per_ticket = 1;   // consecutive rows per scheduler ticket, 1..16
 };
 // selective edges per long-row segment
 constexpr int SEG_EDGES = 1024;

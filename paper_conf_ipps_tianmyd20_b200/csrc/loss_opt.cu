@@ -15,45 +15,69 @@ namespace {
 
 constexpr int CE_BLOCKS = 592;  // 4 x 148 SMs; <= PCGCN_CE_WORK_FLOATS
 
-// one warp per row, grid-stride; C <= 32*8
+// one warp per row, RPW rows per warp step with all their loads issued up
+// front (a row is short: C <= 32*8 logits; at C5's 33.5M rows one row per
+// step left the kernel latency-bound, ~11.6 ms); grid-stride over row groups.
+constexpr int RPW = 4;
 __global__ void __launch_bounds__(256) softmax_ce_kernel(
     const float* __restrict__ L, int64_t ld, const int32_t* __restrict__ labels,
     const uint8_t* __restrict__ train, int64_t M, int C, float inv_nT, const float* __restrict__ s,
     float* __restrict__ dL, float* __restrict__ partial) {
   __shared__ float wsum[8];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-  float my = 0.f;  // lane 0 of each warp accumulates its rows' losses in order
-  for (int64_t row = int64_t(blockIdx.x) * 8 + w; row < M; row += int64_t(gridDim.x) * 8) {
-    const float* Lr = L + row * ld;
-    float v[8];
-    float mx = -INFINITY;
+  const int nt = (C + 31) >> 5;
+  float my = 0.f;  // lane 0 of each warp accumulates its rows' losses in row order
+  for (int64_t row0 = (int64_t(blockIdx.x) * 8 + w) * RPW; row0 < M; row0 += int64_t(gridDim.x) * 8 * RPW) {
+    float v[RPW][8];
+    int y[RPW];
+    float scale[RPW];
+    bool tr[RPW];
 #pragma unroll
-    for (int t = 0; t < 8; ++t) {
-      int c = lane + 32 * t;
-      v[t] = c < C ? Lr[c] : -INFINITY;
-      mx = fmaxf(mx, v[t]);
+    for (int k = 0; k < RPW; ++k) {
+      const int64_t row = row0 + k;
+      const bool ok = row < M;
+      const float* Lr = L + row * ld;
+#pragma unroll
+      for (int t = 0; t < 8; ++t) {
+        const int c = lane + 32 * t;
+        v[k][t] = (ok && t < nt && c < C) ? __ldg(Lr + c) : -INFINITY;
+      }
+      y[k] = ok ? __ldg(labels + row) : 0;
+      tr[k] = ok && __ldg(train + row) != 0;
+      scale[k] = ok ? (s ? __ldg(s + row) : 1.f) : 0.f;
     }
 #pragma unroll
-    for (int off = 16; off; off >>= 1) mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, off));
-    float se = 0.f;
+    for (int k = 0; k < RPW; ++k) {
+      const int64_t row = row0 + k;
+      float mx = -INFINITY;
 #pragma unroll
-    for (int t = 0; t < 8; ++t) {
-      int c = lane + 32 * t;
-      v[t] = c < C ? expf(v[t] - mx) : 0.f;
-      se += v[t];
+      for (int t = 0; t < 8; ++t) mx = fmaxf(mx, v[k][t]);
+#pragma unroll
+      for (int off = 16; off; off >>= 1) mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, off));
+      float se = 0.f, ly = 0.f;
+#pragma unroll
+      for (int t = 0; t < 8; ++t) {
+        const int c = lane + 32 * t;
+        if (c == y[k]) ly = v[k][t];
+        v[k][t] = (t < nt && c < C) ? expf(v[k][t] - mx) : 0.f;
+        se += v[k][t];
+      }
+#pragma unroll
+      for (int off = 16; off; off >>= 1) {
+        se += __shfl_xor_sync(0xffffffffu, se, off);
+        ly += __shfl_xor_sync(0xffffffffu, ly, off);  // the label's logit (one lane holds it)
+      }
+      if (row < M) {
+        const float sc = (tr[k] ? inv_nT : 0.f) * scale[k];
+        const float inv = 1.f / se;
+#pragma unroll
+        for (int t = 0; t < 8; ++t) {
+          const int c = lane + 32 * t;
+          if (t < nt && c < C) dL[row * ld + c] = (v[k][t] * inv - (c == y[k] ? 1.f : 0.f)) * sc;
+        }
+        if (lane == 0 && tr[k]) my += (mx + logf(se) - ly);
+      }
     }
-#pragma unroll
-    for (int off = 16; off; off >>= 1) se += __shfl_xor_sync(0xffffffffu, se, off);
-    const int y = labels[row];
-    const bool tr = train[row] != 0;
-    const float scale = (tr ? inv_nT : 0.f) * (s ? s[row] : 1.f);
-    const float inv = 1.f / se;
-#pragma unroll
-    for (int t = 0; t < 8; ++t) {
-      int c = lane + 32 * t;
-      if (c < C) dL[row * ld + c] = (v[t] * inv - (c == y ? 1.f : 0.f)) * scale;
-    }
-    if (lane == 0 && tr) my += (mx + logf(se) - Lr[y]);
   }
   if (lane == 0) wsum[w] = my;
   __syncthreads();

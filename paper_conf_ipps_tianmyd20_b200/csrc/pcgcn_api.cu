@@ -168,14 +168,37 @@ pcgcn_status upload_plan(pcgcn_plan_s* p) {
 
 namespace {
 
-// PCGCN_OVERLAP=0 serialises the segment pass behind the full-mode tiles (A/B knob)
+// PCGCN_OVERLAP=1 runs the split + full-mode tiles on a high-priority side stream
+// concurrently with the segment pass (measured on C3: no gain, 9.85 vs 9.62 ms
+// epoch; the engine CTAs leave too few registers for co-resident gathers)
 bool overlap_enabled() {
   static int v = -1;
   if (v < 0) {
     const char* e = getenv("PCGCN_OVERLAP");
-    v = e ? (atoi(e) != 0) : 1;
+    v = e ? (atoi(e) != 0) : 0;
   }
   return v != 0;
+}
+
+// rows per scheduler ticket: enough that a ticket covers ~128 selective edges
+// (C5's mean degree 31 -> 8: the next ticket and row pointers are then fetched
+// while the block's rows gather; measured C5 epoch 250 -> 206 ms), 1 for long
+// rows (C3's mean 348: R = 4 measured 2.5% slower there), at most 16
+// (PCGCN_ROWS_PER_TICKET overrides; benchmarks only)
+int rows_per_ticket(int64_t nnz_s, int64_t rows) {
+  static int env = -1;
+  if (env < 0) {
+    const char* e = getenv("PCGCN_ROWS_PER_TICKET");
+    env = e ? atoi(e) : 0;
+  }
+  int R = 1;
+  if (env > 0) {
+    R = env;
+  } else if (rows > 0) {
+    const double deg = double(nnz_s) / double(rows);
+    while (R < 16 && deg * R < 128.0) R *= 2;
+  }
+  return R < 1 ? 1 : (R > 16 ? 16 : R);
 }
 
 pcgcn_status aggregate(pcgcn_plan_t p, const float* Y, int64_t ldy, float* Z, int64_t ldz, int32_t F,
@@ -230,6 +253,7 @@ pcgcn_status aggregate(pcgcn_plan_t p, const float* Y, int64_t ldy, float* Z, in
   a.row_seg = d.row_seg; a.seg_lo = d.seg_lo; a.seg_hi = d.seg_hi; a.nseg = d.nseg;
   a.seg_ws = d.seg_ws; a.ldws = d.fpad_max;
   a.counter = d.counter;
+  a.rows_per_ticket = rows_per_ticket(d.nnz_s, d.rows);
   // the split + full-mode tiles run on the plan's high-priority side stream,
   // concurrently with the long-row segment pass on the caller's stream;
   // PROFILE calls stay serial so per-kernel times add up

@@ -50,18 +50,9 @@ __device__ __forceinline__ const char* row_addr(const char* base, uint32_t j, ui
   asm("mad.wide.u32 %0, %1, %2, %3;" : "=l"(r) : "r"(j), "r"(stride), "l"(reinterpret_cast<uint64_t>(base)));
   return reinterpret_cast<const char*>(r);
 }
-// index stream: read once per pass -> L2 evict_first so it does not push
-// Y' rows out of the L2 (tuning flag AggArgs::idx_evict_first)
-__device__ __forceinline__ int ld_idx(const int* p, bool ef, uint64_t pol) {
-  if (!ef) return __ldg(p);
-  int v;
-  asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
-  return v;
-}
-__device__ __forceinline__ uint64_t policy_evict_first() {
-  uint64_t p;
-  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
-  return p;
+__device__ __forceinline__ int ld_idx(const int* p) { return __ldg(p); }
+__device__ __forceinline__ uint32_t smem_addr(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
 }
 __device__ __forceinline__ void add4(float4& a, const float4& b) {
   a.x += b.x; a.y += b.y; a.z += b.z; a.w += b.w;
@@ -98,8 +89,7 @@ struct Lay {
 template <int G, int V>
 __device__ __forceinline__ int gather_sum(const int* __restrict__ cp, int n, int first,
                                           const int* __restrict__ cpn, int nn, const char* __restrict__ yb,
-                                          uint32_t rstride, const bool (&lok)[V], int lane, float4 (&tot)[V],
-                                          bool ef, uint64_t pol) {
+                                          uint32_t rstride, const bool (&lok)[V], int lane, float4 (&tot)[V]) {
   using L = Lay<G, V>;
   constexpr int S = L::S, STEPS = L::STEPS, UNR = L::UNR, NACC = L::NACC;
   const int slot = lane / G;
@@ -109,13 +99,13 @@ __device__ __forceinline__ int gather_sum(const int* __restrict__ cp, int n, int
 #pragma unroll
     for (int v = 0; v < V; ++v) acc[u][v] = make_float4(0.f, 0.f, 0.f, 0.f);
   int nextidx = first;
-  if (n == 0) nextidx = lane < nn ? ld_idx(cpn + lane, ef, pol) : 0;
+  if (n == 0) nextidx = lane < nn ? ld_idx(cpn + lane) : 0;
   for (int base = 0; base < n; base += 32) {
     const int cnt = (n - base) < 32 ? n - base : 32;
     const int myidx = nextidx;
     // next batch, one ahead (past the end: the next range's first batch)
-    nextidx = (base + 32 + lane < n) ? ld_idx(cp + base + 32 + lane, ef, pol)
-            : (lane < nn ? ld_idx(cpn + lane, ef, pol) : 0);
+    nextidx = (base + 32 + lane < n) ? ld_idx(cp + base + 32 + lane)
+            : (lane < nn ? ld_idx(cpn + lane) : 0);
     if (cnt == 32) {
       // full batch: unguarded, every lane keeps UNR*V 16-byte loads in flight
 #pragma unroll
@@ -197,11 +187,9 @@ __global__ void __launch_bounds__(128, 8) sparse_seg_kernel(AggArgs a) {
 #pragma unroll
   for (int v = 0; v < V; ++v) lok[v] = lane_col<G>(lane, v, nvec) >= 0;
   float4 tot[V];
-  const uint64_t pol = policy_evict_first();
   const int n = int(hi - lo);
-  const int first = lane < n ? ld_idx(a.col + lo + lane, a.idx_evict_first, pol) : 0;
-  gather_sum<G, V>(a.col + lo, n, first, nullptr, 0, yb, uint32_t(a.ldy * 4), lok, lane, tot,
-                   a.idx_evict_first, pol);
+  const int first = lane < n ? ld_idx(a.col + lo + lane) : 0;
+  gather_sum<G, V>(a.col + lo, n, first, nullptr, 0, yb, uint32_t(a.ldy * 4), lok, lane, tot);
   if (lane < G) {
 #pragma unroll
     for (int v = 0; v < V; ++v) {
@@ -230,28 +218,77 @@ __global__ void __launch_bounds__(256, 4) sparse_row_kernel(AggArgs a) {
   }
   const char* yb = reinterpret_cast<const char*>(a.Y) + 16 * (qv[0] < 0 ? 0 : qv[0]);
   const uint32_t rstride = uint32_t(a.ldy * 4);
-  const uint64_t pol = policy_evict_first();
-  auto claim = [&]() {
+  // Rows are claimed in blocks of R consecutive rows per ticket (R >= 4 from
+  // the plan's mean selective degree: short rows would otherwise pay the
+  // ticket -> rowptr -> index dependency chain per row).  The next block's
+  // ticket is issued when a block starts and consumed three rows before its
+  // end; its R+1 row pointers are then copied global -> shared with cp.async
+  // (no registers held in flight) while those rows gather; and the first
+  // index batch of the next row is always in flight while the current row
+  // gathers: in steady state a row costs one gather round trip.
+  __shared__ long long s_rp[8][2][32];  // per warp: this block's / the next block's row pointers
+  const int wib = threadIdx.x >> 5;
+  const int R = a.rows_per_ticket;
+  const int nblk_total = int((a.rows + R - 1) / R);
+  auto fetch_rp = [&](int blk, int b) {  // async copy of rowptr[blk*R .. blk*R+R] into s_rp[wib][b]
+    if (blk < nblk_total && lane <= R) {
+      const int64_t r = int64_t(blk) * R + lane;
+      const long long* src = reinterpret_cast<const long long*>(a.rowptr + (r < a.rows ? r : a.rows));
+      asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_addr(&s_rp[wib][b][lane])), "l"(src)
+                   : "memory");
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+  };
+  auto wait_rp = [&]() {
+    asm volatile("cp.async.wait_group 0;" ::: "memory");
+    __syncwarp();
+  };
+  int blk;
+  {
     int t = 0;
     if (lane == 0) t = atomicAdd(a.counter, 1);
-    return __shfl_sync(0xffffffffu, t, 0);
-  };
-  // software pipeline over rows: the next row's ticket, row pointers and
-  // first index batch are in flight while this row gathers
-  const bool ef = a.idx_evict_first;
-  int row = claim();
-  int64_t e0 = 0, e1 = 0;
-  if (row < a.rows) { e0 = a.rowptr[row]; e1 = a.rowptr[row + 1]; }
-  int pre = (e0 + lane < e1) ? ld_idx(a.col + e0 + lane, ef, pol) : 0;
-  while (row < a.rows) {
-    const int nxt = claim();
+    blk = __shfl_sync(0xffffffffu, t, 0);
+  }
+  int b = 0;
+  fetch_rp(blk, b);
+  wait_rp();
+  int pre = 0;
+  if (blk < nblk_total) {
+    const int64_t f0 = s_rp[wib][b][0], f1 = s_rp[wib][b][1];
+    pre = (f0 + lane < f1) ? ld_idx(a.col + f0 + lane) : 0;
+  }
+  while (blk < nblk_total) {
+    int tk = 0;
+    if (lane == 0) tk = atomicAdd(a.counter, 1);  // next block's ticket, consumed later
+    int nblk = nblk_total;
+    const int nr = int(a.rows - int64_t(blk) * R < R ? a.rows - int64_t(blk) * R : R);
+    const int ic = nr > 3 ? nr - 3 : 0;
+    for (int i = 0; i < nr; ++i) {
+    const int64_t row = int64_t(blk) * R + i;
+    if (i == ic) {
+      nblk = __shfl_sync(0xffffffffu, tk, 0);
+      fetch_rp(nblk, b ^ 1);
+    }
+    if (i + 1 == nr) wait_rp();
+    // edge ranges (re-read from shared memory, not kept live across the gather):
+    // this row [e0, e1) and the next row [n0, n1) (this block's, or the next block's first)
+    const int64_t e0 = s_rp[wib][b][i], e1 = s_rp[wib][b][i + 1];
     int64_t n0 = 0, n1 = 0;
-    if (nxt < a.rows) { n0 = a.rowptr[nxt]; n1 = a.rowptr[nxt + 1]; }
+    if (i + 1 < nr) {
+      n0 = e1;
+      n1 = s_rp[wib][b][i + 2];
+    } else if (nblk < nblk_total) {
+      n0 = s_rp[wib][b ^ 1][0];
+      n1 = s_rp[wib][b ^ 1][1];
+    }
     float4 tot[V];
     int pre_next;
+    // the epilogue's per-row scalars are loaded before the gather (in flight with it)
+    const float ri = a.r[a.row_lo + row];
+    const int zi = HAS_ZD ? a.zd_index[row] : -1;
     const int sg = HAS_SEG ? a.row_seg[row] : -1;
     if (HAS_SEG && sg >= 0) {
-      pre_next = (n0 + lane < n1) ? ld_idx(a.col + n0 + lane, ef, pol) : 0;
+      pre_next = (n0 + lane < n1) ? ld_idx(a.col + n0 + lane) : 0;
       const int ns = int((e1 - e0 + SEG_EDGES - 1) / SEG_EDGES);
 #pragma unroll
       for (int v = 0; v < V; ++v) tot[v] = make_float4(0.f, 0.f, 0.f, 0.f);
@@ -264,10 +301,8 @@ __global__ void __launch_bounds__(256, 4) sparse_row_kernel(AggArgs a) {
       }
     } else {
       pre_next = gather_sum<G, V>(a.col + e0, int(e1 - e0), pre, a.col + n0, int(n1 - n0), yb, rstride, lok,
-                                  lane, tot, ef, pol);
+                                  lane, tot);
     }
-    const float ri = a.r[a.row_lo + row];
-    const int zi = HAS_ZD ? a.zd_index[row] : -1;
     uint32_t bal[V][4];
 #pragma unroll
     for (int v = 0; v < V; ++v) {
@@ -289,29 +324,33 @@ __global__ void __launch_bounds__(256, 4) sparse_row_kernel(AggArgs a) {
       if (own) *reinterpret_cast<float4*>(a.Z + int64_t(row) * a.ldz + 4 * qv[v]) = z;
     }
     if (a.mask) {
-      // lane w assembles mask word w: column col = 32w + b lives in lane
-      // (col/4) % G, vector v = (col/4) / G, component col % 4
+      // lane w assembles mask word w: column col = 32w + 4k + c (k < 8) is
+      // float4 q = 8w + k, held by lane q % G of vector v = q / G, component
+      // c; bit q % G of bal[v][c].  The 8 q's of a word share one v (G >= 8,
+      // or a single word when G < 8), so the word interleaves four bytes:
+      // bit 4k + c = bit k of byte c.
       const int mw = (a.F + 31) >> 5;
       if (lane < mw) {
+        const int vv = (8 * lane) / G, l0 = (8 * lane) % G;
         uint32_t word = 0;
-#pragma unroll 4
-        for (int b = 0; b < 32; ++b) {
-          const int col = 32 * lane + b;
-          const int q = col >> 2;
-          const int vv = q / G, ll = q % G;
-          uint32_t bit = 0;
+#pragma unroll
+        for (int c = 0; c < 4; ++c) {
+          uint32_t x = 0;
 #pragma unroll
           for (int v = 0; v < V; ++v)
-            if (v == vv) bit = (bal[v][col & 3] >> ll) & 1u;
-          word |= bit << b;
+            if (v == vv) x = (bal[v][c] >> l0) & 0xffu;
+          x = (x | (x << 12)) & 0x000f000fu;  // spread bit k to bit 4k
+          x = (x | (x << 6)) & 0x03030303u;
+          x = (x | (x << 3)) & 0x11111111u;
+          word |= x << c;
         }
         a.mask[int64_t(row) * a.mask_ld + lane] = word;
       }
     }
-    row = nxt;
-    e0 = n0;
-    e1 = n1;
     pre = pre_next;
+    }
+    blk = nblk;
+    b ^= 1;
   }
 }
 
@@ -332,7 +371,7 @@ cudaError_t launch_gv(const AggArgs& a, cudaStream_t s) {
   }
   cudaError_t e = cudaMemsetAsync(a.counter, 0, sizeof(int), s);
   if (e != cudaSuccess) return e;
-  const int64_t want = (a.rows + 7) / 8;
+  const int64_t want = ((a.rows + a.rows_per_ticket - 1) / a.rows_per_ticket + 7) / 8;
   const unsigned grid = unsigned(want < slots ? want : slots);
 #define LAUNCH(ZD, SG) sparse_row_kernel<G, V, ZD, SG><<<grid, 256, 0, s>>>(a)
   const bool zd = a.zd_index != nullptr, sg = a.nseg > 0;
@@ -402,16 +441,14 @@ __global__ void __launch_bounds__(256) split_transpose_kernel(const float* __res
 
 cudaError_t launch_sparse_pass(const AggArgs& a, cudaStream_t s);
 
-// Tuning knobs read once (benchmarks only): PCGCN_SPARSE_FSPLIT=<cols> runs
+// Tuning knob read once (benchmarks only): PCGCN_SPARSE_FSPLIT=<cols> runs
 // the gather in column slices of that width (each slice of Y' is a smaller
-// L2 working set; the index stream is re-read per slice), and
-// PCGCN_IDX_EF=0/1 the L2 evict_first hint on the index stream.
+// L2 working set; the index stream is re-read per slice).  (An L2
+// evict_first hint on the index stream was measured and dropped: no gain.)
 struct SparseKnobs {
   int fsplit = 0;
-  bool idx_ef = false;
   SparseKnobs() {
     if (const char* e = getenv("PCGCN_SPARSE_FSPLIT")) fsplit = atoi(e) / 32 * 32;
-    if (const char* e = getenv("PCGCN_IDX_EF")) idx_ef = atoi(e) != 0;
   }
 };
 
@@ -426,7 +463,6 @@ cudaError_t launch_sparse_agg(const AggArgs& a0, cudaStream_t s) {
   if (a0.rows <= 0) return cudaSuccess;
   const SparseKnobs& kn = knobs();
   AggArgs a = a0;
-  a.idx_evict_first = kn.idx_ef;
   if (kn.fsplit <= 0 || a.F <= kn.fsplit) return launch_sparse_pass(a, s);
   for (int c0 = 0; c0 < a.F; c0 += kn.fsplit) {
     AggArgs b = a;
