@@ -13,6 +13,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cstdlib>
 #include <cstdint>
 
 #include "kernels.h"
@@ -115,6 +116,16 @@ __global__ void zero_pad_kernel(float* C, int64_t ldc, int64_t M, int N) {
     C[(i / w) * ldc + N + (i % w)] = 0.f;
 }
 
+// PCGCN_XTG_PRESPLIT=1: the feature-major split pass + engine instead of the
+// in-kernel conversion of D (A/B knob, benchmarks only)
+bool xtg_presplit() {
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("PCGCN_XTG_PRESPLIT");
+    v = e ? (atoi(e) != 0) : 0;
+  }
+  return v != 0;
+}
 int xtg_slices(int64_t M) { return int(std::min<int64_t>(296, std::max<int64_t>(1, (M + 1023) / 1024))); }
 
 }  // namespace
@@ -175,9 +186,15 @@ cudaError_t launch_gemm_xtg(const float* X, int64_t ldx, const float* D, int64_t
     float* hi = work;
     float* lo = work + int64_t(np) * ldT;
     float* part = lo + int64_t(np) * ldT;
-    cudaError_t e = launch_split_transpose(D, ldd, M, N, np, hi, lo, ldT, st);
-    if (e != cudaSuccess) return e;
-    e = launch_tc_gemm_xtg(X, ldx, hi, lo, ldT, part, M, K, N, st);
+    cudaError_t e;
+    if (np <= 128 && !xtg_presplit()) {
+      // B converted inside the engine (D read once; no split pass)
+      e = launch_tc_gemm_xtg_raw(X, ldx, D, ldd, part, M, K, N, st);
+    } else {
+      e = launch_split_transpose(D, ldd, M, N, np, hi, lo, ldT, st);
+      if (e != cudaSuccess) return e;
+      e = launch_tc_gemm_xtg(X, ldx, hi, lo, ldT, part, M, K, N, st);
+    }
     if (e != cudaSuccess) return e;
     const int64_t cnt = int64_t(K) * N;
     reduce_slices_ld_kernel<<<unsigned(std::max<int64_t>(1, std::min<int64_t>(1024, (cnt + 255) / 256))), 256, 0, st>>>(

@@ -83,6 +83,8 @@ cudaError_t launch_tc_gemm_xw(const float* X, int64_t ldx, const float* wThi, co
                               const float* rs, float* Y, int64_t ldy, int64_t M, int K, int N, cudaStream_t s,
                               const uint32_t* mask = nullptr, int64_t mask_ld = 0);
 int64_t tc_xtg_slices(int64_t M, int K);
+cudaError_t launch_tc_gemm_xtg_raw(const float* X, int64_t ldx, const float* D, int64_t ldd, float* partial,
+                                   int64_t M, int K, int N, cudaStream_t s);
 cudaError_t launch_tc_gemm_xtg(const float* X, int64_t ldx, const float* dThi, const float* dTlo, int64_t lddT,
                                float* partial, int64_t M, int K, int N, cudaStream_t s);
 int64_t gemm_xtg_work_floats(int64_t M, int K, int N);

@@ -13,22 +13,23 @@
 namespace pcgcn {
 namespace {
 
-constexpr int CE_BLOCKS = 592;  // 4 x 148 SMs; <= PCGCN_CE_WORK_FLOATS
+constexpr int CE_BLOCKS = 592;  // 4 x 148 SMs, all resident (launch bounds: 4 CTAs/SM); <= PCGCN_CE_WORK_FLOATS
 
 // one warp per row, RPW rows per warp step with all their loads issued up
 // front (a row is short: C <= 32*8 logits; at C5's 33.5M rows one row per
 // step left the kernel latency-bound, ~11.6 ms); grid-stride over row groups.
 constexpr int RPW = 4;
-__global__ void __launch_bounds__(256) softmax_ce_kernel(
+template <int NT>  // 32-logit slices per row (C <= 32 * NT)
+__global__ void __launch_bounds__(256, 4) softmax_ce_kernel(
     const float* __restrict__ L, int64_t ld, const int32_t* __restrict__ labels,
     const uint8_t* __restrict__ train, int64_t M, int C, float inv_nT, const float* __restrict__ s,
     float* __restrict__ dL, float* __restrict__ partial) {
   __shared__ float wsum[8];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-  const int nt = (C + 31) >> 5;
+  constexpr int nt = NT;
   float my = 0.f;  // lane 0 of each warp accumulates its rows' losses in row order
   for (int64_t row0 = (int64_t(blockIdx.x) * 8 + w) * RPW; row0 < M; row0 += int64_t(gridDim.x) * 8 * RPW) {
-    float v[RPW][8];
+    float v[RPW][NT];
     int y[RPW];
     float scale[RPW];
     bool tr[RPW];
@@ -38,9 +39,9 @@ __global__ void __launch_bounds__(256) softmax_ce_kernel(
       const bool ok = row < M;
       const float* Lr = L + row * ld;
 #pragma unroll
-      for (int t = 0; t < 8; ++t) {
+      for (int t = 0; t < NT; ++t) {
         const int c = lane + 32 * t;
-        v[k][t] = (ok && t < nt && c < C) ? __ldg(Lr + c) : -INFINITY;
+        v[k][t] = (ok && c < C) ? __ldg(Lr + c) : -INFINITY;
       }
       y[k] = ok ? __ldg(labels + row) : 0;
       tr[k] = ok && __ldg(train + row) != 0;
@@ -51,15 +52,15 @@ __global__ void __launch_bounds__(256) softmax_ce_kernel(
       const int64_t row = row0 + k;
       float mx = -INFINITY;
 #pragma unroll
-      for (int t = 0; t < 8; ++t) mx = fmaxf(mx, v[k][t]);
+      for (int t = 0; t < NT; ++t) mx = fmaxf(mx, v[k][t]);
 #pragma unroll
       for (int off = 16; off; off >>= 1) mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, off));
       float se = 0.f, ly = 0.f;
 #pragma unroll
-      for (int t = 0; t < 8; ++t) {
+      for (int t = 0; t < NT; ++t) {
         const int c = lane + 32 * t;
         if (c == y[k]) ly = v[k][t];
-        v[k][t] = (t < nt && c < C) ? expf(v[k][t] - mx) : 0.f;
+        v[k][t] = c < C ? expf(v[k][t] - mx) : 0.f;
         se += v[k][t];
       }
 #pragma unroll
@@ -71,9 +72,9 @@ __global__ void __launch_bounds__(256) softmax_ce_kernel(
         const float sc = (tr[k] ? inv_nT : 0.f) * scale[k];
         const float inv = 1.f / se;
 #pragma unroll
-        for (int t = 0; t < 8; ++t) {
+        for (int t = 0; t < NT; ++t) {
           const int c = lane + 32 * t;
-          if (t < nt && c < C) dL[row * ld + c] = (v[k][t] * inv - (c == y[k] ? 1.f : 0.f)) * sc;
+          if (c < C) dL[row * ld + c] = (v[k][t] * inv - (c == y[k] ? 1.f : 0.f)) * sc;
         }
         if (lane == 0 && tr[k]) my += (mx + logf(se) - ly);
       }
@@ -133,7 +134,11 @@ cudaError_t launch_softmax_ce(const float* L, int64_t ld, const int32_t* labels,
                               const uint8_t* train, int64_t M, int C, float inv_nT, const float* s,
                               float* dL, float* loss, float* work, cudaStream_t st) {
   if (C > 256) return cudaErrorInvalidValue;
-  softmax_ce_kernel<<<CE_BLOCKS, 256, 0, st>>>(L, ld, labels, train, M, C, inv_nT, s, dL, work);
+  const int nt = (C + 31) / 32;
+  if (nt <= 1) softmax_ce_kernel<1><<<CE_BLOCKS, 256, 0, st>>>(L, ld, labels, train, M, C, inv_nT, s, dL, work);
+  else if (nt <= 2) softmax_ce_kernel<2><<<CE_BLOCKS, 256, 0, st>>>(L, ld, labels, train, M, C, inv_nT, s, dL, work);
+  else if (nt <= 4) softmax_ce_kernel<4><<<CE_BLOCKS, 256, 0, st>>>(L, ld, labels, train, M, C, inv_nT, s, dL, work);
+  else softmax_ce_kernel<8><<<CE_BLOCKS, 256, 0, st>>>(L, ld, labels, train, M, C, inv_nT, s, dL, work);
   finish_loss_kernel<<<1, 1024, 0, st>>>(work, CE_BLOCKS, inv_nT, loss);
   return cudaGetLastError();
 }

@@ -53,22 +53,28 @@ using namespace tc;
 // issue bookkeeping are paid once per U chunks.
 struct Layout {
   int npad, stages, nacc, U, a_cols;  // a_cols: TMEM columns of one A stage (U*32, or 64 for hi+lo)
+  uint32_t out_bytes;                 // A_ROWMAJOR: epilogue staging (4 warps x 32 rows x (64+4) floats)
+  uint32_t raw_bytes;                 // A_TRANS + raw B: one row-major [32 x npad] D box per stage
   int gst;                            // stages per TMEM accumulation group (<= 8 chunks)
   uint32_t a_bytes, b_bytes, stage_bytes, a_load_bytes;  // b_bytes: ONE chunk of ONE operand
   uint32_t tmem_cols, a_col0;
 };
 
-Layout make_layout(int mode, int npad, int max_stages, int max_u) {
+Layout make_layout(int mode, int npad, int max_stages, int max_u, bool b_raw = false) {
   Layout L;
+  L.raw_bytes = (mode == A_TRANS && b_raw) ? uint32_t(npad) * BK * 4 : 0u;
   L.npad = npad;
   L.b_bytes = uint32_t(npad) * BK * 4;
+  // transform GEMM outputs (N x npad rows, HBM-bound at scale) leave through a
+  // shared-memory transpose so each store instruction writes whole row pieces
+  L.out_bytes = (mode == A_ROWMAJOR && npad <= 128) ? 4u * 32u * (64u + 4u) * 4u : 0u;
   for (int U = (mode == A_BITS ? max_u : 1); U >= 1; U = U > 1 ? U / 2 : 0) {
     L.U = U;
     L.a_cols = mode == A_BITS ? U * BK : 2 * BK;
     L.a_bytes = mode == A_BITS ? uint32_t((U * BM * 4 + 1023) / 1024 * 1024) : BM * BK * 4;
     L.a_load_bytes = mode == A_BITS ? BM * 4 : BM * BK * 4;  // per chunk
-    L.stage_bytes = L.a_bytes + 2 * uint32_t(U) * L.b_bytes;
-    int st = int((200 * 1024) / L.stage_bytes);
+    L.stage_bytes = L.a_bytes + 2 * uint32_t(U) * L.b_bytes + L.raw_bytes;
+    int st = int((200 * 1024 - L.out_bytes) / L.stage_bytes);
     st = st > max_stages ? max_stages : st;
     L.nacc = 2;
     while (st >= 2 && L.nacc * npad + st * L.a_cols > 512) {
@@ -117,6 +123,8 @@ struct Work {
   int64_t split_stride;
   int b_fused;       // B lo rows follow the hi rows in memory: one TMA box {32, 2*npad} per chunk
   int single;        // A_BITS: B hi only (bf16-rounded input), one MMA per K-step (PCGCN_DENSE_BF16X1)
+  int b_raw;         // A_TRANS: B = row-major D box; the builders split + transpose it into the
+                     // K-major SWIZZLE_128B hi/lo layout in smem (no feature-major pre-split pass)
 };
 
 template <int MODE>
@@ -149,7 +157,8 @@ __global__ void __launch_bounds__(NTHREADS, 1)
                      const __grid_constant__ CUtensorMap map_a, const Work w, const Layout L) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-  uint64_t* bar = reinterpret_cast<uint64_t*>(smem + L.stages * L.stage_bytes);
+  float* stage_out = reinterpret_cast<float*>(smem + L.stages * L.stage_bytes);
+  uint64_t* bar = reinterpret_cast<uint64_t*>(smem + L.stages * L.stage_bytes + L.out_bytes);
   uint64_t* full = bar;                     // [stages] A + B landed
   uint64_t* a_full = bar + L.stages;        // [stages] A written to TMEM (128 arrivals)
   uint64_t* empty = bar + 2 * L.stages;     // [stages] MMAs done with the stage
@@ -194,7 +203,8 @@ __global__ void __launch_bounds__(NTHREADS, 1)
           const int nu = int(nch - i < L.U ? nch - i : L.U);
           mbar_wait(&empty[s], ph ^ 1u);
           uint8_t* st = smem + s * L.stage_bytes;
-          mbar_expect_tx(&full[s], uint32_t(nu) * (L.a_load_bytes + (w.single ? 1u : 2u) * L.b_bytes));
+          mbar_expect_tx(&full[s], uint32_t(nu) * (L.a_load_bytes +
+                                                   (w.b_raw ? L.raw_bytes : (w.single ? 1u : 2u) * L.b_bytes)));
           // the bits of a tile's chunks are contiguous: one bulk copy per stage
           if (MODE == A_BITS) bulk_load(st, w.bits + (kb + i) * BM, uint32_t(nu) * BM * 4, &full[s]);
           for (int u = 0; u < nu; ++u) {
@@ -210,7 +220,10 @@ __global__ void __launch_bounds__(NTHREADS, 1)
             }
             // chunk u's B tile in smem: [hi: npad rows][lo: npad rows] x 128 B
             uint8_t* bdst = st + L.a_bytes + u * 2 * L.b_bytes;
-            if (w.b_fused || w.single) {
+            if (MODE == A_TRANS && w.b_raw) {
+              // row-major D rows [k0, k0+32) x features [0, npad) (OOB columns zero-filled)
+              tma_load_2d(&map_bhi, &full[s], st + L.a_bytes + 2 * L.b_bytes, 0, k0);
+            } else if (w.b_fused || w.single) {
               tma_load_2d(&map_bhi, &full[s], bdst, k0, 0);  // one box {32, 2*npad}: hi rows then lo rows
             } else {
               tma_load_2d(&map_bhi, &full[s], bdst, k0, 0);
@@ -316,6 +329,34 @@ __global__ void __launch_bounds__(NTHREADS, 1)
           }
           sttm32(taddr, v);
           sttm32(taddr + BK, lo);
+          if (MODE == A_TRANS && w.b_raw && m < npad) {
+            // B: thread m owns feature m; raw[k][m] (k = 32 rows of the chunk)
+            // -> hi/lo rows m of the K-major SWIZZLE_128B tiles: 16-byte chunk
+            // j (k = 4j..4j+3) of row m lives at m*128 + ((j ^ (m & 7)) * 16)
+            const float* raw = reinterpret_cast<const float*>(st + L.a_bytes + 2 * L.b_bytes);
+            uint8_t* bh = const_cast<uint8_t*>(st) + L.a_bytes;
+            uint8_t* bl = bh + L.b_bytes;
+#pragma unroll
+            for (int j = 0; j < 8; ++j) {
+              float4 h4, l4;
+              float xv[4];
+#pragma unroll
+              for (int e = 0; e < 4; ++e) xv[e] = raw[(4 * j + e) * npad + m];
+              float hv[4], lv[4];
+#pragma unroll
+              for (int e = 0; e < 4; ++e) {
+                hv[e] = __uint_as_float(__float_as_uint(xv[e]) & 0xffffe000u);
+                lv[e] = xv[e] - hv[e];
+              }
+              h4 = make_float4(hv[0], hv[1], hv[2], hv[3]);
+              l4 = make_float4(lv[0], lv[1], lv[2], lv[3]);
+              const uint32_t off = uint32_t(m) * 128u + uint32_t((j ^ (m & 7)) * 16);
+              *reinterpret_cast<float4*>(bh + off) = h4;
+              *reinterpret_cast<float4*>(bl + off) = l4;
+            }
+            // generic-proxy smem writes -> visible to the tensor core (async proxy)
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+          }
         }
         asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
         tc_fence_before();
@@ -384,10 +425,38 @@ __global__ void __launch_bounds__(NTHREADS, 1)
         tc_fence_before();
         mbar_arrive(&acc_empty[ab]);
       }
-      if (live) {
-        const uint32_t* mrow = (MODE == A_ROWMAJOR && w.mask) ? w.mask + row * w.mask_ld : nullptr;
+      // (all 32 lanes take the staged path: rows past M are written to smem
+      // only, never to global)
+      if (live || (NPC > 0 && MODE == A_ROWMAJOR && L.out_bytes)) {
+        const uint32_t* mrow = (MODE == A_ROWMAJOR && w.mask && live) ? w.mask + row * w.mask_ld : nullptr;
         auto mk = [&](int c) { return mrow ? ((mrow[c >> 5] >> (c & 31)) & 1u ? sc : 0.f) : sc; };
-        if (NPC > 0) {
+        if (NPC > 0 && MODE == A_ROWMAJOR && L.out_bytes) {
+          // staged store: each thread holds one row; 64-column halves go
+          // through this warp's [32 rows][68] smem tile and leave as two rows
+          // of 16 float4 per store instruction (whole 256-byte row pieces)
+          float* sb = stage_out + (warp & 3) * 32 * 68;
+          const int64_t rbase = m0 + ((warp & 3) << 5);
+#pragma unroll
+          for (int h = 0; h < (NPC > 0 ? NPC : 1); h += 64) {
+#pragma unroll
+            for (int c = 0; c < 64; c += 4)
+              if (h + c < (NPC > 0 ? NPC : 1))
+                *reinterpret_cast<float4*>(sb + lane * 68 + c) =
+                    make_float4(racc[h + c] * mk(h + c), racc[h + c + 1] * mk(h + c + 1),
+                                racc[h + c + 2] * mk(h + c + 2), racc[h + c + 3] * mk(h + c + 3));
+            __syncwarp();
+            const int q = lane & 15;
+#pragma unroll 4
+            for (int r = 0; r < 32; r += 2) {
+              const int rr = r + (lane >> 4);
+              const int64_t grow = rbase + rr;
+              if (grow < w.mdim && h + 4 * q < w.ncols)
+                *reinterpret_cast<float4*>(w.out + grow * w.ldo + h + 4 * q) =
+                    *reinterpret_cast<const float4*>(sb + rr * 68 + 4 * q);
+            }
+            __syncwarp();
+          }
+        } else if (NPC > 0) {
 #pragma unroll
           for (int c0 = 0; c0 < (NPC > 0 ? NPC : 1); c0 += 4)
             if (c0 < w.ncols)
@@ -490,8 +559,8 @@ template <int MODE>
 cudaError_t launch_engine(const CUtensorMap& bhi, const CUtensorMap& blo, const CUtensorMap& amap, const Work& w,
                           int npad, cudaStream_t s) {
   if (w.ntiles <= 0) return cudaSuccess;
-  const Layout L = make_layout(MODE, npad, max_stages_env(), max_u_env());
-  const size_t smem = 1024 + size_t(L.stages) * L.stage_bytes + (3 * L.stages + 4) * 8 + 16;
+  const Layout L = make_layout(MODE, npad, max_stages_env(), max_u_env(), w.b_raw != 0);
+  const size_t smem = 1024 + size_t(L.stages) * L.stage_bytes + L.out_bytes + (3 * L.stages + 4) * 8 + 16;
   if (smem > 227 * 1024) return cudaErrorInvalidValue;
   static int grid_cap = -1;  // PCGCN_TC_GRID: full-mode CTAs (tuning override, benchmarks only)
   if (grid_cap < 0) {
@@ -584,6 +653,31 @@ int64_t tc_xtg_slices(int64_t M, int K) {
   sl = sl < cap ? sl : cap;
   return sl < 1 ? 1 : (sl > 148 ? 148 : sl);
 }
+// ---- partial[sp] = X[rows of slice sp]ᵀ · D with D row-major (ld ldd, N <= 128):
+//      B converted in the kernel (no split pass; D read once from HBM) ----
+cudaError_t launch_tc_gemm_xtg_raw(const float* X, int64_t ldx, const float* D, int64_t ldd, float* partial,
+                                   int64_t M, int K, int N, cudaStream_t s) {
+  const int npad = (N + 15) / 16 * 16;
+  if (ldx % 4 || ldd % 4 || npad > 128) return cudaErrorInvalidValue;
+  CUtensorMap mr, ma;
+  // D as a [M x N] tensor (row pitch ldd): the box {npad, 32} zero-fills columns >= N
+  if (!make_map(&mr, D, N, M, ldd, npad, BK, false) || !make_map(&ma, X, K, M, ldx, BM, BK, false))
+    return cudaErrorInvalidValue;
+  const int64_t ns = tc_xtg_slices(M, K);
+  Work w{};
+  w.mtiles = (K + BM - 1) / BM;
+  w.ntiles = int64_t(w.mtiles) * ns;
+  w.kdim = M;
+  w.kslice = ((M + ns - 1) / ns + BK - 1) / BK * BK;
+  w.mdim = K;
+  w.out = partial;
+  w.ldo = npad;
+  w.ncols = npad;
+  w.split_stride = int64_t(K) * npad;
+  w.b_raw = 1;
+  return launch_engine<A_TRANS>(mr, mr, ma, w, npad, s);
+}
+
 cudaError_t launch_tc_gemm_xtg(const float* X, int64_t ldx, const float* dThi, const float* dTlo, int64_t lddT,
                                float* partial, int64_t M, int K, int N, cudaStream_t s) {
   const int npad = (N + 15) / 16 * 16;

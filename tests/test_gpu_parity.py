@@ -520,3 +520,78 @@ def test_epoch_parity_deep(wname, theta, nl):
         assert rel(_np(model.gTh[l]).ravel(), grads[l].ravel()) < 1e-4, l
         step = (Ths[l].astype(np.float64) - _np(model.Th[l])) / 0.1          # the SGD update applied
         assert rel(step.ravel(), grads[l].ravel()) < 1e-3, l
+
+
+_KNOB_CODE = r'''
+import sys, numpy as np, torch
+sys.path.insert(0, ".")
+from paper_conf_ipps_tianmyd20_b200 import _lib as L
+from paper_conf_ipps_tianmyd20_b200.gcn import GCN2
+from synth import configs as C, graphs as G
+out = {}
+# selective rows of every length class (hub rows with long-row segments, short
+# rows) next to dense tiles (cliques)
+edges, base = [], 0
+for leaves in (5000, 1100, 2047, 1025):
+    edges += [(base, base + i) for i in range(1, leaves + 1)]
+    base += leaves + 1
+for sz in (300, 200, 129, 64):
+    ii, jj = np.triu_indices(sz, 1)
+    edges += list(zip((base + ii).tolist(), (base + jj).tolist()))
+    base += sz
+e = np.random.default_rng(7).integers(0, base, size=(3 * base, 2))
+edges += [tuple(x) for x in e.tolist() if x[0] != x[1]]
+g = G.from_edges(base, edges)
+rng = np.random.default_rng(11)
+for F, theta in ((128, 0.02), (41, 0.04), (32, 2.0)):
+    pl = L.Plan(g.n, g.rowptr, g.col, 8, theta)
+    Y = torch.from_numpy(rng.standard_normal((g.n, (F + 3) // 4 * 4)).astype(np.float32)).cuda()
+    Z = torch.zeros_like(Y)
+    M = torch.zeros(g.n, (F + 31) // 32, dtype=torch.int32, device="cuda")
+    pl.forward(Y, Z, F=F, flags=L.RELU | L.MASK_OUT, mask=M)
+    torch.cuda.synchronize()
+    out[f"agg{F}"] = Z.cpu().numpy()
+    out[f"mask{F}"] = M.cpu().numpy()
+# one epoch (the xtg / dwt GEMMs included)
+w = C.PUBMED
+gp = C.graph(w)
+X = C.features(w, gp.n)
+Th0, Th1 = C.thetas(w)
+T = C.train_mask(gp.n, w.theta_seed)
+pl = L.Plan(gp.n, gp.rowptr, gp.col, w.P, 0.02)
+perm = pl.perm()
+m = GCN2(pl, X[perm], gp.labels[perm], T[perm], Th0, Th1, optimizer="sgd", lr=0.1)
+m.epoch()
+torch.cuda.synchronize()
+out["gTh0"] = m.gTh0.cpu().numpy()
+out["gTh1"] = m.gTh1.cpu().numpy()
+out["loss"] = np.array([m.loss.item()])
+np.savez(sys.argv[1], **out)
+'''
+
+
+@pytest.mark.parametrize("knob,bitwise", [({"PCGCN_ROWS_PER_TICKET": "1"}, True),
+                                          ({"PCGCN_ROWS_PER_TICKET": "16"}, True),
+                                          ({"PCGCN_OVERLAP": "1"}, True),
+                                          ({"PCGCN_XTG_PRESPLIT": "1"}, True)])
+def test_scheduling_knobs_do_not_change_results(tmp_path, knob, bitwise):
+    """Row-block tickets, the full-mode/segment overlap and the in-kernel xtg
+    B conversion change only scheduling (every output row is still reduced by
+    one warp in the same order; the MMA sequence and the hi/lo split are the
+    same), so aggregation outputs, masks, gradients and the loss must be
+    bitwise identical to the default configuration."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    res = {}
+    for tag, extra in (("default", {}), ("knob", knob)):
+        env = {k: v for k, v in os.environ.items() if not k.startswith("PCGCN_")}
+        env.update(extra)
+        f = str(tmp_path / f"{tag}.npz")
+        subprocess.run([sys.executable, "-c", _KNOB_CODE, f], check=True, env=env, cwd=root, capture_output=True,
+                       text=True, timeout=600)
+        res[tag] = np.load(f)
+    for k in res["default"].files:
+        a, b = res["default"][k], res["knob"][k]
+        assert np.array_equal(a, b), (knob, k, float(np.max(np.abs(a.astype(np.float64) - b))))
