@@ -633,13 +633,14 @@ def main():
         tc_peak = float(json.load(open(MEASURED_PEAKS))["bf16_tflops"]) / 2
     except Exception:
         tc_peak = 1590.0 / 2
-    traffic = l2_read = None
+    traffic = l2_read = lts_pct = None
     tpath = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tpath):
         try:
             tj = json.load(open(tpath)).get(w.name, {})
             traffic = tj.get("sparse_agg_F%d" % w.hidden)
             l2_read = tj.get("sparse_agg_F%d_l2_read_bytes" % w.hidden)
+            lts_pct = tj.get("sparse_agg_F%d_lts_pct" % w.hidden)
         except Exception:
             traffic = None
 
@@ -801,10 +802,14 @@ def main():
                          "traffic_source": "profiles/traffic.json (ncu --set full, dram read+write per launch)",
                          "l2_view": {"l2_read_bytes": l2_read,
                                      "achieved": (l2_read / (t_sp * 1e-3) / 1e9) if l2_read else None,
-                                     "peak": l2_gbs, "unit": "GB/s",
-                                     "frac": (l2_read / (t_sp * 1e-3) / 1e9 / l2_gbs) if l2_read else None,
+                                     "unit": "GB/s",
+                                     "ncu_lts_throughput_pct": lts_pct,
                                      "bytes_source": "ncu lts__t_sectors_srcunit_tex_op_read x 32 per launch "
-                                                     "(profiles/traffic.json); the L1 serves the rest of the gather",
+                                                     "(profiles/traffic.json); ncu_lts_throughput_pct = the L2's "
+                                                     "own %-of-peak (lts__throughput), time-weighted over the pass",
+                                     "probe_peak": l2_gbs,
+                                     "probe_note": "streaming-read probe; the gather's L2->L1 rate exceeds it "
+                                                   "(partition-ordered rows), so the ncu % is the L2 roofline",
                                      "gather_bytes": st["shard_nnz_sparse"] * fp4 * 4,
                                      "gather_GBs": gather,
                                      "peak_source": "measured: max of pcgcn_probe_read_gbs over 16-64 MiB L2-resident buffers, 3 reps each"},

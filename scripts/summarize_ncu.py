@@ -115,6 +115,12 @@ def main(csv_path, rep_path, out_path):
                     l2 += 32.0 * float(d[hdr.index(m)].replace(",", "")) * scale.get(units[hdr.index(m)], 1)
             tr[key] = int(tot)
             tr[key + "_l2_read_bytes"] = int(l2) if l2 else None
+            # time-weighted L2 (LTS) throughput, % of its sustained peak (ncu's own roofline of the L2)
+            m, tm = "lts__throughput.avg.pct_of_peak_sustained_elapsed", "gpu__time_duration.sum"
+            if m in hdr and tm in hdr:
+                ts = [float(d[hdr.index(tm)].replace(",", "")) for d in grp]
+                ps = [float(d[hdr.index(m)].replace(",", "")) for d in grp]
+                tr[key + "_lts_pct"] = round(sum(t * p for t, p in zip(ts, ps)) / max(sum(ts), 1e-30), 2)
             tr[key + "_kernels"] = [short(d[hdr.index("Kernel Name")]) for d in grp]
         tr["source"] = rep_path
         tp = os.path.join(os.path.dirname(out_path), "traffic.json")
