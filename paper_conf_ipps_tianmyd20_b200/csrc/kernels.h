@@ -65,7 +65,12 @@ struct DenseArgs {
   float* zd;                 // [nrt*128 x ldzd]
   int64_t ldzd;
   int npad;                  // UMMA N (multiple of 16, >= F)
+  const int32_t* rt_order = nullptr;  // engine tile order (position i of CTA b: tile rt_order[b + i*G])
+  const float* blk = nullptr;  // source-window blocks (launch_split_windows); nullptr: hiT/loT maps
+  int64_t blk_floats = 0;      // floats per window block
 };
+cudaError_t launch_split_windows(const float* Y, int64_t ldy, int64_t n, int F, int npad, bool single, float* blk,
+                                 int64_t nwin, cudaStream_t s);
 cudaError_t launch_dense_tc(const DenseArgs& a, cudaStream_t s);
 // CTA-pair (cta_group::2) variant of the full mode (tc_pair.cu); map_b covers [hi rows; lo rows]
 bool dense_pair_eligible(int npad);

@@ -26,7 +26,6 @@ __global__ void __launch_bounds__(256, 4) softmax_ce_kernel(
     float* __restrict__ dL, float* __restrict__ partial) {
   __shared__ float wsum[8];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-  constexpr int nt = NT;
   float my = 0.f;  // lane 0 of each warp accumulates its rows' losses in row order
   for (int64_t row0 = (int64_t(blockIdx.x) * 8 + w) * RPW; row0 < M; row0 += int64_t(gridDim.x) * 8 * RPW) {
     float v[RPW][NT];

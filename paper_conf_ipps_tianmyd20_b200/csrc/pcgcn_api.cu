@@ -111,6 +111,29 @@ pcgcn_status upload_plan(pcgcn_plan_s* p) {
     std::vector<int64_t> cp(d.nrt + 1);
     for (int64_t t = 0; t <= d.nrt; ++t) cp[t] = p->rt_cptr[p->rt_lo + t] - ch_lo;
     UP(&d.rt_cptr, cp.data(), d.nrt + 1);
+    {
+      // engine tile order: largest tiles first, dealt to the persistent CTAs
+      // in snake order (CTA b takes positions b, 2G-1-b, 2G+b, ...), so the
+      // static round-robin of the engine sees balanced chunk counts (plain
+      // plan order left 8-18% of the full mode in the slowest CTA on C3)
+      int dev = 0, sms = 148;
+      cudaGetDevice(&dev);
+      cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+      const int64_t G = std::min<int64_t>(d.nrt, sms > 0 ? sms : 148);
+      std::vector<int32_t> bysize(d.nrt);
+      for (int64_t t = 0; t < d.nrt; ++t) bysize[t] = int32_t(t);
+      std::stable_sort(bysize.begin(), bysize.end(), [&](int32_t a, int32_t b) {
+        return cp[a + 1] - cp[a] > cp[b + 1] - cp[b];
+      });
+      std::vector<int32_t> order(d.nrt);
+      for (int64_t i = 0; i < d.nrt; ++i) {
+        const int64_t round = i / G, k = i % G;
+        const bool full_round = (round + 1) * G <= d.nrt;  // a partial last round stays in forward order
+        const int64_t b = ((round & 1) && full_round) ? G - 1 - k : k;  // CTA receiving the i-th largest tile
+        order[round * G + b] = bysize[i];
+      }
+      UP(&d.rt_order, order.data(), d.nrt);
+    }
     UP(&d.ch_col0, p->ch_col0.data() + ch_lo, d.nch);
     UP(&d.bits, p->bits.data() + ch_lo * TILE_M, d.nch * TILE_M);
     UP(&d.zd, (float*)nullptr, d.nrt * TILE_M * d.fpad_max);
@@ -176,6 +199,17 @@ bool overlap_enabled() {
   if (v < 0) {
     const char* e = getenv("PCGCN_OVERLAP");
     v = e ? (atoi(e) != 0) : 0;
+  }
+  return v != 0;
+}
+
+// PCGCN_DENSE_BLOCKED=0: full-mode B through strided TMA boxes of the
+// feature-major split instead of window blocks (A/B knob, benchmarks only)
+bool dense_blocked_enabled() {
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("PCGCN_DENSE_BLOCKED");
+    v = e ? (atoi(e) != 0) : 1;
   }
   return v != 0;
 }
@@ -268,9 +302,14 @@ pcgcn_status aggregate(pcgcn_plan_t p, const float* Y, int64_t ldy, float* Z, in
     ms = side;
   }
   float* ylo = d.yhi ? d.yhi + int64_t(npad) * d.n_pad : nullptr;
+  // full mode's B: source-window blocks fetched by one bulk copy per chunk
+  // (default), or the feature-major split read by strided TMA boxes (the
+  // CTA-pair kernel, or PCGCN_DENSE_BLOCKED=0)
+  const bool blocked = tc && dense_blocked_enabled() && !dense_pair_eligible(npad);
   if (dense && tc) {
     if (prof) d.ev_used[1] = true;
-    e = launch_split_transpose(src, ldsrc, p->n, F, npad, d.yhi, bf16 ? nullptr : ylo, d.n_pad, ms);
+    e = blocked ? launch_split_windows(src, ldsrc, p->n, F, npad, bf16, d.yhi, d.n_pad / 32, ms)
+                : launch_split_transpose(src, ldsrc, p->n, F, npad, d.yhi, bf16 ? nullptr : ylo, d.n_pad, ms);
     if (e != cudaSuccess) return cuda_fail(e, "split_transpose");
   }
   mark(2);
@@ -278,6 +317,11 @@ pcgcn_status aggregate(pcgcn_plan_t p, const float* Y, int64_t ldy, float* Z, in
     if (prof) d.ev_used[2] = true;
     DenseArgs da{d.yhi, bf16 ? nullptr : ylo, d.n_pad, d.n_pad, d.rt_row0, d.rt_nrows, d.rt_cptr, d.ch_col0,
                  d.bits, d.nrt, d.zd, npad, npad};
+    da.rt_order = d.rt_order;
+    if (blocked) {
+      da.blk = d.yhi;
+      da.blk_floats = int64_t(bf16 ? 1 : 2) * npad * 32;
+    }
     e = tc ? launch_dense_tc(da, ms) : launch_dense_simt_y(da, src, ldsrc, F, ms);
     if (e != cudaSuccess) return cuda_fail(e, "dense-mode kernel");
   }

@@ -437,7 +437,55 @@ __global__ void __launch_bounds__(256) split_transpose_kernel(const float* __res
   }
 }
 
+// tf32 split of the (prescaled) input into source-window blocks for the full
+// mode's B operand: window w (sources 32w..32w+31) is one contiguous block of
+// R = 2*npad rows (hi rows 0..npad-1, lo rows npad..2npad-1; R = npad for the
+// bf16-rounded single mode) x 32 sources, each 128-byte row stored already in
+// the UMMA K-major SWIZZLE_128B image (16-byte chunk j of row r at j ^ (r & 7)),
+// so the engine fetches a chunk's whole B with one contiguous bulk copy
+// instead of an R-row strided TMA box.  Sources >= n and features >= F are 0.
+__global__ void __launch_bounds__(256) split_window_kernel(const float* __restrict__ Y, int64_t ldy, int64_t n,
+                                                           int F, int npad, bool single,
+                                                           float* __restrict__ blk) {
+  __shared__ float tile[32][33];
+  const int64_t w = blockIdx.x;
+  const int f0 = blockIdx.y * 32;
+  const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5;  // 32 x 8
+  for (int rr = ty; rr < 32; rr += 8) {
+    const int64_t j = w * 32 + rr;
+    const int f = f0 + tx;
+    tile[rr][tx] = (j < n && f < F) ? __ldg(Y + j * ldy + f) : 0.f;
+  }
+  __syncthreads();
+  const int R = single ? npad : 2 * npad;
+  float* out = blk + w * int64_t(R) * 32;
+  const int k = tx;  // source within the window
+  for (int ff = ty; ff < 32; ff += 8) {
+    const int f = f0 + ff;
+    if (f >= npad) continue;
+    const float v = tile[k][ff];
+    if (!single) {
+      const float h = __uint_as_float(__float_as_uint(v) & 0xffffe000u);
+      const int rh = f, rl = npad + f;
+      out[rh * 32 + ((((k >> 2) ^ (rh & 7)) << 2) | (k & 3))] = h;
+      out[rl * 32 + ((((k >> 2) ^ (rl & 7)) << 2) | (k & 3))] = v - h;
+    } else {  // bf16 round-to-nearest-even (BF16X1 full mode); exact in tf32
+      uint32_t u = __float_as_uint(v);
+      u = (u + 0x7fffu + ((u >> 16) & 1u)) & 0xffff0000u;
+      out[f * 32 + ((((k >> 2) ^ (f & 7)) << 2) | (k & 3))] = __uint_as_float(u);
+    }
+  }
+}
+
 }  // namespace
+
+cudaError_t launch_split_windows(const float* Y, int64_t ldy, int64_t n, int F, int npad, bool single, float* blk,
+                                 int64_t nwin, cudaStream_t s) {
+  if (nwin <= 0) return cudaSuccess;
+  dim3 grid(unsigned(nwin), unsigned((npad + 31) / 32));
+  split_window_kernel<<<grid, 256, 0, s>>>(Y, ldy, n, F, npad, single, blk);
+  return cudaGetLastError();
+}
 
 cudaError_t launch_sparse_pass(const AggArgs& a, cudaStream_t s);
 

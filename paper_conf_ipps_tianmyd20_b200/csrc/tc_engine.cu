@@ -123,6 +123,9 @@ struct Work {
   int64_t split_stride;
   int b_fused;       // B lo rows follow the hi rows in memory: one TMA box {32, 2*npad} per chunk
   int single;        // A_BITS: B hi only (bf16-rounded input), one MMA per K-step (PCGCN_DENSE_BF16X1)
+  const int32_t* order;  // A_BITS: tile processed at position t (nullptr: t itself)
+  const float* bblk;     // A_BITS: source-window blocks of B (pre-swizzled); nullptr: TMA boxes
+  int64_t bblk_stride;   // floats per window block
   int b_raw;         // A_TRANS: B = row-major D box; the builders split + transpose it into the
                      // K-major SWIZZLE_128B hi/lo layout in smem (no feature-major pre-split pass)
 };
@@ -130,6 +133,7 @@ struct Work {
 template <int MODE>
 __device__ __forceinline__ void tile_range(const Work& w, int64_t t, int64_t& kb, int64_t& nch, int64_t& m0,
                                            int64_t& sp) {
+  if (MODE == A_BITS && w.order) t = w.order[t];
   if (MODE == A_BITS) {
     kb = w.rt_cptr[t];
     nch = w.rt_cptr[t + 1] - kb;
@@ -220,7 +224,11 @@ __global__ void __launch_bounds__(NTHREADS, 1)
             }
             // chunk u's B tile in smem: [hi: npad rows][lo: npad rows] x 128 B
             uint8_t* bdst = st + L.a_bytes + u * 2 * L.b_bytes;
-            if (MODE == A_TRANS && w.b_raw) {
+            if (MODE == A_BITS && w.bblk) {
+              // the window's hi+lo (or hi) rows: one contiguous, pre-swizzled block
+              bulk_load(bdst, w.bblk + int64_t(k0 >> 5) * w.bblk_stride, (w.single ? 1u : 2u) * L.b_bytes,
+                        &full[s]);
+            } else if (MODE == A_TRANS && w.b_raw) {
               // row-major D rows [k0, k0+32) x features [0, npad) (OOB columns zero-filled)
               tma_load_2d(&map_bhi, &full[s], st + L.a_bytes + 2 * L.b_bytes, 0, k0);
             } else if (w.b_fused || w.single) {
@@ -592,6 +600,23 @@ cudaError_t launch_dense_tc(const DenseArgs& a, cudaStream_t s) {
   if (a.nrt <= 0) return cudaSuccess;
   if (a.npad % 16 != 0 || a.npad < 16 || a.npad > 256 || a.ldT % 4 != 0) return cudaErrorInvalidValue;
   CUtensorMap mh, ml;
+  if (a.blk) {
+    // window blocks: B arrives by bulk copies (no tensor maps)
+    Work w{};
+    w.bblk = a.blk;
+    w.bblk_stride = a.blk_floats;
+    w.order = a.rt_order;
+    w.single = a.loT ? 0 : 1;
+    w.ntiles = a.nrt;
+    w.rt_cptr = a.rt_cptr;
+    w.ch_col0 = a.ch_col0;
+    w.bits = a.bits;
+    w.out = a.zd;
+    w.ldo = a.ldzd;
+    w.ncols = a.npad;
+    mh = CUtensorMap{};
+    return launch_engine<A_BITS>(mh, mh, mh, w, a.npad, s);
+  }
   if (dense_pair_eligible(a.npad) && a.loT == a.hiT + int64_t(a.npad) * a.ldT) {
     // CTA-pair kernel (tc_pair.cu): one map over [hi rows; lo rows], box = half the features
     if (!make_map(&mh, a.hiT, a.n, 2 * a.npad, a.ldT, BK, a.npad / 2, true)) return cudaErrorInvalidValue;

@@ -573,10 +573,11 @@ np.savez(sys.argv[1], **out)
 @pytest.mark.parametrize("knob,bitwise", [({"PCGCN_ROWS_PER_TICKET": "1"}, True),
                                           ({"PCGCN_ROWS_PER_TICKET": "16"}, True),
                                           ({"PCGCN_OVERLAP": "1"}, True),
-                                          ({"PCGCN_XTG_PRESPLIT": "1"}, True)])
+                                          ({"PCGCN_XTG_PRESPLIT": "1"}, True),
+                                          ({"PCGCN_DENSE_BLOCKED": "0"}, True)])
 def test_scheduling_knobs_do_not_change_results(tmp_path, knob, bitwise):
-    """Row-block tickets, the full-mode/segment overlap and the in-kernel xtg
-    B conversion change only scheduling (every output row is still reduced by
+    """Row-block tickets, the full-mode/segment overlap, the in-kernel xtg B
+    conversion and the window-blocked full-mode B layout change only scheduling (every output row is still reduced by
     one warp in the same order; the MMA sequence and the hi/lo split are the
     same), so aggregation outputs, masks, gradients and the loss must be
     bitwise identical to the default configuration."""
