@@ -437,7 +437,16 @@ __global__ void __launch_bounds__(NTHREADS, 1)
       // only, never to global)
       if (live || (NPC > 0 && MODE == A_ROWMAJOR && L.out_bytes)) {
         const uint32_t* mrow = (MODE == A_ROWMAJOR && w.mask && live) ? w.mask + row * w.mask_ld : nullptr;
-        auto mk = [&](int c) { return mrow ? ((mrow[c >> 5] >> (c & 31)) & 1u ? sc : 0.f) : sc; };
+        // mask words in registers (loaded once per row, not once per column)
+        constexpr int NMW = NPC > 0 ? (NPC + 31) / 32 : 1;
+        uint32_t mwd[NMW];
+#pragma unroll
+        for (int i = 0; i < NMW; ++i) mwd[i] = (mrow && (NPC > 0) && 32 * i < w.ncols) ? __ldg(mrow + i) : 0xffffffffu;
+        auto mk = [&](int c) {
+          if (!mrow) return sc;
+          const uint32_t wd = NPC > 0 ? mwd[(c >> 5) % NMW] : __ldg(mrow + (c >> 5));
+          return ((wd >> (c & 31)) & 1u) ? sc : 0.f;
+        };
         if (NPC > 0 && MODE == A_ROWMAJOR && L.out_bytes) {
           // staged store: each thread holds one row; 64-column halves go
           // through this warp's [32 rows][68] smem tile and leave as two rows
