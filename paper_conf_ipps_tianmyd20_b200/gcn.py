@@ -165,13 +165,20 @@ class GCN2:
 
     def launches_per_epoch(self) -> int:
         """Kernel launches of libpcgcn per epoch (for the bench's gpu_launches)."""
-        st = self.plan.stats()
-        dense = st["shard_chunks"] > 0
-        # split + dense tiles (full mode), segment pass (long rows), selective rows
-        agg = 1 + (2 if dense else 0) + (1 if st["shard_segments"] > 0 else 0)
-        gemm_xw = 1 + 1                          # tile kernel + pad zeroing (ld > N) — upper bound
-        n = 2 * gemm_xw + 4 * agg + 2 + 2 * 3 + 3  # + softmax(2) + 2 x xtg(split, engine, reduce) + dwt(split, engine, pad)
-        n += 2 if self.optimizer == "adam" else 1
+        def agg(plan):
+            st = plan.stats()
+            # split + full-mode tiles, segment pass (long rows), selective rows
+            return 1 + (2 if st["shard_chunks"] > 0 else 0) + (1 if st["shard_segments"] > 0 else 0)
+
+        np16 = lambda f: (f + 15) // 16 * 16  # noqa: E731
+        xw = lambda ld, f: 2 + (1 if ld > np16(f) else 0)  # noqa: E731  W split + engine (+ pad zeroing)
+        n = xw(self.ldH, self.H) + xw(self.ldC, self.C)      # a4, a7
+        n += 2 * agg(self.plan) + 2 * agg(self.plan_c)       # a5/a6, a8, a10, a12
+        n += 2                                               # a9 softmax-CE + loss reduction
+        xtg = lambda f: 2 if np16(f) <= 128 else 3  # noqa: E731  engine (in-kernel B split) + slice sum
+        n += xtg(self.C) + xtg(self.H)                       # a11, a13
+        n += 2 + (1 if self.ldH > np16(self.H) else 0)       # a11 dwt: W split + engine (+ pad zeroing)
+        n += 2 if self.optimizer == "adam" else 1            # a14
         return n
 
     # -- CUDA graph ------------------------------------------------------
