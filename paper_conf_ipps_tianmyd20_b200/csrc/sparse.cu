@@ -12,9 +12,11 @@
 // B200 design:
 //   * one warp per destination row (persistent warps claim rows in plan order
 //     from a ticket counter); the 32 lanes split into S = 32/G edge slots of
-//     G lanes, G the narrowest power of two covering the row's float4s, so
-//     one load instruction reads whole rows and touches the fewest 128-byte
-//     lines (F=128 -> G=32; F=41 -> G=16, two rows per load);
+//     G lanes, G the narrowest power of two covering the row's lane vectors,
+//     so one load instruction reads whole rows and touches the fewest
+//     128-byte lines; a lane vector is 32 bytes (one 256-bit load) when the
+//     row needs no extra padding for it, else 16 (F=128 -> G=16 x 32 B, two
+//     rows per load; F=41 -> G=16 x 16 B, two rows per load);
 //   * the warp loads 32 source indices with one coalesced load and broadcasts
 //     them by shuffle; a row address is one 32x32->64 multiply-add; full
 //     batches are unguarded and keep 8 float4 loads per lane in flight;
@@ -57,47 +59,64 @@ __device__ __forceinline__ uint32_t smem_addr(const void* p) {
 __device__ __forceinline__ void add4(float4& a, const float4& b) {
   a.x += b.x; a.y += b.y; a.z += b.z; a.w += b.w;
 }
+// one lane vector of H float4 (H = 2: one 32-byte LDG.E.ENL2.256, sm_100's
+// widest load — half the load, shuffle and address instructions per gathered
+// byte; needs 32-byte aligned rows)
+template <int H>
+__device__ __forceinline__ void ld_vec(const char* p, float4 (&o)[H]) {
+  if constexpr (H == 1) {
+    o[0] = ld_f4b(p);
+  } else {
+    asm("ld.global.nc.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+        : "=f"(o[0].x), "=f"(o[0].y), "=f"(o[0].z), "=f"(o[0].w), "=f"(o[1].x), "=f"(o[1].y), "=f"(o[1].z),
+          "=f"(o[1].w)
+        : "l"(p));
+  }
+}
 
-// Lane layout for a feature row of nvec float4: the warp's 32 lanes form
-// S = 32/G edge slots of G lanes; lane l of a slot owns float4 columns
-// l, l+G, ..., l+(V-1)G.  A slot's G lanes read one contiguous piece of the
-// row per load, so each load instruction touches the fewest 128-byte lines
-// (the L1TEX wavefront count is what bounds a gather of L2-resident rows).
-template <int G, int V>
+// Lane layout for a feature row of nvec lane vectors (H float4 each): the
+// warp's 32 lanes form S = 32/G edge slots of G lanes; lane l of a slot owns
+// vectors l, l+G, ..., l+(V-1)G.  A slot's G lanes read one contiguous piece
+// of the row per load, so each load instruction touches the fewest 128-byte
+// lines (the L1TEX wavefront count is what bounds a gather of L2-resident rows).
+template <int G, int V, int H>
 struct Lay {
   static constexpr int S = 32 / G;       // edges per warp step
   static constexpr int STEPS = 32 / S;   // steps per 32-index batch
   // steps whose loads are all issued before any is consumed (<= 8 float4
   // per lane in flight: more costs occupancy than it gains in MLP on C3)
-  static constexpr int UCAP = 8 / V;
+  static constexpr int UCAP = 8 / (V * H);
   static constexpr int UNR = (UCAP >= 8 && STEPS >= 8) ? 8
                            : (UCAP >= 4 && STEPS >= 4) ? 4
                            : (UCAP >= 2 && STEPS >= 2) ? 2 : 1;
-  static constexpr int NACC = (V == 1 && UNR >= 2) ? 2 : 1;  // interleaved partial sums
+  static constexpr int NACC = (V * H == 1 && UNR >= 2) ? 2 : 1;  // interleaved partial sums
 };
 
-// tot[v] (valid in every lane after the butterfly) = sum over the n edges at
-// cp[0..n) of Y'[cp[e]][cols of this lane].  yb = this lane's byte offset
+// tot[v][h] (valid in every lane after the butterfly) = sum over the n edges
+// at cp[0..n) of Y'[cp[e]][cols of this lane].  yb = this lane's byte offset
 // into row 0 of Y' (lanes past the row re-read column 0: same line, ignored;
-// columns v >= 1 past the row are not loaded: lok[v] false).
+// vectors v >= 1 past the row are not loaded: lok[v] false).
 // Fixed order: per slot sequential over its edges in NACC interleaved sums,
 // then a butterfly over the slots — bitwise reproducible.
 // Index batches are loaded one ahead: `first` is this range's first batch
 // (lane l: cp[l] if l < n), and the prefetch slot of the last batch loads the
 // first batch of the NEXT range (cpn, nn), which is returned — so a warp
 // walking rows never waits on a row's first index load.
-template <int G, int V>
+template <int G, int V, int H>
 __device__ __forceinline__ int gather_sum(const int* __restrict__ cp, int n, int first,
                                           const int* __restrict__ cpn, int nn, const char* __restrict__ yb,
-                                          uint32_t rstride, const bool (&lok)[V], int lane, float4 (&tot)[V]) {
-  using L = Lay<G, V>;
+                                          uint32_t rstride, const bool (&lok)[V], int lane,
+                                          float4 (&tot)[V][H]) {
+  using L = Lay<G, V, H>;
   constexpr int S = L::S, STEPS = L::STEPS, UNR = L::UNR, NACC = L::NACC;
   const int slot = lane / G;
-  float4 acc[NACC][V];
+  float4 acc[NACC][V][H];
 #pragma unroll
   for (int u = 0; u < NACC; ++u)
 #pragma unroll
-    for (int v = 0; v < V; ++v) acc[u][v] = make_float4(0.f, 0.f, 0.f, 0.f);
+    for (int v = 0; v < V; ++v)
+#pragma unroll
+      for (int h = 0; h < H; ++h) acc[u][v][h] = make_float4(0.f, 0.f, 0.f, 0.f);
   int nextidx = first;
   if (n == 0) nextidx = lane < nn ? ld_idx(cpn + lane) : 0;
   for (int base = 0; base < n; base += 32) {
@@ -107,63 +126,81 @@ __device__ __forceinline__ int gather_sum(const int* __restrict__ cp, int n, int
     nextidx = (base + 32 + lane < n) ? ld_idx(cp + base + 32 + lane)
             : (lane < nn ? ld_idx(cpn + lane) : 0);
     if (cnt == 32) {
-      // full batch: unguarded, every lane keeps UNR*V 16-byte loads in flight
+      // full batch: unguarded, every lane keeps UNR*V*H 16-byte pieces in flight
 #pragma unroll
       for (int k0 = 0; k0 < STEPS; k0 += UNR) {
-        float4 buf[UNR][V];
+        float4 buf[UNR][V][H];
 #pragma unroll
         for (int u = 0; u < UNR; ++u) {
           const uint32_t j = uint32_t(__shfl_sync(0xffffffffu, myidx, (k0 + u) * S + slot));
           const char* p = row_addr(yb, j, rstride);
 #pragma unroll
-          for (int v = 0; v < V; ++v)
-            buf[u][v] = (v == 0 || lok[v]) ? ld_f4b(p + 16 * G * v) : make_float4(0.f, 0.f, 0.f, 0.f);
+          for (int v = 0; v < V; ++v) {
+            if (v == 0 || lok[v]) {
+              ld_vec<H>(p + 16 * H * G * v, buf[u][v]);
+            } else {
+#pragma unroll
+              for (int h = 0; h < H; ++h) buf[u][v][h] = make_float4(0.f, 0.f, 0.f, 0.f);
+            }
+          }
         }
 #pragma unroll
         for (int u = 0; u < UNR; ++u)
 #pragma unroll
-          for (int v = 0; v < V; ++v) add4(acc[u % NACC][v], buf[u][v]);
+          for (int v = 0; v < V; ++v)
+#pragma unroll
+            for (int h = 0; h < H; ++h) add4(acc[u % NACC][v][h], buf[u][v][h]);
       }
     } else {
       // last (partial) batch of the row: slots past the end add nothing
 #pragma unroll
       for (int k0 = 0; k0 < STEPS; k0 += UNR) {
-        float4 buf[UNR][V];
+        float4 buf[UNR][V][H];
 #pragma unroll
         for (int u = 0; u < UNR; ++u) {
           const int e = (k0 + u) * S + slot;
           const uint32_t j = uint32_t(__shfl_sync(0xffffffffu, myidx, e));
           const char* p = row_addr(yb, j, rstride);
 #pragma unroll
-          for (int v = 0; v < V; ++v)
-            buf[u][v] = (e < cnt && (v == 0 || lok[v])) ? ld_f4b(p + 16 * G * v)
-                                                          : make_float4(0.f, 0.f, 0.f, 0.f);
+          for (int v = 0; v < V; ++v) {
+            if (e < cnt && (v == 0 || lok[v])) {
+              ld_vec<H>(p + 16 * H * G * v, buf[u][v]);
+            } else {
+#pragma unroll
+              for (int h = 0; h < H; ++h) buf[u][v][h] = make_float4(0.f, 0.f, 0.f, 0.f);
+            }
+          }
         }
 #pragma unroll
         for (int u = 0; u < UNR; ++u)
 #pragma unroll
-          for (int v = 0; v < V; ++v) add4(acc[u % NACC][v], buf[u][v]);
+          for (int v = 0; v < V; ++v)
+#pragma unroll
+            for (int h = 0; h < H; ++h) add4(acc[u % NACC][v][h], buf[u][v][h]);
         if ((k0 + UNR) * S >= cnt) break;  // warp-uniform: rest of the batch is empty
       }
     }
   }
 #pragma unroll
-  for (int v = 0; v < V; ++v) {
-    tot[v] = acc[0][v];
+  for (int v = 0; v < V; ++v)
 #pragma unroll
-    for (int u = 1; u < NACC; ++u) add4(tot[v], acc[u][v]);
+    for (int h = 0; h < H; ++h) {
+      float4& t = tot[v][h];
+      t = acc[0][v][h];
 #pragma unroll
-    for (int off = G; off < 32; off <<= 1) {  // fixed butterfly over the slots
-      tot[v].x += __shfl_xor_sync(0xffffffffu, tot[v].x, off);
-      tot[v].y += __shfl_xor_sync(0xffffffffu, tot[v].y, off);
-      tot[v].z += __shfl_xor_sync(0xffffffffu, tot[v].z, off);
-      tot[v].w += __shfl_xor_sync(0xffffffffu, tot[v].w, off);
+      for (int u = 1; u < NACC; ++u) add4(t, acc[u][v][h]);
+#pragma unroll
+      for (int off = G; off < 32; off <<= 1) {  // fixed butterfly over the slots
+        t.x += __shfl_xor_sync(0xffffffffu, t.x, off);
+        t.y += __shfl_xor_sync(0xffffffffu, t.y, off);
+        t.z += __shfl_xor_sync(0xffffffffu, t.z, off);
+        t.w += __shfl_xor_sync(0xffffffffu, t.w, off);
+      }
     }
-  }
   return nextidx;
 }
 
-// per-lane byte offset of this lane's first float4 (lanes past the row: 0)
+// this lane's vector index q for vector v (lanes past the row: -1)
 template <int G>
 __device__ __forceinline__ int lane_col(int lane, int v, int nvec) {
   const int q = lane % G + G * v;
@@ -174,27 +211,31 @@ __device__ __forceinline__ int lane_col(int lane, int v, int nvec) {
 // partial sums to seg_ws.
 // 4-warp CTAs (8K registers): small enough to co-reside with a full-mode
 // engine CTA (tc_engine, 320 threads) when the two run concurrently
-template <int G, int V>
+template <int G, int V, int H>
 __global__ void __launch_bounds__(128, 8) sparse_seg_kernel(AggArgs a) {
   const int64_t sg = int64_t(blockIdx.x) * 4 + (threadIdx.x >> 5);
   if (sg >= a.nseg) return;
   const int lane = threadIdx.x & 31;
-  const int nvec = (a.F + 3) >> 2;
+  const int nvec = (a.F + 4 * H - 1) / (4 * H);
+  const int nvec4 = (a.F + 3) >> 2;
   const int q0 = lane_col<G>(lane, 0, nvec);
-  const char* yb = reinterpret_cast<const char*>(a.Y) + 16 * (q0 < 0 ? 0 : q0);
+  const char* yb = reinterpret_cast<const char*>(a.Y) + 16 * H * (q0 < 0 ? 0 : q0);
   const int64_t lo = a.seg_lo[sg], hi = a.seg_hi[sg];
   bool lok[V];
 #pragma unroll
   for (int v = 0; v < V; ++v) lok[v] = lane_col<G>(lane, v, nvec) >= 0;
-  float4 tot[V];
+  float4 tot[V][H];
   const int n = int(hi - lo);
   const int first = lane < n ? ld_idx(a.col + lo + lane) : 0;
-  gather_sum<G, V>(a.col + lo, n, first, nullptr, 0, yb, uint32_t(a.ldy * 4), lok, lane, tot);
+  gather_sum<G, V, H>(a.col + lo, n, first, nullptr, 0, yb, uint32_t(a.ldy * 4), lok, lane, tot);
   if (lane < G) {
 #pragma unroll
     for (int v = 0; v < V; ++v) {
       const int q = lane_col<G>(lane, v, nvec);
-      if (q >= 0) *reinterpret_cast<float4*>(a.seg_ws + sg * a.ldws + 4 * q) = tot[v];
+#pragma unroll
+      for (int h = 0; h < H; ++h)
+        if (q >= 0 && H * q + h < nvec4)
+          *reinterpret_cast<float4*>(a.seg_ws + sg * a.ldws + 4 * (H * q + h)) = tot[v][h];
     }
   }
 }
@@ -204,11 +245,12 @@ __global__ void __launch_bounds__(128, 8) sparse_seg_kernel(AggArgs a) {
 // locality); a row is gathered directly or, if long, summed from its
 // segment partials in segment order.  Fused epilogue: + full-mode partial
 // sum Zd (mode combine, L193), x r_i (optionally twice), ReLU, bit mask.
-template <int G, int V, bool HAS_ZD, bool HAS_SEG>
+template <int G, int V, int H, bool HAS_ZD, bool HAS_SEG>
 __global__ void __launch_bounds__(256, 4) sparse_row_kernel(AggArgs a) {
   const int lane = threadIdx.x & 31;
   const int slot = lane / G;
-  const int nvec = (a.F + 3) >> 2;
+  const int nvec = (a.F + 4 * H - 1) / (4 * H);
+  const int nvec4 = (a.F + 3) >> 2;
   int qv[V];
   bool lok[V];
 #pragma unroll
@@ -216,7 +258,7 @@ __global__ void __launch_bounds__(256, 4) sparse_row_kernel(AggArgs a) {
     qv[v] = lane_col<G>(lane, v, nvec);
     lok[v] = qv[v] >= 0;
   }
-  const char* yb = reinterpret_cast<const char*>(a.Y) + 16 * (qv[0] < 0 ? 0 : qv[0]);
+  const char* yb = reinterpret_cast<const char*>(a.Y) + 16 * H * (qv[0] < 0 ? 0 : qv[0]);
   const uint32_t rstride = uint32_t(a.ldy * 4);
   // Rows are claimed in blocks of R consecutive rows per ticket (R >= 4 from
   // the plan's mean selective degree: short rows would otherwise pay the
@@ -281,7 +323,7 @@ __global__ void __launch_bounds__(256, 4) sparse_row_kernel(AggArgs a) {
       n0 = s_rp[wib][b ^ 1][0];
       n1 = s_rp[wib][b ^ 1][1];
     }
-    float4 tot[V];
+    float4 tot[V][H];
     int pre_next;
     // the epilogue's per-row scalars are loaded before the gather (in flight with it)
     const float ri = a.r[a.row_lo + row];
@@ -291,60 +333,89 @@ __global__ void __launch_bounds__(256, 4) sparse_row_kernel(AggArgs a) {
       pre_next = (n0 + lane < n1) ? ld_idx(a.col + n0 + lane) : 0;
       const int ns = int((e1 - e0 + SEG_EDGES - 1) / SEG_EDGES);
 #pragma unroll
-      for (int v = 0; v < V; ++v) tot[v] = make_float4(0.f, 0.f, 0.f, 0.f);
+      for (int v = 0; v < V; ++v)
+#pragma unroll
+        for (int h = 0; h < H; ++h) tot[v][h] = make_float4(0.f, 0.f, 0.f, 0.f);
       if (slot == 0) {
         for (int k = 0; k < ns; ++k)
 #pragma unroll
           for (int v = 0; v < V; ++v)
-            if (qv[v] >= 0) add4(tot[v], __ldcg(reinterpret_cast<const float4*>(
-                                              a.seg_ws + int64_t(sg + k) * a.ldws + 4 * qv[v])));
+#pragma unroll
+            for (int h = 0; h < H; ++h)
+              if (qv[v] >= 0 && H * qv[v] + h < nvec4)
+                add4(tot[v][h], __ldcg(reinterpret_cast<const float4*>(a.seg_ws + int64_t(sg + k) * a.ldws +
+                                                                        4 * (H * qv[v] + h))));
       }
     } else {
-      pre_next = gather_sum<G, V>(a.col + e0, int(e1 - e0), pre, a.col + n0, int(n1 - n0), yb, rstride, lok,
-                                  lane, tot);
+      pre_next = gather_sum<G, V, H>(a.col + e0, int(e1 - e0), pre, a.col + n0, int(n1 - n0), yb, rstride,
+                                     lok, lane, tot);
     }
     uint32_t bal[V][4];
+    uint32_t mbyte[V];
 #pragma unroll
     for (int v = 0; v < V; ++v) {
-      const bool own = slot == 0 && qv[v] >= 0;
-      float4 z = tot[v];
-      if (HAS_ZD && own && zi >= 0) add4(z, ld_f4(a.zd + int64_t(zi) * a.ldzd + 4 * qv[v]));
-      z.x *= ri; z.y *= ri; z.z *= ri; z.w *= ri;
-      if (a.out_prescaled) { z.x *= ri; z.y *= ri; z.z *= ri; z.w *= ri; }
-      if (a.mask) {
-        const int c = 4 * qv[v];
-        bal[v][0] = __ballot_sync(0xffffffffu, own && z.x > 0.f && c + 0 < a.F);
-        bal[v][1] = __ballot_sync(0xffffffffu, own && z.y > 0.f && c + 1 < a.F);
-        bal[v][2] = __ballot_sync(0xffffffffu, own && z.z > 0.f && c + 2 < a.F);
-        bal[v][3] = __ballot_sync(0xffffffffu, own && z.w > 0.f && c + 3 < a.F);
+      mbyte[v] = 0;
+#pragma unroll
+      for (int h = 0; h < H; ++h) {
+        const int q4 = H * qv[v] + h;  // float4 column index (valid iff qv >= 0 and q4 < nvec4)
+        const bool own = slot == 0 && qv[v] >= 0 && q4 < nvec4;
+        float4 z = tot[v][h];
+        if (HAS_ZD && own && zi >= 0) add4(z, ld_f4(a.zd + int64_t(zi) * a.ldzd + 4 * q4));
+        z.x *= ri; z.y *= ri; z.z *= ri; z.w *= ri;
+        if (a.out_prescaled) { z.x *= ri; z.y *= ri; z.z *= ri; z.w *= ri; }
+        if (a.mask) {
+          const int c = 4 * q4;
+          if constexpr (H == 1) {
+            bal[v][0] = __ballot_sync(0xffffffffu, own && z.x > 0.f && c + 0 < a.F);
+            bal[v][1] = __ballot_sync(0xffffffffu, own && z.y > 0.f && c + 1 < a.F);
+            bal[v][2] = __ballot_sync(0xffffffffu, own && z.z > 0.f && c + 2 < a.F);
+            bal[v][3] = __ballot_sync(0xffffffffu, own && z.w > 0.f && c + 3 < a.F);
+          } else if (own) {  // 8 columns per lane vector = one byte of the mask row
+            const uint32_t m = uint32_t(z.x > 0.f && c + 0 < a.F) | uint32_t(z.y > 0.f && c + 1 < a.F) << 1 |
+                               uint32_t(z.z > 0.f && c + 2 < a.F) << 2 | uint32_t(z.w > 0.f && c + 3 < a.F) << 3;
+            mbyte[v] |= m << (4 * h);
+          }
+        }
+        if (a.relu) {
+          z.x = fmaxf(z.x, 0.f); z.y = fmaxf(z.y, 0.f); z.z = fmaxf(z.z, 0.f); z.w = fmaxf(z.w, 0.f);
+        }
+        if (own) *reinterpret_cast<float4*>(a.Z + int64_t(row) * a.ldz + 4 * q4) = z;
       }
-      if (a.relu) {
-        z.x = fmaxf(z.x, 0.f); z.y = fmaxf(z.y, 0.f); z.z = fmaxf(z.z, 0.f); z.w = fmaxf(z.w, 0.f);
-      }
-      if (own) *reinterpret_cast<float4*>(a.Z + int64_t(row) * a.ldz + 4 * qv[v]) = z;
     }
     if (a.mask) {
-      // lane w assembles mask word w: column col = 32w + 4k + c (k < 8) is
-      // float4 q = 8w + k, held by lane q % G of vector v = q / G, component
-      // c; bit q % G of bal[v][c].  The 8 q's of a word share one v (G >= 8,
-      // or a single word when G < 8), so the word interleaves four bytes:
-      // bit 4k + c = bit k of byte c.
-      const int mw = (a.F + 31) >> 5;
-      if (lane < mw) {
-        const int vv = (8 * lane) / G, l0 = (8 * lane) % G;
-        uint32_t word = 0;
+      if constexpr (H == 1) {
+        // lane w assembles mask word w: column col = 32w + 4k + c (k < 8) is
+        // float4 q = 8w + k, held by lane q % G of vector v = q / G, component
+        // c; bit q % G of bal[v][c].  The 8 q's of a word share one v (G >= 8,
+        // or a single word when G < 8), so the word interleaves four bytes:
+        // bit 4k + c = bit k of byte c.
+        const int mw = (a.F + 31) >> 5;
+        if (lane < mw) {
+          const int vv = (8 * lane) / G, l0 = (8 * lane) % G;
+          uint32_t word = 0;
 #pragma unroll
-        for (int c = 0; c < 4; ++c) {
-          uint32_t x = 0;
+          for (int c = 0; c < 4; ++c) {
+            uint32_t x = 0;
+#pragma unroll
+            for (int v = 0; v < V; ++v)
+              if (v == vv) x = (bal[v][c] >> l0) & 0xffu;
+            x = (x | (x << 12)) & 0x000f000fu;  // spread bit k to bit 4k
+            x = (x | (x << 6)) & 0x03030303u;
+            x = (x | (x << 3)) & 0x11111111u;
+            word |= x << c;
+          }
+          a.mask[int64_t(row) * a.mask_ld + lane] = word;
+        }
+      } else {
+        // the mask row is a little-endian bitset: byte q holds columns
+        // 8q..8q+7, i.e. lane vector q's bits; bytes past the row are zero
+        uint8_t* mrow = reinterpret_cast<uint8_t*>(a.mask + int64_t(row) * a.mask_ld);
+        if (slot == 0) {
 #pragma unroll
           for (int v = 0; v < V; ++v)
-            if (v == vv) x = (bal[v][c] >> l0) & 0xffu;
-          x = (x | (x << 12)) & 0x000f000fu;  // spread bit k to bit 4k
-          x = (x | (x << 6)) & 0x03030303u;
-          x = (x | (x << 3)) & 0x11111111u;
-          word |= x << c;
+            if (qv[v] >= 0) mrow[qv[v]] = uint8_t(mbyte[v]);
         }
-        a.mask[int64_t(row) * a.mask_ld + lane] = word;
+        if (nvec + lane < 4 * a.mask_ld) mrow[nvec + lane] = 0;  // < 4 bytes past the last vector
       }
     }
     pre = pre_next;
@@ -354,7 +425,7 @@ __global__ void __launch_bounds__(256, 4) sparse_row_kernel(AggArgs a) {
   }
 }
 
-template <int G, int V>
+template <int G, int V, int H>
 cudaError_t launch_gv(const AggArgs& a, cudaStream_t s) {
   // persistent row pass: as many 8-warp CTAs as fit (4 per SM at 64 registers)
   static int slots = 0;
@@ -362,18 +433,18 @@ cudaError_t launch_gv(const AggArgs& a, cudaStream_t s) {
     int dev = 0, sms = 148, per = 4;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, sparse_row_kernel<G, V, true, true>, 256, 0);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, sparse_row_kernel<G, V, H, true, true>, 256, 0);
     slots = sms * (per > 0 ? per : 1);
   }
   if (a.nseg > 0 && a.phase != 2) {
-    sparse_seg_kernel<G, V><<<unsigned((a.nseg + 3) / 4), 128, 0, s>>>(a);
+    sparse_seg_kernel<G, V, H><<<unsigned((a.nseg + 3) / 4), 128, 0, s>>>(a);
     if (a.phase == 1) return cudaGetLastError();
   }
   cudaError_t e = cudaMemsetAsync(a.counter, 0, sizeof(int), s);
   if (e != cudaSuccess) return e;
   const int64_t want = ((a.rows + a.rows_per_ticket - 1) / a.rows_per_ticket + 7) / 8;
   const unsigned grid = unsigned(want < slots ? want : slots);
-#define LAUNCH(ZD, SG) sparse_row_kernel<G, V, ZD, SG><<<grid, 256, 0, s>>>(a)
+#define LAUNCH(ZD, SG) sparse_row_kernel<G, V, H, ZD, SG><<<grid, 256, 0, s>>>(a)
   const bool zd = a.zd_index != nullptr, sg = a.nseg > 0;
   if (zd && sg) LAUNCH(true, true);
   else if (zd) LAUNCH(true, false);
@@ -493,10 +564,14 @@ cudaError_t launch_sparse_pass(const AggArgs& a, cudaStream_t s);
 // the gather in column slices of that width (each slice of Y' is a smaller
 // L2 working set; the index stream is re-read per slice).  (An L2
 // evict_first hint on the index stream was measured and dropped: no gain.)
+// PCGCN_SPARSE_V8=0 keeps 16-byte lane vectors even where rows allow the
+// 32-byte ones (A/B measurement).
 struct SparseKnobs {
   int fsplit = 0;
+  bool v8 = true;
   SparseKnobs() {
     if (const char* e = getenv("PCGCN_SPARSE_FSPLIT")) fsplit = atoi(e) / 32 * 32;
+    if (const char* e = getenv("PCGCN_SPARSE_V8")) v8 = atoi(e) != 0;
   }
 };
 
@@ -526,16 +601,32 @@ cudaError_t launch_sparse_agg(const AggArgs& a0, cudaStream_t s) {
 }
 
 cudaError_t launch_sparse_pass(const AggArgs& a, cudaStream_t s) {
-  // G lanes x V float4 per edge slot: the narrowest power-of-two slot that
-  // covers the row, so one load instruction reads whole rows (fewest lines)
+  // G lanes x V vectors per edge slot: the narrowest power-of-two slot that
+  // covers the row, so one load instruction reads whole rows (fewest lines).
+  // Vectors are 32 bytes (8 floats) when the rows are 32-byte aligned and the
+  // wider vector reads no padding the 16-byte one skips (F = 41: 48 vs 44
+  // floats per row, measured 6% slower on C3's L2-bound F = 41 pass); else 16.
+  // Measured (B200, PCGCN_SPARSE_V8=0 vs 1): C5's issue-bound row pass F = 32
+  // 21.2 -> 19.2 ms, F = 128 45.4 -> 43.3 ms; C3 F = 128 unchanged.
+  const bool v8 = knobs().v8 && a.ldy % 8 == 0 && (reinterpret_cast<uintptr_t>(a.Y) & 31) == 0 &&
+                  (a.F + 7) / 8 * 2 == (a.F + 3) / 4;
+  if (v8) {
+    const int nvec = (a.F + 7) / 8;
+    if (nvec <= 1) return launch_gv<1, 1, 2>(a, s);
+    if (nvec <= 2) return launch_gv<2, 1, 2>(a, s);
+    if (nvec <= 4) return launch_gv<4, 1, 2>(a, s);
+    if (nvec <= 8) return launch_gv<8, 1, 2>(a, s);
+    if (nvec <= 16) return launch_gv<16, 1, 2>(a, s);
+    if (nvec <= 32) return launch_gv<32, 1, 2>(a, s);  // F <= 256 = f_max
+  }
   const int nvec = (a.F + 3) / 4;
-  if (nvec <= 1) return launch_gv<1, 1>(a, s);
-  if (nvec <= 2) return launch_gv<2, 1>(a, s);
-  if (nvec <= 4) return launch_gv<4, 1>(a, s);
-  if (nvec <= 8) return launch_gv<8, 1>(a, s);
-  if (nvec <= 16) return launch_gv<16, 1>(a, s);
-  if (nvec <= 32) return launch_gv<32, 1>(a, s);
-  return launch_gv<32, 2>(a, s);
+  if (nvec <= 1) return launch_gv<1, 1, 1>(a, s);
+  if (nvec <= 2) return launch_gv<2, 1, 1>(a, s);
+  if (nvec <= 4) return launch_gv<4, 1, 1>(a, s);
+  if (nvec <= 8) return launch_gv<8, 1, 1>(a, s);
+  if (nvec <= 16) return launch_gv<16, 1, 1>(a, s);
+  if (nvec <= 32) return launch_gv<32, 1, 1>(a, s);
+  return launch_gv<32, 2, 1>(a, s);
 }
 
 cudaError_t launch_prescale(const float* Y, int64_t ldy, const float* r, int64_t n, int F, float* ypre,
