@@ -92,13 +92,13 @@ def main(csv_path, rep_path, out_path):
         wl = sys.argv[6] if len(sys.argv) > 6 else "reddit"
         # the selective pass = segment kernel + row kernel; the capture holds the
         # layer-1 forward (F=H) launches first, then the layer-2 ones (F=C):
-        # group by the lane-slot template argument G of the kernel name
+        # group by the lane layout template arguments <G, V, H> of the kernel name
         sp = [d for d in rows[2:] if "sparse_" in d[hdr.index("Kernel Name")]]
         scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9,
                  "sector": 1, "Ksector": 1e3, "Msector": 1e6, "Gsector": 1e9}
         def g_of(d):
             nm = d[hdr.index("Kernel Name")]
-            return nm.split("<", 1)[1].split(",", 1)[0]
+            return ",".join(a.strip() for a in nm.rsplit("_kernel<", 1)[1].split(">", 1)[0].split(",")[:3])
         tr = {}
         groups = []
         for d in sp:
