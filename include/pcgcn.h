@@ -26,6 +26,9 @@
  *   - Dense matrices are row-major fp32 with an explicit leading dimension
  *     (elements); ld >= roundup(F, 4) and rows 16-byte aligned.  Pad columns
  *     of inputs must be zero; pad columns of outputs are written as zero.
+ *     Inputs with 32-byte aligned rows (ld % 8 == 0, 32-byte aligned base)
+ *     let the selective pass read 32-byte lane vectors when roundup(F, 8) ==
+ *     roundup(F, 4) (same results within tolerance; a different fixed order).
  *   - Device buffers are in PLAN ORDER: row v of Y/Z is the vertex
  *     perm[v] of the input graph (pcgcn_plan_perm).  The caller permutes its
  *     features / labels once, outside any timed region.
