@@ -221,12 +221,10 @@ def epoch_l(Ahat, X, Ths, labels, train):
     return dict(Ps=Ps, Hs=Hs, loss=loss, dL=dL, grads=grads, Gs=Gs)
 
 
-def sgd(Th, g, lr):
-    return np.asarray(Th, dtype=np.float64) - lr * g
-
-
 def adam(Th, g, m, v, t, lr=0.01, b1=0.9, b2=0.999, eps=1e-8):
-    """Adam (Kingma & Ba, Alg. 1) with bias correction; t starts at 1."""
+    """Adam (Kingma & Ba, Alg. 1) with bias correction; t starts at 1.
+    (Reading #14: the paper's model is Kipf's, trained with Adam; SGD needs
+    no oracle — the parity tests read the SGD step back as (Θ - Θ')/lr.)"""
     m = b1 * m + (1 - b1) * g
     v = b2 * v + (1 - b2) * g * g
     mh = m / (1 - b1 ** t)

@@ -35,7 +35,7 @@ __global__ void __launch_bounds__(256) dense_simt_kernel(DenseArgs a, const floa
     for (int e = tid; e < 32 * nvec; e += 256) {
       int b = e / nvec, q = e % nvec;
       int64_t src = col0 + b;
-      sm[e] = src < a.n ? *reinterpret_cast<const float4*>(y + src * ldy + 4 * q)
+      sm[e] = src < a.n_src ? *reinterpret_cast<const float4*>(y + src * ldy + 4 * q)
                         : make_float4(0.f, 0.f, 0.f, 0.f);
     }
     __syncthreads();

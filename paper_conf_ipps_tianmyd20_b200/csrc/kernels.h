@@ -68,6 +68,7 @@ struct DenseArgs {
   const int32_t* rt_order = nullptr;  // engine tile order (position i of CTA b: tile rt_order[b + i*G])
   const float* blk = nullptr;  // source-window blocks (launch_split_windows); nullptr: hiT/loT maps
   int64_t blk_floats = 0;      // floats per window block
+  int64_t n_src = 0;           // real source rows (vertices); rows [n_src, n) of the input are never read
 };
 cudaError_t launch_split_windows(const float* Y, int64_t ldy, int64_t n, int F, int npad, bool single, float* blk,
                                  int64_t nwin, cudaStream_t s);

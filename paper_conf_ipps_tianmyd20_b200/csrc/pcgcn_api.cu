@@ -318,6 +318,7 @@ pcgcn_status aggregate(pcgcn_plan_t p, const float* Y, int64_t ldy, float* Z, in
     DenseArgs da{d.yhi, bf16 ? nullptr : ylo, d.n_pad, d.n_pad, d.rt_row0, d.rt_nrows, d.rt_cptr, d.ch_col0,
                  d.bits, d.nrt, d.zd, npad, npad};
     da.rt_order = d.rt_order;
+    da.n_src = p->n;
     if (blocked) {
       da.blk = d.yhi;
       da.blk_floats = int64_t(bf16 ? 1 : 2) * npad * 32;

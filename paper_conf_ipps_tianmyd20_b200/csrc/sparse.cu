@@ -415,7 +415,10 @@ __global__ void __launch_bounds__(256, 4) sparse_row_kernel(AggArgs a) {
           for (int v = 0; v < V; ++v)
             if (qv[v] >= 0) mrow[qv[v]] = uint8_t(mbyte[v]);
         }
-        if (nvec + lane < 4 * a.mask_ld) mrow[nvec + lane] = 0;  // < 4 bytes past the last vector
+        // zero this row's bytes past the last vector, up to the end of ITS mask
+        // words (ceil(F/32) words: a column slice of PCGCN_SPARSE_FSPLIT owns only
+        // its own words of a wider row)
+        if (nvec + lane < 4 * ((a.F + 31) >> 5)) mrow[nvec + lane] = 0;
       }
     }
     pre = pre_next;

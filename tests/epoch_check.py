@@ -1,0 +1,251 @@
+"""Shared check of one 2-layer GCN epoch on the GPU against the fp64 oracle,
+with condition-scaled gates on EVERY output (tests only).
+
+Each quantity q of the epoch is compared as
+    err(q) = max |q_gpu - q*| / s_q      (gate 1e-5; reading #18)
+where q* is the oracle's fp64 value and s_q its first-order condition scale:
+the bound on |q_gpu - q*| / u when every fp32 operation of the CUDA path and
+every error already present in its inputs contributes u times the absolute
+value of what it touches.  Â = D̃^-½ÃD̃^-½ is nonnegative, so |Â| = Â, and
+(oracle.gcn's notation, Eq. 1, Alg. 1):
+
+    s_P1  = Â (|X| |Θ0|)                           P1 = Â X Θ0
+    s_L   = Â (s_P1 |Θ1|)                          L  = Â ReLU(P1) Θ1   (|H1| <= s_P1)
+    s_dL  = [i∈T] (2 p_ic max_k s_L,ik + p_ic + [c = y_i]) / |T|
+                                                   dL = (softmax(L) - onehot) [i∈T] / |T|
+            (∂softmax_c/∂L_k = p_c(δ_ck - p_k): |δp_c| <= 2 p_c max_k |δL_k|)
+    s_G1  = Â s_dL                                 G1 = Â dL
+    s_gΘ1 = s_P1ᵀ s_G1                             ∇Θ1 = H1ᵀ G1
+    s_dP1 = (s_G1 |Θ1|ᵀ) ⊙ mask1                   dP1 = (G1 Θ1ᵀ) ⊙ [P1 > 0]
+    s_G0  = Â s_dP1                                G0 = Â dP1
+    s_gΘ0 = |X|ᵀ s_G0                              ∇Θ0 = Xᵀ G0
+    s_loss = mean_T(2 max_k s_L,ik + |lse_i| + |L_i,y_i|)
+
+The ReLU mask is a decision taken in floating point (reading #19): entries
+with |P1*| <= BAND · s_P1 may go either way and both are correct results.
+With at most ENUM such entries the oracle's backward is computed for every
+combination and the GPU must match one of them; with more, the GPU's own
+decisions (its bit mask) are taken inside the band — each is a correct result
+by the error bound that defines the band — and the band must stay a small
+minority of the decisions (non-vacuity), everything outside it must agree.
+"""
+from __future__ import annotations
+
+import numpy as np
+
+from oracle import gcn as O
+
+TOL = 1e-5
+BAND = 1e-6
+ENUM = 8
+
+
+def _np(t):
+    return t.detach().cpu().numpy().astype(np.float64)
+
+
+def mask_bits(mask_t, F, inv):
+    m = mask_t.cpu().numpy().view(np.uint32)
+    mw = m.shape[1]
+    bits = ((m[:, :, None] >> np.arange(32, dtype=np.uint32)) & 1).reshape(m.shape[0], 32 * mw)[:, :F]
+    return bits[inv].astype(bool)
+
+
+class OracleEpoch:
+    """fp64 oracle epoch + condition scales (everything in vertex-id order)."""
+
+    def __init__(self, g, X, Th0, Th1, y, T):
+        self.Ahat = O.normalized_adjacency(g.n, g.rowptr, g.col)[0]
+        A = self.Ahat
+        assert A.data.min() >= 0
+        X64 = np.asarray(X, dtype=np.float64)
+        self.absX = np.abs(X64)
+        self.Th0 = np.asarray(Th0, dtype=np.float64)
+        self.Th1 = np.asarray(Th1, dtype=np.float64)
+        self.y = np.asarray(y)
+        self.T = np.asarray(T, dtype=bool)
+        self.nT = int(self.T.sum())
+        self.X64 = X64
+        P1, H1, L = O.forward(A, X64, self.Th0, self.Th1)
+        self.P1, self.H1, self.L = P1, H1, L
+        self.loss, self.dL = O.softmax_ce(L, self.y, self.T)
+        self.sP1 = O.aggregate(A, self.absX @ np.abs(self.Th0))
+        self.sL = O.aggregate(A, self.sP1 @ np.abs(self.Th1))
+        m = L.max(axis=1, keepdims=True)
+        p = np.exp(L - m)
+        p /= p.sum(axis=1, keepdims=True)
+        onehot = np.zeros_like(L)
+        onehot[np.arange(g.n), self.y] = 1.0
+        smax = self.sL.max(axis=1, keepdims=True)
+        self.s_dL = self.T[:, None] * (2 * p * smax + p + onehot) / self.nT
+        self.sG1 = O.aggregate(A, self.s_dL)
+        self.s_gTh1 = self.sP1.T @ self.sG1
+        lse = (m + np.log(np.exp(L - m).sum(axis=1, keepdims=True))).ravel()
+        Ly = L[np.arange(g.n), self.y]
+        self.s_loss = float(((2 * smax.ravel() + np.abs(lse) + np.abs(Ly)) * self.T).sum() / self.nT)
+        self._sG0 = None
+
+    def backward(self, P1v):
+        return O.backward(self.Ahat, self.X64, self.Th0, self.Th1, P1v, self.H1, self.dL)
+
+    def backward_scales(self):
+        """s_dP1, s_G0, s_gΘ0 with the ReLU pattern [P1 > 0] widened by the
+        error band (an upper bound for every admissible decision pattern)."""
+        if self._sG0 is None:
+            keep = (self.P1 > 0) | (np.abs(self.P1) <= BAND * self.sP1)
+            s_dP1 = (self.sG1 @ np.abs(self.Th1).T) * keep
+            sG0 = O.aggregate(self.Ahat, s_dP1)
+            self._sG0 = (s_dP1, sG0, self.absX.T @ sG0)
+        return self._sG0
+
+
+def cerr(a, b, s):
+    return float(np.max(np.abs(a - b) / np.maximum(s, 1e-300)))
+
+
+class OracleEpochL:
+    """The ℓ-layer generalisation (oracle.gcn.forward_l/backward_l) with the
+    same condition scales, layer by layer:
+        s_P[0] = Â(|X||Θ0|),  s_P[l] = Â(s_P[l-1]|Θl|),  s_H[0] = |X|, s_H[l] = s_P[l-1]
+        s_G[ℓ-1] = Â s_dL,    s_∇Θl = s_H[l]ᵀ s_G[l],
+        s_dP[l-1] = (s_G[l]|Θl|ᵀ) ⊙ keep_{l-1},  s_G[l-1] = Â s_dP[l-1]."""
+
+    def __init__(self, g, X, Ths, y, T):
+        self.Ahat = A = O.normalized_adjacency(g.n, g.rowptr, g.col)[0]
+        self.X64 = np.asarray(X, dtype=np.float64)
+        self.Ths = [np.asarray(t, dtype=np.float64) for t in Ths]
+        self.y, self.T = np.asarray(y), np.asarray(T, dtype=bool)
+        self.nT = int(self.T.sum())
+        self.Ps, self.Hs = O.forward_l(A, self.X64, self.Ths)
+        self.sP, sH = [], np.abs(self.X64)
+        for Th in self.Ths:
+            self.sP.append(O.aggregate(A, sH @ np.abs(Th)))
+            sH = self.sP[-1]
+        Lg = self.Ps[-1]
+        self.loss, self.dL = O.softmax_ce(Lg, self.y, self.T)
+        m = Lg.max(axis=1, keepdims=True)
+        p = np.exp(Lg - m)
+        p /= p.sum(axis=1, keepdims=True)
+        onehot = np.zeros_like(Lg)
+        onehot[np.arange(g.n), self.y] = 1.0
+        smax = self.sP[-1].max(axis=1, keepdims=True)
+        self.s_dL = self.T[:, None] * (2 * p * smax + p + onehot) / self.nT
+        lse = (m + np.log(np.exp(Lg - m).sum(axis=1, keepdims=True))).ravel()
+        Ly = Lg[np.arange(g.n), self.y]
+        self.s_loss = float(((2 * smax.ravel() + np.abs(lse) + np.abs(Ly)) * self.T).sum() / self.nT)
+
+    def band(self, l):
+        return np.abs(self.Ps[l]) <= BAND * self.sP[l]
+
+    def backward_scales(self):
+        nl = len(self.Ths)
+        sG = [None] * nl
+        sgrad = [None] * nl
+        G = O.aggregate(self.Ahat, self.s_dL)
+        for l in range(nl - 1, -1, -1):
+            sG[l] = G
+            sH = np.abs(self.X64) if l == 0 else self.sP[l - 1]
+            sgrad[l] = sH.T @ G
+            if l > 0:
+                keep = (self.Ps[l - 1] > 0) | self.band(l - 1)
+                G = O.aggregate(self.Ahat, (G @ np.abs(self.Ths[l]).T) * keep)
+        return sG, sgrad
+
+
+def check_gcnl_epoch(model, ref: OracleEpochL, perm, lr=None, report=None):
+    """The ℓ-layer model (gcn.GCNL) after one epoch vs OracleEpochL.  ReLU
+    decisions: everything outside the band must agree; inside it the GPU's
+    decisions (its bit masks) are the admissible ones taken (module doc)."""
+    inv = np.argsort(perm)
+    dims = [ref.X64.shape[1]] + [t.shape[1] for t in ref.Ths]
+    nl = len(ref.Ths)
+    errs = {}
+    Ps = list(ref.Ps)
+    for l in range(nl - 1):
+        gbits = mask_bits(model.mask[l], dims[l + 1], inv)
+        band = ref.band(l)
+        assert np.all((gbits == (ref.Ps[l] > 0)) | band), f"layer {l}: ReLU decisions differ outside the band"
+        assert band.mean() <= 1e-3, (l, band.mean())
+        errs[f"relu_band_entries_{l}"] = int(band.sum())
+        errs[f"H{l + 1}"] = cerr(_np(model.H[l])[:, :dims[l + 1]][inv], np.maximum(ref.Ps[l], 0), ref.sP[l])
+        Ps[l] = np.where(band, np.where(gbits, 1e-300, -1e-300), ref.Ps[l])
+    errs["logits"] = cerr(_np(model.Lg)[:, :dims[-1]][inv], ref.Ps[-1], ref.sP[-1])
+    errs["loss"] = abs(model.loss.item() - ref.loss) / ref.s_loss
+    grads, Gs = O.backward_l(ref.Ahat, ref.Ths, Ps, ref.Hs, ref.dL)
+    sG, sgrad = ref.backward_scales()
+    for l in range(nl):
+        errs[f"G{l}"] = cerr(_np(model.G[l])[:, :dims[l + 1]][inv], Gs[l], sG[l])
+        errs[f"grad{l}"] = cerr(_np(model.gTh[l]), grads[l], sgrad[l])
+    if lr is not None:
+        th = np.concatenate([t.ravel() for t in ref.Ths])
+        g = _np(model.grad)
+        errs["sgd_step"] = cerr((th - _np(model.theta)) / lr, g, np.abs(th) / lr + np.abs(g))
+    if report is not None:
+        report.update(errs)
+    for k, v in errs.items():
+        if k.startswith("relu"):
+            continue
+        assert v <= (1e-6 if k == "sgd_step" else TOL), (k, errs)
+    return errs
+
+
+def check_gcn2_epoch(model, ref: OracleEpoch, perm, lr=None, Th0=None, Th1=None, report=None):
+    """Compare a GCN2 (one epoch already run, eager or graph replay) with the
+    oracle epoch.  ``lr``/``Th0``/``Th1``: also check the SGD update the model
+    applied, (Θ - Θ')/lr = ∇Θ.  Returns the dict of condition-scaled errors."""
+    inv = np.argsort(perm)
+    H, C = ref.Th0.shape[1], ref.Th1.shape[1]
+
+    def up(t, F):
+        return _np(t)[:, :F][inv]
+
+    errs = {}
+    errs["H1"] = cerr(up(model.H1, H), ref.H1, ref.sP1)
+    errs["L"] = cerr(up(model.Lg, C), ref.L, ref.sL)
+    errs["loss"] = abs(model.loss.item() - ref.loss) / ref.s_loss
+    errs["G1"] = cerr(up(model.G1, C), O.aggregate(ref.Ahat, ref.dL), ref.sG1)
+    # ReLU decisions
+    gbits = mask_bits(model.mask1, H, inv)
+    band = np.abs(ref.P1) <= BAND * ref.sP1
+    outside_ok = (gbits == (ref.P1 > 0)) | band
+    assert outside_ok.all(), f"{int((~outside_ok).sum())} ReLU decisions differ outside the error band"
+    amb = np.argwhere(band)
+    errs["relu_band_entries"] = int(len(amb))
+    variants = []
+    if len(amb) <= ENUM:
+        for bits in range(2 ** len(amb)):
+            P1v = ref.P1.copy()
+            for t, (i, f) in enumerate(amb):
+                P1v[i, f] = 1e-300 if (bits >> t) & 1 else -1e-300
+            variants.append(P1v)
+    else:
+        assert band.mean() <= 1e-3, f"ReLU band holds {band.mean():.2e} of the decisions: vacuous check"
+        variants.append(np.where(band, np.where(gbits, 1e-300, -1e-300), ref.P1))
+    gTh1 = _np(model.gTh1)
+    errs["gTh1"] = cerr(gTh1, ref.H1.T @ O.aggregate(ref.Ahat, ref.dL), ref.s_gTh1)
+    G0 = up(model.G0, H)
+    gTh0 = _np(model.gTh0)
+    best = None
+    for P1v in variants:
+        b = ref.backward(P1v)
+        s_dP1, sG0, s_gTh0 = ref.backward_scales()
+        e = {"G0": cerr(G0, b["G0"], sG0), "gTh0": cerr(gTh0, b["gTh0"], s_gTh0)}
+        # information only: the same error against the plain |X|ᵀ|G0| scale
+        e["gTh0_vs_plain_scale"] = cerr(gTh0, b["gTh0"], ref.absX.T @ np.abs(b["G0"]))
+        if best is None or max(e["G0"], e["gTh0"]) < max(best[0]["G0"], best[0]["gTh0"]):
+            best = (e, b)
+    errs.update(best[0])
+    if lr is not None:
+        # the SGD step Θ' = fl(Θ - fl(lr·g)) applied the gradient the model holds:
+        # (Θ - Θ')/lr recovers it up to u·(|Θ|/lr + |g|)
+        new = _np(model.theta)
+        th = np.concatenate([np.asarray(Th0, np.float64).ravel(), np.asarray(Th1, np.float64).ravel()])
+        g = _np(model.grad)
+        errs["sgd_step"] = cerr((th - new) / lr, g, np.abs(th) / lr + np.abs(g))
+    if report is not None:
+        report.update(errs)
+    for k in ("H1", "L", "loss", "G1", "gTh1", "G0", "gTh0"):
+        assert errs[k] <= TOL, (k, errs)
+    if lr is not None:
+        assert errs["sgd_step"] <= 1e-6, errs
+    return errs

@@ -38,7 +38,7 @@ def _exchange_worker(rank, world, port, ranges, q):
     n = ranges[-1][1]
     full = torch.full((n, 3), -1.0)
     full[lo:hi] = torch.arange(lo, hi, dtype=torch.float32)[:, None] * 10 + rank
-    ex = RowExchange(lo, hi)
+    ex = RowExchange(lo, hi, n=n)
     ex.gather(full)
     g = torch.full((4,), float(rank + 1))
     ex.allreduce(g)
@@ -65,9 +65,17 @@ def test_row_exchange_gloo_world2():
 
 
 def test_row_exchange_rejects_gaps():
-    # ranges must tile the rows: checked locally without a process group
-    from paper_conf_ipps_tianmyd20_b200 import dist as D
-    assert hasattr(D, "RowExchange")
+    """Shard ranges must tile [0, n) in rank order (checked without a process group)."""
+    from paper_conf_ipps_tianmyd20_b200.dist import check_ranges
+    check_ranges([(0, 7), (7, 19)], 19)
+    check_ranges([(0, 0), (0, 5)], 5)                 # an empty shard is allowed
+    for bad, n in (([(0, 7), (8, 19)], 19),          # gap
+                   ([(0, 8), (7, 19)], 19),          # overlap
+                   ([(1, 7), (7, 19)], 19),          # does not start at 0
+                   ([(0, 7), (7, 18)], 19),          # does not reach n
+                   ([(0, 7), (9, 7)], None)):        # negative range
+        with pytest.raises(ValueError):
+            check_ranges(bad, n)
 
 
 # ---------------------------------------------------------------------------

@@ -293,6 +293,38 @@ def test_adam_first_step_closed_form():
     np.testing.assert_allclose(new, -0.01 * g / (np.abs(g) + 1e-8), rtol=1e-12)
 
 
+def test_adam_constant_gradient_any_step():
+    """For a constant gradient the bias corrections are exact at every t:
+    m_t = (1-b1^t) g and v_t = (1-b2^t) g^2, so m̂ = g, v̂ = g^2 and every step
+    moves by lr·g/(|g|+eps) (Kingma & Ba, §2-3).  Checks t = 1..6, including
+    the t = 2 state the GPU Adam is compared against."""
+    g = np.array([0.3, -2.0, 1e-3, 0.0, 7.5])
+    Th, m, v = np.zeros_like(g), np.zeros_like(g), np.zeros_like(g)
+    for t in range(1, 7):
+        Th, m, v = O.adam(Th, g, m, v, t, lr=0.01)
+        np.testing.assert_allclose(m, (1 - 0.9 ** t) * g, rtol=1e-12)
+        np.testing.assert_allclose(v, (1 - 0.999 ** t) * g * g, rtol=1e-12)
+        np.testing.assert_allclose(Th, -0.01 * t * g / (np.abs(g) + 1e-8), rtol=1e-12, atol=1e-300)
+
+
+def test_adam_two_steps_sign_flip_and_scale_invariance():
+    """t = 2 with g2 = -g1: m_2 = b1(1-b1) g - (1-b1) g = -(1-b1)^2 g, so
+    m̂_2 = -(1-b1)^2/(1-b1^2) g = -(0.01/0.19) g, while v̂_2 = g^2 (both terms
+    carry g^2).  And Adam is invariant to a positive rescaling of all
+    gradients up to eps (a wrong power of v or a missing sqrt breaks it)."""
+    g = np.array([0.5, -3.0, 2e-2])
+    Th1, m, v = O.adam(np.zeros_like(g), g, np.zeros_like(g), np.zeros_like(g), 1)
+    Th2, m, v = O.adam(Th1, -g, m, v, 2)
+    step2 = Th2 - Th1
+    np.testing.assert_allclose(step2, 0.01 * (0.01 / 0.19) * g / np.abs(g), rtol=1e-6)
+    for c in (1e-2, 10.0, 1e3):
+        a, ma, va = O.adam(np.ones(3), c * g, np.zeros(3), np.zeros(3), 1, eps=0.0)
+        a, _, _ = O.adam(a, c * 0.5 * g, ma, va, 2, eps=0.0)
+        b, mb, vb = O.adam(np.ones(3), g, np.zeros(3), np.zeros(3), 1, eps=0.0)
+        b, _, _ = O.adam(b, 0.5 * g, mb, vb, 2, eps=0.0)
+        np.testing.assert_allclose(a, b, rtol=1e-12)
+
+
 # P16: Table I counting convention (nnz(A+I) = 2m + n), PAPER.md L216
 def test_p16_counting_convention():
     g = G.sbm(C.PUBMED.spec)
