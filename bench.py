@@ -43,6 +43,10 @@ def parse():
     ap.add_argument("--workload", default="reddit")
     ap.add_argument("--theta", default="auto")
     ap.add_argument("--P", type=int, default=0)
+    ap.add_argument("--order", default="id", choices=["id", "degree"],
+                    help="vertex order inside a partition (pcgcn_opts.vertex_order)")
+    ap.add_argument("--grain", default="block", choices=["block", "tile"],
+                    help="unit of the selective/full decision (pcgcn_opts.mode_grain)")
     ap.add_argument("--oracle-frac", type=float, default=0.02)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
@@ -417,6 +421,12 @@ def run_f2(args):
 # ---------------------------------------------------------------------------
 # our arm
 # ---------------------------------------------------------------------------
+def plan_kw(args):
+    from paper_conf_ipps_tianmyd20_b200 import _lib as L
+    return dict(order=L.ORDER_DEGREE if args.order == "degree" else L.ORDER_ID,
+                grain=L.GRAIN_TILE if args.grain == "tile" else L.GRAIN_BLOCK)
+
+
 def main():
     args = parse()
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -465,7 +475,7 @@ def main():
         theta_src += "single plan (C5-sized graph: no in-situ refinement / grid)"
     elif args.theta == "auto":
         # 2) in-situ refinement per width on this workload (pcgcn_refine_theta)
-        pl0 = L.Plan(g.n, g.rowptr, g.col, P, theta0, f_max=fmax, rank=rank, world=world)
+        pl0 = L.Plan(g.n, g.rowptr, g.col, P, theta0, f_max=fmax, rank=rank, world=world, **plan_kw(args))
         perm = pl0.perm()
         Xp = np.ascontiguousarray(X[perm])
         m0 = GCN2(pl0, Xp, labels[perm], T[perm], Th0, Th1, optimizer="sgd", lr=0.0, device=dev,
@@ -481,14 +491,16 @@ def main():
         # 3) measured choice: time both widths on plans over a θ grid, keep the fastest per width
         #    (large graphs: the in-situ estimates plus the L161 value only — each plan costs seconds)
         if g.nnz < 200_000_000:
-            grid = sorted({round(x, 4) for x in (0.01, 0.014, 0.02, 0.028, 0.04, 0.056, 0.08, thH, thC) if x > 0})
+            base = ((0.02, 0.03, 0.045, 0.06, 0.08, 0.11, 0.15) if args.grain == "tile"
+                    else (0.01, 0.014, 0.02, 0.028, 0.04, 0.056, 0.08))
+            grid = sorted({round(x, 4) for x in (*base, thH, thC) if x > 0})
         else:
             grid = sorted({round(x, 5) for x in (thH, thC, theta0) if x > 0})
         ZH = torch.empty(g.n, Y0.shape[1], device=dev)
         ZC = torch.empty(g.n, Y1.shape[1], device=dev)
         best = {}
         for th in grid:
-            pt = L.Plan(g.n, g.rowptr, g.col, P, th, f_max=fmax, rank=rank, world=world)
+            pt = L.Plan(g.n, g.rowptr, g.col, P, th, f_max=fmax, rank=rank, world=world, **plan_kw(args))
             for F, Yin, Zout in ((w.hidden, Y0, ZH), (w.classes, Y1, ZC)):
                 ts = []
                 for it in range(4):
@@ -514,8 +526,8 @@ def main():
     else:
         theta, theta_src = float(args.theta), "fixed"
     t0 = time.time()
-    pl = L.Plan(g.n, g.rowptr, g.col, P, theta, f_max=fmax, rank=rank, world=world)
-    pl_c = L.Plan(g.n, g.rowptr, g.col, P, theta_c, f_max=fmax, rank=rank, world=world) if theta_c else None
+    pl = L.Plan(g.n, g.rowptr, g.col, P, theta, f_max=fmax, rank=rank, world=world, **plan_kw(args))
+    pl_c = L.Plan(g.n, g.rowptr, g.col, P, theta_c, f_max=fmax, rank=rank, world=world, **plan_kw(args)) if theta_c else None
     st = pl.stats()
     st_c = pl_c.stats() if pl_c else st
     log(f"[bench] plans in {time.time() - t0:.1f}s theta={theta:.4g} theta_c={theta_c} ({theta_src}) stats={st}")
@@ -747,7 +759,7 @@ def main():
         ZC = torch.empty(model.Lg.shape, device=dev)
         for th in [float(x) for x in args.sweep.split(",")]:
             try:
-                pt = L.Plan(g.n, g.rowptr, g.col, P, th, f_max=fmax, rank=rank, world=world)
+                pt = L.Plan(g.n, g.rowptr, g.col, P, th, f_max=fmax, rank=rank, world=world, **plan_kw(args))
             except Exception as e:  # e.g. a full-mode plan that does not fit (the paper's "oom", L276)
                 sweep.append({"theta": th, "error": str(e)[:120]})
                 continue

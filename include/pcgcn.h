@@ -86,7 +86,22 @@ typedef struct {
   const int32_t* part;    /* HOST [n] optional partition override (0 <= part < P); NULL => LP + packing */
   int32_t build_device;   /* 1 (default): upload to the current CUDA device; 0: host-only plan (tests) */
   int32_t rank, world;    /* destination-partition shard of this process; default 0, 1 */
+  int32_t vertex_order;   /* PCGCN_ORDER_*: order of the vertices inside a partition; default ID */
+  int32_t mode_grain;     /* PCGCN_GRAIN_*: unit of the selective/full decision; default BLOCK */
 } pcgcn_opts;
+
+/* Vertex order inside a vertex block V_k (the paper fixes only the blocks, L95-L97):
+ *   ID     — ascending original id (plan spec of DESIGN.md §3a);
+ *   DEGREE — descending degree, ties by id: high-degree rows and sources gather at the
+ *            start of every block, so the 128x32 sub-blocks of a dense region are denser
+ *            (reading #24). */
+enum { PCGCN_ORDER_ID = 0, PCGCN_ORDER_DEGREE = 1 };
+/* Unit of the mode decision (θ rule of L161):
+ *   BLOCK — the partition pair E_{k,i}: full iff nnz(E_ki)/(|V_k||V_i|) > θ (the paper);
+ *   TILE  — the 128-row x 32-source sub-block the full mode executes as one chunk (a row
+ *           tile of V_k against a 32-aligned source window): full iff its nnz/(rows·cols) > θ,
+ *           the same rule at the granularity of the B200 kernel (reading #25). */
+enum { PCGCN_GRAIN_BLOCK = 0, PCGCN_GRAIN_TILE = 1 };
 
 /* Plan statistics (L304-style mode usage + cost model inputs). */
 typedef struct {
@@ -112,7 +127,10 @@ void pcgcn_opts_default(pcgcn_opts* o);
  *          nnz(E_ki)/(|V_k||V_i|) > θ (strict, reading #10).
  *          θ = 0  => every non-empty block dense  ("PCGCN-full", Table III)
  *          θ >= 1 => every block sparse           ("PCGCN-sel", Table III)
- *          θ < 0  => PCGCN_EINVAL here; use pcgcn_calibrate() first.
+ *          θ < 0  => calibrate first on the current device (pcgcn_calibrate at width
+ *                    f_max, p = 0.05, blocks of the mean partition size; L161), then plan
+ *                    with that θ (the value lands in pcgcn_stats.theta); needs
+ *                    build_device = 1, else PCGCN_EINVAL.  NaN => PCGCN_EINVAL.
  *   P: number of vertex blocks K (Alg. 1 "Partition G -> {S_k}", L112), 1..n.
  * On success *out owns host + device memory until pcgcn_destroy. */
 pcgcn_status pcgcn_plan(const pcgcn_csr* A, int32_t P, float theta, const pcgcn_opts* o,

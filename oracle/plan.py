@@ -1,7 +1,7 @@
 """Plan oracle — TEST INFRASTRUCTURE ONLY (same import rule as oracle/gcn.py).
 
 An independent numpy re-derivation, from the written spec (SURVEY.md §8(c)
-item 4 and DESIGN.md "Plan spec"), of everything the host planner exports.
+item 4 and DESIGN.md §3a "Plan spec"), of everything the host planner exports.
 The tests compare it bit-exactly with ``pcgcn_plan_export``.
 
 Paper passages it follows:
@@ -80,8 +80,16 @@ def pack(labels: np.ndarray, P: int) -> np.ndarray:
     return part
 
 
-def build(n: int, rowptr, col, P: int, theta: float, part=None, norm: str = "sym"):
-    """Every plan array, in export order.  ``part`` overrides the partitioner."""
+def build(n: int, rowptr, col, P: int, theta: float, part=None, norm: str = "sym", order: str = "id",
+          grain: str = "block"):
+    """Every plan array, in export order.  ``part`` overrides the partitioner.
+
+    order: "id" — vertices of a block by ascending id; "degree" — by descending
+           degree, ties by id (reading #24).
+    grain: "block" — the paper's rule per partition pair E_{k,i} (L161):
+           full iff nnz/(|V_k||V_i|) > θ; "tile" — the same rule per chunk
+           (128-row tile of V_k x 32-aligned source window), density =
+           nnz/(tile rows · min(32, n - window start)) (reading #25)."""
     A = binary_adjacency(n, rowptr, col)
     deg = np.diff(A.indptr).astype(np.int64)
     dt = deg + 1
@@ -93,7 +101,10 @@ def build(n: int, rowptr, col, P: int, theta: float, part=None, norm: str = "sym
         lab, sweeps = label_propagation(A)
         part = pack(lab, P)
     part = np.asarray(part, dtype=np.int32)
-    perm = np.lexsort((np.arange(n), part)).astype(np.int32)  # new -> old
+    if order == "degree":
+        perm = np.lexsort((np.arange(n), -deg, part)).astype(np.int32)  # new -> old
+    else:
+        perm = np.lexsort((np.arange(n), part)).astype(np.int32)
     inv = np.empty(n, dtype=np.int64)
     inv[perm] = np.arange(n)
     psize = np.bincount(part, minlength=P).astype(np.int64)
@@ -119,8 +130,31 @@ def build(n: int, rowptr, col, P: int, theta: float, part=None, norm: str = "sym
     blk_dense = (dens > np.float64(np.float32(theta))).astype(np.uint8)
 
     # split edges by mode
-    dense_of = dict(zip(ub.tolist(), blk_dense.tolist()))
-    emode = np.array([dense_of[b] for b in bkey.tolist()], dtype=np.uint8) if len(bkey) else np.zeros(0, np.uint8)
+    if grain == "tile":
+        # chunk of an edge: (destination row tile inside its partition, 32-aligned source window)
+        tkey = pd * (n // TILE_M + 2) + (dst - pstart[pd]) // TILE_M
+        ckey = tkey * ((n + TILE_K - 1) // TILE_K) + src // TILE_K
+        uc, cinv, ccnt = np.unique(ckey, return_inverse=True, return_counts=True)
+        c_pd = np.zeros(len(uc), dtype=np.int64)
+        c_pd[cinv] = pd
+        c_dst = np.zeros(len(uc), dtype=np.int64)
+        c_dst[cinv] = dst
+        c_src = np.zeros(len(uc), dtype=np.int64)
+        c_src[cinv] = src
+        t0 = pstart[c_pd] + (c_dst - pstart[c_pd]) // TILE_M * TILE_M
+        rows_t = np.minimum(t0 + TILE_M, pstart[c_pd + 1]) - t0
+        w0 = c_src // TILE_K * TILE_K
+        cols_w = np.minimum(TILE_K, n - w0)
+        cdense = ccnt.astype(np.float64) / (rows_t.astype(np.float64) * cols_w.astype(np.float64)) \
+            > np.float64(np.float32(theta))
+        emode = cdense[cinv].astype(np.uint8)
+        # a block is marked full-mode iff it holds full-mode edges
+        blk_dense = np.zeros(len(ub), dtype=np.uint8)
+        blk_dense[np.searchsorted(ub, bkey[emode == 1])] = 1
+    else:
+        dense_of = dict(zip(ub.tolist(), blk_dense.tolist()))
+        emode = (np.array([dense_of[b] for b in bkey.tolist()], dtype=np.uint8) if len(bkey)
+                 else np.zeros(0, np.uint8))
     sm = emode == 0
     sp_rowptr = np.zeros(n + 1, dtype=np.int64)
     np.cumsum(np.bincount(dst[sm], minlength=n), out=sp_rowptr[1:])

@@ -26,6 +26,8 @@ c_i32, c_i64, c_f32, c_u32, c_vp = ctypes.c_int32, ctypes.c_int64, ctypes.c_floa
 OK, EINVAL, ENOTSYM, ECUDA, ENOMEM, ENCCL, EUNSUP = range(7)
 NORM_SYM, NORM_NONE = 0, 1
 DENSE_TF32X2, DENSE_FP32_SIMT, DENSE_BF16X1 = 0, 1, 2
+ORDER_ID, ORDER_DEGREE = 0, 1
+GRAIN_BLOCK, GRAIN_TILE = 0, 1
 IN_PRESCALED, RELU, MASK_OUT, OUT_PRESCALED, PROFILE = 1, 2, 4, 8, 16
 TIMING_NAMES = ("prescale", "split", "dense_tc", "sparse")
 X_NAMES = ["part", "perm", "pstart", "r", "blk_k", "blk_i", "blk_nnz", "blk_dense", "sp_rowptr", "sp_col",
@@ -41,7 +43,8 @@ class Csr(ctypes.Structure):
 
 class Opts(ctypes.Structure):
     _fields_ = [("norm", c_i32), ("dense_prec", c_i32), ("f_max", c_i32), ("lp_sweeps", c_i32),
-                ("part", c_vp), ("build_device", c_i32), ("rank", c_i32), ("world", c_i32)]
+                ("part", c_vp), ("build_device", c_i32), ("rank", c_i32), ("world", c_i32),
+                ("vertex_order", c_i32), ("mode_grain", c_i32)]
 
 
 class Stats(ctypes.Structure):
@@ -121,7 +124,8 @@ class Plan:
     """pcgcn_plan / pcgcn_forward / pcgcn_backward / pcgcn_destroy."""
 
     def __init__(self, n, rowptr, col, P, theta, *, norm=NORM_SYM, dense_prec=DENSE_TF32X2, f_max=128,
-                 lp_sweeps=10, part=None, build_device=True, rank=0, world=1):
+                 lp_sweeps=10, part=None, build_device=True, rank=0, world=1, order=ORDER_ID,
+                 grain=GRAIN_BLOCK):
         self._h = None
         self.n = int(n)
         rowptr = np.ascontiguousarray(rowptr, dtype=np.int64)
@@ -135,12 +139,14 @@ class Plan:
             o.part = part.ctypes.data
         o.build_device = 1 if build_device else 0
         o.rank, o.world = rank, world
+        o.vertex_order, o.mode_grain = order, grain
         h = c_vp()
         check(lib.pcgcn_plan(ctypes.byref(A), int(P), float(theta), ctypes.byref(o), ctypes.byref(h)), "pcgcn_plan")
         self._h = h
         self.P = int(P)
         self.f_max = f_max
         st = self.stats()
+        self.theta = st["theta"]
         self.row_lo, self.row_hi = st["row_lo"], st["row_hi"]
 
     def __del__(self):

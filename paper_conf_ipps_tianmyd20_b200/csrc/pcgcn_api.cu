@@ -6,6 +6,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cmath>
 #include <cstdlib>
 #include <cstring>
 #include <new>
@@ -352,7 +353,7 @@ using namespace pcgcn;
 
 extern "C" {
 
-int32_t pcgcn_abi_version(void) { return 1; }
+int32_t pcgcn_abi_version(void) { return 2; }
 
 const char* pcgcn_last_error(void) { return g_err.c_str(); }
 
@@ -387,6 +388,25 @@ pcgcn_status pcgcn_plan(const pcgcn_csr* A, int32_t P, float theta, const pcgcn_
       o->dense_prec != PCGCN_DENSE_BF16X1) {
     set_error("unknown dense_prec");
     return PCGCN_EUNSUP;
+  }
+  if ((o->vertex_order != PCGCN_ORDER_ID && o->vertex_order != PCGCN_ORDER_DEGREE) ||
+      (o->mode_grain != PCGCN_GRAIN_BLOCK && o->mode_grain != PCGCN_GRAIN_TILE)) {
+    set_error("unknown vertex_order / mode_grain");
+    return PCGCN_EUNSUP;
+  }
+  if (!(theta >= 0.f)) {
+    // θ < 0: the L161 procedure on this device first (synthetic p = 0.05 blocks
+    // of the plan's mean partition size, width f_max)
+    if (!o->build_device || std::isnan(theta)) {
+      set_error("theta < 0 (calibrate on the device) needs build_device = 1");
+      return PCGCN_EINVAL;
+    }
+    const int64_t rows = A->n / (P > 0 ? P : 1);
+    float th = 0.f, tf = 0.f, ts = 0.f;
+    pcgcn_status cs = pcgcn_calibrate(o->f_max, int32_t(std::max<int64_t>(64, std::min<int64_t>(8192, rows))),
+                                      0.05f, &th, &tf, &ts);
+    if (cs != PCGCN_OK) return cs;
+    theta = th;
   }
   if (o->dense_prec == PCGCN_DENSE_FP32_SIMT && o->f_max > 128) {
     set_error("FP32_SIMT full mode supports F <= 128");

@@ -8,7 +8,7 @@
 //   4. the K×K edge-block table with densities and mode bits (θ rule, L161)
 //   5. the merged selective CSR (L179) and the full-mode tiles (L175) as
 //      128×32 bit chunks grouped per 128-row destination tile.
-// The plan spec it implements is DESIGN.md "Plan spec"; oracle/plan.py is an
+// The plan spec it implements is DESIGN.md §3a; oracle/plan.py is an
 // independent re-derivation and tests/test_plan_abi.py compares them bit-exactly.
 #include <algorithm>
 #include <chrono>
@@ -175,6 +175,10 @@ pcgcn_status build_host_plan(const pcgcn_csr* A, int32_t P, float theta, const p
   for (int64_t v = 0; v < n; ++v)
     if (A->rowptr[v + 1] < A->rowptr[v]) { set_error("rowptr not monotone"); return PCGCN_EINVAL; }
   if (!(theta >= 0.f)) { set_error("theta must be >= 0 (calibrate first)"); return PCGCN_EINVAL; }
+  if (o->vertex_order != PCGCN_ORDER_ID && o->vertex_order != PCGCN_ORDER_DEGREE) {
+    set_error("unknown vertex_order");
+    return PCGCN_EINVAL;
+  }
   if (o->world < 1 || o->rank < 0 || o->rank >= o->world) { set_error("bad rank/world"); return PCGCN_EINVAL; }
   p->n = n; p->P = P; p->theta = theta; p->opts = *o;
 
@@ -205,7 +209,7 @@ pcgcn_status build_host_plan(const pcgcn_csr* A, int32_t P, float theta, const p
   }
   double part_ms = ms_since(tp);
 
-  // permutation: sort by (part, id)
+  // permutation: sort by (part, id), or by (part, -degree, id) (vertex_order DEGREE)
   std::vector<int64_t> psize(P, 0);
   for (int64_t v = 0; v < n; ++v) psize[p->part[v]]++;
   p->pstart.assign(P + 1, 0);
@@ -214,11 +218,17 @@ pcgcn_status build_host_plan(const pcgcn_csr* A, int32_t P, float theta, const p
   std::vector<int64_t> inv(n);
   {
     std::vector<int64_t> fill(p->pstart.begin(), p->pstart.end() - 1);
-    for (int64_t v = 0; v < n; ++v) {
-      int64_t pos = fill[p->part[v]]++;
-      p->perm[pos] = int32_t(v);
-      inv[v] = pos;
+    for (int64_t v = 0; v < n; ++v) p->perm[fill[p->part[v]]++] = int32_t(v);  // (part, id)
+    if (o->vertex_order == PCGCN_ORDER_DEGREE) {
+      parallel_for(P, [&](int, int64_t a, int64_t b) {
+        for (int64_t k = a; k < b; ++k)
+          std::stable_sort(p->perm.begin() + p->pstart[k], p->perm.begin() + p->pstart[k + 1],
+                           [&](int32_t x, int32_t y) {
+                             return C.ptr[x + 1] - C.ptr[x] > C.ptr[y + 1] - C.ptr[y];
+                           });
+      });
     }
+    for (int64_t pos = 0; pos < n; ++pos) inv[p->perm[pos]] = pos;
   }
   p->r.resize(n);
   for (int64_t v = 0; v < n; ++v) p->r[v] = r_orig[p->perm[v]];
@@ -267,6 +277,7 @@ pcgcn_status build_host_plan(const pcgcn_csr* A, int32_t P, float theta, const p
   const int64_t nb = bptr[P];
   p->blk_k.resize(nb); p->blk_i.resize(nb); p->blk_nnz.resize(nb); p->blk_dense.resize(nb);
   const double th = double(theta);
+  const bool tile_grain = o->mode_grain == PCGCN_GRAIN_TILE;
   int64_t nb_dense = 0, intra = 0;
   for (int32_t k = 0; k < P; ++k)
     for (size_t j = 0; j < blocks[k].size(); ++j) {
@@ -275,12 +286,16 @@ pcgcn_status build_host_plan(const pcgcn_csr* A, int32_t P, float theta, const p
       int64_t z = blocks[k][j].second;
       p->blk_k[b] = k; p->blk_i[b] = i; p->blk_nnz[b] = z;
       double dens = double(z) / (double(psize[k]) * double(psize[i]));
-      p->blk_dense[b] = dens > th ? 1 : 0;
-      nb_dense += p->blk_dense[b];
+      p->blk_dense[b] = (!tile_grain && dens > th) ? 1 : 0;
       if (i == k) intra += z;
     }
 
-  // mode of each edge -> merged selective CSR + dense chunks, per partition
+  // mode of each edge -> merged selective CSR + dense chunks, per partition.
+  // A chunk is the 128-row destination tile x 32-aligned global source window
+  // the full mode executes as one unit (TMA box starts must be 16-byte aligned,
+  // so windows are global, not partition-relative).  BLOCK grain: the edges of
+  // full-mode blocks, grouped into chunks (blocks sharing a window share its
+  // chunk); TILE grain: every chunk whose own density nnz/(rows·cols) > θ.
   std::vector<int64_t> sp_cnt(n, 0);
   struct TileOut {
     int32_t row0, nrows;
@@ -288,19 +303,26 @@ pcgcn_status build_host_plan(const pcgcn_csr* A, int32_t P, float theta, const p
     std::vector<uint32_t> bits;
   };
   std::vector<std::vector<TileOut>> tiles(P);
+  auto win_cols = [&](int64_t c0) { return double(std::min<int64_t>(TILE_K, n - c0)); };
   parallel_for(P, [&](int, int64_t a, int64_t b) {
     std::vector<uint8_t> dense_i(P, 0);
+    std::vector<int64_t> blk_pos(P, -1);
     std::vector<std::pair<int32_t, int32_t>> ent;  // (col0, (rr<<5)|bit)
     for (int64_t k = a; k < b; ++k) {
-      bool any_dense = false;
+      bool any_dense = tile_grain;
       for (int64_t j = bptr[k]; j < bptr[k + 1]; ++j) {
         dense_i[p->blk_i[j]] = p->blk_dense[j];
+        blk_pos[p->blk_i[j]] = j;
         any_dense |= p->blk_dense[j] != 0;
       }
-      for (int64_t v = p->pstart[k]; v < p->pstart[k + 1]; ++v) {
-        int64_t c = 0;
-        for (int64_t e = tptr[v]; e < tptr[v + 1]; ++e) c += dense_i[pid[tcol[e]]] ? 0 : 1;
-        sp_cnt[v] = c;
+      if (!tile_grain) {
+        for (int64_t v = p->pstart[k]; v < p->pstart[k + 1]; ++v) {
+          int64_t c = 0;
+          for (int64_t e = tptr[v]; e < tptr[v + 1]; ++e) c += dense_i[pid[tcol[e]]] ? 0 : 1;
+          sp_cnt[v] = c;
+        }
+      } else {
+        for (int64_t v = p->pstart[k]; v < p->pstart[k + 1]; ++v) sp_cnt[v] = tptr[v + 1] - tptr[v];
       }
       if (any_dense) {
         for (int64_t r0 = p->pstart[k]; r0 < p->pstart[k + 1]; r0 += TILE_M) {
@@ -309,10 +331,7 @@ pcgcn_status build_host_plan(const pcgcn_csr* A, int32_t P, float theta, const p
           for (int64_t v = r0; v < r1; ++v)
             for (int64_t e = tptr[v]; e < tptr[v + 1]; ++e) {
               int32_t j = tcol[e];
-              int32_t i = pid[j];
-              if (!dense_i[i]) continue;
-              // 32-aligned global source window (TMA box starts must be 16-byte
-              // aligned); dense blocks sharing a window share one chunk
+              if (!tile_grain && !dense_i[pid[j]]) continue;
               int64_t c0 = (int64_t(j) / TILE_K) * TILE_K;
               ent.push_back({int32_t(c0), int32_t(((v - r0) << 5) | (j - c0))});
             }
@@ -322,19 +341,35 @@ pcgcn_status build_host_plan(const pcgcn_csr* A, int32_t P, float theta, const p
           T.row0 = int32_t(r0);
           T.nrows = int32_t(r1 - r0);
           for (size_t q = 0; q < ent.size();) {
-            int32_t c0 = ent[q].first;
+            const int32_t c0 = ent[q].first;
+            size_t q1 = q;
+            while (q1 < ent.size() && ent[q1].first == c0) ++q1;
+            if (tile_grain && !(double(q1 - q) / (double(r1 - r0) * win_cols(c0)) > th)) {
+              q = q1;  // a selective chunk: its edges stay in the merged CSR
+              continue;
+            }
             size_t base = T.bits.size();
             T.col0.push_back(c0);
             T.bits.resize(base + TILE_M, 0u);
-            for (; q < ent.size() && ent[q].first == c0; ++q)
-              T.bits[base + (ent[q].second >> 5)] |= 1u << (ent[q].second & 31);
+            for (; q < q1; ++q) {
+              const int32_t rr = ent[q].second >> 5, bit = ent[q].second & 31;
+              T.bits[base + rr] |= 1u << bit;
+              if (tile_grain) {
+                sp_cnt[r0 + rr]--;
+                p->blk_dense[blk_pos[pid[c0 + bit]]] = 1;  // block holds full-mode edges
+              }
+            }
           }
-          tiles[k].push_back(std::move(T));
+          if (!T.col0.empty()) tiles[k].push_back(std::move(T));
         }
       }
-      for (int64_t j = bptr[k]; j < bptr[k + 1]; ++j) dense_i[p->blk_i[j]] = 0;
+      for (int64_t j = bptr[k]; j < bptr[k + 1]; ++j) {
+        dense_i[p->blk_i[j]] = 0;
+        blk_pos[p->blk_i[j]] = -1;
+      }
     }
   });
+  for (int64_t b2 = 0; b2 < nb; ++b2) nb_dense += p->blk_dense[b2];
   p->sp_rowptr.assign(n + 1, 0);
   for (int64_t v = 0; v < n; ++v) p->sp_rowptr[v + 1] = p->sp_rowptr[v] + sp_cnt[v];
   p->sp_col.resize(p->sp_rowptr[n]);
@@ -342,10 +377,30 @@ pcgcn_status build_host_plan(const pcgcn_csr* A, int32_t P, float theta, const p
     std::vector<uint8_t> dense_i(P, 0);
     for (int64_t k = a; k < b; ++k) {
       for (int64_t j = bptr[k]; j < bptr[k + 1]; ++j) dense_i[p->blk_i[j]] = p->blk_dense[j];
+      const TileOut* T = tiles[k].empty() ? nullptr : tiles[k].data();
+      size_t tn = tiles[k].size(), ti = 0;
       for (int64_t v = p->pstart[k]; v < p->pstart[k + 1]; ++v) {
         int64_t o2 = p->sp_rowptr[v];
-        for (int64_t e = tptr[v]; e < tptr[v + 1]; ++e)
-          if (!dense_i[pid[tcol[e]]]) p->sp_col[o2++] = tcol[e];
+        if (!tile_grain) {
+          for (int64_t e = tptr[v]; e < tptr[v + 1]; ++e)
+            if (!dense_i[pid[tcol[e]]]) p->sp_col[o2++] = tcol[e];
+          continue;
+        }
+        // TILE grain: the edge is selective unless its window is a chunk of v's tile
+        while (ti < tn && T[ti].row0 + T[ti].nrows <= v) ++ti;
+        const bool has = ti < tn && T[ti].row0 <= v;
+        const int32_t rr = has ? int32_t(v - T[ti].row0) : 0;
+        for (int64_t e = tptr[v]; e < tptr[v + 1]; ++e) {
+          const int32_t j = tcol[e];
+          bool dense = false;
+          if (has) {
+            const int32_t c0 = (j / TILE_K) * TILE_K;
+            auto it = std::lower_bound(T[ti].col0.begin(), T[ti].col0.end(), c0);
+            dense = it != T[ti].col0.end() && *it == c0 &&
+                    ((T[ti].bits[size_t(it - T[ti].col0.begin()) * TILE_M + rr] >> (j - c0)) & 1u);
+          }
+          if (!dense) p->sp_col[o2++] = j;
+        }
       }
       for (int64_t j = bptr[k]; j < bptr[k + 1]; ++j) dense_i[p->blk_i[j]] = 0;
     }

@@ -35,10 +35,10 @@ def _ld(F):
 
 
 def aggregate_gpu(g, Y, P, theta, *, dense=L.DENSE_TF32X2, norm=L.NORM_SYM, part=None, backward=False,
-                  flags=0, f_max=None):
+                  flags=0, f_max=None, **plan_kw):
     F = Y.shape[1]
     f_max = f_max or max(128, F)
-    pl = L.Plan(g.n, g.rowptr, g.col, P, theta, norm=norm, dense_prec=dense, part=part, f_max=f_max)
+    pl = L.Plan(g.n, g.rowptr, g.col, P, theta, norm=norm, dense_prec=dense, part=part, f_max=f_max, **plan_kw)
     perm = pl.perm()
     Yp = np.zeros((g.n, _ld(F)), dtype=np.float32)
     Yp[:, :F] = Y[perm]
@@ -81,15 +81,17 @@ SMALL = {
 
 
 @pytest.mark.parametrize("name", list(SMALL))
-@pytest.mark.parametrize("mode", ["sparse", "dense_tc", "dense_simt", "hybrid", "dense_bf16"])
+@pytest.mark.parametrize("mode", ["sparse", "dense_tc", "dense_simt", "hybrid", "dense_bf16", "hybrid_tile"])
 @pytest.mark.parametrize("F", [1, 7, 16, 33, 41, 48, 64, 128])
 def test_aggregation_parity(name, mode, F):
     g = SMALL[name]()
     P = max(1, min(8, g.n // 40))
-    theta = {"sparse": 2.0, "dense_tc": 0.0, "dense_simt": 0.0, "hybrid": 0.05, "dense_bf16": 0.0}[mode]
+    theta = {"sparse": 2.0, "dense_tc": 0.0, "dense_simt": 0.0, "hybrid": 0.05, "dense_bf16": 0.0,
+             "hybrid_tile": 0.05}[mode]
     dense = {"dense_simt": L.DENSE_FP32_SIMT, "dense_bf16": L.DENSE_BF16X1}.get(mode, L.DENSE_TF32X2)
+    kw = dict(order=L.ORDER_DEGREE, grain=L.GRAIN_TILE) if mode == "hybrid_tile" else {}
     Y = _feat(g.n, F, 11)
-    Z, pl, _ = aggregate_gpu(g, Y, P, theta, dense=dense)
+    Z, pl, _ = aggregate_gpu(g, Y, P, theta, dense=dense, **kw)
     err, _ = cond_err(g, Y, Z)
     # bf16 inputs (PCGCN_DENSE_BF16X1): |rounding| <= 2^-9 per term; gate 2e-2 (north star)
     tol = 2e-2 if mode == "dense_bf16" else TOL
@@ -112,16 +114,17 @@ def test_closed_forms_complete_and_cycle_dense():
     np.testing.assert_allclose(Z, exp, rtol=1e-5, atol=1e-6)
 
 
-@pytest.mark.parametrize("mode", ["sparse", "dense_tc", "dense_simt", "hybrid"])
+@pytest.mark.parametrize("mode", ["sparse", "dense_tc", "dense_simt", "hybrid", "hybrid_tile"])
 def test_integer_exact_bitwise(mode):
     """Pin P9: Ã unnormalised, small integers -> every order gives the exact
-    sum, so GPU (either mode, any partition) == oracle bitwise."""
+    sum, so GPU (either mode, any partition, any grain) == oracle bitwise."""
     g = G.cliques([300, 129, 64, 33, 2], seed=5)
     rng = np.random.default_rng(9)
     Y = rng.integers(-1000, 1000, size=(g.n, 40)).astype(np.float32)
-    theta = {"sparse": 2.0, "dense_tc": 0.0, "dense_simt": 0.0, "hybrid": 0.3}[mode]
+    theta = {"sparse": 2.0, "dense_tc": 0.0, "dense_simt": 0.0, "hybrid": 0.3, "hybrid_tile": 0.3}[mode]
     dense = L.DENSE_FP32_SIMT if mode == "dense_simt" else L.DENSE_TF32X2
-    Z, _, _ = aggregate_gpu(g, Y, 5, theta, dense=dense, norm=L.NORM_NONE)
+    kw = dict(order=L.ORDER_DEGREE, grain=L.GRAIN_TILE) if mode == "hybrid_tile" else {}
+    Z, _, _ = aggregate_gpu(g, Y, 5, theta, dense=dense, norm=L.NORM_NONE, **kw)
     exp = O.aggregate(O.normalized_adjacency(g.n, g.rowptr, g.col, "none")[0], Y.astype(np.float64))
     assert np.array_equal(Z, exp)
 
@@ -323,9 +326,11 @@ def test_epoch_parity(wname, theta, theta_c):
     check_gcn2_epoch(model, ref, perm, lr=0.1, Th0=Th0, Th1=Th1)
 
 
-@pytest.mark.parametrize("d,theta,theta_c", [(1.0, 0.05, 0.1), (1.0, 0.02, 0.02), (10.0, 0.1, 0.2),
-                                             (10.0, 0.0, 2.0), (5.0, 0.4, 0.1)])
-def test_rmat_hybrid_epoch_parity(d, theta, theta_c):
+@pytest.mark.parametrize("d,theta,theta_c,grain", [(1.0, 0.02, 0.02, "block"), (5.0, 0.1, 2.0, "block"),
+                                                   (10.0, 0.2, 0.1, "block"), (10.0, 0.0, 2.0, "block"),
+                                                   (1.0, 0.1, 0.05, "tile"), (5.0, 0.2, 0.3, "tile"),
+                                                   (10.0, 0.3, 0.2, "tile")])
+def test_rmat_hybrid_epoch_parity(d, theta, theta_c, grain):
     """SURVEY F1 / Table III workloads (RMAT-1, -5, -10: n = 10,240, 128 -> 64 -> 32,
     P = 16): mixed selective/full plans, one per
     width, as bench.py --table3 runs them — a full epoch vs the oracle."""
@@ -337,8 +342,9 @@ def test_rmat_hybrid_epoch_parity(d, theta, theta_c):
     Th0, Th1 = C.thetas(w)
     y = C.labels(w, g)
     T = C.train_mask(g.n, w.theta_seed)
-    pl = L.Plan(g.n, g.rowptr, g.col, w.P, theta, f_max=128)
-    pl_c = L.Plan(g.n, g.rowptr, g.col, w.P, theta_c, f_max=128)
+    kw = dict(f_max=128, order=L.ORDER_DEGREE, grain=L.GRAIN_TILE) if grain == "tile" else dict(f_max=128)
+    pl = L.Plan(g.n, g.rowptr, g.col, w.P, theta, **kw)
+    pl_c = L.Plan(g.n, g.rowptr, g.col, w.P, theta_c, **kw)
     st, st_c = pl.stats(), pl_c.stats()
     if 0 < theta < 1:
         assert 0 < st["nnz_dense"] < st["nnz"], st            # a mixed plan

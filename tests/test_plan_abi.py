@@ -1,6 +1,7 @@
 """Host planner (libpcgcn.so, C++) vs the plan oracle (oracle/plan.py):
 bit-exact on every exported array.  CPU only (plans built with
 build_device=0), plus ABI symbol / error-path checks."""
+import functools
 import os
 import re
 
@@ -16,6 +17,14 @@ L = pytest.importorskip("paper_conf_ipps_tianmyd20_b200._lib")
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
+@functools.lru_cache(maxsize=None)
+def _reddit_small():
+    """C3's recipe at 1% (2,328 vertices, 573K edges: dense, so the numpy
+    generator would loop over duplicate draws for a minute; the C++ twin is
+    bit-identical, tests/test_synth.py)."""
+    return C.graph(C.scaled(C.REDDIT, 0.01), impl="c")
+
+
 def test_exports_every_header_symbol():
     hdr = open(os.path.join(ROOT, "include", "pcgcn.h")).read()
     names = set(re.findall(r"\b(pcgcn_[a-z0-9_]+)\s*\(", hdr))
@@ -24,10 +33,12 @@ def test_exports_every_header_symbol():
         assert hasattr(L.lib, nm), nm
 
 
-def _compare(g, P, theta, part=None, norm="sym"):
+def _compare(g, P, theta, part=None, norm="sym", order="id", grain="block"):
     pl = L.Plan(g.n, g.rowptr, g.col, P, theta, part=part, build_device=False,
-                norm=L.NORM_NONE if norm == "none" else L.NORM_SYM)
-    ref = PL.build(g.n, g.rowptr, g.col, P, theta, part=part, norm=norm)
+                norm=L.NORM_NONE if norm == "none" else L.NORM_SYM,
+                order=L.ORDER_DEGREE if order == "degree" else L.ORDER_ID,
+                grain=L.GRAIN_TILE if grain == "tile" else L.GRAIN_BLOCK)
+    ref = PL.build(g.n, g.rowptr, g.col, P, theta, part=part, norm=norm, order=order, grain=grain)
     for name in L.X_NAMES:
         got = pl.export(name)
         exp = np.asarray(ref[name]).reshape(-1)
@@ -50,6 +61,16 @@ def test_bitexact_cora(theta):
     _compare(G.sbm(C.CORA.spec), 8, theta)
 
 
+@pytest.mark.parametrize("order,grain", [("degree", "block"), ("id", "tile"), ("degree", "tile")])
+@pytest.mark.parametrize("theta", [0.0, 0.03, 0.1, 0.3, 2.0])
+def test_bitexact_order_and_tile_grain(theta, order, grain):
+    """Vertex order DEGREE and the per-chunk (TILE) mode decision (DESIGN.md
+    readings #24, #25): bit-exact vs the oracle's independent derivation."""
+    _compare(G.sbm(C.CORA.spec), 8, theta, order=order, grain=grain)
+    _compare(_reddit_small(), 12, theta, order=order, grain=grain)
+    _compare(G.messy_random(700, 4000, 3), 5, theta, order=order, grain=grain)
+
+
 @pytest.mark.parametrize("theta", [0.0, 0.05, 2.0])
 def test_bitexact_pubmed_scaled(theta):
     w = C.scaled(C.PUBMED, 0.25)
@@ -57,8 +78,7 @@ def test_bitexact_pubmed_scaled(theta):
 
 
 def test_bitexact_reddit_scaled():
-    w = C.scaled(C.REDDIT, 0.01)
-    _compare(C.graph(w), 13, 0.03)
+    _compare(_reddit_small(), 13, 0.03)
 
 
 def test_bitexact_messy_input_and_override():

@@ -121,3 +121,62 @@ def test_r_bits():
     pl = PL.build(g.n, g.rowptr, g.col, P=1, theta=2.0)
     assert pl["r"][0] == np.float32(1 / np.sqrt(6.0))
     assert pl["r"][1] == np.float32(1 / np.sqrt(2.0))
+
+
+def _dense_matrix_from_plan(pl, n):
+    """Ã in plan order rebuilt from the selective CSR and the bit chunks, with
+    the mode of every entry (1 = full mode)."""
+    M = np.zeros((n, n), dtype=np.int64)
+    mode = np.zeros((n, n), dtype=np.int64)
+    for v in range(n):
+        for j in pl["sp_col"][pl["sp_rowptr"][v]:pl["sp_rowptr"][v + 1]]:
+            M[v, j] += 1
+    for t, (r0, nr) in enumerate(zip(pl["rt_row0"], pl["rt_nrows"])):
+        for c in range(pl["rt_cptr"][t], pl["rt_cptr"][t + 1]):
+            w = pl["bits"][c * 128:(c + 1) * 128]
+            for rr in range(nr):
+                for b in range(32):
+                    if (int(w[rr]) >> b) & 1:
+                        M[r0 + rr, pl["ch_col0"][c] + b] += 1
+                        mode[r0 + rr, pl["ch_col0"][c] + b] = 1
+    return M, mode
+
+
+@pytest.mark.parametrize("theta", [0.0, 0.05, 0.2, 0.6, 2.0])
+def test_degree_order_and_tile_grain_invariants(theta):
+    """Readings #24/#25 by brute force on the reassembled matrix: (a) inside
+    every partition the vertices run by descending degree (ties by id); (b)
+    every 128-row tile x 32-aligned window sub-block of Ã (in plan order) is
+    wholly full-mode iff its density nnz/(rows·min(32, n-c0)) > θ, else wholly
+    selective; (c) bits + CSR reassemble Ã exactly."""
+    g = G.cliques([40, 150, 7, 90, 300], seed=3)
+    rng = np.random.default_rng(5)
+    # sprinkle random edges so sub-block densities vary
+    e = rng.integers(0, g.n, size=(2000, 2))
+    g = G.from_edges(g.n, list(zip(*np.nonzero(
+        O.normalized_adjacency(g.n, g.rowptr, g.col, "none")[0].toarray() - np.eye(g.n)))) +
+        [tuple(x) for x in e.tolist() if x[0] != x[1]])
+    n = g.n
+    pl = PL.build(g.n, g.rowptr, g.col, P=3, theta=theta, order="degree", grain="tile")
+    deg = np.diff(O.binary_adjacency(n, g.rowptr, g.col).indptr)
+    perm = pl["perm"]
+    for k in range(3):
+        seg = perm[pl["pstart"][k]:pl["pstart"][k + 1]]
+        key = list(zip((-deg[seg]).tolist(), seg.tolist()))
+        assert key == sorted(key)
+    M, mode = _dense_matrix_from_plan(pl, n)
+    At = O.normalized_adjacency(n, g.rowptr, g.col, "none")[0].toarray()
+    inv = np.argsort(perm)
+    Ap = np.zeros_like(M)
+    Ap[np.ix_(inv, inv)] = At
+    assert np.array_equal(M, Ap)
+    for k in range(3):
+        for r0 in range(pl["pstart"][k], pl["pstart"][k + 1], 128):
+            r1 = min(r0 + 128, pl["pstart"][k + 1])
+            for c0 in range(0, n, 32):
+                sub = M[r0:r1, c0:c0 + 32]
+                if sub.sum() == 0:
+                    continue
+                dense = sub.sum() / (sub.shape[0] * sub.shape[1]) > np.float32(theta)
+                md = mode[r0:r1, c0:c0 + 32][sub > 0]
+                assert md.all() if dense else not md.any(), (k, r0, c0, theta)
