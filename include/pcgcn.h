@@ -118,6 +118,10 @@ typedef struct {
   double partition_ms, plan_ms; /* host time of LP+packing, and of the whole plan */
   int64_t device_bytes;         /* device memory owned by the plan */
   int64_t shard_segments;       /* long selective rows' segments (> 1024 edges per row, reading #22) */
+  int64_t src_rows_pc;          /* Σ_k |distinct sources of V_k's selective edges| (B_pc model) */
+  int64_t shard_src_rows_pc;    /* the same over this shard's partitions */
+  int64_t halo_recv_rows;       /* rows of other shards this shard reads (0 unsharded) */
+  int64_t halo_send_rows;       /* Σ_q rows of this shard that shard q reads */
 } pcgcn_stats;
 
 void pcgcn_opts_default(pcgcn_opts* o);
@@ -180,6 +184,25 @@ pcgcn_status pcgcn_forward(pcgcn_plan_t p, const float* Y, int64_t ldy, float* Z
  * reuses the forward plan.  Same argument rules as pcgcn_forward (mask unused). */
 pcgcn_status pcgcn_backward(pcgcn_plan_t p, const float* dZ, int64_t ldz, float* dY, int64_t ldy,
                             int32_t F, uint32_t flags, void* stream);
+
+/* ---- halo exchange of a sharded plan (world > 1) ----
+ * Shard r owns plan rows [row0[r], row0[r+1]).  Before an aggregation it needs the
+ * rows of other shards that its selective edges read and every row of the 32-source
+ * windows of its full-mode chunks: the halo.  The planner lists them per peer q
+ * (ascending plan rows): RECV = rows of shard q this shard reads, SEND = rows of this
+ * shard that shard q reads (= q's RECV list for this rank; every rank builds the same
+ * deterministic plan).  A shard's own rows are never listed; world = 1 => empty. */
+pcgcn_status pcgcn_plan_shard_rows(pcgcn_plan_t p, int64_t* row0 /* HOST [world+1] */);
+int64_t pcgcn_plan_halo_rows(pcgcn_plan_t p, int32_t q, int32_t send);  /* list length; -1 on bad args */
+pcgcn_status pcgcn_plan_halo_export(pcgcn_plan_t p, int32_t q, int32_t send, int32_t* host_buf, int64_t cap);
+/* pack: buf[i] = Y[send row i] for the concatenated SEND lists (peers in rank order),
+ * unpack: Y[recv row i] = buf[i] for the concatenated RECV lists.  Y DEVICE [n x ldy]
+ * (full height, plan order), buf DEVICE [rows x w] dense; w floats are copied per row
+ * (multiple of 4, <= ldy: pass the activation stride to move pad columns too).
+ * Bitwise copies; stream-ordered, graph-capturable.  The transport between the two
+ * (NCCL grouped send/recv, or an all-to-all) is the caller's (dist.py). */
+pcgcn_status pcgcn_halo_pack(pcgcn_plan_t p, const float* Y, int64_t ldy, int32_t w, float* buf, void* stream);
+pcgcn_status pcgcn_halo_unpack(pcgcn_plan_t p, const float* buf, float* Y, int64_t ldy, int32_t w, void* stream);
 
 /* ---- dense helpers of the 2-layer GCN step (Alg. 1 transform, L114) ---- */
 

@@ -53,7 +53,8 @@ class Stats(ctypes.Structure):
                 ("nnz_dense", c_i64), ("intra_edges", c_i64), ("row_tiles", c_i64), ("chunks", c_i64),
                 ("row_lo", c_i64), ("row_hi", c_i64), ("shard_nnz_sparse", c_i64), ("shard_chunks", c_i64),
                 ("theta", ctypes.c_double), ("partition_ms", ctypes.c_double), ("plan_ms", ctypes.c_double),
-                ("device_bytes", c_i64), ("shard_segments", c_i64)]
+                ("device_bytes", c_i64), ("shard_segments", c_i64), ("src_rows_pc", c_i64),
+                ("shard_src_rows_pc", c_i64), ("halo_recv_rows", c_i64), ("halo_send_rows", c_i64)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -92,6 +93,11 @@ _sig("pcgcn_refine_theta", c_i32, c_vp, c_vp, c_i64, c_vp, c_i64, c_i32, ctypes.
      ctypes.POINTER(c_f32), ctypes.POINTER(c_f32))
 _sig("pcgcn_probe_read_gbs", c_i32, c_i64, c_i32, ctypes.POINTER(c_f32))
 _sig("pcgcn_probe_gather_gbs", c_i32, c_i64, c_i32, c_i32, ctypes.POINTER(c_f32))
+_sig("pcgcn_plan_shard_rows", c_i32, c_vp, c_vp)
+_sig("pcgcn_plan_halo_rows", c_i64, c_vp, c_i32, c_i32)
+_sig("pcgcn_plan_halo_export", c_i32, c_vp, c_i32, c_i32, c_vp, c_i64)
+_sig("pcgcn_halo_pack", c_i32, c_vp, c_vp, c_i64, c_i32, c_vp, c_vp)
+_sig("pcgcn_halo_unpack", c_i32, c_vp, c_vp, c_vp, c_i64, c_i32, c_vp)
 _sig("pcgcn_last_error", ctypes.c_char_p)
 _sig("pcgcn_abi_version", c_i32)
 
@@ -175,6 +181,32 @@ class Plan:
         if nbytes:
             check(lib.pcgcn_plan_export(self._h, w, out.ctypes.data, nbytes), "pcgcn_plan_export")
         return out
+
+    def shard_rows(self, world):
+        out = np.zeros(world + 1, dtype=np.int64)
+        check(lib.pcgcn_plan_shard_rows(self._h, out.ctypes.data), "pcgcn_plan_shard_rows")
+        return out
+
+    def halo(self, q, send):
+        """Plan rows of the halo list for peer q (send: rows of this shard q reads;
+        else rows of shard q this shard reads)."""
+        k = lib.pcgcn_plan_halo_rows(self._h, int(q), int(bool(send)))
+        if k < 0:
+            raise ValueError(f"bad peer {q}")
+        out = np.empty(k, dtype=np.int32)
+        if k:
+            check(lib.pcgcn_plan_halo_export(self._h, int(q), int(bool(send)), out.ctypes.data, k),
+                  "pcgcn_plan_halo_export")
+        return out
+
+    def halo_pack(self, Y, buf, w=None, stream=None):
+        w = Y.shape[1] if w is None else w
+        check(lib.pcgcn_halo_pack(self._h, _ptr(Y), Y.stride(0), w, _ptr(buf), _stream(stream)), "pcgcn_halo_pack")
+
+    def halo_unpack(self, buf, Y, w=None, stream=None):
+        w = Y.shape[1] if w is None else w
+        check(lib.pcgcn_halo_unpack(self._h, _ptr(buf), _ptr(Y), Y.stride(0), w, _stream(stream)),
+              "pcgcn_halo_unpack")
 
     def rowscale_ptr(self):
         return lib.pcgcn_plan_rowscale(self._h)

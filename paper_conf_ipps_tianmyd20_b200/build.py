@@ -18,7 +18,7 @@ OUT = os.path.join(HERE, "libpcgcn.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 CU_SOURCES = ["pcgcn_api.cu", "sparse.cu", "tc_engine.cu", "dense_simt.cu", "gemm.cu", "loss_opt.cu",
-              "calibrate.cu", "probe.cu", "tc_pair.cu"]
+              "calibrate.cu", "probe.cu", "tc_pair.cu", "halo.cu"]
 CXX_SOURCES = ["planner.cpp"]
 
 

@@ -101,6 +101,10 @@ cudaError_t launch_gemm_dwt(const float* D, int64_t ldd, const float* W, const u
                             const float* s, float* O, int64_t ldo, int64_t M, int N, int K,
                             float* work, cudaStream_t st);
 
+// ---- halo exchange of a sharded plan (halo.cu) ----
+cudaError_t launch_halo_copy(bool pack, const float* src, int64_t lds, float* dst, int64_t ldd, const int32_t* idx,
+                             int64_t rows, int w, cudaStream_t s);
+
 // ---- loss / optimiser (loss_opt.cu) ----
 cudaError_t launch_softmax_ce(const float* L, int64_t ld, const int32_t* labels,
                               const uint8_t* train, int64_t M, int C, float inv_nT, const float* s,

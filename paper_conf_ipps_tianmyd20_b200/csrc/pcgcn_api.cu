@@ -143,6 +143,15 @@ pcgcn_status upload_plan(pcgcn_plan_s* p) {
   }
   UP(&d.ypre, (float*)nullptr, n * d.fpad_max);
   UP(&d.zrow, (float*)nullptr, 256);
+  if (p->opts.world > 1) {
+    std::vector<int32_t> sl, rl;
+    for (auto& l : p->halo_send) sl.insert(sl.end(), l.begin(), l.end());
+    for (auto& l : p->halo_recv) rl.insert(rl.end(), l.begin(), l.end());
+    d.halo_nsend = int64_t(sl.size());
+    d.halo_nrecv = int64_t(rl.size());
+    UP(&d.halo_send, sl.data(), d.halo_nsend);
+    UP(&d.halo_recv, rl.data(), d.halo_nrecv);
+  }
   UP(&d.counter, (int*)nullptr, 32);
   {
     // long selective rows -> segments of SEG_EDGES edges (reading #22)
@@ -450,6 +459,49 @@ pcgcn_status pcgcn_backward(pcgcn_plan_t p, const float* dZ, int64_t ldz, float*
                             int32_t F, uint32_t flags, void* stream) {
   // Âᵀ = Â for a symmetric input: the forward plan serves the backward.
   return aggregate(p, dZ, ldz, dY, ldy, F, flags & ~uint32_t(PCGCN_MASK_OUT), nullptr, stream);
+}
+
+int64_t pcgcn_plan_halo_rows(pcgcn_plan_t p, int32_t q, int32_t send) {
+  if (!p || q < 0 || q >= p->opts.world) return -1;
+  if (p->opts.world == 1) return 0;
+  return int64_t((send ? p->halo_send : p->halo_recv)[q].size());
+}
+
+pcgcn_status pcgcn_plan_halo_export(pcgcn_plan_t p, int32_t q, int32_t send, int32_t* buf, int64_t cap) {
+  const int64_t n = pcgcn_plan_halo_rows(p, q, send);
+  if (n < 0 || (n > 0 && (!buf || cap < n))) { set_error("plan_halo_export: bad peer / buffer"); return PCGCN_EINVAL; }
+  if (n > 0) std::memcpy(buf, (send ? p->halo_send : p->halo_recv)[q].data(), sizeof(int32_t) * size_t(n));
+  return PCGCN_OK;
+}
+
+pcgcn_status pcgcn_plan_shard_rows(pcgcn_plan_t p, int64_t* row0) {
+  if (!p || !row0) { set_error("null argument"); return PCGCN_EINVAL; }
+  if (p->shard_row0.empty()) { row0[0] = 0; row0[1] = p->n; return PCGCN_OK; }
+  std::memcpy(row0, p->shard_row0.data(), sizeof(int64_t) * p->shard_row0.size());
+  return PCGCN_OK;
+}
+
+static pcgcn_status halo_copy(pcgcn_plan_t p, bool pack, const float* src, int64_t lds, float* dst, int64_t ldd,
+                              int32_t w, void* stream) {
+  if (!p || !p->d.built) { set_error("plan has no device structures"); return PCGCN_EINVAL; }
+  const int64_t rows = pack ? p->d.halo_nsend : p->d.halo_nrecv;
+  if (rows == 0) return PCGCN_OK;
+  if (!src || !dst || w < 4 || (w & 3) || lds < w || ldd < w || (lds & 3) || (ldd & 3) ||
+      (reinterpret_cast<uintptr_t>(src) & 15) || (reinterpret_cast<uintptr_t>(dst) & 15)) {
+    set_error("halo pack/unpack: bad buffers (w multiple of 4, ld >= w, 16-byte aligned rows)");
+    return PCGCN_EINVAL;
+  }
+  cudaError_t e = launch_halo_copy(pack, src, lds, dst, ldd, pack ? p->d.halo_send : p->d.halo_recv, rows, w,
+                                   static_cast<cudaStream_t>(stream));
+  return e == cudaSuccess ? PCGCN_OK : cuda_fail(e, pack ? "halo_pack" : "halo_unpack");
+}
+
+pcgcn_status pcgcn_halo_pack(pcgcn_plan_t p, const float* Y, int64_t ldy, int32_t w, float* buf, void* stream) {
+  return halo_copy(p, true, Y, ldy, buf, w, w, stream);
+}
+
+pcgcn_status pcgcn_halo_unpack(pcgcn_plan_t p, const float* buf, float* Y, int64_t ldy, int32_t w, void* stream) {
+  return halo_copy(p, false, buf, w, Y, ldy, w, stream);
 }
 
 pcgcn_status pcgcn_plan_perm(pcgcn_plan_t p, int32_t* perm) {

@@ -34,6 +34,9 @@ struct DevicePlan {
   int64_t* seg_hi = nullptr;
   float* seg_ws = nullptr;        // [nseg x fpad_max] segment partial sums
   int* counter = nullptr;         // [32] selective-pass row ticket
+  int32_t* halo_send = nullptr;   // [Σ_q send rows] plan rows of this shard, peers in rank order
+  int32_t* halo_recv = nullptr;   // [Σ_q recv rows] plan rows of other shards, peers in rank order
+  int64_t halo_nsend = 0, halo_nrecv = 0;
   int64_t rows = 0, nnz_s = 0, nrt = 0, nch = 0, nseg = 0;
   int64_t n_pad = 0;
   int fpad_max = 0;
@@ -72,6 +75,10 @@ struct pcgcn_plan_s {
   // shard
   int32_t k_lo = 0, k_hi = 0;
   int64_t row_lo = 0, row_hi = 0, rt_lo = 0, rt_hi = 0;
+  std::vector<int64_t> shard_row0;                 // [world+1] first plan row of every shard
+  std::vector<std::vector<int32_t>> halo_recv;     // [world] rows of shard q this shard reads
+  std::vector<std::vector<int32_t>> halo_send;     // [world] rows of this shard that shard q reads
+  int64_t stats_src_rows_pc = 0, stats_shard_src_rows_pc = 0;
   pcgcn_stats stats{};
   pcgcn::DevicePlan d;
 };

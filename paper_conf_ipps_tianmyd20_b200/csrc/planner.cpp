@@ -448,6 +448,63 @@ pcgcn_status build_host_plan(const pcgcn_csr* A, int32_t P, float theta, const p
     p->row_hi = p->pstart[p->k_hi];
     p->rt_lo = part_rt[p->k_lo];
     p->rt_hi = part_rt[p->k_hi];
+    p->shard_row0.assign(o->world + 1, 0);
+    for (int32_t q = 0; q <= o->world; ++q) p->shard_row0[q] = p->pstart[bound(q)];
+    // halo lists (L99: a shard reads the source rows its
+    // blocks touch): rows of shard q that shard r reads — the sources of r's
+    // selective edges and every row of the 32-source windows of r's chunks —
+    // for r = this rank (recv, one list per q) and q = this rank (send, one
+    // list per r).  Lists are ascending; a shard's own rows are never listed.
+    const int32_t W = o->world;
+    if (W > 1) {
+      std::vector<std::vector<uint64_t>> need(W, std::vector<uint64_t>((n + 63) / 64, 0));
+      parallel_for(W, [&](int, int64_t a, int64_t b) {
+        for (int64_t r = a; r < b; ++r) {
+          auto& bm = need[r];
+          const int32_t ka = bound(int32_t(r)), kb = bound(int32_t(r) + 1);
+          for (int64_t v = p->pstart[ka]; v < p->pstart[kb]; ++v)
+            for (int64_t e = p->sp_rowptr[v]; e < p->sp_rowptr[v + 1]; ++e) {
+              const int64_t j = p->sp_col[e];
+              bm[j >> 6] |= 1ull << (j & 63);
+            }
+          for (int64_t t = part_rt[ka]; t < part_rt[kb]; ++t)
+            for (int64_t c = p->rt_cptr[t]; c < p->rt_cptr[t + 1]; ++c) {
+              const int64_t c0 = p->ch_col0[c];
+              for (int64_t j = c0; j < std::min<int64_t>(c0 + TILE_K, n); ++j) bm[j >> 6] |= 1ull << (j & 63);
+            }
+        }
+      });
+      auto rows_in = [&](const std::vector<uint64_t>& bm, int64_t lo, int64_t hi, std::vector<int32_t>& out) {
+        for (int64_t j = lo; j < hi; ++j)
+          if ((bm[j >> 6] >> (j & 63)) & 1ull) out.push_back(int32_t(j));
+      };
+      p->halo_recv.assign(W, {});
+      p->halo_send.assign(W, {});
+      for (int32_t q = 0; q < W; ++q) {
+        if (q == o->rank) continue;
+        rows_in(need[o->rank], p->shard_row0[q], p->shard_row0[q + 1], p->halo_recv[q]);
+        rows_in(need[q], p->row_lo, p->row_hi, p->halo_send[q]);
+      }
+    }
+  }
+
+  // partition-centric source rows (SURVEY.md §8(d) B_pc): Σ_k |distinct sources
+  // of V_k's selective edges| — the rows a destination partition must fetch if
+  // each of its blocks' source slices were read once (L129 §III-A.b)
+  {
+    std::vector<int64_t> upc(P, 0);
+    parallel_for(P, [&](int, int64_t a, int64_t b) {
+      std::vector<int32_t> buf;
+      for (int64_t k = a; k < b; ++k) {
+        buf.assign(p->sp_col.begin() + p->sp_rowptr[p->pstart[k]], p->sp_col.begin() + p->sp_rowptr[p->pstart[k + 1]]);
+        std::sort(buf.begin(), buf.end());
+        upc[k] = std::unique(buf.begin(), buf.end()) - buf.begin();
+      }
+    });
+    for (int32_t k = 0; k < P; ++k) {
+      p->stats_src_rows_pc += upc[k];
+      if (k >= p->k_lo && k < p->k_hi) p->stats_shard_src_rows_pc += upc[k];
+    }
   }
 
   // stats
@@ -462,6 +519,10 @@ pcgcn_status build_host_plan(const pcgcn_csr* A, int32_t P, float theta, const p
   S.shard_nnz_sparse = p->sp_rowptr[p->row_hi] - p->sp_rowptr[p->row_lo];
   S.shard_chunks = p->rt_cptr[p->rt_hi] - p->rt_cptr[p->rt_lo];
   S.theta = theta;
+  S.src_rows_pc = p->stats_src_rows_pc;
+  S.shard_src_rows_pc = p->stats_shard_src_rows_pc;
+  for (auto& l : p->halo_recv) S.halo_recv_rows += int64_t(l.size());
+  for (auto& l : p->halo_send) S.halo_send_rows += int64_t(l.size());
   S.partition_ms = part_ms;
   S.plan_ms = ms_since(t0);
   return PCGCN_OK;

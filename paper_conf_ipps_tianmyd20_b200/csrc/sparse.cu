@@ -79,20 +79,33 @@ __device__ __forceinline__ void ld_vec(const char* p, float4 (&o)[H]) {
 // vectors l, l+G, ..., l+(V-1)G.  A slot's G lanes read one contiguous piece
 // of the row per load, so each load instruction touches the fewest 128-byte
 // lines (the L1TEX wavefront count is what bounds a gather of L2-resident rows).
+// G need not be a power of two: the S = floor(32/G) slots then leave
+// 32 - S·G lanes idle (they issue no loads), an index batch holds S·STEPS
+// <= 32 edges, and the slots are combined by a fixed sequence of shuffles
+// instead of the butterfly.  (F = 41 rows of 48 floats as six 32-byte
+// vectors: G = 6, five rows per load instruction, 30 of 32 lanes busy — vs
+// 11 of 16 lanes with 16-byte vectors.)
 template <int G, int V, int H>
 struct Lay {
+  static constexpr bool POW2 = (G & (G - 1)) == 0;
   static constexpr int S = 32 / G;       // edges per warp step
-  static constexpr int STEPS = 32 / S;   // steps per 32-index batch
-  // steps whose loads are all issued before any is consumed (<= 8 float4
-  // per lane in flight: more costs occupancy than it gains in MLP on C3)
-  static constexpr int UCAP = 8 / (V * H);
-  static constexpr int UNR = (UCAP >= 8 && STEPS >= 8) ? 8
-                           : (UCAP >= 4 && STEPS >= 4) ? 4
-                           : (UCAP >= 2 && STEPS >= 2) ? 2 : 1;
+  static constexpr int STEPS = 32 / S;   // steps per index batch
+  static constexpr int BATCH = S * STEPS;  // edges per coalesced index load (<= 32)
+  // steps whose loads are all issued before any is consumed: <= 8 float4 per
+  // lane in flight for the power-of-two layouts (more costs occupancy than it
+  // gains in MLP on C3); the partial-warp layouts hold up to 12 (they run at
+  // 3 CTAs per SM, see sparse_row_kernel's launch bounds)
+  static constexpr int UCAP = (POW2 ? 8 : 12) / (V * H);
+  static constexpr int UNR = (UCAP >= 8 && STEPS % 8 == 0) ? 8
+                           : (UCAP >= 6 && STEPS % 6 == 0) ? 6
+                           : (UCAP >= 4 && STEPS % 4 == 0) ? 4
+                           : (UCAP >= 3 && STEPS % 3 == 0) ? 3
+                           : (UCAP >= 2 && STEPS % 2 == 0) ? 2 : 1;
   static constexpr int NACC = (V * H == 1 && UNR >= 2) ? 2 : 1;  // interleaved partial sums
+  static constexpr int MINB = POW2 ? 4 : 3;  // resident 256-thread CTAs per SM
 };
 
-// tot[v][h] (valid in every lane after the butterfly) = sum over the n edges
+// tot[v][h] (valid in lanes < G; in every lane for power-of-two G) = sum over the n edges
 // at cp[0..n) of Y'[cp[e]][cols of this lane].  yb = this lane's byte offset
 // into row 0 of Y' (lanes past the row re-read column 0: same line, ignored;
 // vectors v >= 1 past the row are not loaded: lok[v] false).
@@ -108,8 +121,9 @@ __device__ __forceinline__ int gather_sum(const int* __restrict__ cp, int n, int
                                           uint32_t rstride, const bool (&lok)[V], int lane,
                                           float4 (&tot)[V][H]) {
   using L = Lay<G, V, H>;
-  constexpr int S = L::S, STEPS = L::STEPS, UNR = L::UNR, NACC = L::NACC;
+  constexpr int S = L::S, STEPS = L::STEPS, UNR = L::UNR, NACC = L::NACC, BATCH = L::BATCH;
   const int slot = lane / G;
+  const bool active = L::POW2 || slot < S;  // idle lanes of a partial-warp layout load nothing
   float4 acc[NACC][V][H];
 #pragma unroll
   for (int u = 0; u < NACC; ++u)
@@ -119,13 +133,13 @@ __device__ __forceinline__ int gather_sum(const int* __restrict__ cp, int n, int
       for (int h = 0; h < H; ++h) acc[u][v][h] = make_float4(0.f, 0.f, 0.f, 0.f);
   int nextidx = first;
   if (n == 0) nextidx = lane < nn ? ld_idx(cpn + lane) : 0;
-  for (int base = 0; base < n; base += 32) {
-    const int cnt = (n - base) < 32 ? n - base : 32;
+  for (int base = 0; base < n; base += BATCH) {
+    const int cnt = (n - base) < BATCH ? n - base : BATCH;
     const int myidx = nextidx;
     // next batch, one ahead (past the end: the next range's first batch)
-    nextidx = (base + 32 + lane < n) ? ld_idx(cp + base + 32 + lane)
+    nextidx = (base + BATCH + lane < n) ? ld_idx(cp + base + BATCH + lane)
             : (lane < nn ? ld_idx(cpn + lane) : 0);
-    if (cnt == 32) {
+    if (cnt == BATCH) {
       // full batch: unguarded, every lane keeps UNR*V*H 16-byte pieces in flight
 #pragma unroll
       for (int k0 = 0; k0 < STEPS; k0 += UNR) {
@@ -136,7 +150,7 @@ __device__ __forceinline__ int gather_sum(const int* __restrict__ cp, int n, int
           const char* p = row_addr(yb, j, rstride);
 #pragma unroll
           for (int v = 0; v < V; ++v) {
-            if (v == 0 || lok[v]) {
+            if (active && (v == 0 || lok[v])) {
               ld_vec<H>(p + 16 * H * G * v, buf[u][v]);
             } else {
 #pragma unroll
@@ -163,7 +177,7 @@ __device__ __forceinline__ int gather_sum(const int* __restrict__ cp, int n, int
           const char* p = row_addr(yb, j, rstride);
 #pragma unroll
           for (int v = 0; v < V; ++v) {
-            if (e < cnt && (v == 0 || lok[v])) {
+            if (active && e < cnt && (v == 0 || lok[v])) {
               ld_vec<H>(p + 16 * H * G * v, buf[u][v]);
             } else {
 #pragma unroll
@@ -189,12 +203,25 @@ __device__ __forceinline__ int gather_sum(const int* __restrict__ cp, int n, int
       t = acc[0][v][h];
 #pragma unroll
       for (int u = 1; u < NACC; ++u) add4(t, acc[u][v][h]);
+      if constexpr (L::POW2) {
 #pragma unroll
-      for (int off = G; off < 32; off <<= 1) {  // fixed butterfly over the slots
-        t.x += __shfl_xor_sync(0xffffffffu, t.x, off);
-        t.y += __shfl_xor_sync(0xffffffffu, t.y, off);
-        t.z += __shfl_xor_sync(0xffffffffu, t.z, off);
-        t.w += __shfl_xor_sync(0xffffffffu, t.w, off);
+        for (int off = G; off < 32; off <<= 1) {  // fixed butterfly over the slots
+          t.x += __shfl_xor_sync(0xffffffffu, t.x, off);
+          t.y += __shfl_xor_sync(0xffffffffu, t.y, off);
+          t.z += __shfl_xor_sync(0xffffffffu, t.z, off);
+          t.w += __shfl_xor_sync(0xffffffffu, t.w, off);
+        }
+      } else {
+        // slots 1..S-1 added to slot 0 in slot order (valid in lanes < G only)
+        const float4 mine = t;
+#pragma unroll
+        for (int k = 1; k < S; ++k) {
+          const int src = lane + k * G;
+          t.x += __shfl_sync(0xffffffffu, mine.x, src);
+          t.y += __shfl_sync(0xffffffffu, mine.y, src);
+          t.z += __shfl_sync(0xffffffffu, mine.z, src);
+          t.w += __shfl_sync(0xffffffffu, mine.w, src);
+        }
       }
     }
   return nextidx;
@@ -212,7 +239,7 @@ __device__ __forceinline__ int lane_col(int lane, int v, int nvec) {
 // 4-warp CTAs (8K registers): small enough to co-reside with a full-mode
 // engine CTA (tc_engine, 320 threads) when the two run concurrently
 template <int G, int V, int H>
-__global__ void __launch_bounds__(128, 8) sparse_seg_kernel(AggArgs a) {
+__global__ void __launch_bounds__(128, 2 * Lay<G, V, H>::MINB) sparse_seg_kernel(AggArgs a) {
   const int64_t sg = int64_t(blockIdx.x) * 4 + (threadIdx.x >> 5);
   if (sg >= a.nseg) return;
   const int lane = threadIdx.x & 31;
@@ -246,7 +273,7 @@ __global__ void __launch_bounds__(128, 8) sparse_seg_kernel(AggArgs a) {
 // segment partials in segment order.  Fused epilogue: + full-mode partial
 // sum Zd (mode combine, L193), x r_i (optionally twice), ReLU, bit mask.
 template <int G, int V, int H, bool HAS_ZD, bool HAS_SEG>
-__global__ void __launch_bounds__(256, 4) sparse_row_kernel(AggArgs a) {
+__global__ void __launch_bounds__(256, Lay<G, V, H>::MINB) sparse_row_kernel(AggArgs a) {
   const int lane = threadIdx.x & 31;
   const int slot = lane / G;
   const int nvec = (a.F + 4 * H - 1) / (4 * H);
@@ -572,9 +599,11 @@ cudaError_t launch_sparse_pass(const AggArgs& a, cudaStream_t s);
 struct SparseKnobs {
   int fsplit = 0;
   bool v8 = true;
+  bool g6 = true;  // PCGCN_SPARSE_G6=0: F = 41..48 keeps the 16-byte G = 16 layout (A/B)
   SparseKnobs() {
     if (const char* e = getenv("PCGCN_SPARSE_FSPLIT")) fsplit = atoi(e) / 32 * 32;
     if (const char* e = getenv("PCGCN_SPARSE_V8")) v8 = atoi(e) != 0;
+    if (const char* e = getenv("PCGCN_SPARSE_G6")) g6 = atoi(e) != 0;
   }
 };
 
@@ -611,8 +640,12 @@ cudaError_t launch_sparse_pass(const AggArgs& a, cudaStream_t s) {
   // floats per row, measured 6% slower on C3's L2-bound F = 41 pass); else 16.
   // Measured (B200, PCGCN_SPARSE_V8=0 vs 1): C5's issue-bound row pass F = 32
   // 21.2 -> 19.2 ms, F = 128 45.4 -> 43.3 ms; C3 F = 128 unchanged.
-  const bool v8 = knobs().v8 && a.ldy % 8 == 0 && (reinterpret_cast<uintptr_t>(a.Y) & 31) == 0 &&
-                  (a.F + 7) / 8 * 2 == (a.F + 3) / 4;
+  const bool al32 = knobs().v8 && a.ldy % 8 == 0 && (reinterpret_cast<uintptr_t>(a.Y) & 31) == 0;
+  const bool v8 = al32 && (a.F + 7) / 8 * 2 == (a.F + 3) / 4;
+  // 41..48 features in 32-byte aligned rows (C3's class width, ld 48): six
+  // 32-byte vectors per row read the row's 192 bytes (6 sectors, as many as the
+  // 44 floats of the 16-byte layout touch) with 5 rows per load instruction
+  if (al32 && knobs().g6 && (a.F + 7) / 8 == 6) return launch_gv<6, 1, 2>(a, s);
   if (v8) {
     const int nvec = (a.F + 7) / 8;
     if (nvec <= 1) return launch_gv<1, 1, 2>(a, s);

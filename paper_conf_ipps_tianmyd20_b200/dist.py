@@ -2,12 +2,20 @@
 
 Destination partitions are sharded over ranks in contiguous plan-row ranges
 (the planner's cost-balanced split).  Each aggregation needs the prescaled
-source rows of every partition its blocks touch; Reddit-shaped graphs touch
-all remote rows, so the exchange is an all-gather of the producer's output
-rows into the full-height input buffer (one broadcast per owner into its row
-range — ranges are uneven).  ∇Θ (one flat buffer) and the loss are summed
-with one all-reduce each.  torch.distributed (NCCL on GPUs, gloo in the CPU
-tests) is the transport; the arithmetic stays in libpcgcn.
+source rows of the partitions its blocks touch (§III-A.b):
+
+* HaloExchange — the planner's halo lists (pcgcn_plan_halo_*): libpcgcn packs
+  the rows each peer reads into one send buffer, one all-to-all with per-peer
+  split sizes (NCCL grouped send/recv over NVLink) moves only those rows, and
+  libpcgcn scatters the received rows into the full-height input.  When a
+  plan's halo exceeds half of the remote rows on some rank (Reddit-shaped
+  graphs touch ~100% of them) the exchange falls back to
+* RowExchange — an all-gather of every owner's range (one broadcast per
+  owner, ranges are uneven).
+
+∇Θ (one flat buffer) and the loss are summed with one all-reduce each.
+torch.distributed (NCCL on GPUs, gloo in the tests) is the transport; the
+arithmetic and the row packing stay in libpcgcn.
 """
 from __future__ import annotations
 
@@ -43,13 +51,79 @@ class RowExchange:
         # broadcast() takes GLOBAL ranks; map the group-local owner index
         self.src = [q if group is None else dist.get_global_rank(group, q) for q in range(self.world)]
 
-    def gather(self, full: torch.Tensor, lo: int = None, hi: int = None):
+    def gather(self, full: torch.Tensor, lo: int = None, hi: int = None, plan=None):
         """full[lo_q:hi_q] of every rank q becomes visible on every rank."""
         if full.shape[0] != self.ranges[-1][1]:
             raise ValueError(f"full buffer has {full.shape[0]} rows, ranges cover {self.ranges[-1][1]}")
         for q, (a, b) in enumerate(self.ranges):
             if b > a:
                 dist.broadcast(full[a:b], src=self.src[q], group=self.group)
+
+    def allreduce(self, t: torch.Tensor):
+        dist.all_reduce(t, op=dist.ReduceOp.SUM, group=self.group)
+
+
+class HaloExchange:
+    """Halo-only exchange (see the module doc).  ``plans``: the plans whose
+    aggregations consume exchanged buffers (per-width plans have their own
+    lists); ``gather(full, lo, hi, plan)`` refreshes the rows of ``full`` that
+    ``plan``'s local rows read.  Falls back to the all-gather per plan when
+    its halo exceeds ``threshold`` of the remote rows on any rank."""
+
+    def __init__(self, plans, group=None, threshold: float = 0.5):
+        self.group = group
+        self.world = dist.get_world_size(group)
+        self.rank = dist.get_rank(group)
+        self.backend = dist.get_backend(group)
+        p0 = plans[0]
+        self.ranges = [(int(a), int(b)) for a, b in zip(p0.shard_rows(self.world)[:-1], p0.shard_rows(self.world)[1:])]
+        check_ranges(self.ranges, p0.n)
+        assert self.ranges[self.rank] == (p0.row_lo, p0.row_hi)
+        self.rowx = RowExchange(p0.row_lo, p0.row_hi, group=group, n=p0.n)
+        self.info = {}
+        for pl in plans:
+            recv = [len(pl.halo(q, False)) if q != self.rank else 0 for q in range(self.world)]
+            send = [len(pl.halo(q, True)) if q != self.rank else 0 for q in range(self.world)]
+            remote = pl.n - (pl.row_hi - pl.row_lo)
+            frac = torch.tensor([sum(recv) / max(remote, 1)], dtype=torch.float64)
+            dist.all_reduce(frac, op=dist.ReduceOp.MAX, group=group)
+            mode = "allgather" if float(frac) > threshold else "halo"
+            self.info[id(pl)] = dict(plan=pl, recv=recv, send=send, mode=mode, frac=float(frac))
+        self._bufs = {}
+        self.bytes_moved = 0   # rows x stride x 4 received by this rank, summed over gather calls
+
+    def mode(self, plan):
+        return self.info[id(plan)]["mode"]
+
+    def _buf(self, key, rows, w, like):
+        b = self._bufs.get(key)
+        if b is None or b.shape[0] < rows or b.shape[1] != w:
+            b = torch.empty(max(rows, 1), w, dtype=like.dtype, device=like.device)
+            self._bufs[key] = b
+        return b[:rows]
+
+    def gather(self, full: torch.Tensor, lo: int = None, hi: int = None, plan=None):
+        inf = self.info[id(plan)] if plan is not None else None
+        if inf is None or inf["mode"] == "allgather":
+            self.rowx.gather(full)
+            self.bytes_moved += (full.shape[0] - (self.ranges[self.rank][1] - self.ranges[self.rank][0])) \
+                * full.shape[1] * 4
+            return
+        pl, w = inf["plan"], full.shape[1]
+        assert full.is_contiguous() and full.shape[0] == pl.n
+        send = self._buf(("s", id(pl), w), sum(inf["send"]), w, full)
+        recv = self._buf(("r", id(pl), w), sum(inf["recv"]), w, full)
+        pl.halo_pack(full, send, w)
+        if self.backend == "gloo" and full.is_cuda:   # gloo moves host tensors only (tests)
+            r_h = torch.empty(recv.shape, dtype=recv.dtype)
+            dist.all_to_all_single(r_h, send.cpu(), output_split_sizes=inf["recv"], input_split_sizes=inf["send"],
+                                   group=self.group)
+            recv.copy_(r_h)
+        else:
+            dist.all_to_all_single(recv, send, output_split_sizes=inf["recv"], input_split_sizes=inf["send"],
+                                   group=self.group)
+        pl.halo_unpack(recv, full, w)
+        self.bytes_moved += recv.shape[0] * w * 4
 
     def allreduce(self, t: torch.Tensor):
         dist.all_reduce(t, op=dist.ReduceOp.SUM, group=self.group)

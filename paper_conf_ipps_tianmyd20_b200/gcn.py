@@ -22,6 +22,8 @@ diag(r)·Y (r = d̃^-½) and the aggregation applies r_i once in its epilogue:
 """
 from __future__ import annotations
 
+import ctypes
+
 import numpy as np
 import torch
 
@@ -38,12 +40,18 @@ def _ld(F: int) -> int:
 class GCN2:
     def __init__(self, plan: L.Plan, X_plan: np.ndarray, labels_plan: np.ndarray, train_plan: np.ndarray,
                  Th0: np.ndarray, Th1: np.ndarray, *, optimizer: str = "adam", lr: float = 0.01,
-                 device: str | torch.device = "cuda", exchange=None, plan_c: L.Plan | None = None):
+                 device: str | torch.device = "cuda", exchange=None, plan_c: L.Plan | None = None,
+                 narrow: bool = False):
         """All row-indexed host arrays are already in plan order (X_plan = X[perm]).
-        ``exchange`` (sharded runs): object with ``gather(local, full)`` and
-        ``allreduce(t)``; rows owned here are plan.row_lo:plan.row_hi.
+        ``exchange`` (sharded runs): object with ``gather(full, lo, hi, plan=)``
+        and ``allreduce(t)``; rows owned here are plan.row_lo:plan.row_hi.
         ``plan_c`` (optional): plan of the same graph and partition with its own
-        θ, used for the width-C aggregations (per-width mode choice)."""
+        θ, used for the width-C aggregations (per-width mode choice).
+        ``narrow`` (sharded runs, SURVEY.md §8(e) "narrowest-width exchange"):
+        every rank keeps X for all n rows and computes Y0' for all of them (no
+        width-H exchange before layer 1); the backward exchanges G1 (width C)
+        and the ReLU bit mask instead of dP1' (width H), and recomputes
+        dP1' = diag(r)((G1Θ1ᵀ)⊙mask1) for all rows."""
         self.plan = plan
         self.plan_c = plan_c if plan_c is not None else plan
         assert (self.plan_c.row_lo, self.plan_c.row_hi) == (plan.row_lo, plan.row_hi)
@@ -57,14 +65,17 @@ class GCN2:
         self.optimizer = optimizer
         self.lr = lr
         self.exchange = exchange
+        self.narrow = bool(narrow and exchange is not None)
         assert max(self.H, self.C) <= plan.f_max
         d, f32 = self.dev, torch.float32
         n, rows, H, C = self.n, self.rows, self.H, self.C
         self.ldH, self.ldC = _ld(H), _ld(C)
         # X rows padded to a multiple of 4 floats (16-byte rows: TMA-loadable)
         self.ldX = _ld(self.f_in)
-        self.X = torch.zeros(self.rows, self.ldX, dtype=f32, device=d)
-        self.X[:, :self.f_in] = torch.from_numpy(np.ascontiguousarray(X_plan[self.lo:self.hi], dtype=np.float32)).to(d)
+        xr = slice(0, n) if self.narrow else slice(self.lo, self.hi)
+        self.X_all = torch.zeros(xr.stop - xr.start, self.ldX, dtype=f32, device=d)
+        self.X_all[:, :self.f_in] = torch.from_numpy(np.ascontiguousarray(X_plan[xr], dtype=np.float32)).to(d)
+        self.X = self.X_all[self.lo:self.hi] if self.narrow else self.X_all
         self.labels = torch.from_numpy(np.ascontiguousarray(labels_plan[self.lo:self.hi], dtype=np.int32)).to(d)
         self.train = torch.from_numpy(np.ascontiguousarray(train_plan[self.lo:self.hi], dtype=np.uint8)).to(d)
         self.inv_nT = 1.0 / float(np.count_nonzero(train_plan))
@@ -81,11 +92,15 @@ class GCN2:
         # activations: inputs of aggregations span all n rows (sources), outputs the shard
         self.Y0 = torch.zeros(n, self.ldH, dtype=f32, device=d)
         self.H1 = torch.zeros(rows, self.ldH, dtype=f32, device=d)
-        self.mask1 = torch.zeros(rows, (H + 31) // 32, dtype=torch.int32, device=d)
+        mw = (H + 31) // 32
+        # narrow: full-height mask / G1 (exchanged), the local rows are views
+        self.mask1_all = torch.zeros(n if self.narrow else rows, mw, dtype=torch.int32, device=d)
+        self.mask1 = self.mask1_all[self.lo:self.hi] if self.narrow else self.mask1_all
         self.Y1 = torch.zeros(n, self.ldC, dtype=f32, device=d)
         self.Lg = torch.zeros(rows, self.ldC, dtype=f32, device=d)
         self.dL = torch.zeros(n, self.ldC, dtype=f32, device=d)
-        self.G1 = torch.zeros(rows, self.ldC, dtype=f32, device=d)
+        self.G1_all = torch.zeros(n if self.narrow else rows, self.ldC, dtype=f32, device=d)
+        self.G1 = self.G1_all[self.lo:self.hi] if self.narrow else self.G1_all
         self.dP1 = torch.zeros(n, self.ldH, dtype=f32, device=d)
         self.G0 = torch.zeros(rows, self.ldH, dtype=f32, device=d)
         self.loss = torch.zeros(1, dtype=f32, device=d)
@@ -94,6 +109,9 @@ class GCN2:
         self.xtg_work = torch.zeros(max(wk, 1), dtype=f32, device=d)
         wk = max(L.gemm_xw_work_floats(self.f_in, H), L.gemm_xw_work_floats(H, C), L.gemm_dwt_work_floats(H, C))
         self.xw_work = torch.zeros(wk, dtype=f32, device=d)
+        if self.narrow:
+            wk = max(wk, L.gemm_xw_work_floats(self.f_in, H))
+            self.xw_work = torch.zeros(wk, dtype=f32, device=d)
         self.r = plan.rowscale_ptr()  # device [n]
         self.r_local = None if self.lo == 0 else self.r + 4 * self.lo
         self._graph = None
@@ -106,9 +124,9 @@ class GCN2:
     def _local(self, full):
         return full[self.lo:self.hi]
 
-    def _gather(self, full):
+    def _gather(self, full, plan):
         if self.exchange is not None:
-            self.exchange.gather(full, self.lo, self.hi)
+            self.exchange.gather(full, self.lo, self.hi, plan=plan)
 
     def epoch(self, stream=None, hook=None, agg_flags=0):
         """One epoch; ``hook(name)`` (optional) is called after every step so a
@@ -117,10 +135,15 @@ class GCN2:
         rr = self._r_rows()
         H, C, p = self.H, self.C, self.plan
         # layer 1
-        L.gemm_xw(self.X, self.Th0, rr, self._local(self.Y0), M=self.rows, K=self.f_in, N=H, work=self.xw_work,
-                  stream=stream)
+        if self.narrow:   # Y0' for all n rows from the replicated X: no width-H exchange
+            L.gemm_xw(self.X_all, self.Th0, ctypes.c_void_p(self.r), self.Y0, M=self.n, K=self.f_in, N=H,
+                      work=self.xw_work, stream=stream)
+        else:
+            L.gemm_xw(self.X, self.Th0, rr, self._local(self.Y0), M=self.rows, K=self.f_in, N=H, work=self.xw_work,
+                      stream=stream)
         mark("a4_gemm_xw0")
-        self._gather(self.Y0)
+        if not self.narrow:
+            self._gather(self.Y0, p)
         mark("x_gather_y0")
         p.forward(self.Y0, self.H1, F=H, flags=L.IN_PRESCALED | L.RELU | L.MASK_OUT | agg_flags, mask=self.mask1,
                   stream=stream)
@@ -129,7 +152,7 @@ class GCN2:
         L.gemm_xw(self.H1, self.Th1, rr, self._local(self.Y1), M=self.rows, K=H, N=C, work=self.xw_work,
                   stream=stream)
         mark("a7_gemm_xw1")
-        self._gather(self.Y1)
+        self._gather(self.Y1, self.plan_c)
         mark("x_gather_y1")
         self.plan_c.forward(self.Y1, self.Lg, F=C, flags=L.IN_PRESCALED | agg_flags, stream=stream)
         mark("a8_agg_fwd_C")
@@ -137,16 +160,23 @@ class GCN2:
         L.softmax_ce(self.Lg, self.labels, self.train, self.inv_nT, rr, self._local(self.dL), self.loss,
                      self.ce_work, M=self.rows, C=C, stream=stream)
         mark("a9_softmax_ce")
-        self._gather(self.dL)
+        self._gather(self.dL, self.plan_c)
         mark("x_gather_dl")
         # backward
         self.plan_c.backward(self.dL, self.G1, F=C, flags=L.IN_PRESCALED | agg_flags, stream=stream)
         mark("a10_agg_bwd_C")
         L.gemm_xtg(self.H1, self.G1, self.gTh1, self.xtg_work, M=self.rows, K=H, N=C, stream=stream)
-        L.gemm_dwt(self.G1, self.Th1, self.mask1, rr, self._local(self.dP1), M=self.rows, N=C, K=H,
-                   work=self.xw_work, stream=stream)
+        if self.narrow:   # exchange G1 (width C) and the mask, recompute dP1' for all rows
+            self.exchange.gather(self.G1_all, self.lo, self.hi, plan=None)
+            self.exchange.gather(self.mask1_all.view(torch.float32), self.lo, self.hi, plan=None)
+            L.gemm_dwt(self.G1_all, self.Th1, self.mask1_all, ctypes.c_void_p(self.r), self.dP1, M=self.n, N=C, K=H,
+                       work=self.xw_work, stream=stream)
+        else:
+            L.gemm_dwt(self.G1, self.Th1, self.mask1, rr, self._local(self.dP1), M=self.rows, N=C, K=H,
+                       work=self.xw_work, stream=stream)
         mark("a11_gemm_xtg1_dwt")
-        self._gather(self.dP1)
+        if not self.narrow:
+            self._gather(self.dP1, p)
         mark("x_gather_dp1")
         p.backward(self.dP1, self.G0, F=H, flags=L.IN_PRESCALED | agg_flags, stream=stream)
         mark("a12_agg_bwd_H")
@@ -179,6 +209,10 @@ class GCN2:
         n += xtg(self.C) + xtg(self.H)                       # a11, a13
         n += 2 + (1 if self.ldH > np16(self.H) else 0)       # a11 dwt: W split + engine (+ pad zeroing)
         n += 2 if self.optimizer == "adam" else 1            # a14
+        ex = self.exchange
+        if ex is not None and hasattr(ex, "mode"):            # halo pack + unpack per halo-mode gather
+            gathered = [self.plan_c, self.plan_c] + ([] if self.narrow else [self.plan, self.plan])
+            n += sum(2 for pl in gathered if ex.mode(pl) == "halo")
         return n
 
     # -- CUDA graph ------------------------------------------------------

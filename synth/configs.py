@@ -77,6 +77,13 @@ PL32M = Workload(
                      alpha=2.2, cap=16_000.0, seed=5001),
     f_in=128, hidden=128, classes=32, P=16384, feat_kind="normal", feat_seed=5002, theta_seed=5003)
 
+# C5's recipe at test size (sharded-path tests): 256 communities of 128 vertices,
+# 90% of draws inside the community, Pareto(2.2) propensities, 250K edges.
+PL_SMALL = Workload(
+    "pl-small", SBMSpec([128] * 256, sub_size=0, p_sub=0.0, p_class=0.9, m_target=250_000,
+                        alpha=2.2, cap=1_000.0, seed=5101),
+    f_in=128, hidden=128, classes=32, P=64, feat_kind="normal", feat_seed=5102, theta_seed=5103)
+
 # RMAT-{0.1,0.5,1,5,10}: the paper's synthetic density series (L251, Table I
 # L223-L227: 10,240 vertices, density = m / n^2, 128 features, 32 labels),
 # regenerated for the Table III (L263-L281) sel / full / hybrid replica.  The
@@ -86,7 +93,7 @@ RMAT = {d: Workload(f"rmat-{d:g}", RMATSpec(10_240, int(round(d / 100 * 10_240 *
                     theta_seed=6201 + i)
         for i, d in enumerate((0.1, 0.5, 1.0, 5.0, 10.0))}
 
-WORKLOADS = {w.name: w for w in (CORA, PUBMED, REDDIT, SBM4M, PL32M, *RMAT.values())}
+WORKLOADS = {w.name: w for w in (CORA, PUBMED, REDDIT, SBM4M, PL32M, PL_SMALL, *RMAT.values())}
 
 
 def labels(w: Workload, g: Graph) -> np.ndarray:

@@ -145,3 +145,172 @@ def test_sharded_epoch_matches_unsharded():
         # relative gate as the single-GPU gradient parity (test_gpu_parity)
         assert np.max(np.abs(grad - gr)) <= 1e-4 * np.max(np.abs(gr))
     assert np.array_equal(res[0][7], res[1][7])       # replicas agree after the update
+
+
+# ---------------------------------------------------------------------------
+# halo lists and the halo exchange
+# ---------------------------------------------------------------------------
+
+def _halo_brute(pl_r, n, ranges, r):
+    """Rows of other shards that shard r reads: selective sources of its rows
+    and every row of its chunks' 32-source windows (from the exported plan)."""
+    lo, hi = ranges[r]
+    rp, col = pl_r.export("sp_rowptr"), pl_r.export("sp_col")
+    need = set(col[rp[lo]:rp[hi]].tolist())
+    r0, nr, cp, c0 = pl_r.export("rt_row0"), pl_r.export("rt_nrows"), pl_r.export("rt_cptr"), pl_r.export("ch_col0")
+    for t in range(len(r0)):
+        if lo <= r0[t] < hi:
+            for c in range(cp[t], cp[t + 1]):
+                need.update(range(c0[c], min(c0[c] + 32, n)))
+    return {q: sorted(j for j in need if ranges[q][0] <= j < ranges[q][1]) for q in range(len(ranges)) if q != r}
+
+
+@pytest.mark.parametrize("world,theta", [(2, 0.05), (3, 0.0), (4, 2.0)])
+def test_halo_lists_match_brute_force(world, theta):
+    from paper_conf_ipps_tianmyd20_b200 import _lib as L
+    from synth import configs as C
+    w = C.PUBMED
+    g = C.graph(w)
+    pls = [L.Plan(g.n, g.rowptr, g.col, w.P, theta, build_device=False, rank=r, world=world) for r in range(world)]
+    row0 = pls[0].shard_rows(world)
+    ranges = list(zip(row0[:-1].tolist(), row0[1:].tolist()))
+    for r, pl in enumerate(pls):
+        assert (pl.row_lo, pl.row_hi) == ranges[r]
+        assert np.array_equal(pl.shard_rows(world), row0)
+        exp = _halo_brute(pl, g.n, ranges, r)
+        for q in range(world):
+            if q == r:
+                assert len(pl.halo(q, False)) == 0 and len(pl.halo(q, True)) == 0
+                continue
+            assert pl.halo(q, False).tolist() == exp[q], (r, q)
+            # what r sends to q is exactly what q receives from r
+            assert np.array_equal(pl.halo(q, True), pls[q].halo(r, False))
+        st = pl.stats()
+        assert st["halo_recv_rows"] == sum(len(v) for v in exp.values())
+
+
+def _halo_worker(rank, world, port, q):
+    """HaloExchange over gloo with host-only plans: the plan's pack/unpack
+    (device kernels in the product) are replaced by their definition on host
+    tensors, so this checks the split sizes, peer order and transport."""
+    import sys
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    from paper_conf_ipps_tianmyd20_b200 import _lib as L
+    from paper_conf_ipps_tianmyd20_b200.dist import HaloExchange
+    from synth import configs as C
+    _init(rank, world, port)
+    w = C.PUBMED
+    g = C.graph(w)
+    pl = L.Plan(g.n, g.rowptr, g.col, w.P, 0.05, build_device=False, rank=rank, world=world)
+    send_rows = np.concatenate([pl.halo(p, True) for p in range(world)]).astype(np.int64)
+    recv_rows = np.concatenate([pl.halo(p, False) for p in range(world)]).astype(np.int64)
+    pl.halo_pack = lambda Y, buf, w_: buf.copy_(Y[torch.from_numpy(send_rows)])
+    pl.halo_unpack = lambda buf, Y, w_: Y.index_copy_(0, torch.from_numpy(recv_rows), buf)
+    ex = HaloExchange([pl], threshold=1.1)
+    full = torch.full((g.n, 4), -1.0)
+    full[pl.row_lo:pl.row_hi] = torch.arange(pl.row_lo, pl.row_hi, dtype=torch.float32)[:, None]
+    ex.gather(full, pl.row_lo, pl.row_hi, plan=pl)
+    q.put((rank, ex.mode(pl), recv_rows, full.numpy().copy(), pl.row_lo, pl.row_hi))
+    dist.destroy_process_group()
+
+
+def test_halo_exchange_gloo_world2():
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    ps = [ctx.Process(target=_halo_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in ps:
+        p.start()
+    out = [q.get(timeout=180) for _ in ps]
+    for p in ps:
+        p.join(timeout=60)
+    for rank, mode, recv_rows, full, lo, hi in out:
+        assert mode == "halo"
+        got = full[:, 0]
+        assert np.array_equal(got[lo:hi], np.arange(lo, hi))               # own rows untouched
+        assert np.array_equal(got[recv_rows], recv_rows.astype(np.float32))  # halo rows arrived
+        rest = np.setdiff1d(np.setdiff1d(np.arange(len(got)), np.arange(lo, hi)), recv_rows)
+        assert np.all(got[rest] == -1.0)                                   # nothing else moved
+
+
+def _halo_epoch_worker(rank, world, port, q, wname, theta, narrow, threshold):
+    import sys
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    from paper_conf_ipps_tianmyd20_b200 import _lib as L
+    from paper_conf_ipps_tianmyd20_b200.dist import HaloExchange
+    from paper_conf_ipps_tianmyd20_b200.gcn import GCN2
+    from synth import configs as C
+    _init(rank, world, port)
+    torch.cuda.set_device(0)
+    w = C.WORKLOADS[wname]
+    g = C.graph(w)
+    X = C.features(w, g.n)
+    Th0, Th1 = C.thetas(w)
+    T = C.train_mask(g.n, w.theta_seed)
+    y = C.labels(w, g)
+    pl = L.Plan(g.n, g.rowptr, g.col, w.P, theta, rank=rank, world=world)
+    pl_c = L.Plan(g.n, g.rowptr, g.col, w.P, theta * 2 if theta < 1 else theta, rank=rank, world=world)
+    perm = pl.perm()
+    ex = HaloExchange([pl, pl_c], threshold=threshold)
+    model = GCN2(pl, X[perm], y[perm], T[perm], Th0, Th1, optimizer="sgd", lr=0.1, exchange=ex, plan_c=pl_c,
+                 narrow=narrow)
+    model.epoch()
+    torch.cuda.synchronize()
+    q.put((rank, pl.row_lo, pl.row_hi, model.H1.cpu().numpy(), model.Lg.cpu().numpy(), model.G0.cpu().numpy(),
+           model.loss.item(), model.grad.cpu().numpy(), model.theta.cpu().numpy(), ex.mode(pl), ex.mode(pl_c),
+           ex.bytes_moved))
+    dist.destroy_process_group()
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("wname,theta,narrow,threshold", [("pl-small", 0.05, False, 1.1),
+                                                          ("pubmed", 0.02, False, 1.1),
+                                                          ("pubmed", 0.02, True, 0.5),
+                                                          ("pl-small", 0.05, True, 1.1)])
+def test_sharded_halo_epoch_matches_unsharded(wname, theta, narrow, threshold):
+    """Halo exchange (only the rows each shard reads move) and the narrow
+    variant (Y0' recomputed from replicated X, G1 + mask exchanged instead of
+    dP1'): output rows bitwise equal to the unsharded epoch, gradients within
+    the all-reduce reassociation tolerance; on the clustered power-law graph
+    (C5's recipe at test size, synth.configs.PL_SMALL) the halo moves a fraction of the remote rows."""
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    from paper_conf_ipps_tianmyd20_b200 import _lib as L
+    from paper_conf_ipps_tianmyd20_b200.gcn import GCN2
+    from synth import configs as C
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    ps = [ctx.Process(target=_halo_epoch_worker, args=(r, 2, port, q, wname, theta, narrow, threshold))
+          for r in range(2)]
+    for p in ps:
+        p.start()
+    res = sorted([q.get(timeout=900) for _ in ps], key=lambda t: t[0])
+    for p in ps:
+        p.join(timeout=60)
+    w = C.WORKLOADS[wname]
+    g = C.graph(w)
+    X = C.features(w, g.n)
+    Th0, Th1 = C.thetas(w)
+    T = C.train_mask(g.n, w.theta_seed)
+    y = C.labels(w, g)
+    pl = L.Plan(g.n, g.rowptr, g.col, w.P, theta)
+    pl_c = L.Plan(g.n, g.rowptr, g.col, w.P, theta * 2 if theta < 1 else theta)
+    perm = pl.perm()
+    ref = GCN2(pl, X[perm], y[perm], T[perm], Th0, Th1, optimizer="sgd", lr=0.1, plan_c=pl_c)
+    ref.epoch()
+    torch.cuda.synchronize()
+    H1, Lg, G0 = ref.H1.cpu().numpy(), ref.Lg.cpu().numpy(), ref.G0.cpu().numpy()
+    gr = ref.grad.cpu().numpy()
+    for rank, lo, hi, h1, lg, g0, loss, grad, theta_new, m_h, m_c, moved in res:
+        if threshold > 1:
+            assert m_h == "halo" and m_c == "halo"
+        assert np.array_equal(h1, H1[lo:hi])
+        assert np.array_equal(lg, Lg[lo:hi])
+        assert np.array_equal(g0, G0[lo:hi])
+        assert abs(loss - ref.loss.item()) <= 1e-6 * abs(ref.loss.item())
+        assert np.max(np.abs(grad - gr)) <= 1e-5 * np.max(np.abs(gr))
+        if wname.startswith("pl") and not narrow:
+            full_ag = 4 * (g.n - (hi - lo)) * (ref.ldH * 2 + ref.ldC * 2)
+            assert moved < 0.5 * full_ag, (moved, full_ag)
+    assert np.array_equal(res[0][8], res[1][8])

@@ -488,6 +488,42 @@ def test_long_rows_segments(F, ldpad):
     assert torch.equal(Z2[:, :F], Zd[:, :F])
 
 
+@pytest.mark.parametrize("F,ld", [(41, 48), (42, 48), (47, 48), (48, 48), (41, 56), (48, 64)])
+@pytest.mark.parametrize("gname", ["hubs", "cora", "cliques"])
+def test_partial_warp_layout(gname, F, ld):
+    """41..48 features in 32-byte aligned rows take the G = 6 lane layout (five
+    rows per load instruction, two idle lanes, slots combined by a fixed
+    shuffle sequence): values, ReLU, mask (incl. its zero tail) vs the oracle,
+    long-row segments included, and run-to-run bitwise."""
+    g = {"hubs": _hubs, "cora": lambda: G.sbm(C.CORA.spec),
+         "cliques": lambda: G.cliques([130, 70, 200, 5, 1], seed=2)}[gname]()
+    pl = L.Plan(g.n, g.rowptr, g.col, 4, 0.05 if gname != "hubs" else 2.0, f_max=128)
+    perm = pl.perm()
+    Y = _feat(g.n, F, 23)
+    Yp = np.zeros((g.n, ld), np.float32)
+    Yp[:, :F] = Y[perm]
+    Yd = torch.from_numpy(Yp).cuda()
+    assert Yd.data_ptr() % 32 == 0
+    Zd = torch.full((g.n, ld), float("nan"), device="cuda")
+    mw = (F + 31) // 32
+    mask = torch.full((g.n, mw), -1, dtype=torch.int32, device="cuda")
+    pl.forward(Yd, Zd, F=F, flags=L.RELU | L.MASK_OUT, mask=mask)
+    torch.cuda.synchronize()
+    Ahat = O.normalized_adjacency(g.n, g.rowptr, g.col)[0]
+    Zs = O.aggregate(Ahat, Y.astype(np.float64))[perm]
+    scale = np.maximum(O.aggregate(abs(Ahat), np.abs(Y.astype(np.float64)))[perm], 1e-30)
+    Zc = Zd.cpu().numpy()[:, :F].astype(np.float64)
+    assert np.max(np.abs(Zc - np.maximum(Zs, 0)) / scale) <= TOL
+    m = mask.cpu().numpy().view(np.uint32)
+    bits = ((m[:, :, None] >> np.arange(32, dtype=np.uint32)) & 1).reshape(g.n, 32 * mw)
+    assert np.all((bits[:, :F].astype(bool) == (Zs > 0)) | (np.abs(Zs) < 1e-6 * scale))
+    assert np.all(bits[:, F:] == 0)
+    Z2 = torch.full_like(Zd, float("nan"))
+    pl.forward(Yd, Z2, F=F, flags=L.RELU | L.MASK_OUT, mask=mask)
+    torch.cuda.synchronize()
+    assert torch.equal(Z2[:, :F], Zd[:, :F])
+
+
 @pytest.mark.parametrize("wname,theta,nl", [("cora", 0.05, 4), ("pubmed", 0.0, 4), ("cora", 2.0, 3),
                                             ("pubmed", 0.02, 2)])
 def test_epoch_parity_deep(wname, theta, nl):
@@ -534,7 +570,7 @@ e = np.random.default_rng(7).integers(0, base, size=(3 * base, 2))
 edges += [tuple(x) for x in e.tolist() if x[0] != x[1]]
 g = G.from_edges(base, edges)
 rng = np.random.default_rng(11)
-for F, theta, ld in ((128, 0.02, 128), (41, 0.04, 44), (40, 0.04, 48), (32, 2.0, 32)):
+for F, theta, ld in ((128, 0.02, 128), (41, 0.04, 44), (40, 0.04, 48), (32, 2.0, 32), (41, 0.03, 48)):
     pl = L.Plan(g.n, g.rowptr, g.col, 8, theta)
     Y = torch.from_numpy(rng.standard_normal((g.n, ld)).astype(np.float32)).cuda()
     Y[:, F:] = 0
@@ -542,8 +578,8 @@ for F, theta, ld in ((128, 0.02, 128), (41, 0.04, 44), (40, 0.04, 48), (32, 2.0,
     M = torch.zeros(g.n, (F + 31) // 32, dtype=torch.int32, device="cuda")
     pl.forward(Y, Z, F=F, flags=L.RELU | L.MASK_OUT, mask=M)
     torch.cuda.synchronize()
-    out[f"agg{F}"] = Z.cpu().numpy()
-    out[f"mask{F}"] = M.cpu().numpy()
+    out[f"agg{F}_{ld}"] = Z.cpu().numpy()
+    out[f"mask{F}_{ld}"] = M.cpu().numpy()
 # one epoch (the xtg / dwt GEMMs included)
 w = C.PUBMED
 gp = C.graph(w)
@@ -568,7 +604,8 @@ np.savez(sys.argv[1], **out)
                                           ({"PCGCN_XTG_PRESPLIT": "1"}, True),
                                           ({"PCGCN_DENSE_BLOCKED": "0"}, True),
                                           ({"PCGCN_SPARSE_V8": "0"}, False),
-                                          ({"PCGCN_SPARSE_FSPLIT": "32"}, False)])
+                                          ({"PCGCN_SPARSE_FSPLIT": "32"}, False),
+                                          ({"PCGCN_SPARSE_G6": "0"}, False)])
 def test_scheduling_knobs_do_not_change_results(tmp_path, knob, bitwise):
     """Row-block tickets, the full-mode/segment overlap, the in-kernel xtg B
     conversion and the window-blocked full-mode B layout change only scheduling (every output row is still reduced by
@@ -594,9 +631,9 @@ def test_scheduling_knobs_do_not_change_results(tmp_path, knob, bitwise):
         elif k.startswith("mask"):
             # 16- vs 32-byte lane vectors sum a row's edges in another (fixed)
             # order: each run's mask must be exactly its own [Z > 0]
-            F = int(k[4:])
+            F, ld = (int(x) for x in k[4:].split("_"))
             for tag in ("default", "knob"):
-                Z = res[tag][f"agg{F}"][:, :F]
+                Z = res[tag][f"agg{F}_{ld}"][:, :F]
                 want = np.zeros_like(res[tag][k])
                 for c in range(F):
                     want[:, c // 32] |= ((Z[:, c] > 0).astype(np.int64) << (c % 32)).astype(np.uint32).view(np.int32)
