@@ -43,10 +43,12 @@ def parse():
     ap.add_argument("--workload", default="reddit")
     ap.add_argument("--theta", default="auto")
     ap.add_argument("--P", type=int, default=0)
-    ap.add_argument("--order", default="id", choices=["id", "degree"],
+    ap.add_argument("--order", default="degree", choices=["id", "degree"],
                     help="vertex order inside a partition (pcgcn_opts.vertex_order)")
-    ap.add_argument("--grain", default="block", choices=["block", "tile"],
+    ap.add_argument("--grain", default="tile", choices=["block", "tile"],
                     help="unit of the selective/full decision (pcgcn_opts.mode_grain)")
+    ap.add_argument("--dense", default="tf32x2", choices=["tf32x2", "bf16x3"],
+                    help="full-mode arithmetic (pcgcn_opts.dense_prec)")
     ap.add_argument("--oracle-frac", type=float, default=0.02)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
@@ -130,6 +132,14 @@ def load_workload(name):
     return w, g, X, Th0, Th1, C.labels(w, g), T
 
 
+def workload_str(w, g):
+    """config.workload of both arms (the generator emits no duplicates or
+    self-loops, so nnz(A+I) = nnz(A) + n)."""
+    idx = {'cora': 0, 'pubmed': 1, 'reddit': 2, 'sbm4m': 3, 'pl32m': 4}.get(w.name)
+    return (f"{w.name}-shaped DC-SBM (BASELINE configs[{idx}]) n={g.n} nnz(A+I)={g.nnz + g.n} "
+            f"F={w.f_in}->{w.hidden}->{w.classes}")
+
+
 HUGE_NNZ = 500_000_000  # C5-sized graphs: single calibrated plan, row-wise oracle sample, serial e2e
 
 
@@ -153,6 +163,19 @@ def agg_bytes(st, n, rows, F, dense_rows, nchunks):
     nnz_s = st["shard_nnz_sparse"]
     b = nnz_s * 4 + (rows + 1) * 8 + rows * 4 + n * F * 4 + rows * F * 4
     b += 2 * dense_rows * F * 4 + nchunks * (512 + 4)
+    return int(b)
+
+
+def agg_bpc(st, rows, F, dense_rows, nchunks, bf3=False):
+    """Partition-centric bytes model of one aggregation (SURVEY.md §8(d) B_pc;
+    PAPER.md L129 §III-A.b): structure (indices, row pointers, r) + every
+    destination partition's distinct selective source rows read once
+    (stats shard_src_rows_pc) + the output + the full mode's bit tiles and
+    B windows (one per chunk) + the Zd round trip of rows with chunks."""
+    npad = (F + 15) // 16 * 16
+    b = st["shard_nnz_sparse"] * 4 + (rows + 1) * 8 + rows * 4
+    b += 4 * F * (st["shard_src_rows_pc"] + rows)
+    b += nchunks * (516 + (6 if bf3 else 8) * 32 * npad) + 2 * dense_rows * F * 4
     return int(b)
 
 
@@ -242,14 +265,17 @@ def run_reference(args, rank, world):
     v = float(np.mean(ts))
     blas, cores = osamp.cores()
     sample = (f"{len(osamp.rows)} seeded random output rows ({osamp.frac:.2%} of n) of every epoch op "
-              f"(4 aggregations scipy fp64 single-threaded, GEMMs numpy BLAS {blas} threads), x1/frac")
+              f"(4 aggregations scipy fp64 single-threaded, GEMMs numpy BLAS {blas} threads), x1/frac: each "
+              f"step times the sample and reports the epoch it extrapolates to (the full, unextrapolated "
+              f"oracle epoch is profiles/r2_oracle_epoch.json)")
     line = {
-        "impl": "reference", "metric": "2-layer GCN epoch ms (oracle, extrapolated from a row sample)",
+        "impl": "reference", "metric": "2-layer GCN epoch ms",
         "value": v, "unit": "ms", "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
         "ms_per_step": v, "higher_is_better": False, "scaling": "strong", "vs_baseline": None,
         "dtype": "f64", "data": "synthetic",
-        "config": {"workload": f"{w.name}-shaped DC-SBM n={g.n} nnz(A+I)={g.nnz + g.n} F={w.f_in}->{w.hidden}->{w.classes}",
-                   "parallelism": "cpu"},
+        "config": {"workload": workload_str(w, g),
+                   "parallelism": "cpu", "extrapolated": True,
+                   "sample_seconds_per_step": float(np.mean(ts)) * osamp.frac / 1e3},
         "cpu_baseline": {"value": v, "unit": "ms", "cores": blas, "host_cores": cores, "kind": "oracle",
                          "sample": sample},
         "e2e": {"value": v, "unit": "ms", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
@@ -424,7 +450,8 @@ def run_f2(args):
 def plan_kw(args):
     from paper_conf_ipps_tianmyd20_b200 import _lib as L
     return dict(order=L.ORDER_DEGREE if args.order == "degree" else L.ORDER_ID,
-                grain=L.GRAIN_TILE if args.grain == "tile" else L.GRAIN_BLOCK)
+                grain=L.GRAIN_TILE if args.grain == "tile" else L.GRAIN_BLOCK,
+                dense_prec=L.DENSE_BF16X3 if args.dense == "bf16x3" else L.DENSE_TF32X2)
 
 
 def main():
@@ -639,12 +666,14 @@ def main():
     gather = st["shard_nnz_sparse"] * fp4 * 4 / (t_sp * 1e-3) / 1e9
     t_tc = kern["a5a6_agg_fwd_H"]["dense_tc"]
     npad = (w.hidden + 15) // 16 * 16
-    tc_flops = st["shard_chunks"] * 2 * 128 * 32 * npad * 2  # 2 MMAs (hi, lo) per chunk
+    bf3 = args.dense == "bf16x3"
+    # executed MMA flops per chunk: 2 (hi, lo) tf32 products, or 3 bf16 parts
+    tc_flops = st["shard_chunks"] * 2 * 128 * 32 * npad * (3 if bf3 else 2)
     tc_tf = tc_flops / (t_tc * 1e-3) / 1e12 if t_tc > 0 else None
     try:
-        tc_peak = float(json.load(open(MEASURED_PEAKS))["bf16_tflops"]) / 2
+        tc_peak = float(json.load(open(MEASURED_PEAKS))["bf16_tflops"]) / (1 if bf3 else 2)
     except Exception:
-        tc_peak = 1590.0 / 2
+        tc_peak = 1590.0 / (1 if bf3 else 2)
     traffic = l2_read = lts_pct = None
     tpath = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tpath):
@@ -797,8 +826,7 @@ def main():
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": False,
             "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
             "config": {
-                "workload": f"{w.name}-shaped DC-SBM (BASELINE configs[{ {'cora': 0, 'pubmed': 1, 'reddit': 2, 'sbm4m': 3, 'pl32m': 4}.get(w.name)}]) n={g.n} nnz(A+I)={st['nnz']} "
-                            f"F={w.f_in}->{w.hidden}->{w.classes}",
+                "workload": workload_str(w, g),
                 "P": P, "theta": theta, "theta_c": theta_c if theta_c else theta, "theta_source": theta_src, "optimizer": "adam",
                 "parallelism": f"dp-rows{world}" if world > 1 else "single",
                 "l2": "flushed (256 MiB write) between timed steps",
@@ -835,10 +863,19 @@ def main():
                                          "source": "pcgcn_probe_gather_gbs: the kernel's access pattern (random "
                                                    "rows of row_bytes, 8 in flight per lane, 32 warps/SM) from "
                                                    "64 KB / 64 MB / 4 GB buffers, best of 3"}},
+            "bytes_views": {
+                "aggregation": f"layer-1 forward, F={w.hidden} (selective + full mode)",
+                "B_min": bH, "B_pc": agg_bpc(st, rows, w.hidden, dense_rows, st["shard_chunks"], args.dense == "bf16x3"),
+                "ncu_dram_selective": traffic,
+                "dram_over_B_min_selective": (traffic / b_sp) if traffic else None,
+                "src_rows_pc": st["shard_src_rows_pc"],
+                "note": "B_min = compulsory bytes; B_pc = each destination partition reads its distinct selective "
+                        "sources once; ncu DRAM bytes of the selective kernels per launch (cold cache)"},
             "tensor_view": {"kernel": "tc_engine<A_BITS> full-mode tiles, layer-1 forward",
-                            "ms": t_tc, "achieved": tc_tf, "unit": "TFLOP/s (tf32)", "peak": tc_peak,
-                            "frac": (tc_tf / tc_peak) if tc_tf else None,
-                            "peak_source": "measured bf16 dense (MEASURED_PEAKS.json) x 0.5 (tf32:bf16 nominal ratio)"},
+                            "ms": t_tc, "achieved": tc_tf, "unit": "TFLOP/s (bf16)" if bf3 else "TFLOP/s (tf32)",
+                            "peak": tc_peak, "frac": (tc_tf / tc_peak) if tc_tf else None,
+                            "peak_source": ("measured bf16 dense (MEASURED_PEAKS.json)" if bf3 else
+                                            "measured bf16 dense (MEASURED_PEAKS.json) x 0.5 (tf32:bf16 nominal ratio)")},
             "agg_kernels_ms": kern,
             "agg_GBs": {"fwd_H": bH / (per["a5a6_agg_fwd_H"] * 1e-3) / 1e9,
                         "fwd_C": bC / (per["a8_agg_fwd_C"] * 1e-3) / 1e9,

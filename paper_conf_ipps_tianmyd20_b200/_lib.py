@@ -25,7 +25,7 @@ c_i32, c_i64, c_f32, c_u32, c_vp = ctypes.c_int32, ctypes.c_int64, ctypes.c_floa
 # status codes
 OK, EINVAL, ENOTSYM, ECUDA, ENOMEM, ENCCL, EUNSUP = range(7)
 NORM_SYM, NORM_NONE = 0, 1
-DENSE_TF32X2, DENSE_FP32_SIMT, DENSE_BF16X1 = 0, 1, 2
+DENSE_TF32X2, DENSE_FP32_SIMT, DENSE_BF16X1, DENSE_BF16X3 = 0, 1, 2, 3
 ORDER_ID, ORDER_DEGREE = 0, 1
 GRAIN_BLOCK, GRAIN_TILE = 0, 1
 IN_PRESCALED, RELU, MASK_OUT, OUT_PRESCALED, PROFILE = 1, 2, 4, 8, 16

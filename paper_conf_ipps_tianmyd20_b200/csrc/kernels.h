@@ -69,8 +69,10 @@ struct DenseArgs {
   const float* blk = nullptr;  // source-window blocks (launch_split_windows); nullptr: hiT/loT maps
   int64_t blk_floats = 0;      // floats per window block
   int64_t n_src = 0;           // real source rows (vertices); rows [n_src, n) of the input are never read
+  int bf3 = 0;                 // PCGCN_DENSE_BF16X3: window blocks hold 3 bf16 parts (kind::f16 MMAs)
 };
-cudaError_t launch_split_windows(const float* Y, int64_t ldy, int64_t n, int F, int npad, bool single, float* blk,
+// mode 0: tf32 hi/lo, 1: bf16 single (BF16X1), 2: three bf16 parts (BF16X3)
+cudaError_t launch_split_windows(const float* Y, int64_t ldy, int64_t n, int F, int npad, int mode, float* blk,
                                  int64_t nwin, cudaStream_t s);
 cudaError_t launch_dense_tc(const DenseArgs& a, cudaStream_t s);
 // CTA-pair (cta_group::2) variant of the full mode (tc_pair.cu); map_b covers [hi rows; lo rows]

@@ -264,7 +264,8 @@ pcgcn_status aggregate(pcgcn_plan_t p, const float* Y, int64_t ldy, float* Z, in
   const float* src = Y;
   int64_t ldsrc = ldy;
   const bool bf16 = p->opts.dense_prec == PCGCN_DENSE_BF16X1;
-  const bool tc = p->opts.dense_prec == PCGCN_DENSE_TF32X2 || bf16;
+  const bool bf3 = p->opts.dense_prec == PCGCN_DENSE_BF16X3;
+  const bool tc = p->opts.dense_prec == PCGCN_DENSE_TF32X2 || bf16 || bf3;
   const bool prof = (flags & PCGCN_PROFILE) != 0;
   auto mark = [&](int k) {
     if (!prof) return;
@@ -315,10 +316,10 @@ pcgcn_status aggregate(pcgcn_plan_t p, const float* Y, int64_t ldy, float* Z, in
   // full mode's B: source-window blocks fetched by one bulk copy per chunk
   // (default), or the feature-major split read by strided TMA boxes (the
   // CTA-pair kernel, or PCGCN_DENSE_BLOCKED=0)
-  const bool blocked = tc && dense_blocked_enabled() && !dense_pair_eligible(npad);
+  const bool blocked = bf3 || (tc && dense_blocked_enabled() && !dense_pair_eligible(npad));
   if (dense && tc) {
     if (prof) d.ev_used[1] = true;
-    e = blocked ? launch_split_windows(src, ldsrc, p->n, F, npad, bf16, d.yhi, d.n_pad / 32, ms)
+    e = blocked ? launch_split_windows(src, ldsrc, p->n, F, npad, bf3 ? 2 : (bf16 ? 1 : 0), d.yhi, d.n_pad / 32, ms)
                 : launch_split_transpose(src, ldsrc, p->n, F, npad, d.yhi, bf16 ? nullptr : ylo, d.n_pad, ms);
     if (e != cudaSuccess) return cuda_fail(e, "split_transpose");
   }
@@ -331,7 +332,8 @@ pcgcn_status aggregate(pcgcn_plan_t p, const float* Y, int64_t ldy, float* Z, in
     da.n_src = p->n;
     if (blocked) {
       da.blk = d.yhi;
-      da.blk_floats = int64_t(bf16 ? 1 : 2) * npad * 32;
+      da.blk_floats = bf3 ? int64_t(npad) * 48 : int64_t(bf16 ? 1 : 2) * npad * 32;
+      da.bf3 = bf3 ? 1 : 0;
     }
     e = tc ? launch_dense_tc(da, ms) : launch_dense_simt_y(da, src, ldsrc, F, ms);
     if (e != cudaSuccess) return cuda_fail(e, "dense-mode kernel");
@@ -394,7 +396,7 @@ pcgcn_status pcgcn_plan(const pcgcn_csr* A, int32_t P, float theta, const pcgcn_
   if (!o) o = &def;
   if (o->f_max < 1 || o->f_max > 256) { set_error("f_max must be in [1, 256]"); return PCGCN_EINVAL; }
   if (o->dense_prec != PCGCN_DENSE_TF32X2 && o->dense_prec != PCGCN_DENSE_FP32_SIMT &&
-      o->dense_prec != PCGCN_DENSE_BF16X1) {
+      o->dense_prec != PCGCN_DENSE_BF16X1 && o->dense_prec != PCGCN_DENSE_BF16X3) {
     set_error("unknown dense_prec");
     return PCGCN_EUNSUP;
   }

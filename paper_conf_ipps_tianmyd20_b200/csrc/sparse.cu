@@ -545,8 +545,18 @@ __global__ void __launch_bounds__(256) split_transpose_kernel(const float* __res
 // the UMMA K-major SWIZZLE_128B image (16-byte chunk j of row r at j ^ (r & 7)),
 // so the engine fetches a chunk's whole B with one contiguous bulk copy
 // instead of an R-row strided TMA box.  Sources >= n and features >= F are 0.
+// mode 2 (BF16X3): y = b0 + b1 + b2 with b0 = bf16(y), b1 = bf16(y - b0),
+// b2 = bf16(y - b0 - b1) (round to nearest even; each residual is exact in
+// fp32, |y - b0 - b1 - b2| <= 2^-24 |y|), as three parts of npad rows x 32
+// bf16 = 64-byte rows in the K-major SWIZZLE_64B image (16-byte chunk j of
+// row r at j ^ ((r >> 1) & 3)).
+__device__ __forceinline__ uint32_t bf16_rn_bits(float v) {
+  const uint32_t u = __float_as_uint(v);
+  return (u + 0x7fffu + ((u >> 16) & 1u)) & 0xffff0000u;
+}
+
 __global__ void __launch_bounds__(256) split_window_kernel(const float* __restrict__ Y, int64_t ldy, int64_t n,
-                                                           int F, int npad, bool single,
+                                                           int F, int npad, int mode,
                                                            float* __restrict__ blk) {
   __shared__ float tile[32][33];
   const int64_t w = blockIdx.x;
@@ -558,9 +568,27 @@ __global__ void __launch_bounds__(256) split_window_kernel(const float* __restri
     tile[rr][tx] = (j < n && f < F) ? __ldg(Y + j * ldy + f) : 0.f;
   }
   __syncthreads();
+  const int k = tx;  // source within the window
+  if (mode == 2) {
+    uint16_t* out = reinterpret_cast<uint16_t*>(blk + w * int64_t(npad) * 48);  // 3 parts x npad x 64 B
+    for (int ff = ty; ff < 32; ff += 8) {
+      const int f = f0 + ff;
+      if (f >= npad) continue;
+      const float v = tile[k][ff];
+      const uint32_t h0 = bf16_rn_bits(v);
+      const float r1 = v - __uint_as_float(h0);
+      const uint32_t h1 = bf16_rn_bits(r1);
+      const uint32_t h2 = bf16_rn_bits(r1 - __uint_as_float(h1));
+      const int pos = f * 32 + ((((k >> 3) ^ ((f >> 1) & 3)) << 3) | (k & 7));  // bf16 element offset
+      out[pos] = uint16_t(h0 >> 16);
+      out[npad * 32 + pos] = uint16_t(h1 >> 16);
+      out[2 * npad * 32 + pos] = uint16_t(h2 >> 16);
+    }
+    return;
+  }
+  const bool single = mode == 1;
   const int R = single ? npad : 2 * npad;
   float* out = blk + w * int64_t(R) * 32;
-  const int k = tx;  // source within the window
   for (int ff = ty; ff < 32; ff += 8) {
     const int f = f0 + ff;
     if (f >= npad) continue;
@@ -571,20 +599,18 @@ __global__ void __launch_bounds__(256) split_window_kernel(const float* __restri
       out[rh * 32 + ((((k >> 2) ^ (rh & 7)) << 2) | (k & 3))] = h;
       out[rl * 32 + ((((k >> 2) ^ (rl & 7)) << 2) | (k & 3))] = v - h;
     } else {  // bf16 round-to-nearest-even (BF16X1 full mode); exact in tf32
-      uint32_t u = __float_as_uint(v);
-      u = (u + 0x7fffu + ((u >> 16) & 1u)) & 0xffff0000u;
-      out[f * 32 + ((((k >> 2) ^ (f & 7)) << 2) | (k & 3))] = __uint_as_float(u);
+      out[f * 32 + ((((k >> 2) ^ (f & 7)) << 2) | (k & 3))] = __uint_as_float(bf16_rn_bits(v));
     }
   }
 }
 
 }  // namespace
 
-cudaError_t launch_split_windows(const float* Y, int64_t ldy, int64_t n, int F, int npad, bool single, float* blk,
+cudaError_t launch_split_windows(const float* Y, int64_t ldy, int64_t n, int F, int npad, int mode, float* blk,
                                  int64_t nwin, cudaStream_t s) {
   if (nwin <= 0) return cudaSuccess;
   dim3 grid(unsigned(nwin), unsigned((npad + 31) / 32));
-  split_window_kernel<<<grid, 256, 0, s>>>(Y, ldy, n, F, npad, single, blk);
+  split_window_kernel<<<grid, 256, 0, s>>>(Y, ldy, n, F, npad, mode, blk);
   return cudaGetLastError();
 }
 

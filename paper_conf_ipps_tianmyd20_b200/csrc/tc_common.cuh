@@ -78,12 +78,44 @@ __device__ __forceinline__ void sttm32(uint32_t taddr, const uint32_t (&v)[32]) 
       : "memory");
 }
 
+// D[tmem] (+)= A[tmem] · B[smem desc], kind::f16 (bf16 operands, fp32 accumulation)
+__device__ __forceinline__ void mma_ts_f16(uint32_t d, uint32_t a, uint64_t bdesc, uint32_t idesc, uint32_t acc) {
+  asm volatile(
+      "{\n"
+      ".reg .pred p;\n"
+      "setp.ne.b32 p, %4, 0;\n"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, p;\n"
+      "}\n" ::"r"(d),
+      "r"(a), "l"(bdesc), "r"(idesc), "r"(acc)
+      : "memory");
+}
+__device__ __forceinline__ void sttm16(uint32_t taddr, const uint32_t (&v)[16]) {
+  asm volatile(
+      "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};" ::"r"(
+          taddr),
+      "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7]), "r"(v[8]), "r"(v[9]),
+      "r"(v[10]), "r"(v[11]), "r"(v[12]), "r"(v[13]), "r"(v[14]), "r"(v[15])
+      : "memory");
+}
+
 // UMMA shared-memory matrix descriptor (sm_100): start>>4 [0,14), LBO>>4
 // [16,30), SBO>>4 [32,46), version=1 [46,48), layout type [61,64) (2=SW128).
 // K-major SW128: 8-row groups 1024 B apart; K advance = +32 B per 8 tf32.
 __device__ __forceinline__ uint64_t sdesc_kmajor_sw128(uint32_t saddr) {
   return uint64_t((saddr >> 4) & 0x3FFFu) | (uint64_t(1) << 16) | (uint64_t(1024 >> 4) << 32) |
          (uint64_t(1) << 46) | (uint64_t(2) << 61);
+}
+// K-major SW64 (layout type 4): 64-byte rows (32 bf16), 8-row groups 512 B
+// apart; 16-byte chunk j of row r stored at j ^ ((r >> 1) & 3); K advance =
+// +32 B per 16 bf16.  Regions must be 512-byte aligned.
+__device__ __forceinline__ uint64_t sdesc_kmajor_sw64(uint32_t saddr) {
+  return uint64_t((saddr >> 4) & 0x3FFFu) | (uint64_t(1) << 16) | (uint64_t(512 >> 4) << 32) |
+         (uint64_t(1) << 46) | (uint64_t(4) << 61);
+}
+// instruction descriptor, kind::f16 with bf16 A and B (format 1), D f32,
+// both K-major, N>>3 [17,23), M>>4 [24,29)
+__host__ __device__ constexpr uint32_t idesc_bf16(int M, int N) {
+  return (1u << 4) | (1u << 7) | (1u << 10) | (uint32_t(N >> 3) << 17) | (uint32_t(M >> 4) << 24);
 }
 // instruction descriptor, kind::tf32: D f32 [4,6), A tf32 [7,10), B tf32
 // [10,13), A and B K-major (bits 15/16 = 0), N>>3 [17,23), M>>4 [24,29).

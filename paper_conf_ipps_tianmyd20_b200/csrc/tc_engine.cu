@@ -52,7 +52,8 @@ using namespace tc;
 // small): per-stage barrier round trips, the TMEM-store wait and the MMA
 // issue bookkeeping are paid once per U chunks.
 struct Layout {
-  int npad, stages, nacc, U, a_cols;  // a_cols: TMEM columns of one A stage (U*32, or 64 for hi+lo)
+  int npad, stages, nacc, U, a_cols;  // a_cols: TMEM columns of one A stage (U*32, U*16 bf16x3, or 64 for hi+lo)
+  uint32_t bchunk;                    // smem bytes of ONE chunk's B (all parts)
   uint32_t out_bytes;                 // A_ROWMAJOR: epilogue staging (4 warps x 32 rows x (64+4) floats)
   uint32_t raw_bytes;                 // A_TRANS + raw B: one row-major [32 x npad] D box per stage
   int gst;                            // stages per TMEM accumulation group (<= 8 chunks)
@@ -60,20 +61,22 @@ struct Layout {
   uint32_t tmem_cols, a_col0;
 };
 
-Layout make_layout(int mode, int npad, int max_stages, int max_u, bool b_raw = false) {
+Layout make_layout(int mode, int npad, int max_stages, int max_u, bool b_raw = false, bool bf3 = false) {
   Layout L;
   L.raw_bytes = (mode == A_TRANS && b_raw) ? uint32_t(npad) * BK * 4 : 0u;
   L.npad = npad;
   L.b_bytes = uint32_t(npad) * BK * 4;
+  // bf16x3 full mode: three K-major SW64 parts of npad rows x 64 B; else hi + lo tf32 (128 B rows)
+  L.bchunk = bf3 ? 3u * uint32_t(npad) * 64u : 2u * L.b_bytes;
   // transform GEMM outputs (N x npad rows, HBM-bound at scale) leave through a
   // shared-memory transpose so each store instruction writes whole row pieces
   L.out_bytes = (mode == A_ROWMAJOR && npad <= 128) ? 4u * 32u * (64u + 4u) * 4u : 0u;
   for (int U = (mode == A_BITS ? max_u : 1); U >= 1; U = U > 1 ? U / 2 : 0) {
     L.U = U;
-    L.a_cols = mode == A_BITS ? U * BK : 2 * BK;
+    L.a_cols = mode == A_BITS ? U * (bf3 ? BK / 2 : BK) : 2 * BK;
     L.a_bytes = mode == A_BITS ? uint32_t((U * BM * 4 + 1023) / 1024 * 1024) : BM * BK * 4;
     L.a_load_bytes = mode == A_BITS ? BM * 4 : BM * BK * 4;  // per chunk
-    L.stage_bytes = L.a_bytes + 2 * uint32_t(U) * L.b_bytes + L.raw_bytes;
+    L.stage_bytes = L.a_bytes + uint32_t(U) * L.bchunk + L.raw_bytes;
     int st = int((200 * 1024 - L.out_bytes) / L.stage_bytes);
     st = st > max_stages ? max_stages : st;
     L.nacc = 2;
@@ -123,6 +126,7 @@ struct Work {
   int64_t split_stride;
   int b_fused;       // B lo rows follow the hi rows in memory: one TMA box {32, 2*npad} per chunk
   int single;        // A_BITS: B hi only (bf16-rounded input), one MMA per K-step (PCGCN_DENSE_BF16X1)
+  int bf3;           // A_BITS: kind::f16, B = three bf16 parts (PCGCN_DENSE_BF16X3), window blocks only
   const int32_t* order;  // A_BITS: tile processed at position t (nullptr: t itself)
   const float* bblk;     // A_BITS: source-window blocks of B (pre-swizzled); nullptr: TMA boxes
   int64_t bblk_stride;   // floats per window block
@@ -208,7 +212,8 @@ __global__ void __launch_bounds__(NTHREADS, 1)
           mbar_wait(&empty[s], ph ^ 1u);
           uint8_t* st = smem + s * L.stage_bytes;
           mbar_expect_tx(&full[s], uint32_t(nu) * (L.a_load_bytes +
-                                                   (w.b_raw ? L.raw_bytes : (w.single ? 1u : 2u) * L.b_bytes)));
+                                                   (w.b_raw ? L.raw_bytes
+                                                            : w.bf3 ? L.bchunk : (w.single ? 1u : 2u) * L.b_bytes)));
           // the bits of a tile's chunks are contiguous: one bulk copy per stage
           if (MODE == A_BITS) bulk_load(st, w.bits + (kb + i) * BM, uint32_t(nu) * BM * 4, &full[s]);
           for (int u = 0; u < nu; ++u) {
@@ -223,11 +228,11 @@ __global__ void __launch_bounds__(NTHREADS, 1)
               tma_load_2d(&map_a, &full[s], st, int(m0), k0);
             }
             // chunk u's B tile in smem: [hi: npad rows][lo: npad rows] x 128 B
-            uint8_t* bdst = st + L.a_bytes + u * 2 * L.b_bytes;
+            uint8_t* bdst = st + L.a_bytes + u * L.bchunk;
             if (MODE == A_BITS && w.bblk) {
-              // the window's hi+lo (or hi) rows: one contiguous, pre-swizzled block
-              bulk_load(bdst, w.bblk + int64_t(k0 >> 5) * w.bblk_stride, (w.single ? 1u : 2u) * L.b_bytes,
-                        &full[s]);
+              // the window's hi+lo (or hi, or 3 bf16 parts) rows: one contiguous, pre-swizzled block
+              bulk_load(bdst, w.bblk + int64_t(k0 >> 5) * w.bblk_stride,
+                        w.bf3 ? L.bchunk : (w.single ? 1u : 2u) * L.b_bytes, &full[s]);
             } else if (MODE == A_TRANS && w.b_raw) {
               // row-major D rows [k0, k0+32) x features [0, npad) (OOB columns zero-filled)
               tma_load_2d(&map_bhi, &full[s], st + L.a_bytes + 2 * L.b_bytes, 0, k0);
@@ -245,7 +250,7 @@ __global__ void __launch_bounds__(NTHREADS, 1)
   } else if (warp == 1) {
     if (lane == 0) {
       // ---- MMA issuer ----
-      const uint32_t idesc = idesc_tf32(BM, npad);
+      const uint32_t idesc = (MODE == A_BITS && w.bf3) ? idesc_bf16(BM, npad) : idesc_tf32(BM, npad);
       int s = 0;
       uint32_t ph = 0, gc = 0;  // gc: accumulation-group counter (shared enumeration with the epilogue)
       for (int64_t t = blockIdx.x; t < w.ntiles; t += gridDim.x) {
@@ -270,7 +275,22 @@ __global__ void __launch_bounds__(NTHREADS, 1)
           const uint32_t sb = smem_u32(smem + s * L.stage_bytes + L.a_bytes);
           const uint32_t sa = tmem + L.a_col0 + uint32_t(s) * uint32_t(L.a_cols);
           for (int u = 0; u < nu; ++u) {
-            const uint32_t bh0 = sb + uint32_t(u) * 2u * L.b_bytes;
+            if (MODE == A_BITS && w.bf3) {
+              // A (0/1 as bf16, 16 TMEM columns) against the 3 bf16 parts of the
+              // window: 2 K=16 MMAs per part, fp32 accumulation in TMEM
+              const uint32_t b0 = sb + uint32_t(u) * L.bchunk;
+              const uint32_t a0 = sa + uint32_t(u) * (BK / 2);
+#pragma unroll
+              for (int part = 0; part < 3; ++part)
+#pragma unroll
+                for (int kk = 0; kk < 2; ++kk) {
+                  const uint64_t bd = sdesc_kmajor_sw64(b0 + uint32_t(part) * uint32_t(npad) * 64u + kk * 32u);
+                  mma_ts_f16(d, a0 + kk * 8u, bd, idesc, acc);
+                  acc = 1u;
+                }
+              continue;
+            }
+            const uint32_t bh0 = sb + uint32_t(u) * L.bchunk;
             const uint32_t bl0 = bh0 + L.b_bytes;
             const uint32_t a0 = sa + uint32_t(u) * BK;
 #pragma unroll
@@ -305,7 +325,17 @@ __global__ void __launch_bounds__(NTHREADS, 1)
         const uint8_t* st = smem + s * L.stage_bytes;
         const uint32_t taddr = tmem + lane_base + L.a_col0 + uint32_t(s) * uint32_t(L.a_cols);
         uint32_t v[32];
-        if (MODE == A_BITS) {
+        if (MODE == A_BITS && w.bf3) {
+          // bf16 A: two elements per TMEM column, element 2j in the low half
+          for (int u = 0; u < nu; ++u) {
+            const uint32_t wd = reinterpret_cast<const uint32_t*>(st + u * BM * 4)[m];
+            uint32_t h[16];
+#pragma unroll
+            for (int j = 0; j < 16; ++j)
+              h[j] = (((wd >> (2 * j)) & 1u) ? 0x3f80u : 0u) | (((wd >> (2 * j + 1)) & 1u) ? 0x3f800000u : 0u);
+            sttm16(taddr + uint32_t(u) * (BK / 2), h);
+          }
+        } else if (MODE == A_BITS) {
           for (int u = 0; u < nu; ++u) {
             const uint32_t wd = reinterpret_cast<const uint32_t*>(st + u * BM * 4)[m];
 #pragma unroll
@@ -576,7 +606,7 @@ template <int MODE>
 cudaError_t launch_engine(const CUtensorMap& bhi, const CUtensorMap& blo, const CUtensorMap& amap, const Work& w,
                           int npad, cudaStream_t s) {
   if (w.ntiles <= 0) return cudaSuccess;
-  const Layout L = make_layout(MODE, npad, max_stages_env(), max_u_env(), w.b_raw != 0);
+  const Layout L = make_layout(MODE, npad, max_stages_env(), max_u_env(), w.b_raw != 0, w.bf3 != 0);
   const size_t smem = 1024 + size_t(L.stages) * L.stage_bytes + L.out_bytes + (3 * L.stages + 4) * 8 + 16;
   if (smem > 227 * 1024) return cudaErrorInvalidValue;
   static int grid_cap = -1;  // PCGCN_TC_GRID: full-mode CTAs (tuning override, benchmarks only)
@@ -615,7 +645,8 @@ cudaError_t launch_dense_tc(const DenseArgs& a, cudaStream_t s) {
     w.bblk = a.blk;
     w.bblk_stride = a.blk_floats;
     w.order = a.rt_order;
-    w.single = a.loT ? 0 : 1;
+    w.single = (a.loT || a.bf3) ? 0 : 1;
+    w.bf3 = a.bf3;
     w.ntiles = a.nrt;
     w.rt_cptr = a.rt_cptr;
     w.ch_col0 = a.ch_col0;

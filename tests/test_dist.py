@@ -256,9 +256,12 @@ def _halo_epoch_worker(rank, world, port, q, wname, theta, narrow, threshold):
                  narrow=narrow)
     model.epoch()
     torch.cuda.synchronize()
+    # bytes a halo-mode epoch must move into this rank: Y0', dP1' (width ldH, plan's
+    # halo) and Y1', dL' (width ldC, plan_c's halo)
+    expect = 4 * (2 * model.ldH * pl.stats()["halo_recv_rows"] + 2 * model.ldC * pl_c.stats()["halo_recv_rows"])
     q.put((rank, pl.row_lo, pl.row_hi, model.H1.cpu().numpy(), model.Lg.cpu().numpy(), model.G0.cpu().numpy(),
            model.loss.item(), model.grad.cpu().numpy(), model.theta.cpu().numpy(), ex.mode(pl), ex.mode(pl_c),
-           ex.bytes_moved))
+           (ex.bytes_moved, expect)))
     dist.destroy_process_group()
 
 
@@ -310,7 +313,9 @@ def test_sharded_halo_epoch_matches_unsharded(wname, theta, narrow, threshold):
         assert np.array_equal(g0, G0[lo:hi])
         assert abs(loss - ref.loss.item()) <= 1e-6 * abs(ref.loss.item())
         assert np.max(np.abs(grad - gr)) <= 1e-5 * np.max(np.abs(gr))
-        if wname.startswith("pl") and not narrow:
+        if threshold > 1 and not narrow:
             full_ag = 4 * (g.n - (hi - lo)) * (ref.ldH * 2 + ref.ldC * 2)
-            assert moved < 0.5 * full_ag, (moved, full_ag)
+            assert moved[0] == moved[1], moved           # exactly the planner's halo rows moved
+            if wname.startswith("pl"):
+                assert moved[0] < 0.75 * full_ag, (moved, full_ag)   # clustered graph: well below an all-gather
     assert np.array_equal(res[0][8], res[1][8])

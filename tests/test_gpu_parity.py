@@ -81,15 +81,17 @@ SMALL = {
 
 
 @pytest.mark.parametrize("name", list(SMALL))
-@pytest.mark.parametrize("mode", ["sparse", "dense_tc", "dense_simt", "hybrid", "dense_bf16", "hybrid_tile"])
+@pytest.mark.parametrize("mode", ["sparse", "dense_tc", "dense_simt", "hybrid", "dense_bf16", "hybrid_tile",
+                                  "dense_bf3", "hybrid_tile_bf3"])
 @pytest.mark.parametrize("F", [1, 7, 16, 33, 41, 48, 64, 128])
 def test_aggregation_parity(name, mode, F):
     g = SMALL[name]()
     P = max(1, min(8, g.n // 40))
     theta = {"sparse": 2.0, "dense_tc": 0.0, "dense_simt": 0.0, "hybrid": 0.05, "dense_bf16": 0.0,
-             "hybrid_tile": 0.05}[mode]
-    dense = {"dense_simt": L.DENSE_FP32_SIMT, "dense_bf16": L.DENSE_BF16X1}.get(mode, L.DENSE_TF32X2)
-    kw = dict(order=L.ORDER_DEGREE, grain=L.GRAIN_TILE) if mode == "hybrid_tile" else {}
+             "hybrid_tile": 0.05, "dense_bf3": 0.0, "hybrid_tile_bf3": 0.05}[mode]
+    dense = {"dense_simt": L.DENSE_FP32_SIMT, "dense_bf16": L.DENSE_BF16X1, "dense_bf3": L.DENSE_BF16X3,
+             "hybrid_tile_bf3": L.DENSE_BF16X3}.get(mode, L.DENSE_TF32X2)
+    kw = dict(order=L.ORDER_DEGREE, grain=L.GRAIN_TILE) if mode.startswith("hybrid_tile") else {}
     Y = _feat(g.n, F, 11)
     Z, pl, _ = aggregate_gpu(g, Y, P, theta, dense=dense, **kw)
     err, _ = cond_err(g, Y, Z)
@@ -114,23 +116,25 @@ def test_closed_forms_complete_and_cycle_dense():
     np.testing.assert_allclose(Z, exp, rtol=1e-5, atol=1e-6)
 
 
-@pytest.mark.parametrize("mode", ["sparse", "dense_tc", "dense_simt", "hybrid", "hybrid_tile"])
+@pytest.mark.parametrize("mode", ["sparse", "dense_tc", "dense_simt", "hybrid", "hybrid_tile", "dense_bf3"])
 def test_integer_exact_bitwise(mode):
     """Pin P9: Ã unnormalised, small integers -> every order gives the exact
     sum, so GPU (either mode, any partition, any grain) == oracle bitwise."""
     g = G.cliques([300, 129, 64, 33, 2], seed=5)
     rng = np.random.default_rng(9)
     Y = rng.integers(-1000, 1000, size=(g.n, 40)).astype(np.float32)
-    theta = {"sparse": 2.0, "dense_tc": 0.0, "dense_simt": 0.0, "hybrid": 0.3, "hybrid_tile": 0.3}[mode]
-    dense = L.DENSE_FP32_SIMT if mode == "dense_simt" else L.DENSE_TF32X2
+    theta = {"sparse": 2.0, "dense_tc": 0.0, "dense_simt": 0.0, "hybrid": 0.3, "hybrid_tile": 0.3,
+             "dense_bf3": 0.0}[mode]
+    dense = {"dense_simt": L.DENSE_FP32_SIMT, "dense_bf3": L.DENSE_BF16X3}.get(mode, L.DENSE_TF32X2)
     kw = dict(order=L.ORDER_DEGREE, grain=L.GRAIN_TILE) if mode == "hybrid_tile" else {}
     Z, _, _ = aggregate_gpu(g, Y, 5, theta, dense=dense, norm=L.NORM_NONE, **kw)
     exp = O.aggregate(O.normalized_adjacency(g.n, g.rowptr, g.col, "none")[0], Y.astype(np.float64))
     assert np.array_equal(Z, exp)
 
 
+@pytest.mark.parametrize("dense", ["tf32x2", "bf16x3"])
 @pytest.mark.parametrize("F", [16, 41, 128, 200])
-def test_dense_long_accumulation_accuracy(F):
+def test_dense_long_accumulation_accuracy(F, dense):
     """Full mode on rows with thousands of dense terms, all-positive values
     whose tf32 lo part matters (1 - 2^-24): the tensor core's biased TMEM
     accumulation must not build up (groups of <= 8 chunks are folded into
@@ -138,7 +142,8 @@ def test_dense_long_accumulation_accuracy(F):
     g = G.cliques([2000, 1500])
     x = np.float32(1.0 - 2.0 ** -24)
     Y = np.full((g.n, F), x, dtype=np.float32)
-    Z, pl, _ = aggregate_gpu(g, Y, 2, 0.0, norm=L.NORM_NONE, f_max=256)
+    Z, pl, _ = aggregate_gpu(g, Y, 2, 0.0, norm=L.NORM_NONE, f_max=256,
+                             dense=L.DENSE_BF16X3 if dense == "bf16x3" else L.DENSE_TF32X2)
     assert pl.stats()["nnz_dense"] == pl.stats()["nnz"]
     size = np.where(g.labels == 0, 2000, 1500)[:, None]
     rel = np.abs(Z - size * float(x)) / (size * float(x))
@@ -329,7 +334,8 @@ def test_epoch_parity(wname, theta, theta_c):
 @pytest.mark.parametrize("d,theta,theta_c,grain", [(1.0, 0.02, 0.02, "block"), (5.0, 0.1, 2.0, "block"),
                                                    (10.0, 0.2, 0.1, "block"), (10.0, 0.0, 2.0, "block"),
                                                    (1.0, 0.1, 0.05, "tile"), (5.0, 0.2, 0.3, "tile"),
-                                                   (10.0, 0.3, 0.2, "tile")])
+                                                   (10.0, 0.3, 0.2, "tile"), (10.0, 0.1, 0.1, "tile_bf3"),
+                                                   (1.0, 0.05, 0.08, "tile_bf3")])
 def test_rmat_hybrid_epoch_parity(d, theta, theta_c, grain):
     """SURVEY F1 / Table III workloads (RMAT-1, -5, -10: n = 10,240, 128 -> 64 -> 32,
     P = 16): mixed selective/full plans, one per
@@ -342,7 +348,9 @@ def test_rmat_hybrid_epoch_parity(d, theta, theta_c, grain):
     Th0, Th1 = C.thetas(w)
     y = C.labels(w, g)
     T = C.train_mask(g.n, w.theta_seed)
-    kw = dict(f_max=128, order=L.ORDER_DEGREE, grain=L.GRAIN_TILE) if grain == "tile" else dict(f_max=128)
+    kw = dict(f_max=128, order=L.ORDER_DEGREE, grain=L.GRAIN_TILE) if grain.startswith("tile") else dict(f_max=128)
+    if grain.endswith("bf3"):
+        kw["dense_prec"] = L.DENSE_BF16X3
     pl = L.Plan(g.n, g.rowptr, g.col, w.P, theta, **kw)
     pl_c = L.Plan(g.n, g.rowptr, g.col, w.P, theta_c, **kw)
     st, st_c = pl.stats(), pl_c.stats()

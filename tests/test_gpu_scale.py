@@ -45,8 +45,10 @@ def c3_epoch(c3):
 
 # θ pairs (F = H plan, F = C plan): the pair BENCH_r01 selected with its measured
 # grid (0.0418, 0.056), the grid's neighbours, and all-selective
-@pytest.mark.parametrize("theta,theta_c", [(0.0418, 0.056), (0.028, 0.04), (0.02, 0.0575), (2.0, 2.0)])
-def test_c3_bench_epoch_all_rows(c3_epoch, theta, theta_c):
+@pytest.mark.parametrize("theta,theta_c,cfg", [(0.0418, 0.056, "block"), (0.028, 0.04, "block"), (2.0, 2.0, "block"),
+                                               (0.066, 0.066, "tile"), (0.045, 0.08, "tile"),
+                                               (0.066, 0.066, "tile_bf3"), (0.04, 0.05, "tile_bf3")])
+def test_c3_bench_epoch_all_rows(c3_epoch, theta, theta_c, cfg):
     """The exact launch configuration bench.py times on C3 (two plans, one per
     width; activation strides 128 / 48; one CUDA-graph replay of the epoch),
     with SGD so the update can be read back: H1, logits, loss, G1, G0, ∇Θ1,
@@ -55,8 +57,13 @@ def test_c3_bench_epoch_all_rows(c3_epoch, theta, theta_c):
     from epoch_check import check_gcn2_epoch
     w, g, X, Th0, Th1, y, T, ref = c3_epoch
     fmax = max(w.hidden, w.classes)
-    pl = L.Plan(g.n, g.rowptr, g.col, w.P, theta, f_max=fmax)
-    pl_c = L.Plan(g.n, g.rowptr, g.col, w.P, theta_c, f_max=fmax)
+    kw = dict(f_max=fmax)
+    if cfg.startswith("tile"):     # bench.py's default: degree order, per-chunk modes
+        kw.update(order=L.ORDER_DEGREE, grain=L.GRAIN_TILE)
+    if cfg.endswith("bf3"):
+        kw.update(dense_prec=L.DENSE_BF16X3)
+    pl = L.Plan(g.n, g.rowptr, g.col, w.P, theta, **kw)
+    pl_c = L.Plan(g.n, g.rowptr, g.col, w.P, theta_c, **kw)
     if theta < 1:
         assert pl.stats()["nnz_dense"] > 0 and pl_c.stats()["nnz_dense"] > 0
     perm = pl.perm()
@@ -68,7 +75,7 @@ def test_c3_bench_epoch_all_rows(c3_epoch, theta, theta_c):
     torch.cuda.synchronize()
     rep = {}
     check_gcn2_epoch(model, ref, perm, lr=0.1, Th0=Th0, Th1=Th1, report=rep)
-    print("c3 bench epoch", theta, theta_c, rep)
+    print("c3 bench epoch", theta, theta_c, cfg, rep)
 
 
 @pytest.fixture(scope="module")
