@@ -42,12 +42,13 @@ def parse():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--workload", default="reddit")
     ap.add_argument("--theta", default="auto")
+    ap.add_argument("--theta-c", type=float, default=None, help="fixed θ of the width-C plan (with a fixed --theta)")
     ap.add_argument("--P", type=int, default=0)
     ap.add_argument("--order", default="degree", choices=["id", "degree"],
                     help="vertex order inside a partition (pcgcn_opts.vertex_order)")
     ap.add_argument("--grain", default="tile", choices=["block", "tile"],
                     help="unit of the selective/full decision (pcgcn_opts.mode_grain)")
-    ap.add_argument("--dense", default="tf32x2", choices=["tf32x2", "bf16x3"],
+    ap.add_argument("--dense", default="bf16x3", choices=["tf32x2", "bf16x3"],
                     help="full-mode arithmetic (pcgcn_opts.dense_prec)")
     ap.add_argument("--oracle-frac", type=float, default=0.02)
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -58,6 +59,8 @@ def parse():
                     help="F2 sensitivity: 'L1,L2,..:H1,H2,..' epoch ms of the l-layer GCN over layers x hidden")
     ap.add_argument("--f3", type=int, default=0,
                     help="F3 convergence study (§V-E): epochs of Adam training, fp32 vs bf16 full mode")
+    ap.add_argument("--f3-signal", type=float, default=0.015, help="F3: class-signal strength of the features")
+    ap.add_argument("--f3-seeds", type=int, default=3, help="F3: initialisations")
     ap.add_argument("--table3", action="store_true",
                     help="Table III replica on RMAT-{0.1..10}: epoch ms of PCGCN-sel / -full / hybrid")
     return ap.parse_args()
@@ -312,7 +315,7 @@ def run_table3(args):
                "theta_L161": th0}
 
         def epoch_ms(theta):
-            pl = L.Plan(g.n, g.rowptr, g.col, w.P, theta, f_max=max(w.hidden, w.classes))
+            pl = L.Plan(g.n, g.rowptr, g.col, w.P, theta, f_max=max(w.hidden, w.classes), **plan_kw(args))
             perm = pl.perm()
             m = GCN2(pl, np.ascontiguousarray(X[perm]), lab[perm], T[perm], Th0, Th1, optimizer="adam", lr=0.01,
                      device=dev)
@@ -336,10 +339,14 @@ def run_table3(args):
         ent["hybrid_ms"], ent["hybrid_dense_frac"] = epoch_ms(th0)
         grid = {}
         for th in (0.01, 0.02, 0.05, 0.1, 0.2, 0.4):
-            grid[th] = epoch_ms(th)[0]
+            grid[th] = epoch_ms(th)
+        ent["grid"] = {str(k): {"ms": v[0], "dense_frac": v[1]} for k, v in grid.items()}
+        grid = {k: v[0] for k, v in grid.items()}
         bt = min(grid, key=grid.get)
         ent["hybrid_grid_best"] = {"theta": bt, "ms": grid[bt]}
         ent["ordering_holds"] = ent["hybrid_ms"] <= 1.05 * min(ent["sel_ms"], ent["full_ms"])
+        ent["ordering_holds_grid"] = grid[bt] <= min(ent["sel_ms"], ent["full_ms"])
+        ent["plan"] = {"order": args.order, "grain": args.grain, "dense": args.dense}
         log(f"[table3] {ent}")
         rows.append(ent)
     print(json.dumps({"table3": rows, "metric": "2-layer GCN epoch ms", "unit": "ms", "steps": args.steps,
@@ -348,49 +355,64 @@ def run_table3(args):
 
 
 def run_f3(args):
-    """SURVEY F3 / PAPER.md §V-E (L330-L334, Fig. 9): per-epoch test accuracy
-    of the same 2-layer GCN trained with the exact fp32 selective mode
-    (θ = 2), the fp32-accurate hybrid (tf32 hi/lo full mode) and the bf16
-    full mode (PCGCN_DENSE_BF16X1, hybrid θ and every block full), on the
-    workload's graph with an 80/20 train/test split.  The synthetic features
-    carry a weak class signal here (class mean vectors, 0.5 x N(0,1)) so
-    that the task is learnable; same seed and init for every variant."""
+    """SURVEY F3 / PAPER.md §V-E (L330-L334, Fig. 9): test accuracy of the
+    same 2-layer GCN trained with the exact fp32 selective mode (θ = 2), the
+    fp32-accurate hybrid (tf32 hi/lo full mode), the bf16 hybrid and the bf16
+    all-full executor (PCGCN_DENSE_BF16X1: the paper's 16-bit tensor-core
+    policy), 80/20 split, over ``--f3-seeds`` initialisations.  The features
+    carry a WEAK class signal (class mean vectors x ``--f3-signal`` added to
+    the synthetic features; 0.015 puts the fp32 test accuracy of C2 in the
+    70-90% band, tuned with the fp64 oracle) so the task does not saturate and
+    a precision effect could show.  Reports each variant's accuracy delta to
+    fp32 per seed and its mean / max."""
     import torch
     from paper_conf_ipps_tianmyd20_b200 import _lib as L
     from paper_conf_ipps_tianmyd20_b200.gcn import GCN2
+    from synth import configs as C
     dev = torch.device("cuda", 0)
     torch.cuda.set_device(dev)
     w, g, X, Th0, Th1, labels, T = load_workload(args.workload)
-    mu = np.random.default_rng([w.feat_seed, 99]).standard_normal((w.classes, w.f_in)).astype(np.float32) * 0.5
-    X = (X + mu[labels]).astype(np.float32)
+    mu = np.random.default_rng([w.feat_seed, 99]).standard_normal((w.classes, w.f_in)).astype(np.float32)
+    X = (X + args.f3_signal * mu[labels]).astype(np.float32)
     theta_h = float(args.theta) if args.theta != "auto" else 0.05
     variants = [("fp32_selective", 2.0, L.DENSE_TF32X2), ("tf32x2_hybrid", theta_h, L.DENSE_TF32X2),
                 ("bf16_hybrid", theta_h, L.DENSE_BF16X1), ("bf16_full", 0.0, L.DENSE_BF16X1)]
-    curves = {}
-    for name, th, prec in variants:
-        pl = L.Plan(g.n, g.rowptr, g.col, args.P or w.P, th, dense_prec=prec, f_max=max(w.hidden, w.classes))
-        perm = pl.perm()
-        lab = labels[perm]
-        test = torch.from_numpy(~T[perm]).to(dev)
-        labd = torch.from_numpy(lab.astype(np.int64)).to(dev)
-        m = GCN2(pl, np.ascontiguousarray(X[perm]), lab, T[perm], Th0, Th1, optimizer="adam", lr=0.01, device=dev)
-        acc, losses = [], []
-        for ep in range(args.f3):
-            m.epoch()
-            if ep % 10 == 9 or ep == args.f3 - 1:
-                pred = m.Lg[:, :w.classes].argmax(dim=1)   # logits of the forward just run
-                acc.append(float((pred[test] == labd[test]).float().mean().item()))
-                losses.append(float(m.loss.item()))
-        st = pl.stats()
-        curves[name] = {"theta": th, "dense_edge_frac": st["nnz_dense"] / st["nnz"], "test_acc_every10": acc,
-                        "loss_every10": losses, "final_test_acc": acc[-1]}
-        log(f"[f3] {name}: {curves[name]['final_test_acc']:.4f} dense={curves[name]['dense_edge_frac']:.3f}")
-        del m
-        pl.destroy()
-    base = curves["fp32_selective"]["final_test_acc"]
-    for k in curves:
-        curves[k]["acc_delta_vs_fp32"] = curves[k]["final_test_acc"] - base
+    seeds = list(range(args.f3_seeds))
+    curves = {name: {"per_seed": []} for name, _, _ in variants}
+    for sd in seeds:
+        th0 = C.glorot(w.f_in, w.hidden, w.theta_seed + 100 * sd, 0)
+        th1 = C.glorot(w.hidden, w.classes, w.theta_seed + 100 * sd, 1)
+        for name, th, prec in variants:
+            kw = plan_kw(args)
+            kw["dense_prec"] = prec
+            pl = L.Plan(g.n, g.rowptr, g.col, args.P or w.P, th, f_max=max(w.hidden, w.classes), **kw)
+            perm = pl.perm()
+            lab = labels[perm]
+            test = torch.from_numpy(~T[perm]).to(dev)
+            labd = torch.from_numpy(lab.astype(np.int64)).to(dev)
+            m = GCN2(pl, np.ascontiguousarray(X[perm]), lab, T[perm], th0, th1, optimizer="adam", lr=0.01,
+                     device=dev)
+            acc = []
+            for ep in range(args.f3):
+                m.epoch()
+                if ep % 10 == 9 or ep == args.f3 - 1:
+                    pred = m.Lg[:, :w.classes].argmax(dim=1)   # logits of the forward just run
+                    acc.append(float((pred[test] == labd[test]).float().mean().item()))
+            st = pl.stats()
+            curves[name]["per_seed"].append({"seed": sd, "final_test_acc": acc[-1], "test_acc_every10": acc,
+                                             "dense_edge_frac": st["nnz_dense"] / st["nnz"], "theta": th})
+            log(f"[f3] seed {sd} {name}: {acc[-1]:.4f} dense={st['nnz_dense'] / st['nnz']:.3f}")
+            del m
+            pl.destroy()
+    for name in curves:
+        d = [curves[name]["per_seed"][i]["final_test_acc"] - curves["fp32_selective"]["per_seed"][i]["final_test_acc"]
+             for i in range(len(seeds))]
+        curves[name]["acc_delta_vs_fp32"] = d
+        curves[name]["acc_delta_mean"] = float(np.mean(d))
+        curves[name]["acc_delta_max_abs"] = float(np.max(np.abs(d)))
+        curves[name]["final_test_acc_mean"] = float(np.mean([e["final_test_acc"] for e in curves[name]["per_seed"]]))
     print(json.dumps({"f3": curves, "workload": w.name, "epochs": args.f3, "optimizer": "adam lr 0.01",
+                      "signal": args.f3_signal, "seeds": len(seeds),
                       "paper": "§V-E: PCGCN-TC accuracy drop 0.08% (pubmed), 0.19% (reddit-s) — context"}), flush=True)
 
 
@@ -552,6 +574,7 @@ def main():
         del Y0, Y1, ZH, ZC
     else:
         theta, theta_src = float(args.theta), "fixed"
+        theta_c = args.theta_c
     t0 = time.time()
     pl = L.Plan(g.n, g.rowptr, g.col, P, theta, f_max=fmax, rank=rank, world=world, **plan_kw(args))
     pl_c = L.Plan(g.n, g.rowptr, g.col, P, theta_c, f_max=fmax, rank=rank, world=world, **plan_kw(args)) if theta_c else None

@@ -133,6 +133,11 @@ pcgcn_status upload_plan(pcgcn_plan_s* p) {
         const int64_t b = ((round & 1) && full_round) ? G - 1 - k : k;  // CTA receiving the i-th largest tile
         order[round * G + b] = bysize[i];
       }
+      // PCGCN_TC_ORDER=plan (A/B knob): tiles in plan order, so the CTAs work on
+      // neighbouring row tiles at the same time and share their source windows in L2
+      if (const char* e = getenv("PCGCN_TC_ORDER"))
+        if (std::string(e) == "plan")
+          for (int64_t i = 0; i < d.nrt; ++i) order[i] = int32_t(i);
       UP(&d.rt_order, order.data(), d.nrt);
     }
     UP(&d.ch_col0, p->ch_col0.data() + ch_lo, d.nch);
