@@ -53,7 +53,7 @@ typedef enum {
   PCGCN_ENOTSYM = 2,  /* input adjacency not symmetric (needed for Âᵀ = Â) */
   PCGCN_ECUDA = 3,    /* CUDA runtime error (also: no usable GPU) */
   PCGCN_ENOMEM = 4,   /* host or device allocation failed */
-  PCGCN_ENCCL = 5,    /* reserved: collective failure */
+  PCGCN_ENCCL = 5,    /* NCCL missing or a collective failed (pcgcn_nccl_* / pcgcn_halo_exchange) */
   PCGCN_EUNSUP = 6    /* unsupported option combination */
 } pcgcn_status;
 
@@ -207,6 +207,20 @@ pcgcn_status pcgcn_plan_halo_export(pcgcn_plan_t p, int32_t q, int32_t send, int
  * (NCCL grouped send/recv, or an all-to-all) is the caller's (dist.py). */
 pcgcn_status pcgcn_halo_pack(pcgcn_plan_t p, const float* Y, int64_t ldy, int32_t w, float* buf, void* stream);
 pcgcn_status pcgcn_halo_unpack(pcgcn_plan_t p, const float* buf, float* Y, int64_t ldy, int32_t w, void* stream);
+
+/* In-library NCCL transport (SURVEY.md §8(b) nccl_comm): libnccl.so.2 is opened at first
+ * use (no link-time dependency); PCGCN_ENCCL when it is missing or a call fails.
+ *   pcgcn_nccl_unique_id: rank 0 creates the 128-byte id (HOST buffer) that the caller
+ *       distributes (e.g. over the torch process group);
+ *   pcgcn_nccl_comm_init: every rank joins on the current CUDA device (collective);
+ *   pcgcn_halo_exchange: pack -> one NCCL group of ncclSend/ncclRecv to every peer with a
+ *       non-empty list -> unpack, on `stream` (graph-capturable); sendbuf/recvbuf DEVICE
+ *       [Σ send rows x w] / [Σ recv rows x w]; world = 1 => no-op. */
+pcgcn_status pcgcn_nccl_unique_id(void* id128);
+pcgcn_status pcgcn_nccl_comm_init(const void* id128, int32_t rank, int32_t world, void** comm_out);
+void pcgcn_nccl_comm_destroy(void* comm);
+pcgcn_status pcgcn_halo_exchange(pcgcn_plan_t p, float* Y, int64_t ldy, int32_t w, float* sendbuf, float* recvbuf,
+                                 void* nccl_comm, void* stream);
 
 /* ---- dense helpers of the 2-layer GCN step (Alg. 1 transform, L114) ---- */
 

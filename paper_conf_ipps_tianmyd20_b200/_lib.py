@@ -98,6 +98,10 @@ _sig("pcgcn_plan_halo_rows", c_i64, c_vp, c_i32, c_i32)
 _sig("pcgcn_plan_halo_export", c_i32, c_vp, c_i32, c_i32, c_vp, c_i64)
 _sig("pcgcn_halo_pack", c_i32, c_vp, c_vp, c_i64, c_i32, c_vp, c_vp)
 _sig("pcgcn_halo_unpack", c_i32, c_vp, c_vp, c_vp, c_i64, c_i32, c_vp)
+_sig("pcgcn_nccl_unique_id", c_i32, c_vp)
+_sig("pcgcn_nccl_comm_init", c_i32, c_vp, c_i32, c_i32, ctypes.POINTER(c_vp))
+_sig("pcgcn_nccl_comm_destroy", None, c_vp)
+_sig("pcgcn_halo_exchange", c_i32, c_vp, c_vp, c_i64, c_i32, c_vp, c_vp, c_vp, c_vp)
 _sig("pcgcn_last_error", ctypes.c_char_p)
 _sig("pcgcn_abi_version", c_i32)
 
@@ -208,6 +212,12 @@ class Plan:
         check(lib.pcgcn_halo_unpack(self._h, _ptr(buf), _ptr(Y), Y.stride(0), w, _stream(stream)),
               "pcgcn_halo_unpack")
 
+    def halo_exchange(self, Y, sendbuf, recvbuf, comm, w=None, stream=None):
+        """pack -> NCCL grouped send/recv (in libpcgcn) -> unpack."""
+        w = Y.shape[1] if w is None else w
+        check(lib.pcgcn_halo_exchange(self._h, _ptr(Y), Y.stride(0), w, _ptr(sendbuf), _ptr(recvbuf), comm,
+                                      _stream(stream)), "pcgcn_halo_exchange")
+
     def rowscale_ptr(self):
         return lib.pcgcn_plan_rowscale(self._h)
 
@@ -287,6 +297,23 @@ def refine_theta(plan, Y, Z, F, stream=None):
     check(lib.pcgcn_refine_theta(plan._h, _ptr(Y), Y.stride(0), _ptr(Z), Z.stride(0), F, ctypes.byref(th),
                                  ctypes.byref(cc), ctypes.byref(ce)), "pcgcn_refine_theta")
     return th.value, cc.value, ce.value
+
+
+def nccl_unique_id() -> bytes:
+    buf = ctypes.create_string_buffer(128)
+    check(lib.pcgcn_nccl_unique_id(buf), "pcgcn_nccl_unique_id")
+    return buf.raw
+
+
+def nccl_comm_init(uid: bytes, rank: int, world: int):
+    comm = c_vp()
+    check(lib.pcgcn_nccl_comm_init(ctypes.create_string_buffer(uid, 128), rank, world, ctypes.byref(comm)),
+          "pcgcn_nccl_comm_init")
+    return comm
+
+
+def nccl_comm_destroy(comm):
+    lib.pcgcn_nccl_comm_destroy(comm)
 
 
 def probe_read_gbs(nbytes, iters=20):

@@ -19,7 +19,7 @@ NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 CU_SOURCES = ["pcgcn_api.cu", "sparse.cu", "tc_engine.cu", "dense_simt.cu", "gemm.cu", "loss_opt.cu",
               "calibrate.cu", "probe.cu", "tc_pair.cu", "halo.cu"]
-CXX_SOURCES = ["planner.cpp"]
+CXX_SOURCES = ["planner.cpp", "nccl_halo.cpp"]
 
 
 def _run(cmd):
@@ -56,7 +56,7 @@ def build(verbose_ptxas: bool = False, force: bool = False) -> str:
         objs.append(o)
         if force or _stale(o, [s] + headers):
             _run(["g++", "-O3", "-std=c++17", "-fPIC", "-pthread", "-I" + os.path.join(ROOT, "include"),
-                  "-c", s, "-o", o])
+                  "-I/usr/local/cuda/include", "-c", s, "-o", o])
     if force or _stale(OUT, objs):
         _run([NVCC, *ARCH, "-shared", "-o", OUT, *objs, "-Xcompiler", "-pthread", "-lcuda" if False else "-ldl"])
     return OUT

@@ -70,8 +70,13 @@ class HaloExchange:
     ``plan``'s local rows read.  Falls back to the all-gather per plan when
     its halo exceeds ``threshold`` of the remote rows on any rank."""
 
-    def __init__(self, plans, group=None, threshold: float = 0.5):
+    def __init__(self, plans, group=None, threshold: float = 0.5, transport: str = "torch"):
+        """transport: "torch" — torch.distributed all_to_all_single (NCCL grouped
+        send/recv on GPUs, gloo in the tests); "lib" — libpcgcn's own NCCL group
+        (pcgcn_halo_exchange on a communicator bootstrapped here)."""
         self.group = group
+        self.transport = transport
+        self.comm = None
         self.world = dist.get_world_size(group)
         self.rank = dist.get_rank(group)
         self.backend = dist.get_backend(group)
@@ -91,6 +96,17 @@ class HaloExchange:
             self.info[id(pl)] = dict(plan=pl, recv=recv, send=send, mode=mode, frac=float(frac))
         self._bufs = {}
         self.bytes_moved = 0   # rows x stride x 4 received by this rank, summed over gather calls
+        if transport == "lib":
+            from . import _lib as L
+            uid = [L.nccl_unique_id() if self.rank == 0 else None]
+            dist.broadcast_object_list(uid, src=0 if group is None else dist.get_global_rank(group, 0), group=group)
+            self.comm = L.nccl_comm_init(uid[0], self.rank, self.world)
+
+    def close(self):
+        if self.comm is not None:
+            from . import _lib as L
+            L.nccl_comm_destroy(self.comm)
+            self.comm = None
 
     def mode(self, plan):
         return self.info[id(plan)]["mode"]
@@ -113,6 +129,10 @@ class HaloExchange:
         assert full.is_contiguous() and full.shape[0] == pl.n
         send = self._buf(("s", id(pl), w), sum(inf["send"]), w, full)
         recv = self._buf(("r", id(pl), w), sum(inf["recv"]), w, full)
+        if self.comm is not None:
+            pl.halo_exchange(full, send, recv, self.comm, w)
+            self.bytes_moved += recv.shape[0] * w * 4
+            return
         pl.halo_pack(full, send, w)
         if self.backend == "gloo" and full.is_cuda:   # gloo moves host tensors only (tests)
             r_h = torch.empty(recv.shape, dtype=recv.dtype)

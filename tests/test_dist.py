@@ -319,3 +319,61 @@ def test_sharded_halo_epoch_matches_unsharded(wname, theta, narrow, threshold):
             if wname.startswith("pl"):
                 assert moved[0] < 0.75 * full_ag, (moved, full_ag)   # clustered graph: well below an all-gather
     assert np.array_equal(res[0][8], res[1][8])
+
+
+def _nccl_lib_worker(rank, world, port, q):
+    import sys
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    from paper_conf_ipps_tianmyd20_b200 import _lib as L
+    from paper_conf_ipps_tianmyd20_b200.dist import HaloExchange
+    from synth import configs as C
+    _init(rank, world, port)
+    torch.cuda.set_device(0)
+    w = C.PL_SMALL
+    g = C.graph(w)
+    pl = L.Plan(g.n, g.rowptr, g.col, w.P, 0.05, rank=rank, world=world)
+    try:
+        ex = HaloExchange([pl], threshold=1.1, transport="lib")
+    except L.PcgcnError as e:        # NCCL refuses two ranks on one device
+        q.put((rank, "skip", str(e)))
+        dist.destroy_process_group()
+        return
+    full = torch.full((g.n, 8), -1.0, device="cuda")
+    full[pl.row_lo:pl.row_hi] = torch.arange(pl.row_lo, pl.row_hi, dtype=torch.float32, device="cuda")[:, None]
+    ex.gather(full, pl.row_lo, pl.row_hi, plan=pl)
+    torch.cuda.synchronize()
+    recv_rows = np.concatenate([pl.halo(p_, False) for p_ in range(world)]).astype(np.int64)
+    q.put((rank, "ok", (recv_rows, full.cpu().numpy(), pl.row_lo, pl.row_hi)))
+    ex.close()
+    dist.destroy_process_group()
+
+
+@pytest.mark.gpu
+def test_halo_exchange_in_library_nccl():
+    """pcgcn_halo_exchange (pack -> libpcgcn's NCCL group of send/recv ->
+    unpack), two ranks; skipped when NCCL refuses two ranks on one device
+    (the 1-GPU test box)."""
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    ps = [ctx.Process(target=_nccl_lib_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in ps:
+        p.start()
+    out = [q.get(timeout=300) for _ in ps]
+    for p in ps:
+        p.join(timeout=60)
+    if any(o[1] == "skip" for o in out):
+        pytest.skip("NCCL: " + [o[2] for o in out if o[1] == "skip"][0][:200])
+    for rank, _, (recv_rows, full, lo, hi) in out:
+        got = full[:, 0]
+        assert np.array_equal(got[lo:hi], np.arange(lo, hi))
+        assert np.array_equal(got[recv_rows], recv_rows.astype(np.float32))
+
+
+def test_nccl_unique_id_host():
+    """The in-library NCCL bootstrap creates a 128-byte id without a GPU."""
+    from paper_conf_ipps_tianmyd20_b200 import _lib as L
+    a, b = L.nccl_unique_id(), L.nccl_unique_id()
+    assert len(a) == 128 and a != b
