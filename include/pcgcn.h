@@ -22,7 +22,9 @@
  *   - "HOST" pointers are read during the call only (borrowed).  "DEVICE"
  *     pointers are CUDA device memory owned by the caller, and every device
  *     call is asynchronous on the given cudaStream_t (passed as void*), never
- *     synchronises the host, allocates nothing, and is CUDA-graph capturable.
+ *     synchronises the host, allocates nothing, and is CUDA-graph capturable
+ *     (one exception: the first forward/backward WITHOUT PCGCN_IN_PRESCALED
+ *     allocates the plan's n x f_max prescale workspace).
  *   - Dense matrices are row-major fp32 with an explicit leading dimension
  *     (elements); ld >= roundup(F, 4) and rows 16-byte aligned.  Pad columns
  *     of inputs must be zero; pad columns of outputs are written as zero.

@@ -159,7 +159,10 @@ cudaError_t launch_gemm_xw(const float* X, int64_t ldx, const float* W, int64_t 
 
 int64_t gemm_xtg_work_floats(int64_t M, int K, int N) {
   const int64_t simt = int64_t(xtg_slices(M)) * K * N;
-  const int64_t tc = 2 * int64_t(npad16(N)) * r32(M) + tc_xtg_slices(M, K) * int64_t(K) * npad16(N);
+  // the in-engine B conversion (npad <= 128) needs only the slice partials; the
+  // pre-split path also a feature-major hi/lo copy of D (2 x npad x M floats)
+  const bool raw = npad16(N) <= 128 && !xtg_presplit();
+  const int64_t tc = (raw ? 0 : 2 * int64_t(npad16(N)) * r32(M)) + tc_xtg_slices(M, K) * int64_t(K) * npad16(N);
   return simt > tc ? simt : tc;
 }
 
@@ -183,11 +186,12 @@ cudaError_t launch_gemm_xtg(const float* X, int64_t ldx, const float* D, int64_t
     // slices, then a fixed-order sum of the slice partials
     const int np = npad16(N);
     const int64_t ldT = r32(M);
+    const bool raw = np <= 128 && !xtg_presplit();
     float* hi = work;
     float* lo = work + int64_t(np) * ldT;
-    float* part = lo + int64_t(np) * ldT;
+    float* part = raw ? work : lo + int64_t(np) * ldT;
     cudaError_t e;
-    if (np <= 128 && !xtg_presplit()) {
+    if (raw) {
       // B converted inside the engine (D read once; no split pass)
       e = launch_tc_gemm_xtg_raw(X, ldx, D, ldd, part, M, K, N, st);
     } else {

@@ -143,10 +143,16 @@ pcgcn_status upload_plan(pcgcn_plan_s* p) {
     UP(&d.ch_col0, p->ch_col0.data() + ch_lo, d.nch);
     UP(&d.bits, p->bits.data() + ch_lo * TILE_M, d.nch * TILE_M);
     UP(&d.zd, (float*)nullptr, d.nrt * TILE_M * d.fpad_max);
-    // hi rows then lo rows of the feature-major split (per call: lo = hi + npad*n_pad)
-    UP(&d.yhi, (float*)nullptr, 2 * d.n_pad * d.fpad_max);
+    // the full mode's B: window blocks (or the feature-major split) of the whole
+    // input — tf32 hi + lo: 2 floats per element, bf16x3: 3 bf16 = 1.5 floats,
+    // bf16x1: 1; the CUDA-core full mode reads the input directly
+    const int dp = p->opts.dense_prec;
+    const int64_t half_floats = dp == PCGCN_DENSE_BF16X3 ? 3 : dp == PCGCN_DENSE_BF16X1 ? 2
+                              : dp == PCGCN_DENSE_FP32_SIMT ? 0 : 4;
+    if (half_floats > 0) UP(&d.yhi, (float*)nullptr, half_floats * d.n_pad * d.fpad_max / 2);
   }
-  UP(&d.ypre, (float*)nullptr, n * d.fpad_max);
+  // (ypre, the prescaled copy of an un-prescaled input, is allocated by the
+  // first forward/backward call without PCGCN_IN_PRESCALED)
   UP(&d.zrow, (float*)nullptr, 256);
   if (p->opts.world > 1) {
     std::vector<int32_t> sl, rl;
@@ -280,6 +286,15 @@ pcgcn_status aggregate(pcgcn_plan_t p, const float* Y, int64_t ldy, float* Z, in
   if (prof) for (int k = 0; k < 4; ++k) d.ev_used[k] = false;
   mark(0);
   if (!prescaled) {
+    if (!d.ypre) {
+      // first un-prescaled call: the prescale workspace (n x fpad_max floats);
+      // not capturable — calls inside a CUDA graph pass prescaled inputs
+      d.ypre = static_cast<float*>(dev_alloc(sizeof(float) * size_t(std::max<int64_t>(p->n * d.fpad_max, 1))));
+      if (!d.ypre) { set_error("device allocation of the prescale workspace failed"); return PCGCN_ENOMEM; }
+      d.owned.push_back(d.ypre);
+      d.bytes += int64_t(sizeof(float)) * p->n * d.fpad_max;
+      p->stats.device_bytes = d.bytes;
+    }
     if (prof) d.ev_used[0] = true;
     e = launch_prescale(Y, ldy, d.r, p->n, F, d.ypre, ld4, s);
     if (e != cudaSuccess) return cuda_fail(e, "prescale");
