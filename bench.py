@@ -44,9 +44,9 @@ def parse():
     ap.add_argument("--theta", default="auto")
     ap.add_argument("--theta-c", type=float, default=None, help="fixed θ of the width-C plan (with a fixed --theta)")
     ap.add_argument("--P", type=int, default=0)
-    ap.add_argument("--order", default="degree", choices=["id", "degree"],
+    ap.add_argument("--order", default="auto", choices=["auto", "id", "degree"],
                     help="vertex order inside a partition (pcgcn_opts.vertex_order)")
-    ap.add_argument("--grain", default="tile", choices=["block", "tile"],
+    ap.add_argument("--grain", default="auto", choices=["auto", "block", "tile"],
                     help="unit of the selective/full decision (pcgcn_opts.mode_grain)")
     ap.add_argument("--dense", default="bf16x3", choices=["tf32x2", "bf16x3"],
                     help="full-mode arithmetic (pcgcn_opts.dense_prec)")
@@ -306,6 +306,7 @@ def run_table3(args):
     rows = []
     for d, w in C.RMAT.items():
         g = C.graph(w)
+        resolve_plan_defaults(args, g)
         X = C.features(w, g.n)
         Th0, Th1 = C.thetas(w)
         T = C.train_mask(g.n, w.theta_seed)
@@ -372,6 +373,7 @@ def run_f3(args):
     dev = torch.device("cuda", 0)
     torch.cuda.set_device(dev)
     w, g, X, Th0, Th1, labels, T = load_workload(args.workload)
+    resolve_plan_defaults(args, g)
     mu = np.random.default_rng([w.feat_seed, 99]).standard_normal((w.classes, w.f_in)).astype(np.float32)
     X = (X + args.f3_signal * mu[labels]).astype(np.float32)
     theta_h = float(args.theta) if args.theta != "auto" else 0.05
@@ -469,6 +471,19 @@ def run_f2(args):
 # ---------------------------------------------------------------------------
 # our arm
 # ---------------------------------------------------------------------------
+def resolve_plan_defaults(args, g):
+    """--order/--grain auto: degree order + per-chunk modes where the full mode
+    pays (C3: 9.6 -> 8.3 ms), the paper's id order + per-block modes on
+    C5-sized graphs, where chunks of hub rows cost a full-height window split
+    (15 ms per F=128 call) for no selective-pass saving (measured: 212 vs 160 ms
+    epoch, profiles/r2_c5_*.json)."""
+    huge = g.nnz > HUGE_NNZ
+    if args.order == "auto":
+        args.order = "id" if huge else "degree"
+    if args.grain == "auto":
+        args.grain = "block" if huge else "tile"
+
+
 def plan_kw(args):
     from paper_conf_ipps_tianmyd20_b200 import _lib as L
     return dict(order=L.ORDER_DEGREE if args.order == "degree" else L.ORDER_ID,
@@ -508,6 +523,7 @@ def main():
     dev = torch.device("cuda", local)
     torch.cuda.set_device(dev)
     w, g, X, Th0, Th1, labels, T = load_workload(args.workload)
+    resolve_plan_defaults(args, g)
     P = args.P or w.P
     fmax = max(w.hidden, w.classes)
     theta_c = None
@@ -851,6 +867,7 @@ def main():
             "config": {
                 "workload": workload_str(w, g),
                 "P": P, "theta": theta, "theta_c": theta_c if theta_c else theta, "theta_source": theta_src, "optimizer": "adam",
+                "plan_options": {"vertex_order": args.order, "mode_grain": args.grain, "dense_prec": args.dense},
                 "parallelism": f"dp-rows{world}" if world > 1 else "single",
                 "l2": "flushed (256 MiB write) between timed steps",
                 "cuda_graph": use_graph,

@@ -70,6 +70,7 @@ struct DenseArgs {
   int64_t blk_floats = 0;      // floats per window block
   int64_t n_src = 0;           // real source rows (vertices); rows [n_src, n) of the input are never read
   int bf3 = 0;                 // PCGCN_DENSE_BF16X3: window blocks hold 3 bf16 parts (kind::f16 MMAs)
+  int* dyn = nullptr;          // zeroed tile ticket: CTAs claim tiles dynamically in rt_order / plan order
 };
 // mode 0: tf32 hi/lo, 1: bf16 single (BF16X1), 2: three bf16 parts (BF16X3)
 cudaError_t launch_split_windows(const float* Y, int64_t ldy, int64_t n, int F, int npad, int mode, float* blk,

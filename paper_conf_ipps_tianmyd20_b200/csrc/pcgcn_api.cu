@@ -235,6 +235,16 @@ bool dense_blocked_enabled() {
   return v != 0;
 }
 
+// PCGCN_TC_DYN=1: full-mode tiles claimed dynamically in plan order (A/B knob)
+bool tc_dyn_enabled() {
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("PCGCN_TC_DYN");
+    v = e ? (atoi(e) != 0) : 0;
+  }
+  return v != 0;
+}
+
 // rows per scheduler ticket: enough that a ticket covers ~128 selective edges
 // (C5's mean degree 31 -> 8: the next ticket and row pointers are then fetched
 // while the block's rows gather; measured C5 epoch 250 -> 206 ms), 1 for long
@@ -350,6 +360,13 @@ pcgcn_status aggregate(pcgcn_plan_t p, const float* Y, int64_t ldy, float* Z, in
                  d.bits, d.nrt, d.zd, npad, npad};
     da.rt_order = d.rt_order;
     da.n_src = p->n;
+    if (blocked && tc_dyn_enabled()) {
+      // tiles claimed dynamically, in plan order: neighbouring row tiles (and
+      // their source windows) are in flight together, balance comes from the claims
+      da.dyn = d.counter + 16;
+      da.rt_order = nullptr;
+      if ((e = cudaMemsetAsync(da.dyn, 0, sizeof(int), ms)) != cudaSuccess) return cuda_fail(e, "memset");
+    }
     if (blocked) {
       da.blk = d.yhi;
       da.blk_floats = bf3 ? int64_t(npad) * 48 : int64_t(bf16 ? 1 : 2) * npad * 32;

@@ -128,6 +128,8 @@ struct Work {
   int single;        // A_BITS: B hi only (bf16-rounded input), one MMA per K-step (PCGCN_DENSE_BF16X1)
   int bf3;           // A_BITS: kind::f16, B = three bf16 parts (PCGCN_DENSE_BF16X3), window blocks only
   const int32_t* order;  // A_BITS: tile processed at position t (nullptr: t itself)
+  int* dyn;              // A_BITS: tile ticket counter (zeroed before the launch): CTAs claim positions
+                         // dynamically, in order, through a smem ring (nullptr: static round robin)
   const float* bblk;     // A_BITS: source-window blocks of B (pre-swizzled); nullptr: TMA boxes
   int64_t bblk_stride;   // floats per window block
   int b_raw;         // A_TRANS: B = row-major D box; the builders split + transpose it into the
@@ -158,6 +160,54 @@ __device__ __forceinline__ void tile_range(const Work& w, int64_t t, int64_t& kb
   }
 }
 
+// Tile sequence of one CTA: static round robin (t = blockIdx.x + i·gridDim.x),
+// or (w.dyn) positions claimed by the producer from a global ticket counter and
+// passed to the MMA issuer, the builders and the epilogue through a ring of TQ
+// smem slots — every role sees the same sequence; a slot is reused once all
+// three consumer roles have read it (tq_empty, 3 arrivals).
+constexpr int TQ = 16;
+
+struct TileIter {
+  int64_t t;       // current position
+  uint32_t qi;     // ring counter
+};
+
+// consumer side: next position, or false when the sequence ends.  `bar_id` > 0:
+// the role's named barrier (all its 128 threads read the slot before one
+// releases it); 0 for the single-thread MMA issuer.
+__device__ __forceinline__ bool tile_next(const Work& w, TileIter& it, bool first, uint64_t* tq_full,
+                                          uint64_t* tq_empty, const int64_t* tq, int bar_id, bool leader) {
+  if (!w.dyn) {
+    it.t = first ? int64_t(blockIdx.x) : it.t + gridDim.x;
+    return it.t < w.ntiles;
+  }
+  const uint32_t slot = it.qi % TQ, par = (it.qi / TQ) & 1u;
+  mbar_wait(&tq_full[slot], par);
+  it.t = *reinterpret_cast<const volatile int64_t*>(&tq[slot]);
+  if (bar_id > 0) asm volatile("bar.sync %0, 128;" ::"r"(bar_id) : "memory");
+  if (leader) mbar_arrive(&tq_empty[slot]);
+  ++it.qi;
+  return it.t >= 0;
+}
+
+// producer side: claim the next position and publish it to the ring
+__device__ __forceinline__ bool tile_claim(const Work& w, TileIter& it, bool first, uint64_t* tq_full,
+                                           uint64_t* tq_empty, int64_t* tq) {
+  if (!w.dyn) {
+    it.t = first ? int64_t(blockIdx.x) : it.t + gridDim.x;
+    return it.t < w.ntiles;
+  }
+  const uint32_t slot = it.qi % TQ, par = (it.qi / TQ) & 1u;
+  mbar_wait(&tq_empty[slot], par ^ 1u);
+  int64_t t = atomicAdd(w.dyn, 1);
+  if (t >= w.ntiles) t = -1;
+  *reinterpret_cast<volatile int64_t*>(&tq[slot]) = t;
+  mbar_arrive(&tq_full[slot]);
+  ++it.qi;
+  it.t = t;
+  return t >= 0;
+}
+
 // NPC: register-accumulator width of the epilogue (>= npad), 0 = accumulate in the output row
 template <int MODE, int NPC>
 __global__ void __launch_bounds__(NTHREADS, 1)
@@ -172,7 +222,10 @@ __global__ void __launch_bounds__(NTHREADS, 1)
   uint64_t* empty = bar + 2 * L.stages;     // [stages] MMAs done with the stage
   uint64_t* acc_full = bar + 3 * L.stages;  // [2]
   uint64_t* acc_empty = acc_full + 2;       // [2] (128 arrivals)
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(acc_empty + 2);
+  uint64_t* tq_full = acc_empty + 2;        // [TQ] tile id written by the producer
+  uint64_t* tq_empty = tq_full + TQ;        // [TQ] tile id read by the 3 consumer roles
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tq_empty + TQ);
+  int64_t* tq = reinterpret_cast<int64_t*>(tmem_slot + 4);  // [TQ] tile positions (-1: done)
   const int npad = L.npad;
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -185,6 +238,10 @@ __global__ void __launch_bounds__(NTHREADS, 1)
     for (int b = 0; b < 2; ++b) {
       mbar_init(&acc_full[b], 1);
       mbar_init(&acc_empty[b], 128);
+    }
+    for (int q = 0; q < TQ; ++q) {
+      mbar_init(&tq_full[q], 1);
+      mbar_init(&tq_empty[q], 3);
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
@@ -204,7 +261,9 @@ __global__ void __launch_bounds__(NTHREADS, 1)
       // ---- producer ----
       int s = 0;
       uint32_t ph = 0;
-      for (int64_t t = blockIdx.x; t < w.ntiles; t += gridDim.x) {
+      TileIter it{0, 0};
+      for (bool f = true; tile_claim(w, it, f, tq_full, tq_empty, tq); f = false) {
+        const int64_t t = it.t;
         int64_t kb, nch, m0, sp;
         tile_range<MODE>(w, t, kb, nch, m0, sp);
         for (int64_t i = 0; i < nch; i += L.U) {
@@ -253,7 +312,9 @@ __global__ void __launch_bounds__(NTHREADS, 1)
       const uint32_t idesc = (MODE == A_BITS && w.bf3) ? idesc_bf16(BM, npad) : idesc_tf32(BM, npad);
       int s = 0;
       uint32_t ph = 0, gc = 0;  // gc: accumulation-group counter (shared enumeration with the epilogue)
-      for (int64_t t = blockIdx.x; t < w.ntiles; t += gridDim.x) {
+      TileIter it{0, 0};
+      for (bool f = true; tile_next(w, it, f, tq_full, tq_empty, tq, 0, true); f = false) {
+        const int64_t t = it.t;
         int64_t kb, nch, m0, sp;
         tile_range<MODE>(w, t, kb, nch, m0, sp);
         const int64_t nst = (nch + L.U - 1) / L.U;
@@ -316,7 +377,9 @@ __global__ void __launch_bounds__(NTHREADS, 1)
     const uint32_t lane_base = uint32_t((warp & 3) * 32) << 16;
     int s = 0;
     uint32_t ph = 0;
-    for (int64_t t = blockIdx.x; t < w.ntiles; t += gridDim.x) {
+    TileIter it{0, 0};
+    for (bool f = true; tile_next(w, it, f, tq_full, tq_empty, tq, 1, m == 0); f = false) {
+      const int64_t t = it.t;
       int64_t kb, nch, m0, sp;
       tile_range<MODE>(w, t, kb, nch, m0, sp);
       for (int64_t i = 0; i < nch; i += L.U) {
@@ -413,7 +476,9 @@ __global__ void __launch_bounds__(NTHREADS, 1)
     const int m = ((warp & 3) << 5) | lane;
     const uint32_t lane_base = uint32_t((warp & 3) * 32) << 16;
     uint32_t gc = 0;
-    for (int64_t t = blockIdx.x; t < w.ntiles; t += gridDim.x) {
+    TileIter it{0, 0};
+    for (bool f = true; tile_next(w, it, f, tq_full, tq_empty, tq, 2, m == 0); f = false) {
+      const int64_t t = it.t;
       int64_t kb, nch, m0, sp;
       tile_range<MODE>(w, t, kb, nch, m0, sp);
       const int64_t nst = (nch + L.U - 1) / L.U;
@@ -607,7 +672,8 @@ cudaError_t launch_engine(const CUtensorMap& bhi, const CUtensorMap& blo, const 
                           int npad, cudaStream_t s) {
   if (w.ntiles <= 0) return cudaSuccess;
   const Layout L = make_layout(MODE, npad, max_stages_env(), max_u_env(), w.b_raw != 0, w.bf3 != 0);
-  const size_t smem = 1024 + size_t(L.stages) * L.stage_bytes + L.out_bytes + (3 * L.stages + 4) * 8 + 16;
+  const size_t smem = 1024 + size_t(L.stages) * L.stage_bytes + L.out_bytes + (3 * L.stages + 4 + 2 * TQ) * 8 + 16 +
+                     TQ * 8;
   if (smem > 227 * 1024) return cudaErrorInvalidValue;
   static int grid_cap = -1;  // PCGCN_TC_GRID: full-mode CTAs (tuning override, benchmarks only)
   if (grid_cap < 0) {
@@ -647,6 +713,7 @@ cudaError_t launch_dense_tc(const DenseArgs& a, cudaStream_t s) {
     w.order = a.rt_order;
     w.single = (a.loT || a.bf3) ? 0 : 1;
     w.bf3 = a.bf3;
+    w.dyn = a.dyn;
     w.ntiles = a.nrt;
     w.rt_cptr = a.rt_cptr;
     w.ch_col0 = a.ch_col0;
