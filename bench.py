@@ -713,7 +713,8 @@ def main():
         tc_peak = float(json.load(open(MEASURED_PEAKS))["bf16_tflops"]) / (1 if bf3 else 2)
     except Exception:
         tc_peak = 1590.0 / (1 if bf3 else 2)
-    traffic = l2_read = lts_pct = None
+    traffic = l2_read = lts_pct = dram_pct = None
+    traffic_cfg = None
     tpath = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tpath):
         try:
@@ -721,8 +722,13 @@ def main():
             traffic = tj.get("sparse_agg_F%d" % w.hidden)
             l2_read = tj.get("sparse_agg_F%d_l2_read_bytes" % w.hidden)
             lts_pct = tj.get("sparse_agg_F%d_lts_pct" % w.hidden)
+            dram_pct = tj.get("sparse_agg_F%d_dram_pct" % w.hidden)
+            traffic_cfg = tj.get("config")
         except Exception:
             traffic = None
+    # the binding unit of the selective gather per its ncu capture: the L2 (LTS)
+    # or HBM, whichever runs closer to its sustained peak
+    l2_bound = lts_pct is not None and l2_read and (dram_pct is None or lts_pct >= dram_pct)
 
     # ---- e2e: host buffers, H2D of the step's inputs and D2H of the loss inside the region ----
     e2e = None
@@ -876,10 +882,21 @@ def main():
                                             "partition_ms", "plan_ms")},
             },
             "roofline": {"kernel": "sparse_agg (selective-mode gather), layer-1 forward, F=%d" % w.hidden,
-                         "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
+                         "bound": "l2" if l2_bound else "hbm",
+                         "achieved": (l2_read / (t_sp * 1e-3) / 1e9) if l2_bound else achieved,
+                         "peak": (l2_read / (t_sp * 1e-3) / 1e9 / (lts_pct / 100.0)) if l2_bound else peak,
+                         "unit": "GB/s",
+                         "frac": (lts_pct / 100.0) if l2_bound else achieved / peak,
+                         "traffic": traffic,
+                         "peak_source": ("L2: achieved L2->L1 bytes per launch (ncu) / live event time, against the "
+                                         "LTS sustained peak ncu reports for this kernel (lts__throughput % of peak, "
+                                         "the most-utilised unit); HBM view below") if l2_bound else peak_src,
+                         "hbm_view": {"algorithmic_bytes": b_sp, "achieved": achieved, "peak": peak, "frac": achieved / peak,
+                                      "peak_source": peak_src, "ncu_dram_pct": dram_pct,
+                                      "dram_bytes_per_launch": traffic},
                          "algorithmic_bytes": b_sp, "ms": t_sp,
                          "traffic_source": "profiles/traffic.json (ncu --set full, dram read+write per launch)",
+                         "traffic_config": traffic_cfg,
                          "l2_view": {"l2_read_bytes": l2_read,
                                      "achieved": (l2_read / (t_sp * 1e-3) / 1e9) if l2_read else None,
                                      "unit": "GB/s",

@@ -153,8 +153,11 @@ enum {
   PCGCN_RELU = 2u,          /* Z = max(Z, 0) */
   PCGCN_MASK_OUT = 4u,      /* write mask bit [Z_pre > 0], 1 bit per element, row stride ceil(F/32) u32 */
   PCGCN_OUT_PRESCALED = 8u, /* Z = diag(r)·Z again (feeds the next aggregation directly) */
-  PCGCN_PROFILE = 16u       /* record CUDA events around each internal kernel (not graph-capturable);
+  PCGCN_PROFILE = 16u,      /* record CUDA events around each internal kernel (not graph-capturable);
                                read them with pcgcn_plan_last_timings after the stream completes */
+  PCGCN_IN_SPLIT = 32u      /* with IN_PRESCALED: the plan's full-mode window blocks already hold this
+                               input (written by pcgcn_gemm_xw_split / pcgcn_gemm_dwt_split with this plan
+                               and F), so the split pass is skipped */
 };
 
 /* Per-kernel times (ms) of the last PCGCN_PROFILE call on this plan:
@@ -235,6 +238,15 @@ int64_t pcgcn_gemm_xw_work_floats(int32_t K, int32_t N);
 pcgcn_status pcgcn_gemm_xw(const float* X, int64_t ldx, const float* W, int64_t ldw, const float* s,
                            float* Y, int64_t ldy, int64_t M, int32_t K, int32_t N, float* work, void* stream);
 
+/* The same transform GEMM with the full mode's split fused into its epilogue:
+ * besides Y it writes plan p's window blocks of Y (p's precision, width N) — bit-identical
+ * to what the split pass of a following forward/backward would write, which then runs
+ * with PCGCN_IN_SPLIT.  p unsharded, M == n, N <= min(f_max, 128), the tcgen05 path
+ * (work, ld multiples of 4); a plan without full-mode chunks writes Y only. */
+pcgcn_status pcgcn_gemm_xw_split(pcgcn_plan_t p, const float* X, int64_t ldx, const float* W, int64_t ldw,
+                                 const float* s, float* Y, int64_t ldy, int64_t M, int32_t K, int32_t N, float* work,
+                                 void* stream);
+
 /* G = Xᵀ·D:  X DEVICE [M x K] ld ldx, D DEVICE [M x N] ld ldd, G DEVICE [K x N] (ld N), fp32.
  * Split over M into fixed slices whose partial products land in `work`
  * (DEVICE, pcgcn_gemm_xtg_work_floats(M,K,N) floats), then summed in a fixed
@@ -255,6 +267,10 @@ int64_t pcgcn_gemm_dwt_work_floats(int32_t K, int32_t N);
 pcgcn_status pcgcn_gemm_dwt(const float* D, int64_t ldd, const float* W, const uint32_t* mask,
                             const float* s, float* O, int64_t ldo, int64_t M, int32_t N, int32_t K,
                             float* work, void* stream);
+/* ... with plan p's window blocks of O written in the epilogue (as pcgcn_gemm_xw_split; width K) */
+pcgcn_status pcgcn_gemm_dwt_split(pcgcn_plan_t p, const float* D, int64_t ldd, const float* W, const uint32_t* mask,
+                                  const float* s, float* O, int64_t ldo, int64_t M, int32_t N, int32_t K, float* work,
+                                  void* stream);
 
 /* Softmax cross-entropy over the train mask (reading #14):
  *   loss = (1/nT) Σ_{i: train_i} [logsumexp(L_i) - L_{i,y_i}]

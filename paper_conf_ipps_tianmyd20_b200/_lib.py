@@ -28,7 +28,7 @@ NORM_SYM, NORM_NONE = 0, 1
 DENSE_TF32X2, DENSE_FP32_SIMT, DENSE_BF16X1, DENSE_BF16X3 = 0, 1, 2, 3
 ORDER_ID, ORDER_DEGREE = 0, 1
 GRAIN_BLOCK, GRAIN_TILE = 0, 1
-IN_PRESCALED, RELU, MASK_OUT, OUT_PRESCALED, PROFILE = 1, 2, 4, 8, 16
+IN_PRESCALED, RELU, MASK_OUT, OUT_PRESCALED, PROFILE, IN_SPLIT = 1, 2, 4, 8, 16, 32
 TIMING_NAMES = ("prescale", "split", "dense_tc", "sparse")
 X_NAMES = ["part", "perm", "pstart", "r", "blk_k", "blk_i", "blk_nnz", "blk_dense", "sp_rowptr", "sp_col",
            "rt_row0", "rt_nrows", "rt_cptr", "ch_col0", "bits", "zd_index", "sweeps"]
@@ -78,6 +78,8 @@ _sig("pcgcn_gemm_xtg_work_floats", c_i64, c_i64, c_i32, c_i32)
 _sig("pcgcn_gemm_xtg", c_i32, c_vp, c_i64, c_vp, c_i64, c_vp, c_i64, c_i32, c_i32, c_vp, c_vp)
 _sig("pcgcn_gemm_dwt", c_i32, c_vp, c_i64, c_vp, c_vp, c_vp, c_vp, c_i64, c_i64, c_i32, c_i32, c_vp, c_vp)
 _sig("pcgcn_gemm_dwt_work_floats", c_i64, c_i32, c_i32)
+_sig("pcgcn_gemm_xw_split", c_i32, c_vp, c_vp, c_i64, c_vp, c_i64, c_vp, c_vp, c_i64, c_i64, c_i32, c_i32, c_vp, c_vp)
+_sig("pcgcn_gemm_dwt_split", c_i32, c_vp, c_vp, c_i64, c_vp, c_vp, c_vp, c_vp, c_i64, c_i64, c_i32, c_i32, c_vp, c_vp)
 _sig("pcgcn_softmax_ce", c_i32, c_vp, c_i64, c_vp, c_vp, c_i64, c_i32, c_f32, c_vp, c_vp, c_vp, c_vp, c_vp)
 _sig("pcgcn_adam", c_i32, c_vp, c_vp, c_vp, c_vp, c_i64, c_f32, c_f32, c_f32, c_f32, c_vp, c_vp)
 _sig("pcgcn_sgd", c_i32, c_vp, c_vp, c_i64, c_f32, c_vp)
@@ -248,6 +250,23 @@ def gemm_xw(X, W, s, Y, M=None, K=None, N=None, work=None, stream=None):
     N = W.shape[1] if N is None else N
     check(lib.pcgcn_gemm_xw(_ptr(X), X.stride(0), _ptr(W), W.stride(0), s, _ptr(Y), Y.stride(0), M, K, N,
                             _ptr(work), _stream(stream)), "pcgcn_gemm_xw")
+
+
+def gemm_xw_split(plan, X, W, s, Y, M=None, K=None, N=None, work=None, stream=None):
+    """gemm_xw + the plan's full-mode window blocks of Y (consume with IN_SPLIT)."""
+    M = X.shape[0] if M is None else M
+    K = X.shape[1] if K is None else K
+    N = W.shape[1] if N is None else N
+    check(lib.pcgcn_gemm_xw_split(plan._h, _ptr(X), X.stride(0), _ptr(W), W.stride(0), s, _ptr(Y), Y.stride(0), M, K,
+                                  N, _ptr(work), _stream(stream)), "pcgcn_gemm_xw_split")
+
+
+def gemm_dwt_split(plan, D, W, mask, s, O, M=None, N=None, K=None, work=None, stream=None):
+    M = D.shape[0] if M is None else M
+    K = W.shape[0] if K is None else K
+    N = W.shape[1] if N is None else N
+    check(lib.pcgcn_gemm_dwt_split(plan._h, _ptr(D), D.stride(0), _ptr(W), _ptr(mask), s, _ptr(O), O.stride(0), M, N,
+                                   K, _ptr(work), _stream(stream)), "pcgcn_gemm_dwt_split")
 
 
 def gemm_xtg_work_floats(M, K, N):

@@ -136,7 +136,8 @@ int npad16(int n) { return (n + 15) / 16 * 16; }
 int64_t gemm_xw_work_floats(int K, int N) { return 2 * int64_t(npad16(N)) * r32(K); }
 
 cudaError_t launch_gemm_xw(const float* X, int64_t ldx, const float* W, int64_t ldw, const float* s,
-                           float* Y, int64_t ldy, int64_t M, int K, int N, float* work, cudaStream_t st) {
+                           float* Y, int64_t ldy, int64_t M, int K, int N, float* work, cudaStream_t st,
+                           const WindowOut* wo) {
   if (work && ldx % 4 == 0 && ldy % 4 == 0 && N <= 256 && M > 0) {
     // tcgen05 3xTF32: Wᵀ split hi/lo (feature-major), then the engine
     const int np = npad16(N);
@@ -145,7 +146,7 @@ cudaError_t launch_gemm_xw(const float* X, int64_t ldx, const float* W, int64_t 
     float* lo = work + int64_t(np) * ldT;
     cudaError_t e = launch_split_transpose(W, ldw, K, N, np, hi, lo, ldT, st);
     if (e != cudaSuccess) return e;
-    e = launch_tc_gemm_xw(X, ldx, hi, lo, ldT, s, Y, ldy, M, K, N, st);
+    e = launch_tc_gemm_xw(X, ldx, hi, lo, ldT, s, Y, ldy, M, K, N, st, nullptr, 0, wo);
     if (e != cudaSuccess) return e;
     if (ldy > np) zero_pad_kernel<<<256, 256, 0, st>>>(Y, ldy, M, np);
     return cudaGetLastError();
@@ -236,7 +237,7 @@ int64_t gemm_dwt_work_floats(int K, int N) { return 2 * int64_t(npad16(K)) * r32
 
 cudaError_t launch_gemm_dwt(const float* D, int64_t ldd, const float* W, const uint32_t* mask,
                             const float* s, float* O, int64_t ldo, int64_t M, int N, int K,
-                            float* work, cudaStream_t st) {
+                            float* work, cudaStream_t st, const WindowOut* wo) {
   if (work && ldd % 4 == 0 && ldo % 4 == 0 && K <= 256 && M > 0) {
     // tcgen05 3xTF32 (the xw engine with D as A, W rows as the feature-major
     // B, and the ReLU' bit mask + row scale in the epilogue)
@@ -246,7 +247,7 @@ cudaError_t launch_gemm_dwt(const float* D, int64_t ldd, const float* W, const u
     float* lo = work + int64_t(np) * ldT;
     split_rows_kernel<<<unsigned(std::min<int64_t>(256, (np * ldT + 255) / 256)), 256, 0, st>>>(
         W, N, K, N, np, ldT, hi, lo);
-    cudaError_t e = launch_tc_gemm_xw(D, ldd, hi, lo, ldT, s, O, ldo, M, N, K, st, mask, (K + 31) / 32);
+    cudaError_t e = launch_tc_gemm_xw(D, ldd, hi, lo, ldT, s, O, ldo, M, N, K, st, mask, (K + 31) / 32, wo);
     if (e != cudaSuccess) return e;
     if (ldo > np) zero_pad_kernel<<<256, 256, 0, st>>>(O, ldo, M, np);
     return cudaGetLastError();

@@ -6,6 +6,14 @@
 
 namespace pcgcn {
 
+// fused split target of a transform GEMM: the full mode's window blocks of the output
+struct WindowOut {
+  float* blk = nullptr;      // window blocks (DevicePlan::yhi)
+  int mode = 0;              // 1 tf32 hi/lo, 2 bf16x1, 3 bf16x3
+  int64_t blk_floats = 0;    // floats per window block
+  int64_t nwin = 0;          // windows in the buffer
+};
+
 // ---- aggregation (sparse.cu) ----
 struct AggArgs {
   const float* Y;            // prescaled input (all n rows), ld ldy
@@ -86,11 +94,12 @@ cudaError_t launch_dense_simt_y(const DenseArgs& a, const float* y, int64_t ldy,
 // ---- GEMMs (gemm.cu) ----
 int64_t gemm_xw_work_floats(int K, int N);
 cudaError_t launch_gemm_xw(const float* X, int64_t ldx, const float* W, int64_t ldw, const float* s,
-                           float* Y, int64_t ldy, int64_t M, int K, int N, float* work, cudaStream_t st);
+                           float* Y, int64_t ldy, int64_t M, int K, int N, float* work, cudaStream_t st,
+                           const WindowOut* wo = nullptr);
 // tcgen05 engine GEMMs (tc_engine.cu)
 cudaError_t launch_tc_gemm_xw(const float* X, int64_t ldx, const float* wThi, const float* wTlo, int64_t ldwT,
                               const float* rs, float* Y, int64_t ldy, int64_t M, int K, int N, cudaStream_t s,
-                              const uint32_t* mask = nullptr, int64_t mask_ld = 0);
+                              const uint32_t* mask = nullptr, int64_t mask_ld = 0, const WindowOut* wo = nullptr);
 int64_t tc_xtg_slices(int64_t M, int K);
 cudaError_t launch_tc_gemm_xtg_raw(const float* X, int64_t ldx, const float* D, int64_t ldd, float* partial,
                                    int64_t M, int K, int N, cudaStream_t s);
@@ -102,7 +111,7 @@ cudaError_t launch_gemm_xtg(const float* X, int64_t ldx, const float* D, int64_t
 int64_t gemm_dwt_work_floats(int K, int N);
 cudaError_t launch_gemm_dwt(const float* D, int64_t ldd, const float* W, const uint32_t* mask,
                             const float* s, float* O, int64_t ldo, int64_t M, int N, int K,
-                            float* work, cudaStream_t st);
+                            float* work, cudaStream_t st, const WindowOut* wo = nullptr);
 
 // ---- halo exchange of a sharded plan (halo.cu) ----
 cudaError_t launch_halo_copy(bool pack, const float* src, int64_t lds, float* dst, int64_t ldd, const int32_t* idx,

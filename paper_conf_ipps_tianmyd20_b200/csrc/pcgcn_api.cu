@@ -266,6 +266,22 @@ int rows_per_ticket(int64_t nnz_s, int64_t rows) {
   return R < 1 ? 1 : (R > 16 ? 16 : R);
 }
 
+// the plan's full-mode window-block target for a producer of width F (fused
+// split); false if the plan has no chunks on this device / precision
+bool window_out(pcgcn_plan_t p, int32_t F, WindowOut* wo) {
+  const DevicePlan& d = p->d;
+  const int dp = p->opts.dense_prec;
+  if (!d.built || d.nch == 0 || !d.yhi || dp == PCGCN_DENSE_FP32_SIMT) return false;
+  if (dp == PCGCN_DENSE_TF32X2 && (!dense_blocked_enabled() || dense_pair_eligible(int(round_up(F, 16)))))
+    return false;
+  const int64_t npad = round_up(F, 16);
+  wo->blk = d.yhi;
+  wo->mode = dp == PCGCN_DENSE_BF16X3 ? 3 : dp == PCGCN_DENSE_BF16X1 ? 2 : 1;
+  wo->blk_floats = dp == PCGCN_DENSE_BF16X3 ? npad * 48 : (dp == PCGCN_DENSE_BF16X1 ? 1 : 2) * npad * 32;
+  wo->nwin = d.n_pad / 32;
+  return true;
+}
+
 pcgcn_status aggregate(pcgcn_plan_t p, const float* Y, int64_t ldy, float* Z, int64_t ldz, int32_t F,
                        uint32_t flags, uint32_t* mask, void* stream) {
   if (!p || !p->d.built) { set_error("plan has no device structures"); return PCGCN_EINVAL; }
@@ -275,6 +291,10 @@ pcgcn_status aggregate(pcgcn_plan_t p, const float* Y, int64_t ldy, float* Z, in
     return PCGCN_EINVAL;
   }
   if ((flags & PCGCN_MASK_OUT) && !mask) { set_error("MASK_OUT needs a mask buffer"); return PCGCN_EINVAL; }
+  if ((flags & PCGCN_IN_SPLIT) && !(flags & PCGCN_IN_PRESCALED)) {
+    set_error("IN_SPLIT requires IN_PRESCALED (the fused split writes the prescaled producer output)");
+    return PCGCN_EINVAL;
+  }
   DevicePlan& d = p->d;
   cudaStream_t s = static_cast<cudaStream_t>(stream);
   cudaError_t e;
@@ -347,7 +367,10 @@ pcgcn_status aggregate(pcgcn_plan_t p, const float* Y, int64_t ldy, float* Z, in
   // (default), or the feature-major split read by strided TMA boxes (the
   // CTA-pair kernel, or PCGCN_DENSE_BLOCKED=0)
   const bool blocked = bf3 || (tc && dense_blocked_enabled() && !dense_pair_eligible(npad));
-  if (dense && tc) {
+  // IN_SPLIT: the producer already wrote the window blocks (pcgcn_gemm_*_split
+  // writes them exactly when the full mode uses window blocks)
+  const bool presplit = (flags & PCGCN_IN_SPLIT) && blocked;
+  if (dense && tc && !presplit) {
     if (prof) d.ev_used[1] = true;
     e = blocked ? launch_split_windows(src, ldsrc, p->n, F, npad, bf3 ? 2 : (bf16 ? 1 : 0), d.yhi, d.n_pad / 32, ms)
                 : launch_split_transpose(src, ldsrc, p->n, F, npad, d.yhi, bf16 ? nullptr : ylo, d.n_pad, ms);
@@ -631,6 +654,55 @@ pcgcn_status pcgcn_gemm_xw(const float* X, int64_t ldx, const float* W, int64_t 
   }
   cudaError_t e = launch_gemm_xw(X, ldx, W, ldw, s, Y, ldy, M, K, N, work, static_cast<cudaStream_t>(stream));
   return e == cudaSuccess ? PCGCN_OK : cuda_fail(e, "gemm_xw");
+}
+
+static pcgcn_status split_target(pcgcn_plan_t p, int64_t M, int32_t F, const float* work, int64_t ldx, int64_t ldy,
+                                 WindowOut* wo, bool* any) {
+  *any = false;
+  if (!p || !p->d.built) { set_error("gemm *_split: plan has no device structures"); return PCGCN_EINVAL; }
+  if (p->opts.world != 1 || M != p->n) {
+    set_error("gemm *_split: unsharded plan and all n rows only (a sharded input is split after its exchange)");
+    return PCGCN_EINVAL;
+  }
+  if (F > p->opts.f_max || F > 128) { set_error("gemm *_split: F > f_max or > 128"); return PCGCN_EINVAL; }
+  *any = window_out(p, F, wo);
+  if (*any && (!work || (ldx & 3) || (ldy & 3))) {
+    set_error("gemm *_split: needs the tcgen05 path (work buffer, ld multiples of 4)");
+    return PCGCN_EINVAL;
+  }
+  return PCGCN_OK;
+}
+
+pcgcn_status pcgcn_gemm_xw_split(pcgcn_plan_t p, const float* X, int64_t ldx, const float* W, int64_t ldw,
+                                 const float* s, float* Y, int64_t ldy, int64_t M, int32_t K, int32_t N, float* work,
+                                 void* stream) {
+  if (!X || !W || !Y || M < 0 || K < 1 || N < 1 || ldx < K || ldw < N || ldy < N) {
+    set_error("gemm_xw_split: bad arguments");
+    return PCGCN_EINVAL;
+  }
+  WindowOut wo;
+  bool any = false;
+  pcgcn_status st = split_target(p, M, N, work, ldx, ldy, &wo, &any);
+  if (st != PCGCN_OK) return st;
+  cudaError_t e = launch_gemm_xw(X, ldx, W, ldw, s, Y, ldy, M, K, N, work, static_cast<cudaStream_t>(stream),
+                                 any ? &wo : nullptr);
+  return e == cudaSuccess ? PCGCN_OK : cuda_fail(e, "gemm_xw_split");
+}
+
+pcgcn_status pcgcn_gemm_dwt_split(pcgcn_plan_t p, const float* D, int64_t ldd, const float* W, const uint32_t* mask,
+                                  const float* s, float* O, int64_t ldo, int64_t M, int32_t N, int32_t K, float* work,
+                                  void* stream) {
+  if (!D || !W || !O || M < 0 || K < 1 || N < 1 || ldd < N || ldo < K) {
+    set_error("gemm_dwt_split: bad arguments");
+    return PCGCN_EINVAL;
+  }
+  WindowOut wo;
+  bool any = false;
+  pcgcn_status st = split_target(p, M, K, work, ldd, ldo, &wo, &any);
+  if (st != PCGCN_OK) return st;
+  cudaError_t e = launch_gemm_dwt(D, ldd, W, mask, s, O, ldo, M, N, K, work, static_cast<cudaStream_t>(stream),
+                                  any ? &wo : nullptr);
+  return e == cudaSuccess ? PCGCN_OK : cuda_fail(e, "gemm_dwt_split");
 }
 
 int64_t pcgcn_gemm_xtg_work_floats(int64_t M, int32_t K, int32_t N) { return gemm_xtg_work_floats(M, K, N); }

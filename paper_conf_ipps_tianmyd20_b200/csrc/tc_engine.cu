@@ -132,6 +132,9 @@ struct Work {
                          // dynamically, in order, through a smem ring (nullptr: static round robin)
   const float* bblk;     // A_BITS: source-window blocks of B (pre-swizzled); nullptr: TMA boxes
   int64_t bblk_stride;   // floats per window block
+  float* wblk;       // A_ROWMAJOR: also write the output as full-mode window blocks (fused split)
+  int wmode;         // 1: tf32 hi/lo (SW128, 2·npad rows), 2: bf16-rounded (BF16X1), 3: bf16x3 (SW64 parts)
+  int64_t wblk_floats, wblk_nwin;  // floats per window block; windows in the buffer
   int b_raw;         // A_TRANS: B = row-major D box; the builders split + transpose it into the
                      // K-major SWIZZLE_128B hi/lo layout in smem (no feature-major pre-split pass)
 };
@@ -568,6 +571,45 @@ __global__ void __launch_bounds__(NTHREADS, 1)
             }
             __syncwarp();
           }
+          if (w.wblk) {
+            // fused split: this warp's 32 rows are one source
+            // window; lane = source k; the same values as the rows just stored,
+            // in the full mode's pre-swizzled window-block image (the layout of
+            // split_window_kernel, so the aggregation reads identical bits)
+            const int64_t win = (m0 >> 5) + (warp & 3);
+            if (win < w.wblk_nwin) {
+              float* blk = w.wblk + win * w.wblk_floats;
+              uint16_t* b16 = reinterpret_cast<uint16_t*>(blk);
+              const int k = lane;
+#pragma unroll
+              for (int f = 0; f < (NPC > 0 ? NPC : 1); ++f) {
+                if (f >= npad) break;
+                const float v = f < w.ncols ? racc[f] * mk(f) : 0.f;
+                if (w.wmode == 3) {
+                  const uint32_t u0 = __float_as_uint(v);
+                  const uint32_t h0 = (u0 + 0x7fffu + ((u0 >> 16) & 1u)) & 0xffff0000u;
+                  const float r1 = v - __uint_as_float(h0);
+                  const uint32_t u1 = __float_as_uint(r1);
+                  const uint32_t h1 = (u1 + 0x7fffu + ((u1 >> 16) & 1u)) & 0xffff0000u;
+                  const uint32_t u2 = __float_as_uint(r1 - __uint_as_float(h1));
+                  const uint32_t h2 = (u2 + 0x7fffu + ((u2 >> 16) & 1u)) & 0xffff0000u;
+                  const int pos = f * 32 + ((((k >> 3) ^ ((f >> 1) & 3)) << 3) | (k & 7));
+                  b16[pos] = uint16_t(h0 >> 16);
+                  b16[npad * 32 + pos] = uint16_t(h1 >> 16);
+                  b16[2 * npad * 32 + pos] = uint16_t(h2 >> 16);
+                } else if (w.wmode == 1) {
+                  const float h = __uint_as_float(__float_as_uint(v) & 0xffffe000u);
+                  const int rh = f, rl = npad + f;
+                  blk[rh * 32 + ((((k >> 2) ^ (rh & 7)) << 2) | (k & 3))] = h;
+                  blk[rl * 32 + ((((k >> 2) ^ (rl & 7)) << 2) | (k & 3))] = v - h;
+                } else {
+                  const uint32_t u = __float_as_uint(v);
+                  blk[f * 32 + ((((k >> 2) ^ (f & 7)) << 2) | (k & 3))] =
+                      __uint_as_float((u + 0x7fffu + ((u >> 16) & 1u)) & 0xffff0000u);
+                }
+              }
+            }
+          }
         } else if (NPC > 0) {
 #pragma unroll
           for (int c0 = 0; c0 < (NPC > 0 ? NPC : 1); c0 += 4)
@@ -752,7 +794,7 @@ cudaError_t launch_dense_tc(const DenseArgs& a, cudaStream_t s) {
 // ---- Y = diag(s)·X·W, W pre-split feature-major (wT hi/lo [npad][ldwT]) ----
 cudaError_t launch_tc_gemm_xw(const float* X, int64_t ldx, const float* wThi, const float* wTlo, int64_t ldwT,
                               const float* rs, float* Y, int64_t ldy, int64_t M, int K, int N, cudaStream_t s,
-                              const uint32_t* mask, int64_t mask_ld) {
+                              const uint32_t* mask, int64_t mask_ld, const WindowOut* wo) {
   const int npad = (N + 15) / 16 * 16;
   if (ldx % 4 || ldwT % 4 || ldy % 4 || npad > 256) return cudaErrorInvalidValue;
   CUtensorMap mh, ml, ma;
@@ -770,6 +812,13 @@ cudaError_t launch_tc_gemm_xw(const float* X, int64_t ldx, const float* wThi, co
   w.rowscale = rs;
   w.mask = mask;
   w.mask_ld = mask_ld;
+  if (wo && wo->blk) {
+    if (npad > 128 || ldy < N) return cudaErrorInvalidValue;  // fused split: staged epilogue path only
+    w.wblk = wo->blk;
+    w.wmode = wo->mode;
+    w.wblk_floats = wo->blk_floats;
+    w.wblk_nwin = wo->nwin;
+  }
   return launch_engine<A_ROWMAJOR>(mh, ml, ma, w, npad, s);
 }
 

@@ -41,7 +41,7 @@ class GCN2:
     def __init__(self, plan: L.Plan, X_plan: np.ndarray, labels_plan: np.ndarray, train_plan: np.ndarray,
                  Th0: np.ndarray, Th1: np.ndarray, *, optimizer: str = "adam", lr: float = 0.01,
                  device: str | torch.device = "cuda", exchange=None, plan_c: L.Plan | None = None,
-                 narrow: bool = False):
+                 narrow: bool = False, fuse_split: bool = True):
         """All row-indexed host arrays are already in plan order (X_plan = X[perm]).
         ``exchange`` (sharded runs): object with ``gather(full, lo, hi, plan=)``
         and ``allreduce(t)``; rows owned here are plan.row_lo:plan.row_hi.
@@ -66,6 +66,9 @@ class GCN2:
         self.lr = lr
         self.exchange = exchange
         self.narrow = bool(narrow and exchange is not None)
+        # single GPU: the transform GEMMs also write the full mode's window blocks
+        # (pcgcn_gemm_*_split) and the aggregations skip their split pass (IN_SPLIT)
+        self.fuse = bool(fuse_split and exchange is None and max(Th0.shape[1], Th1.shape[1]) <= 128)
         assert max(self.H, self.C) <= plan.f_max
         d, f32 = self.dev, torch.float32
         n, rows, H, C = self.n, self.rows, self.H, self.C
@@ -138,6 +141,9 @@ class GCN2:
         if self.narrow:   # Y0' for all n rows from the replicated X: no width-H exchange
             L.gemm_xw(self.X_all, self.Th0, ctypes.c_void_p(self.r), self.Y0, M=self.n, K=self.f_in, N=H,
                       work=self.xw_work, stream=stream)
+        elif self.fuse:
+            L.gemm_xw_split(p, self.X, self.Th0, rr, self.Y0, M=self.rows, K=self.f_in, N=H, work=self.xw_work,
+                            stream=stream)
         else:
             L.gemm_xw(self.X, self.Th0, rr, self._local(self.Y0), M=self.rows, K=self.f_in, N=H, work=self.xw_work,
                       stream=stream)
@@ -145,16 +151,21 @@ class GCN2:
         if not self.narrow:
             self._gather(self.Y0, p)
         mark("x_gather_y0")
-        p.forward(self.Y0, self.H1, F=H, flags=L.IN_PRESCALED | L.RELU | L.MASK_OUT | agg_flags, mask=self.mask1,
+        sf = L.IN_SPLIT if self.fuse else 0
+        p.forward(self.Y0, self.H1, F=H, flags=L.IN_PRESCALED | L.RELU | L.MASK_OUT | sf | agg_flags, mask=self.mask1,
                   stream=stream)
         mark("a5a6_agg_fwd_H")
         # layer 2
-        L.gemm_xw(self.H1, self.Th1, rr, self._local(self.Y1), M=self.rows, K=H, N=C, work=self.xw_work,
-                  stream=stream)
+        if self.fuse:
+            L.gemm_xw_split(self.plan_c, self.H1, self.Th1, rr, self.Y1, M=self.rows, K=H, N=C, work=self.xw_work,
+                            stream=stream)
+        else:
+            L.gemm_xw(self.H1, self.Th1, rr, self._local(self.Y1), M=self.rows, K=H, N=C, work=self.xw_work,
+                      stream=stream)
         mark("a7_gemm_xw1")
         self._gather(self.Y1, self.plan_c)
         mark("x_gather_y1")
-        self.plan_c.forward(self.Y1, self.Lg, F=C, flags=L.IN_PRESCALED | agg_flags, stream=stream)
+        self.plan_c.forward(self.Y1, self.Lg, F=C, flags=L.IN_PRESCALED | sf | agg_flags, stream=stream)
         mark("a8_agg_fwd_C")
         # loss
         L.softmax_ce(self.Lg, self.labels, self.train, self.inv_nT, rr, self._local(self.dL), self.loss,
@@ -171,6 +182,9 @@ class GCN2:
             self.exchange.gather(self.mask1_all.view(torch.float32), self.lo, self.hi, plan=None)
             L.gemm_dwt(self.G1_all, self.Th1, self.mask1_all, ctypes.c_void_p(self.r), self.dP1, M=self.n, N=C, K=H,
                        work=self.xw_work, stream=stream)
+        elif self.fuse:
+            L.gemm_dwt_split(p, self.G1, self.Th1, self.mask1, rr, self.dP1, M=self.rows, N=C, K=H,
+                             work=self.xw_work, stream=stream)
         else:
             L.gemm_dwt(self.G1, self.Th1, self.mask1, rr, self._local(self.dP1), M=self.rows, N=C, K=H,
                        work=self.xw_work, stream=stream)
@@ -178,7 +192,7 @@ class GCN2:
         if not self.narrow:
             self._gather(self.dP1, p)
         mark("x_gather_dp1")
-        p.backward(self.dP1, self.G0, F=H, flags=L.IN_PRESCALED | agg_flags, stream=stream)
+        p.backward(self.dP1, self.G0, F=H, flags=L.IN_PRESCALED | sf | agg_flags, stream=stream)
         mark("a12_agg_bwd_H")
         L.gemm_xtg(self.X, self.G0, self.gTh0, self.xtg_work, M=self.rows, K=self.f_in, N=H, stream=stream)
         mark("a13_gemm_xtg0")
@@ -204,6 +218,8 @@ class GCN2:
         xw = lambda ld, f: 2 + (1 if ld > np16(f) else 0)  # noqa: E731  W split + engine (+ pad zeroing)
         n = xw(self.ldH, self.H) + xw(self.ldC, self.C)      # a4, a7
         n += 2 * agg(self.plan) + 2 * agg(self.plan_c)       # a5/a6, a8, a10, a12
+        if self.fuse:                                        # split passes fused into xw0, xw1, dwt
+            n -= sum(1 for pl in (self.plan, self.plan_c, self.plan) if pl.stats()["shard_chunks"] > 0)
         n += 2                                               # a9 softmax-CE + loss reduction
         xtg = lambda f: 2 if np16(f) <= 128 else 3  # noqa: E731  engine (in-kernel B split) + slice sum
         n += xtg(self.C) + xtg(self.H)                       # a11, a13

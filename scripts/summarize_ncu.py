@@ -3,7 +3,7 @@
 markdown file under profiles/.  Runs here (no GPU needed to read reports).
 
     python scripts/summarize_ncu.py gpurun_out/r1_launch_list.csv gpurun_out/r1_full.ncu-rep profiles/r1_ncu.md \
-        [F_H F_C [workload]]
+        [F_H F_C [workload [config]]]
 
 With F_H F_C it also merges the selective kernel's per-launch DRAM traffic and
 L2->L1 read bytes into profiles/traffic.json under the workload's name (bench.py's
@@ -22,7 +22,7 @@ METRICS = [
     ("lts__t_sector_hit_rate.pct", "L2 hit %"),
     ("lts__t_sectors_srcunit_tex_op_read.sum", "L2->L1 read sectors"),
     ("lts__throughput.avg.pct_of_peak_sustained_elapsed", "L2 thru %"),
-    ("dram__throughput.avg.pct_of_peak_sustained_elapsed", "DRAM thru %"),
+    ("gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed", "DRAM thru %"),
     ("sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_active", "tensor pipe %"),
     ("smsp__issue_active.avg.pct_of_peak_sustained_active", "issue active %"),
     ("sm__warps_active.avg.pct_of_peak_sustained_active", "warps active %"),
@@ -105,6 +105,14 @@ def main(csv_path, rep_path, out_path):
             if not groups or g_of(d) != g_of(groups[-1][0]):
                 groups.append([])
             groups[-1].append(d)
+        def one_call(grp):   # a call = [segment pass] + row pass; later calls of the same layout follow
+            out = []
+            for d in grp:
+                out.append(d)
+                if "sparse_row" in d[hdr.index("Kernel Name")]:
+                    break
+            return out
+        groups = [one_call(g_) for g_ in groups]
         for key, grp in zip(("sparse_agg_F%d" % fH, "sparse_agg_F%d" % fC), groups[:2]):
             tot, l2 = 0.0, 0.0
             for d in grp:
@@ -116,13 +124,18 @@ def main(csv_path, rep_path, out_path):
             tr[key] = int(tot)
             tr[key + "_l2_read_bytes"] = int(l2) if l2 else None
             # time-weighted L2 (LTS) throughput, % of its sustained peak (ncu's own roofline of the L2)
-            m, tm = "lts__throughput.avg.pct_of_peak_sustained_elapsed", "gpu__time_duration.sum"
-            if m in hdr and tm in hdr:
-                ts = [float(d[hdr.index(tm)].replace(",", "")) for d in grp]
-                ps = [float(d[hdr.index(m)].replace(",", "")) for d in grp]
-                tr[key + "_lts_pct"] = round(sum(t * p for t, p in zip(ts, ps)) / max(sum(ts), 1e-30), 2)
+            tm = "gpu__time_duration.sum"
+            for m, suffix in (("lts__throughput.avg.pct_of_peak_sustained_elapsed", "_lts_pct"),
+                              ("gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed", "_dram_pct"),
+                              ("l1tex__throughput.avg.pct_of_peak_sustained_active", "_l1tex_pct")):
+                if m in hdr and tm in hdr:
+                    ts = [float(d[hdr.index(tm)].replace(",", "")) for d in grp]
+                    ps = [float(d[hdr.index(m)].replace(",", "")) for d in grp]
+                    tr[key + suffix] = round(sum(t * p for t, p in zip(ts, ps)) / max(sum(ts), 1e-30), 2)
             tr[key + "_kernels"] = [short(d[hdr.index("Kernel Name")]) for d in grp]
         tr["source"] = rep_path
+        if len(sys.argv) > 7:
+            tr["config"] = sys.argv[7]   # the plan options / θ the capture ran with (bench.py checks it)
         tp = os.path.join(os.path.dirname(out_path), "traffic.json")
         allt = json.load(open(tp)) if os.path.exists(tp) else {}
         allt[wl] = tr

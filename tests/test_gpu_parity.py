@@ -650,3 +650,33 @@ def test_scheduling_knobs_do_not_change_results(tmp_path, knob, bitwise):
         else:
             scale = max(float(np.max(np.abs(a))), 1e-30)
             assert float(np.max(np.abs(a.astype(np.float64) - b))) <= 2e-6 * scale, (knob, k)
+
+
+@pytest.mark.parametrize("wname,theta,dense", [("cora", 0.01, "tf32x2"), ("pubmed", 0.0, "bf16x3"),
+                                               ("cora", 0.005, "bf16x3"), ("pubmed", 2.0, "tf32x2")])
+def test_fused_split_is_bitwise(wname, theta, dense):
+    """pcgcn_gemm_xw_split / pcgcn_gemm_dwt_split write the full mode's window
+    blocks in the GEMM epilogue and the aggregations then skip their split pass
+    (IN_SPLIT): every output of the epoch is bitwise identical to the unfused
+    epoch (same window-block bits, same MMAs)."""
+    from paper_conf_ipps_tianmyd20_b200.gcn import GCN2
+    w = C.WORKLOADS[wname]
+    g = C.graph(w)
+    X = C.features(w, g.n)
+    Th0, Th1 = C.thetas(w)
+    T = C.train_mask(g.n, w.theta_seed)
+    kw = dict(order=L.ORDER_DEGREE, grain=L.GRAIN_TILE,
+              dense_prec=L.DENSE_BF16X3 if dense == "bf16x3" else L.DENSE_TF32X2)
+    pl = L.Plan(g.n, g.rowptr, g.col, w.P, theta, **kw)
+    pl_c = L.Plan(g.n, g.rowptr, g.col, w.P, theta * 2 if theta < 1 else theta, **kw)
+    perm = pl.perm()
+    outs = []
+    for fuse in (True, False):
+        m = GCN2(pl, X[perm], g.labels[perm], T[perm], Th0, Th1, optimizer="sgd", lr=0.1, plan_c=pl_c,
+                 fuse_split=fuse)
+        assert m.fuse == fuse
+        m.epoch()
+        torch.cuda.synchronize()
+        outs.append([t.clone() for t in (m.Y0, m.H1, m.mask1, m.Y1, m.Lg, m.G1, m.dP1, m.G0, m.grad, m.theta)])
+    for a, b in zip(*outs):
+        assert torch.equal(a, b)
