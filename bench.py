@@ -568,7 +568,7 @@ def main():
             pt = L.Plan(g.n, g.rowptr, g.col, P, th, f_max=fmax, rank=rank, world=world, **plan_kw(args))
             for F, Yin, Zout in ((w.hidden, Y0, ZH), (w.classes, Y1, ZC)):
                 ts = []
-                for it in range(4):
+                for it in range(7):
                     a_, b_ = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
                     a_.record()
                     pt.forward(Yin, Zout, F=F, flags=L.IN_PRESCALED)

@@ -614,7 +614,7 @@ np.savez(sys.argv[1], **out)
                                           ({"PCGCN_SPARSE_V8": "0"}, False),
                                           ({"PCGCN_SPARSE_FSPLIT": "32"}, False),
                                           ({"PCGCN_SPARSE_G6": "0"}, False),
-                                          ({"PCGCN_TC_DYN": "1"}, True)])
+                                          ({"PCGCN_TC_DYN": "0"}, True)])
 def test_scheduling_knobs_do_not_change_results(tmp_path, knob, bitwise):
     """Row-block tickets, the full-mode/segment overlap, the in-kernel xtg B
     conversion and the window-blocked full-mode B layout change only scheduling (every output row is still reduced by
