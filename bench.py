@@ -48,6 +48,8 @@ def parse():
                     help="vertex order inside a partition (pcgcn_opts.vertex_order)")
     ap.add_argument("--grain", default="auto", choices=["auto", "block", "tile"],
                     help="unit of the selective/full decision (pcgcn_opts.mode_grain)")
+    ap.add_argument("--fuse-split", default="on", choices=["on", "off"],
+                    help="transform GEMMs write the full mode's window blocks (pcgcn_gemm_*_split)")
     ap.add_argument("--dense", default="bf16x3", choices=["tf32x2", "bf16x3"],
                     help="full-mode arithmetic (pcgcn_opts.dense_prec)")
     ap.add_argument("--oracle-frac", type=float, default=0.02)
@@ -601,7 +603,7 @@ def main():
     Xp = np.ascontiguousarray(X[perm])
     exch = RowExchange(pl.row_lo, pl.row_hi) if world > 1 else None
     model = GCN2(pl, Xp, labels[perm], T[perm], Th0, Th1, optimizer="adam", lr=0.01, device=dev, exchange=exch,
-                 plan_c=pl_c)
+                 plan_c=pl_c, fuse_split=args.fuse_split == "on")
     use_graph = world == 1 and not args.eager
     stream = torch.cuda.current_stream(dev)
     if use_graph:
@@ -873,7 +875,8 @@ def main():
             "config": {
                 "workload": workload_str(w, g),
                 "P": P, "theta": theta, "theta_c": theta_c if theta_c else theta, "theta_source": theta_src, "optimizer": "adam",
-                "plan_options": {"vertex_order": args.order, "mode_grain": args.grain, "dense_prec": args.dense},
+                "plan_options": {"vertex_order": args.order, "mode_grain": args.grain, "dense_prec": args.dense,
+                                 "fused_split": bool(model.fuse)},
                 "parallelism": f"dp-rows{world}" if world > 1 else "single",
                 "l2": "flushed (256 MiB write) between timed steps",
                 "cuda_graph": use_graph,

@@ -569,46 +569,76 @@ __global__ void __launch_bounds__(NTHREADS, 1)
                 *reinterpret_cast<float4*>(w.out + grow * w.ldo + h + 4 * q) =
                     *reinterpret_cast<const float4*>(sb + rr * 68 + 4 * q);
             }
-            __syncwarp();
-          }
-          if (w.wblk) {
-            // fused split: this warp's 32 rows are one source
-            // window; lane = source k; the same values as the rows just stored,
-            // in the full mode's pre-swizzled window-block image (the layout of
-            // split_window_kernel, so the aggregation reads identical bits)
-            const int64_t win = (m0 >> 5) + (warp & 3);
-            if (win < w.wblk_nwin) {
-              float* blk = w.wblk + win * w.wblk_floats;
-              uint16_t* b16 = reinterpret_cast<uint16_t*>(blk);
-              const int k = lane;
+            if (w.wblk) {
+              // fused split: this warp's 32 rows are one source
+              // window and the smem tile holds them transposed-ready: lane l
+              // takes features h+l and h+32+l, reads the 32 sources of each
+              // from a column of the tile, and writes them in the full mode's
+              // pre-swizzled window-block image — the bits split_window_kernel
+              // would write, so the aggregation sees identical input
+              const int64_t win = (m0 >> 5) + (warp & 3);
+              if (win < w.wblk_nwin) {
+                float* blk = w.wblk + win * w.wblk_floats;
 #pragma unroll
-              for (int f = 0; f < (NPC > 0 ? NPC : 1); ++f) {
-                if (f >= npad) break;
-                const float v = f < w.ncols ? racc[f] * mk(f) : 0.f;
-                if (w.wmode == 3) {
-                  const uint32_t u0 = __float_as_uint(v);
-                  const uint32_t h0 = (u0 + 0x7fffu + ((u0 >> 16) & 1u)) & 0xffff0000u;
-                  const float r1 = v - __uint_as_float(h0);
-                  const uint32_t u1 = __float_as_uint(r1);
-                  const uint32_t h1 = (u1 + 0x7fffu + ((u1 >> 16) & 1u)) & 0xffff0000u;
-                  const uint32_t u2 = __float_as_uint(r1 - __uint_as_float(h1));
-                  const uint32_t h2 = (u2 + 0x7fffu + ((u2 >> 16) & 1u)) & 0xffff0000u;
-                  const int pos = f * 32 + ((((k >> 3) ^ ((f >> 1) & 3)) << 3) | (k & 7));
-                  b16[pos] = uint16_t(h0 >> 16);
-                  b16[npad * 32 + pos] = uint16_t(h1 >> 16);
-                  b16[2 * npad * 32 + pos] = uint16_t(h2 >> 16);
-                } else if (w.wmode == 1) {
-                  const float h = __uint_as_float(__float_as_uint(v) & 0xffffe000u);
-                  const int rh = f, rl = npad + f;
-                  blk[rh * 32 + ((((k >> 2) ^ (rh & 7)) << 2) | (k & 3))] = h;
-                  blk[rl * 32 + ((((k >> 2) ^ (rl & 7)) << 2) | (k & 3))] = v - h;
-                } else {
-                  const uint32_t u = __float_as_uint(v);
-                  blk[f * 32 + ((((k >> 2) ^ (f & 7)) << 2) | (k & 3))] =
-                      __uint_as_float((u + 0x7fffu + ((u >> 16) & 1u)) & 0xffff0000u);
+                for (int fh = 0; fh < 64; fh += 32) {
+                  const int f = h + fh + lane;
+                  if (f >= npad) continue;
+                  if (w.wmode == 3) {
+                    uint16_t* b16 = reinterpret_cast<uint16_t*>(blk);
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) {  // sources 8j..8j+7: one 16-byte chunk per part
+                      uint32_t p0[4], p1[4], p2[4];
+#pragma unroll
+                      for (int e = 0; e < 8; e += 2) {
+                        uint32_t hh[2][3];
+#pragma unroll
+                        for (int t = 0; t < 2; ++t) {
+                          const float v = sb[(8 * j + e + t) * 68 + fh + lane];
+                          const uint32_t u0 = __float_as_uint(v);
+                          const uint32_t h0 = (u0 + 0x7fffu + ((u0 >> 16) & 1u)) & 0xffff0000u;
+                          const float r1 = v - __uint_as_float(h0);
+                          const uint32_t u1 = __float_as_uint(r1);
+                          const uint32_t h1 = (u1 + 0x7fffu + ((u1 >> 16) & 1u)) & 0xffff0000u;
+                          const uint32_t u2 = __float_as_uint(r1 - __uint_as_float(h1));
+                          hh[t][0] = h0 >> 16;
+                          hh[t][1] = h1 >> 16;
+                          hh[t][2] = ((u2 + 0x7fffu + ((u2 >> 16) & 1u)) & 0xffff0000u) >> 16;
+                        }
+                        p0[e / 2] = hh[0][0] | (hh[1][0] << 16);
+                        p1[e / 2] = hh[0][1] | (hh[1][1] << 16);
+                        p2[e / 2] = hh[0][2] | (hh[1][2] << 16);
+                      }
+                      const int pos = f * 32 + ((j ^ ((f >> 1) & 3)) << 3);
+                      *reinterpret_cast<uint4*>(b16 + pos) = make_uint4(p0[0], p0[1], p0[2], p0[3]);
+                      *reinterpret_cast<uint4*>(b16 + npad * 32 + pos) = make_uint4(p1[0], p1[1], p1[2], p1[3]);
+                      *reinterpret_cast<uint4*>(b16 + 2 * npad * 32 + pos) = make_uint4(p2[0], p2[1], p2[2], p2[3]);
+                    }
+                  } else {
+#pragma unroll
+                    for (int j = 0; j < 8; ++j) {  // sources 4j..4j+3: one 16-byte chunk
+                      float4 hv, lv;
+                      float* hp = &hv.x;
+                      float* lp = &lv.x;
+#pragma unroll
+                      for (int e = 0; e < 4; ++e) {
+                        const float v = sb[(4 * j + e) * 68 + fh + lane];
+                        if (w.wmode == 1) {
+                          hp[e] = __uint_as_float(__float_as_uint(v) & 0xffffe000u);
+                          lp[e] = v - hp[e];
+                        } else {
+                          const uint32_t u = __float_as_uint(v);
+                          hp[e] = __uint_as_float((u + 0x7fffu + ((u >> 16) & 1u)) & 0xffff0000u);
+                        }
+                      }
+                      const int rh = f, rl = npad + f;
+                      *reinterpret_cast<float4*>(blk + rh * 32 + ((j ^ (rh & 7)) << 2)) = hv;
+                      if (w.wmode == 1) *reinterpret_cast<float4*>(blk + rl * 32 + ((j ^ (rl & 7)) << 2)) = lv;
+                    }
+                  }
                 }
               }
             }
+            __syncwarp();
           }
         } else if (NPC > 0) {
 #pragma unroll
