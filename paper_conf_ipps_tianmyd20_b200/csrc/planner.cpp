@@ -307,7 +307,7 @@ pcgcn_status build_host_plan(const pcgcn_csr* A, int32_t P, float theta, const p
   parallel_for(P, [&](int, int64_t a, int64_t b) {
     std::vector<uint8_t> dense_i(P, 0);
     std::vector<int64_t> blk_pos(P, -1);
-    std::vector<std::pair<int32_t, int32_t>> ent;  // (col0, (rr<<5)|bit)
+    std::vector<int32_t> wcnt((n + TILE_K - 1) / TILE_K, 0), wslot((n + TILE_K - 1) / TILE_K, -1), touched;
     for (int64_t k = a; k < b; ++k) {
       bool any_dense = tile_grain;
       for (int64_t j = bptr[k]; j < bptr[k + 1]; ++j) {
@@ -326,40 +326,49 @@ pcgcn_status build_host_plan(const pcgcn_csr* A, int32_t P, float theta, const p
       }
       if (any_dense) {
         for (int64_t r0 = p->pstart[k]; r0 < p->pstart[k + 1]; r0 += TILE_M) {
-          int64_t r1 = std::min<int64_t>(r0 + TILE_M, p->pstart[k + 1]);
-          ent.clear();
+          const int64_t r1 = std::min<int64_t>(r0 + TILE_M, p->pstart[k + 1]);
+          // count the candidate edges per 32-source window (dense per-thread
+          // counters over the n/32 windows; only the touched ones are reset)
+          touched.clear();
           for (int64_t v = r0; v < r1; ++v)
             for (int64_t e = tptr[v]; e < tptr[v + 1]; ++e) {
-              int32_t j = tcol[e];
+              const int32_t j = tcol[e];
               if (!tile_grain && !dense_i[pid[j]]) continue;
-              int64_t c0 = (int64_t(j) / TILE_K) * TILE_K;
-              ent.push_back({int32_t(c0), int32_t(((v - r0) << 5) | (j - c0))});
+              const int32_t wv = j / TILE_K;
+              if (wcnt[wv]++ == 0) touched.push_back(wv);
             }
-          if (ent.empty()) continue;
-          std::sort(ent.begin(), ent.end());
+          if (touched.empty()) continue;
+          std::sort(touched.begin(), touched.end());
           TileOut T;
           T.row0 = int32_t(r0);
           T.nrows = int32_t(r1 - r0);
-          for (size_t q = 0; q < ent.size();) {
-            const int32_t c0 = ent[q].first;
-            size_t q1 = q;
-            while (q1 < ent.size() && ent[q1].first == c0) ++q1;
-            if (tile_grain && !(double(q1 - q) / (double(r1 - r0) * win_cols(c0)) > th)) {
-              q = q1;  // a selective chunk: its edges stay in the merged CSR
-              continue;
+          for (int32_t wv : touched) {
+            const int64_t c0 = int64_t(wv) * TILE_K;
+            // block grain: every window of a full-mode block is a chunk; tile
+            // grain: the chunk's own density decides (a selective chunk's edges
+            // stay in the merged CSR)
+            if (!tile_grain || double(wcnt[wv]) / (double(r1 - r0) * win_cols(c0)) > th) {
+              wslot[wv] = int32_t(T.col0.size());
+              T.col0.push_back(int32_t(c0));
             }
-            size_t base = T.bits.size();
-            T.col0.push_back(c0);
-            T.bits.resize(base + TILE_M, 0u);
-            for (; q < q1; ++q) {
-              const int32_t rr = ent[q].second >> 5, bit = ent[q].second & 31;
-              T.bits[base + rr] |= 1u << bit;
-              if (tile_grain) {
-                sp_cnt[r0 + rr]--;
-                p->blk_dense[blk_pos[pid[c0 + bit]]] = 1;  // block holds full-mode edges
-              }
-            }
+            wcnt[wv] = 0;
           }
+          T.bits.assign(T.col0.size() * TILE_M, 0u);
+          if (!T.col0.empty()) {
+            for (int64_t v = r0; v < r1; ++v)
+              for (int64_t e = tptr[v]; e < tptr[v + 1]; ++e) {
+                const int32_t j = tcol[e];
+                const int32_t sl = wslot[j / TILE_K];
+                if (sl < 0 || (!tile_grain && !dense_i[pid[j]])) continue;
+                const int32_t bit = j % TILE_K;
+                T.bits[size_t(sl) * TILE_M + size_t(v - r0)] |= 1u << bit;
+                if (tile_grain) {
+                  sp_cnt[v]--;
+                  p->blk_dense[blk_pos[pid[j]]] = 1;  // block holds full-mode edges
+                }
+              }
+          }
+          for (int32_t wv : touched) wslot[wv] = -1;
           if (!T.col0.empty()) tiles[k].push_back(std::move(T));
         }
       }
