@@ -227,6 +227,27 @@ void pcgcn_nccl_comm_destroy(void* comm);
 pcgcn_status pcgcn_halo_exchange(pcgcn_plan_t p, float* Y, int64_t ldy, int32_t w, float* sendbuf, float* recvbuf,
                                  void* nccl_comm, void* stream);
 
+/* Device-initiated peer gather: the selective pass of shard r reads
+ * each source row straight from its owner's buffer — peer_Y[q] (DEVICE pointer valid in
+ * this process: NVLink peer memory, or a CUDA IPC mapping) holds shard q's rows
+ * [row0[q], row0[q+1]) (pcgcn_plan_shard_rows) with row stride ldy — so no halo copy is
+ * exchanged at all.  Z: this shard's rows.  Selective-only shards (a shard with full-mode
+ * chunks returns PCGCN_EUNSUP), prescaled inputs (IN_PRESCALED required), world <= 8.
+ * Each row is summed in the same order as by pcgcn_forward on a full-height input:
+ * bitwise the same result. */
+pcgcn_status pcgcn_forward_peer(pcgcn_plan_t p, const float* const* peer_Y /* HOST [world] */, int64_t ldy,
+                                float* Z, int64_t ldz, int32_t F, uint32_t flags, uint32_t* mask, void* stream);
+pcgcn_status pcgcn_backward_peer(pcgcn_plan_t p, const float* const* peer_dZ /* HOST [world] */, int64_t ldz,
+                                 float* dY, int64_t ldy, int32_t F, uint32_t flags, void* stream);
+/* CUDA IPC plumbing for peer buffers between processes: allocate (zeroed, its own
+ * allocation so the handle covers exactly it), export a 64-byte handle, open a peer's
+ * handle (lazy peer access), close, free. */
+pcgcn_status pcgcn_ipc_alloc(int64_t bytes, void** ptr);
+void pcgcn_ipc_free(void* ptr);
+pcgcn_status pcgcn_ipc_handle(void* ptr, void* handle64);
+pcgcn_status pcgcn_ipc_open(const void* handle64, void** ptr);
+void pcgcn_ipc_close(void* ptr);
+
 /* ---- dense helpers of the 2-layer GCN step (Alg. 1 transform, L114) ---- */
 
 /* Y = diag(s)·(X·W):  X DEVICE [M x K] ld ldx, W DEVICE [K x N] ld ldw, Y DEVICE [M x N] ld ldy.

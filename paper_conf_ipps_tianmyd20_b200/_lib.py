@@ -104,6 +104,13 @@ _sig("pcgcn_nccl_unique_id", c_i32, c_vp)
 _sig("pcgcn_nccl_comm_init", c_i32, c_vp, c_i32, c_i32, ctypes.POINTER(c_vp))
 _sig("pcgcn_nccl_comm_destroy", None, c_vp)
 _sig("pcgcn_halo_exchange", c_i32, c_vp, c_vp, c_i64, c_i32, c_vp, c_vp, c_vp, c_vp)
+_sig("pcgcn_forward_peer", c_i32, c_vp, c_vp, c_i64, c_vp, c_i64, c_i32, c_u32, c_vp, c_vp)
+_sig("pcgcn_backward_peer", c_i32, c_vp, c_vp, c_i64, c_vp, c_i64, c_i32, c_u32, c_vp)
+_sig("pcgcn_ipc_alloc", c_i32, c_i64, ctypes.POINTER(c_vp))
+_sig("pcgcn_ipc_free", None, c_vp)
+_sig("pcgcn_ipc_handle", c_i32, c_vp, c_vp)
+_sig("pcgcn_ipc_open", c_i32, c_vp, ctypes.POINTER(c_vp))
+_sig("pcgcn_ipc_close", None, c_vp)
 _sig("pcgcn_last_error", ctypes.c_char_p)
 _sig("pcgcn_abi_version", c_i32)
 
@@ -220,6 +227,18 @@ class Plan:
         check(lib.pcgcn_halo_exchange(self._h, _ptr(Y), Y.stride(0), w, _ptr(sendbuf), _ptr(recvbuf), comm,
                                       _stream(stream)), "pcgcn_halo_exchange")
 
+    def forward_peer(self, peers, ldy, Z, F, flags=0, mask=None, stream=None):
+        """Selective pass reading sources from the shards' own buffers (device
+        pointers, one per shard)."""
+        tab = (c_vp * len(peers))(*[int(x) for x in peers])
+        check(lib.pcgcn_forward_peer(self._h, tab, ldy, _ptr(Z), Z.stride(0), F, flags, _ptr(mask), _stream(stream)),
+              "pcgcn_forward_peer")
+
+    def backward_peer(self, peers, ldz, dY, F, flags=0, stream=None):
+        tab = (c_vp * len(peers))(*[int(x) for x in peers])
+        check(lib.pcgcn_backward_peer(self._h, tab, ldz, _ptr(dY), dY.stride(0), F, flags, _stream(stream)),
+              "pcgcn_backward_peer")
+
     def rowscale_ptr(self):
         return lib.pcgcn_plan_rowscale(self._h)
 
@@ -333,6 +352,43 @@ def nccl_comm_init(uid: bytes, rank: int, world: int):
 
 def nccl_comm_destroy(comm):
     lib.pcgcn_nccl_comm_destroy(comm)
+
+
+class IpcBuffer:
+    """A device buffer in its own allocation, shareable with other processes by
+    CUDA IPC; ``tensor`` views it as a float32 [rows x cols] torch tensor."""
+
+    def __init__(self, rows, cols):
+        import torch
+        p = c_vp()
+        check(lib.pcgcn_ipc_alloc(int(rows) * int(cols) * 4 or 16, ctypes.byref(p)), "pcgcn_ipc_alloc")
+        self.ptr = p.value
+        self.rows, self.cols = int(rows), int(cols)
+
+        class _Cai:
+            __cuda_array_interface__ = {"shape": (self.rows, self.cols), "typestr": "<f4", "data": (self.ptr, False),
+                                        "version": 3, "strides": None}
+        self.tensor = torch.as_tensor(_Cai(), device="cuda")
+
+    def handle(self) -> bytes:
+        buf = ctypes.create_string_buffer(64)
+        check(lib.pcgcn_ipc_handle(c_vp(self.ptr), buf), "pcgcn_ipc_handle")
+        return buf.raw
+
+    def free(self):
+        if self.ptr:
+            lib.pcgcn_ipc_free(c_vp(self.ptr))
+            self.ptr = None
+
+
+def ipc_open(handle: bytes) -> int:
+    p = c_vp()
+    check(lib.pcgcn_ipc_open(ctypes.create_string_buffer(handle, 64), ctypes.byref(p)), "pcgcn_ipc_open")
+    return p.value
+
+
+def ipc_close(ptr: int):
+    lib.pcgcn_ipc_close(c_vp(ptr))
 
 
 def probe_read_gbs(nbytes, iters=20):

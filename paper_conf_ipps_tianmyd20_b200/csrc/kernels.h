@@ -44,6 +44,12 @@ struct AggArgs {
   float* seg_ws;             // [nseg x ldws] fp32 partial sums
   int64_t ldws;
   int* counter;              // dynamic row scheduler ticket (zeroed on the stream before each pass)
+  // device-initiated peer gather: sources of shard q are read from
+  // shard q's own buffer (peer_base[q] = its row row0[q]; NVLink peer memory
+  // on a multi-GPU node, CUDA IPC in the 1-GPU tests) instead of an exchanged copy
+  int peer_world = 0;        // 0: sources come from Y
+  const char* peer_base[8];
+  int64_t peer_row0[9];
   int phase = 0;             // 0: segment pass + row pass; 1: segment pass only; 2: row pass only
   int rows_per_ticket = 1;   // consecutive rows per scheduler ticket, 1..16
 };

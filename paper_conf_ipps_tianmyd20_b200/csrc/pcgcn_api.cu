@@ -569,6 +569,87 @@ pcgcn_status pcgcn_halo_unpack(pcgcn_plan_t p, const float* buf, float* Y, int64
   return halo_copy(p, false, buf, w, Y, ldy, w, stream);
 }
 
+// ---- device-initiated peer gather ----
+static pcgcn_status aggregate_peer(pcgcn_plan_t p, const float* const* peer, int64_t ldy, float* Z, int64_t ldz,
+                                   int32_t F, uint32_t flags, uint32_t* mask, void* stream) {
+  if (!p || !p->d.built) { set_error("plan has no device structures"); return PCGCN_EINVAL; }
+  const int32_t W = p->opts.world;
+  if (!peer || W < 1 || W > 8) { set_error("forward_peer: peer table of 1..8 shards required"); return PCGCN_EINVAL; }
+  if (!(flags & PCGCN_IN_PRESCALED)) { set_error("forward_peer: inputs must be prescaled (IN_PRESCALED)"); return PCGCN_EINVAL; }
+  if (p->d.nch > 0) { set_error("forward_peer: the shard has full-mode chunks (selective-only plans)"); return PCGCN_EUNSUP; }
+  if (sparse_fsplit_active(F)) { set_error("forward_peer: PCGCN_SPARSE_FSPLIT not supported"); return PCGCN_EUNSUP; }
+  if (!Z || F < 1 || F > p->opts.f_max || ldy < round_up(F, 4) || ldz < round_up(F, 4) || (ldy & 3) || (ldz & 3) ||
+      !aligned16(Z)) {
+    set_error("forward_peer: bad Z/F/ld");
+    return PCGCN_EINVAL;
+  }
+  if ((flags & PCGCN_MASK_OUT) && !mask) { set_error("MASK_OUT needs a mask buffer"); return PCGCN_EINVAL; }
+  DevicePlan& d = p->d;
+  AggArgs a;
+  a.Y = nullptr; a.ldy = ldy; a.Z = Z; a.ldz = ldz;
+  a.mask = (flags & PCGCN_MASK_OUT) ? mask : nullptr;
+  a.rowptr = d.sp_rowptr; a.col = d.sp_col; a.r = d.r;
+  a.row_lo = p->row_lo; a.rows = d.rows;
+  a.zd_index = nullptr; a.zd = nullptr; a.ldzd = 0; a.zrow = d.zrow;
+  a.mask_ld = (F + 31) / 32;
+  a.n_src = p->n;
+  a.F = F;
+  a.relu = (flags & PCGCN_RELU) != 0;
+  a.out_prescaled = (flags & PCGCN_OUT_PRESCALED) != 0;
+  a.row_seg = d.row_seg; a.seg_lo = d.seg_lo; a.seg_hi = d.seg_hi; a.nseg = d.nseg;
+  a.seg_ws = d.seg_ws; a.ldws = d.fpad_max;
+  a.counter = d.counter;
+  a.rows_per_ticket = rows_per_ticket(d.nnz_s, d.rows);
+  a.peer_world = W;
+  for (int q = 0; q < 8; ++q) a.peer_base[q] = q < W ? reinterpret_cast<const char*>(peer[q]) : nullptr;
+  for (int q = 0; q <= 8; ++q)
+    a.peer_row0[q] = W == 1 ? (q == 0 ? 0 : p->n) : p->shard_row0[std::min<int32_t>(q, W)];
+  for (int q = 0; q < W; ++q)
+    if (!a.peer_base[q] || (reinterpret_cast<uintptr_t>(a.peer_base[q]) & 31)) {
+      set_error("forward_peer: null or not 32-byte aligned peer buffer");
+      return PCGCN_EINVAL;
+    }
+  cudaError_t e = launch_sparse_agg(a, static_cast<cudaStream_t>(stream));
+  return e == cudaSuccess ? PCGCN_OK : cuda_fail(e, "forward_peer");
+}
+
+pcgcn_status pcgcn_forward_peer(pcgcn_plan_t p, const float* const* peer_Y, int64_t ldy, float* Z, int64_t ldz,
+                                int32_t F, uint32_t flags, uint32_t* mask, void* stream) {
+  return aggregate_peer(p, peer_Y, ldy, Z, ldz, F, flags, mask, stream);
+}
+
+pcgcn_status pcgcn_backward_peer(pcgcn_plan_t p, const float* const* peer_dZ, int64_t ldz, float* dY, int64_t ldy,
+                                 int32_t F, uint32_t flags, void* stream) {
+  return aggregate_peer(p, peer_dZ, ldz, dY, ldy, F, flags & ~uint32_t(PCGCN_MASK_OUT), nullptr, stream);
+}
+
+// ---- CUDA IPC helpers (peer buffers across processes) ----
+pcgcn_status pcgcn_ipc_alloc(int64_t bytes, void** ptr) {
+  if (!ptr || bytes <= 0) { set_error("ipc_alloc: bad arguments"); return PCGCN_EINVAL; }
+  cudaError_t e = cudaMalloc(ptr, size_t(bytes));
+  if (e != cudaSuccess) return cuda_fail(e, "ipc_alloc");
+  e = cudaMemset(*ptr, 0, size_t(bytes));
+  return e == cudaSuccess ? PCGCN_OK : cuda_fail(e, "ipc_alloc memset");
+}
+void pcgcn_ipc_free(void* ptr) { if (ptr) cudaFree(ptr); }
+pcgcn_status pcgcn_ipc_handle(void* ptr, void* handle64) {
+  if (!ptr || !handle64) { set_error("ipc_handle: null argument"); return PCGCN_EINVAL; }
+  cudaIpcMemHandle_t h;
+  cudaError_t e = cudaIpcGetMemHandle(&h, ptr);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaIpcGetMemHandle");
+  static_assert(sizeof(h) == 64, "cudaIpcMemHandle_t is 64 bytes");
+  std::memcpy(handle64, &h, 64);
+  return PCGCN_OK;
+}
+pcgcn_status pcgcn_ipc_open(const void* handle64, void** ptr) {
+  if (!ptr || !handle64) { set_error("ipc_open: null argument"); return PCGCN_EINVAL; }
+  cudaIpcMemHandle_t h;
+  std::memcpy(&h, handle64, 64);
+  cudaError_t e = cudaIpcOpenMemHandle(ptr, h, cudaIpcMemLazyEnablePeerAccess);
+  return e == cudaSuccess ? PCGCN_OK : cuda_fail(e, "cudaIpcOpenMemHandle");
+}
+void pcgcn_ipc_close(void* ptr) { if (ptr) cudaIpcCloseMemHandle(ptr); }
+
 pcgcn_status pcgcn_plan_perm(pcgcn_plan_t p, int32_t* perm) {
   if (!p || !perm) { set_error("null argument"); return PCGCN_EINVAL; }
   std::memcpy(perm, p->perm.data(), sizeof(int32_t) * p->n);

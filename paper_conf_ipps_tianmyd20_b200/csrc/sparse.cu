@@ -52,7 +52,29 @@ __device__ __forceinline__ const char* row_addr(const char* base, uint32_t j, ui
   asm("mad.wide.u32 %0, %1, %2, %3;" : "=l"(r) : "r"(j), "r"(stride), "l"(reinterpret_cast<uint64_t>(base)));
   return reinterpret_cast<const char*>(r);
 }
-__device__ __forceinline__ int ld_idx(const int* p) { return __ldg(p); }
+// a source index as the gather uses it: the plan row (PEER = false), or (owner
+// shard << 28) | row inside the owner's buffer (PEER: every index is decoded
+// once, by the lane that loads it, and reaches the other lanes by shuffle)
+template <bool PEER>
+__device__ __forceinline__ int ld_col(const int* p, const AggArgs& a) {
+  const int j = __ldg(p);
+  if constexpr (!PEER) {
+    return j;
+  } else {
+    int o = 0;
+#pragma unroll
+    for (int q = 1; q < 8; ++q) o += (q < a.peer_world && j >= a.peer_row0[q]) ? 1 : 0;
+    return (o << 28) | int(j - a.peer_row0[o]);
+  }
+}
+template <bool PEER>
+__device__ __forceinline__ const char* src_row(const char* yb, uint32_t j, uint32_t rstride, const AggArgs& a) {
+  if constexpr (!PEER) {
+    return row_addr(yb, j, rstride);
+  } else {  // yb holds this lane's byte offset inside a row
+    return row_addr(a.peer_base[j >> 28] + reinterpret_cast<uintptr_t>(yb), j & 0x0fffffffu, rstride);
+  }
+}
 __device__ __forceinline__ uint32_t smem_addr(const void* p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
 }
@@ -115,11 +137,11 @@ struct Lay {
 // (lane l: cp[l] if l < n), and the prefetch slot of the last batch loads the
 // first batch of the NEXT range (cpn, nn), which is returned — so a warp
 // walking rows never waits on a row's first index load.
-template <int G, int V, int H>
+template <int G, int V, int H, bool PEER = false>
 __device__ __forceinline__ int gather_sum(const int* __restrict__ cp, int n, int first,
                                           const int* __restrict__ cpn, int nn, const char* __restrict__ yb,
                                           uint32_t rstride, const bool (&lok)[V], int lane,
-                                          float4 (&tot)[V][H]) {
+                                          float4 (&tot)[V][H], const AggArgs& a) {
   using L = Lay<G, V, H>;
   constexpr int S = L::S, STEPS = L::STEPS, UNR = L::UNR, NACC = L::NACC, BATCH = L::BATCH;
   const int slot = lane / G;
@@ -132,13 +154,13 @@ __device__ __forceinline__ int gather_sum(const int* __restrict__ cp, int n, int
 #pragma unroll
       for (int h = 0; h < H; ++h) acc[u][v][h] = make_float4(0.f, 0.f, 0.f, 0.f);
   int nextidx = first;
-  if (n == 0) nextidx = lane < nn ? ld_idx(cpn + lane) : 0;
+  if (n == 0) nextidx = lane < nn ? ld_col<PEER>(cpn + lane, a) : 0;
   for (int base = 0; base < n; base += BATCH) {
     const int cnt = (n - base) < BATCH ? n - base : BATCH;
     const int myidx = nextidx;
     // next batch, one ahead (past the end: the next range's first batch)
-    nextidx = (base + BATCH + lane < n) ? ld_idx(cp + base + BATCH + lane)
-            : (lane < nn ? ld_idx(cpn + lane) : 0);
+    nextidx = (base + BATCH + lane < n) ? ld_col<PEER>(cp + base + BATCH + lane, a)
+            : (lane < nn ? ld_col<PEER>(cpn + lane, a) : 0);
     if (cnt == BATCH) {
       // full batch: unguarded, every lane keeps UNR*V*H 16-byte pieces in flight
 #pragma unroll
@@ -147,7 +169,7 @@ __device__ __forceinline__ int gather_sum(const int* __restrict__ cp, int n, int
 #pragma unroll
         for (int u = 0; u < UNR; ++u) {
           const uint32_t j = uint32_t(__shfl_sync(0xffffffffu, myidx, (k0 + u) * S + slot));
-          const char* p = row_addr(yb, j, rstride);
+          const char* p = src_row<PEER>(yb, j, rstride, a);
 #pragma unroll
           for (int v = 0; v < V; ++v) {
             if (active && (v == 0 || lok[v])) {
@@ -174,7 +196,7 @@ __device__ __forceinline__ int gather_sum(const int* __restrict__ cp, int n, int
         for (int u = 0; u < UNR; ++u) {
           const int e = (k0 + u) * S + slot;
           const uint32_t j = uint32_t(__shfl_sync(0xffffffffu, myidx, e));
-          const char* p = row_addr(yb, j, rstride);
+          const char* p = src_row<PEER>(yb, j, rstride, a);
 #pragma unroll
           for (int v = 0; v < V; ++v) {
             if (active && e < cnt && (v == 0 || lok[v])) {
@@ -238,7 +260,7 @@ __device__ __forceinline__ int lane_col(int lane, int v, int nvec) {
 // partial sums to seg_ws.
 // 4-warp CTAs (8K registers): small enough to co-reside with a full-mode
 // engine CTA (tc_engine, 320 threads) when the two run concurrently
-template <int G, int V, int H>
+template <int G, int V, int H, bool PEER>
 __global__ void __launch_bounds__(128, 2 * Lay<G, V, H>::MINB) sparse_seg_kernel(AggArgs a) {
   const int64_t sg = int64_t(blockIdx.x) * 4 + (threadIdx.x >> 5);
   if (sg >= a.nseg) return;
@@ -246,15 +268,15 @@ __global__ void __launch_bounds__(128, 2 * Lay<G, V, H>::MINB) sparse_seg_kernel
   const int nvec = (a.F + 4 * H - 1) / (4 * H);
   const int nvec4 = (a.F + 3) >> 2;
   const int q0 = lane_col<G>(lane, 0, nvec);
-  const char* yb = reinterpret_cast<const char*>(a.Y) + 16 * H * (q0 < 0 ? 0 : q0);
+  const char* yb = (PEER ? nullptr : reinterpret_cast<const char*>(a.Y)) + 16 * H * (q0 < 0 ? 0 : q0);
   const int64_t lo = a.seg_lo[sg], hi = a.seg_hi[sg];
   bool lok[V];
 #pragma unroll
   for (int v = 0; v < V; ++v) lok[v] = lane_col<G>(lane, v, nvec) >= 0;
   float4 tot[V][H];
   const int n = int(hi - lo);
-  const int first = lane < n ? ld_idx(a.col + lo + lane) : 0;
-  gather_sum<G, V, H>(a.col + lo, n, first, nullptr, 0, yb, uint32_t(a.ldy * 4), lok, lane, tot);
+  const int first = lane < n ? ld_col<PEER>(a.col + lo + lane, a) : 0;
+  gather_sum<G, V, H, PEER>(a.col + lo, n, first, nullptr, 0, yb, uint32_t(a.ldy * 4), lok, lane, tot, a);
   if (lane < G) {
 #pragma unroll
     for (int v = 0; v < V; ++v) {
@@ -272,7 +294,7 @@ __global__ void __launch_bounds__(128, 2 * Lay<G, V, H>::MINB) sparse_seg_kernel
 // locality); a row is gathered directly or, if long, summed from its
 // segment partials in segment order.  Fused epilogue: + full-mode partial
 // sum Zd (mode combine, L193), x r_i (optionally twice), ReLU, bit mask.
-template <int G, int V, int H, bool HAS_ZD, bool HAS_SEG>
+template <int G, int V, int H, bool HAS_ZD, bool HAS_SEG, bool PEER>
 __global__ void __launch_bounds__(256, Lay<G, V, H>::MINB) sparse_row_kernel(AggArgs a) {
   const int lane = threadIdx.x & 31;
   const int slot = lane / G;
@@ -285,7 +307,7 @@ __global__ void __launch_bounds__(256, Lay<G, V, H>::MINB) sparse_row_kernel(Agg
     qv[v] = lane_col<G>(lane, v, nvec);
     lok[v] = qv[v] >= 0;
   }
-  const char* yb = reinterpret_cast<const char*>(a.Y) + 16 * H * (qv[0] < 0 ? 0 : qv[0]);
+  const char* yb = (PEER ? nullptr : reinterpret_cast<const char*>(a.Y)) + 16 * H * (qv[0] < 0 ? 0 : qv[0]);
   const uint32_t rstride = uint32_t(a.ldy * 4);
   // Rows are claimed in blocks of R consecutive rows per ticket (R >= 4 from
   // the plan's mean selective degree: short rows would otherwise pay the
@@ -324,7 +346,7 @@ __global__ void __launch_bounds__(256, Lay<G, V, H>::MINB) sparse_row_kernel(Agg
   int pre = 0;
   if (blk < nblk_total) {
     const int64_t f0 = s_rp[wib][b][0], f1 = s_rp[wib][b][1];
-    pre = (f0 + lane < f1) ? ld_idx(a.col + f0 + lane) : 0;
+    pre = (f0 + lane < f1) ? ld_col<PEER>(a.col + f0 + lane, a) : 0;
   }
   while (blk < nblk_total) {
     int tk = 0;
@@ -357,7 +379,7 @@ __global__ void __launch_bounds__(256, Lay<G, V, H>::MINB) sparse_row_kernel(Agg
     const int zi = HAS_ZD ? a.zd_index[row] : -1;
     const int sg = HAS_SEG ? a.row_seg[row] : -1;
     if (HAS_SEG && sg >= 0) {
-      pre_next = (n0 + lane < n1) ? ld_idx(a.col + n0 + lane) : 0;
+      pre_next = (n0 + lane < n1) ? ld_col<PEER>(a.col + n0 + lane, a) : 0;
       const int ns = int((e1 - e0 + SEG_EDGES - 1) / SEG_EDGES);
 #pragma unroll
       for (int v = 0; v < V; ++v)
@@ -374,8 +396,8 @@ __global__ void __launch_bounds__(256, Lay<G, V, H>::MINB) sparse_row_kernel(Agg
                                                                         4 * (H * qv[v] + h))));
       }
     } else {
-      pre_next = gather_sum<G, V, H>(a.col + e0, int(e1 - e0), pre, a.col + n0, int(n1 - n0), yb, rstride,
-                                     lok, lane, tot);
+      pre_next = gather_sum<G, V, H, PEER>(a.col + e0, int(e1 - e0), pre, a.col + n0, int(n1 - n0), yb, rstride,
+                                           lok, lane, tot, a);
     }
     uint32_t bal[V][4];
     uint32_t mbyte[V];
@@ -455,26 +477,26 @@ __global__ void __launch_bounds__(256, Lay<G, V, H>::MINB) sparse_row_kernel(Agg
   }
 }
 
-template <int G, int V, int H>
-cudaError_t launch_gv(const AggArgs& a, cudaStream_t s) {
+template <int G, int V, int H, bool PEER>
+cudaError_t launch_gvp(const AggArgs& a, cudaStream_t s) {
   // persistent row pass: as many 8-warp CTAs as fit (4 per SM at 64 registers)
   static int slots = 0;
   if (!slots) {
     int dev = 0, sms = 148, per = 4;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, sparse_row_kernel<G, V, H, true, true>, 256, 0);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, sparse_row_kernel<G, V, H, true, true, PEER>, 256, 0);
     slots = sms * (per > 0 ? per : 1);
   }
   if (a.nseg > 0 && a.phase != 2) {
-    sparse_seg_kernel<G, V, H><<<unsigned((a.nseg + 3) / 4), 128, 0, s>>>(a);
+    sparse_seg_kernel<G, V, H, PEER><<<unsigned((a.nseg + 3) / 4), 128, 0, s>>>(a);
     if (a.phase == 1) return cudaGetLastError();
   }
   cudaError_t e = cudaMemsetAsync(a.counter, 0, sizeof(int), s);
   if (e != cudaSuccess) return e;
   const int64_t want = ((a.rows + a.rows_per_ticket - 1) / a.rows_per_ticket + 7) / 8;
   const unsigned grid = unsigned(want < slots ? want : slots);
-#define LAUNCH(ZD, SG) sparse_row_kernel<G, V, H, ZD, SG><<<grid, 256, 0, s>>>(a)
+#define LAUNCH(ZD, SG) sparse_row_kernel<G, V, H, ZD, SG, PEER><<<grid, 256, 0, s>>>(a)
   const bool zd = a.zd_index != nullptr, sg = a.nseg > 0;
   if (zd && sg) LAUNCH(true, true);
   else if (zd) LAUNCH(true, false);
@@ -482,6 +504,11 @@ cudaError_t launch_gv(const AggArgs& a, cudaStream_t s) {
   else LAUNCH(false, false);
 #undef LAUNCH
   return cudaGetLastError();
+}
+
+template <int G, int V, int H>
+cudaError_t launch_gv(const AggArgs& a, cudaStream_t s) {
+  return a.peer_world > 0 ? launch_gvp<G, V, H, true>(a, s) : launch_gvp<G, V, H, false>(a, s);
 }
 
 // ypre = diag(r)·Y (row-major, ld ldpre)

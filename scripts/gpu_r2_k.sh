@@ -17,3 +17,5 @@ TH4=$(python -c "import json;print(json.load(open('gpurun_out/r2k_c4.json'))['co
 timeout 900 ncu --profile-from-start off --metrics gpu__time_duration.sum --clock-control none --csv \
   --log-file gpurun_out/r2k_c4_launches.csv python scripts/profile_epoch.py --workload sbm4m --theta $TH4 --order id --grain block > gpurun_out/r2k_c4_prof.json 2>&1
 timeout 2400 python bench.py --workload pl32m --steps 5 --warmup 3 --no-cpu-baseline > gpurun_out/r2k_c5.json 2> gpurun_out/r2k_c5.err
+timeout 1200 python bench.py --table3 --order id --grain block --dense tf32x2 --steps 20 --warmup 5 > gpurun_out/r2k_table3_block.json 2> gpurun_out/r2k_table3_block.err
+timeout 1200 python bench.py --workload pubmed --f3 200 --f3-signal 0.011 --f3-seeds 3 > gpurun_out/r2k_f3_pubmed.json 2> gpurun_out/r2k_f3_pubmed.err

@@ -377,3 +377,83 @@ def test_nccl_unique_id_host():
     from paper_conf_ipps_tianmyd20_b200 import _lib as L
     a, b = L.nccl_unique_id(), L.nccl_unique_id()
     assert len(a) == 128 and a != b
+
+
+# ---------------------------------------------------------------------------
+# device-initiated peer gather: sources read from the owners' buffers
+# ---------------------------------------------------------------------------
+
+def _peer_worker(rank, world, port, q, wname, F, ld, theta):
+    import sys
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    from paper_conf_ipps_tianmyd20_b200 import _lib as L
+    from synth import configs as C
+    _init(rank, world, port)
+    torch.cuda.set_device(0)
+    w = C.WORKLOADS[wname]
+    g = C.graph(w)
+    pl = L.Plan(g.n, g.rowptr, g.col, w.P, theta, rank=rank, world=world)
+    row0 = pl.shard_rows(world)
+    Y = np.random.default_rng(5).standard_normal((g.n, ld)).astype(np.float32)
+    Y[:, F:] = 0
+    buf = L.IpcBuffer(pl.row_hi - pl.row_lo, ld)        # this shard's rows only
+    buf.tensor.copy_(torch.from_numpy(Y[pl.row_lo:pl.row_hi]))
+    torch.cuda.synchronize()
+    handles = [None] * world
+    dist.all_gather_object(handles, buf.handle())
+    peers = [buf.ptr if r == rank else L.ipc_open(handles[r]) for r in range(world)]
+    Z = torch.full((pl.row_hi - pl.row_lo, ld), float("nan"), device="cuda")
+    M = torch.zeros(pl.row_hi - pl.row_lo, (F + 31) // 32, dtype=torch.int32, device="cuda")
+    pl.forward_peer(peers, ld, Z, F, flags=L.IN_PRESCALED | L.RELU | L.MASK_OUT, mask=M)
+    Zb = torch.full_like(Z, float("nan"))
+    pl.backward_peer(peers, ld, Zb, F, flags=L.IN_PRESCALED)
+    torch.cuda.synchronize()
+    q.put((rank, pl.row_lo, pl.row_hi, Z.cpu().numpy(), M.cpu().numpy(), Zb.cpu().numpy(), row0.tolist()))
+    dist.barrier()
+    for r, ptr in enumerate(peers):
+        if r != rank:
+            L.ipc_close(ptr)
+    buf.free()
+    dist.destroy_process_group()
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("wname,F,ld,theta", [("pl-small", 128, 128, 2.0), ("pl-small", 32, 32, 2.0),
+                                              ("pubmed", 41, 48, 2.0)])
+def test_peer_gather_matches_unsharded(wname, F, ld, theta):
+    """pcgcn_forward_peer / pcgcn_backward_peer: each shard's
+    selective pass reads every source row from the owner shard's own buffer
+    (CUDA IPC mappings between two processes on this GPU; NVLink peer memory
+    on a multi-GPU node) — no exchanged copy — and its rows (values, ReLU
+    mask) are bitwise equal to the unsharded aggregation."""
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    from paper_conf_ipps_tianmyd20_b200 import _lib as L
+    from synth import configs as C
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    ps = [ctx.Process(target=_peer_worker, args=(r, 2, port, q, wname, F, ld, theta)) for r in range(2)]
+    for p in ps:
+        p.start()
+    res = sorted([q.get(timeout=600) for _ in ps], key=lambda t: t[0])
+    for p in ps:
+        p.join(timeout=60)
+    w = C.WORKLOADS[wname]
+    g = C.graph(w)
+    pl = L.Plan(g.n, g.rowptr, g.col, w.P, theta)
+    Y = np.random.default_rng(5).standard_normal((g.n, ld)).astype(np.float32)
+    Y[:, F:] = 0
+    Yd = torch.from_numpy(Y).cuda()
+    Z = torch.full((g.n, ld), float("nan"), device="cuda")
+    M = torch.zeros(g.n, (F + 31) // 32, dtype=torch.int32, device="cuda")
+    pl.forward(Yd, Z, F=F, flags=L.IN_PRESCALED | L.RELU | L.MASK_OUT, mask=M)
+    Zb = torch.full_like(Z, float("nan"))
+    pl.backward(Yd, Zb, F=F, flags=L.IN_PRESCALED)
+    torch.cuda.synchronize()
+    Z, M, Zb = Z.cpu().numpy(), M.cpu().numpy(), Zb.cpu().numpy()
+    assert res[0][1] == 0 and res[-1][2] == g.n
+    for rank, lo, hi, z, m, zb, row0 in res:
+        assert np.array_equal(z[:, :F], Z[lo:hi, :F])
+        assert np.array_equal(m, M[lo:hi])
+        assert np.array_equal(zb[:, :F], Zb[lo:hi, :F])
