@@ -147,3 +147,68 @@ class HaloExchange:
 
     def allreduce(self, t: torch.Tensor):
         dist.all_reduce(t, op=dist.ReduceOp.SUM, group=self.group)
+
+
+class PeerExchange:
+    """Device-initiated peer gather: no rows are copied.
+    Each shard keeps its aggregation inputs (Y0', Y1', dL', dP1') in buffers of
+    its own rows that every other shard maps — NVLink peer memory across the
+    GPUs of a node, CUDA IPC between processes — and the selective pass
+    (pcgcn_forward_peer) reads each source row from its owner.  Before an
+    aggregation the shards only synchronise (every producer must have written
+    its rows): ``gather`` is a barrier.  Selective-only plans (the full mode's
+    window split would need the remote rows)."""
+
+    peer = True
+
+    def __init__(self, plan, group=None):
+        from . import _lib as L
+        self.L = L
+        self.group = group
+        self.world = dist.get_world_size(group)
+        self.rank = dist.get_rank(group)
+        row0 = plan.shard_rows(self.world)
+        self.ranges = [(int(a), int(b)) for a, b in zip(row0[:-1], row0[1:])]
+        check_ranges(self.ranges, plan.n)
+        self._bufs, self._peers, self._opened = {}, {}, []
+        self._flag = torch.zeros(1, device="cuda") if dist.get_backend(group) == "nccl" else torch.zeros(1)
+
+    def local_buffer(self, key, rows, cols):
+        """This shard's buffer for input ``key`` (collective: all ranks call it
+        in the same order); returns the torch view of its rows."""
+        buf = self.L.IpcBuffer(rows, cols)
+        handles = [None] * self.world
+        dist.all_gather_object(handles, buf.handle(), group=self.group)
+        peers = []
+        for q in range(self.world):
+            if q == self.rank:
+                peers.append(buf.ptr)
+            else:
+                ptr = self.L.ipc_open(handles[q])
+                self._opened.append(ptr)
+                peers.append(ptr)
+        self._bufs[key], self._peers[key] = buf, peers
+        return buf.tensor
+
+    def peers(self, key):
+        return self._peers[key]
+
+    def gather(self, full, lo=None, hi=None, plan=None):
+        # the producers of every shard must be done before anyone reads: a
+        # (stream-ordered, for NCCL) all-reduce of one float is the barrier
+        if self._flag.is_cuda:
+            dist.all_reduce(self._flag, group=self.group)
+        else:
+            torch.cuda.synchronize()
+            dist.barrier(group=self.group)
+
+    def allreduce(self, t: torch.Tensor):
+        dist.all_reduce(t, op=dist.ReduceOp.SUM, group=self.group)
+
+    def close(self):
+        dist.barrier(group=self.group)
+        for ptr in self._opened:
+            self.L.ipc_close(ptr)
+        for b in self._bufs.values():
+            b.free()
+        self._opened, self._bufs = [], {}

@@ -93,18 +93,26 @@ class GCN2:
         self.v = torch.zeros_like(self.theta)
         self.step_ctr = torch.zeros(1, dtype=torch.int32, device=d)
         # activations: inputs of aggregations span all n rows (sources), outputs the shard
-        self.Y0 = torch.zeros(n, self.ldH, dtype=f32, device=d)
+        # peer mode (dist.PeerExchange): the aggregation inputs hold only
+        # this shard's rows, in IPC/peer-mapped buffers the other shards read directly
+        self.peer = exchange is not None and getattr(exchange, "peer", False)
+        if self.peer:
+            self.narrow = False
+            self.fuse = False
+        ain = (lambda key, w: exchange.local_buffer(key, rows, w)) if self.peer else \
+            (lambda key, w: torch.zeros(n, w, dtype=f32, device=d))
+        self.Y0 = ain("Y0", self.ldH)
         self.H1 = torch.zeros(rows, self.ldH, dtype=f32, device=d)
         mw = (H + 31) // 32
         # narrow: full-height mask / G1 (exchanged), the local rows are views
         self.mask1_all = torch.zeros(n if self.narrow else rows, mw, dtype=torch.int32, device=d)
         self.mask1 = self.mask1_all[self.lo:self.hi] if self.narrow else self.mask1_all
-        self.Y1 = torch.zeros(n, self.ldC, dtype=f32, device=d)
+        self.Y1 = ain("Y1", self.ldC)
         self.Lg = torch.zeros(rows, self.ldC, dtype=f32, device=d)
-        self.dL = torch.zeros(n, self.ldC, dtype=f32, device=d)
+        self.dL = ain("dL", self.ldC)
         self.G1_all = torch.zeros(n if self.narrow else rows, self.ldC, dtype=f32, device=d)
         self.G1 = self.G1_all[self.lo:self.hi] if self.narrow else self.G1_all
-        self.dP1 = torch.zeros(n, self.ldH, dtype=f32, device=d)
+        self.dP1 = ain("dP1", self.ldH)
         self.G0 = torch.zeros(rows, self.ldH, dtype=f32, device=d)
         self.loss = torch.zeros(1, dtype=f32, device=d)
         self.ce_work = torch.zeros(L.CE_WORK_FLOATS, dtype=f32, device=d)
@@ -125,11 +133,25 @@ class GCN2:
         return ctypes.c_void_p(self.r + 4 * self.lo) if self.lo else ctypes.c_void_p(self.r)
 
     def _local(self, full):
-        return full[self.lo:self.hi]
+        return full if self.peer else full[self.lo:self.hi]
 
     def _gather(self, full, plan):
         if self.exchange is not None:
             self.exchange.gather(full, self.lo, self.hi, plan=plan)
+
+    def _agg(self, plan, key, Y, Z, F, flags, mask=None, backward=False, stream=None):
+        """One aggregation: from the full-height input, or (peer mode) from every
+        shard's own buffer through the peer table."""
+        if self.peer:
+            peers, ld = self.exchange.peers(key), Y.shape[1]
+            if backward:
+                plan.backward_peer(peers, ld, Z, F, flags=flags, stream=stream)
+            else:
+                plan.forward_peer(peers, ld, Z, F, flags=flags, mask=mask, stream=stream)
+        elif backward:
+            plan.backward(Y, Z, F=F, flags=flags, stream=stream)
+        else:
+            plan.forward(Y, Z, F=F, flags=flags, mask=mask, stream=stream)
 
     def epoch(self, stream=None, hook=None, agg_flags=0):
         """One epoch; ``hook(name)`` (optional) is called after every step so a
@@ -152,7 +174,7 @@ class GCN2:
             self._gather(self.Y0, p)
         mark("x_gather_y0")
         sf = L.IN_SPLIT if self.fuse else 0
-        p.forward(self.Y0, self.H1, F=H, flags=L.IN_PRESCALED | L.RELU | L.MASK_OUT | sf | agg_flags, mask=self.mask1,
+        self._agg(p, "Y0", self.Y0, self.H1, H, L.IN_PRESCALED | L.RELU | L.MASK_OUT | sf | agg_flags, mask=self.mask1,
                   stream=stream)
         mark("a5a6_agg_fwd_H")
         # layer 2
@@ -165,7 +187,7 @@ class GCN2:
         mark("a7_gemm_xw1")
         self._gather(self.Y1, self.plan_c)
         mark("x_gather_y1")
-        self.plan_c.forward(self.Y1, self.Lg, F=C, flags=L.IN_PRESCALED | sf | agg_flags, stream=stream)
+        self._agg(self.plan_c, "Y1", self.Y1, self.Lg, C, L.IN_PRESCALED | sf | agg_flags, stream=stream)
         mark("a8_agg_fwd_C")
         # loss
         L.softmax_ce(self.Lg, self.labels, self.train, self.inv_nT, rr, self._local(self.dL), self.loss,
@@ -174,7 +196,7 @@ class GCN2:
         self._gather(self.dL, self.plan_c)
         mark("x_gather_dl")
         # backward
-        self.plan_c.backward(self.dL, self.G1, F=C, flags=L.IN_PRESCALED | agg_flags, stream=stream)
+        self._agg(self.plan_c, "dL", self.dL, self.G1, C, L.IN_PRESCALED | agg_flags, backward=True, stream=stream)
         mark("a10_agg_bwd_C")
         L.gemm_xtg(self.H1, self.G1, self.gTh1, self.xtg_work, M=self.rows, K=H, N=C, stream=stream)
         if self.narrow:   # exchange G1 (width C) and the mask, recompute dP1' for all rows
@@ -192,7 +214,7 @@ class GCN2:
         if not self.narrow:
             self._gather(self.dP1, p)
         mark("x_gather_dp1")
-        p.backward(self.dP1, self.G0, F=H, flags=L.IN_PRESCALED | sf | agg_flags, stream=stream)
+        self._agg(p, "dP1", self.dP1, self.G0, H, L.IN_PRESCALED | sf | agg_flags, backward=True, stream=stream)
         mark("a12_agg_bwd_H")
         L.gemm_xtg(self.X, self.G0, self.gTh0, self.xtg_work, M=self.rows, K=self.f_in, N=H, stream=stream)
         mark("a13_gemm_xtg0")

@@ -457,3 +457,72 @@ def test_peer_gather_matches_unsharded(wname, F, ld, theta):
         assert np.array_equal(z[:, :F], Z[lo:hi, :F])
         assert np.array_equal(m, M[lo:hi])
         assert np.array_equal(zb[:, :F], Zb[lo:hi, :F])
+
+
+def _peer_epoch_worker(rank, world, port, q):
+    import sys
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    from paper_conf_ipps_tianmyd20_b200 import _lib as L
+    from paper_conf_ipps_tianmyd20_b200.dist import PeerExchange
+    from paper_conf_ipps_tianmyd20_b200.gcn import GCN2
+    from synth import configs as C
+    _init(rank, world, port)
+    torch.cuda.set_device(0)
+    w = C.PL_SMALL
+    g = C.graph(w)
+    X = C.features(w, g.n)
+    Th0, Th1 = C.thetas(w)
+    T = C.train_mask(g.n, w.theta_seed)
+    y = C.labels(w, g)
+    pl = L.Plan(g.n, g.rowptr, g.col, w.P, 2.0, rank=rank, world=world)
+    perm = pl.perm()
+    ex = PeerExchange(pl)
+    model = GCN2(pl, X[perm], y[perm], T[perm], Th0, Th1, optimizer="sgd", lr=0.1, exchange=ex)
+    assert model.peer and model.Y0.shape[0] == pl.row_hi - pl.row_lo
+    model.epoch()
+    torch.cuda.synchronize()
+    q.put((rank, pl.row_lo, pl.row_hi, model.H1.cpu().numpy(), model.Lg.cpu().numpy(), model.G0.cpu().numpy(),
+           model.loss.item(), model.grad.cpu().numpy(), model.theta.cpu().numpy()))
+    ex.close()
+    dist.destroy_process_group()
+
+
+@pytest.mark.gpu
+def test_sharded_peer_epoch_matches_unsharded():
+    """A whole sharded 2-layer GCN epoch in peer mode (dist.PeerExchange: the
+    aggregation inputs live in per-shard IPC buffers, every selective pass
+    reads remote rows from their owners; no halo copies): rows bitwise equal
+    to the unsharded epoch, gradients within the all-reduce tolerance."""
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    from paper_conf_ipps_tianmyd20_b200 import _lib as L
+    from paper_conf_ipps_tianmyd20_b200.gcn import GCN2
+    from synth import configs as C
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    ps = [ctx.Process(target=_peer_epoch_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in ps:
+        p.start()
+    res = sorted([q.get(timeout=600) for _ in ps], key=lambda t: t[0])
+    for p in ps:
+        p.join(timeout=60)
+    w = C.PL_SMALL
+    g = C.graph(w)
+    X = C.features(w, g.n)
+    Th0, Th1 = C.thetas(w)
+    T = C.train_mask(g.n, w.theta_seed)
+    y = C.labels(w, g)
+    pl = L.Plan(g.n, g.rowptr, g.col, w.P, 2.0)
+    perm = pl.perm()
+    ref = GCN2(pl, X[perm], y[perm], T[perm], Th0, Th1, optimizer="sgd", lr=0.1)
+    ref.epoch()
+    torch.cuda.synchronize()
+    H1, Lg, G0, gr = ref.H1.cpu().numpy(), ref.Lg.cpu().numpy(), ref.G0.cpu().numpy(), ref.grad.cpu().numpy()
+    for rank, lo, hi, h1, lg, g0, loss, grad, theta in res:
+        assert np.array_equal(h1, H1[lo:hi])
+        assert np.array_equal(lg, Lg[lo:hi])
+        assert np.array_equal(g0, G0[lo:hi])
+        assert abs(loss - ref.loss.item()) <= 1e-6 * abs(ref.loss.item())
+        assert np.max(np.abs(grad - gr)) <= 1e-5 * np.max(np.abs(gr))
+    assert np.array_equal(res[0][8], res[1][8])
