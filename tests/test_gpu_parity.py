@@ -680,3 +680,19 @@ def test_fused_split_is_bitwise(wname, theta, dense):
         outs.append([t.clone() for t in (m.Y0, m.H1, m.mask1, m.Y1, m.Lg, m.G1, m.dP1, m.G0, m.grad, m.theta)])
     for a, b in zip(*outs):
         assert torch.equal(a, b)
+
+
+def test_plan_with_negative_theta_calibrates_first():
+    """θ < 0 in pcgcn_plan: the L161 calibration runs on the device first and
+    the plan uses the θ it returns (reported in the stats); the plan then
+    aggregates within the usual gate."""
+    g = G.sbm(C.PUBMED.spec)
+    pl = L.Plan(g.n, g.rowptr, g.col, 32, -1.0, f_max=64)
+    th = pl.stats()["theta"]
+    assert 0.0 < th < 1.0 and pl.theta == th
+    Y = _feat(g.n, 48, 3)
+    Z, _, _ = aggregate_gpu(g, Y, 32, th, f_max=64)
+    err, _ = cond_err(g, Y, Z)
+    assert err <= TOL
+    with pytest.raises(L.PcgcnError):
+        L.Plan(g.n, g.rowptr, g.col, 32, -1.0, build_device=False)
