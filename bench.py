@@ -50,7 +50,7 @@ def parse():
                     help="unit of the selective/full decision (pcgcn_opts.mode_grain)")
     ap.add_argument("--fuse-split", default="on", choices=["on", "off"],
                     help="transform GEMMs write the full mode's window blocks (pcgcn_gemm_*_split)")
-    ap.add_argument("--dense", default="bf16x3", choices=["tf32x2", "bf16x3"],
+    ap.add_argument("--dense", default="bf16x3", choices=["tf32x2", "bf16x3", "bf16x1"],
                     help="full-mode arithmetic (pcgcn_opts.dense_prec)")
     ap.add_argument("--oracle-frac", type=float, default=0.02)
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -171,7 +171,7 @@ def agg_bytes(st, n, rows, F, dense_rows, nchunks):
     return int(b)
 
 
-def agg_bpc(st, rows, F, dense_rows, nchunks, bf3=False):
+def agg_bpc(st, rows, F, dense_rows, nchunks, bf3=False, bf1=False):
     """Partition-centric bytes model of one aggregation (SURVEY.md §8(d) B_pc;
     PAPER.md L129 §III-A.b): structure (indices, row pointers, r) + every
     destination partition's distinct selective source rows read once
@@ -180,7 +180,7 @@ def agg_bpc(st, rows, F, dense_rows, nchunks, bf3=False):
     npad = (F + 15) // 16 * 16
     b = st["shard_nnz_sparse"] * 4 + (rows + 1) * 8 + rows * 4
     b += 4 * F * (st["shard_src_rows_pc"] + rows)
-    b += nchunks * (516 + (6 if bf3 else 8) * 32 * npad) + 2 * dense_rows * F * 4
+    b += nchunks * (516 + (6 if bf3 else 2 if bf1 else 8) * 32 * npad) + 2 * dense_rows * F * 4
     return int(b)
 
 
@@ -490,7 +490,7 @@ def plan_kw(args):
     from paper_conf_ipps_tianmyd20_b200 import _lib as L
     return dict(order=L.ORDER_DEGREE if args.order == "degree" else L.ORDER_ID,
                 grain=L.GRAIN_TILE if args.grain == "tile" else L.GRAIN_BLOCK,
-                dense_prec=L.DENSE_BF16X3 if args.dense == "bf16x3" else L.DENSE_TF32X2)
+                dense_prec={"bf16x3": L.DENSE_BF16X3, "bf16x1": L.DENSE_BF16X1}.get(args.dense, L.DENSE_TF32X2))
 
 
 def main():
@@ -727,13 +727,14 @@ def main():
     t_tc = kern["a5a6_agg_fwd_H"]["dense_tc"]
     npad = (w.hidden + 15) // 16 * 16
     bf3 = args.dense == "bf16x3"
-    # executed MMA flops per chunk: 2 (hi, lo) tf32 products, or 3 bf16 parts
-    tc_flops = st["shard_chunks"] * 2 * 128 * 32 * npad * (3 if bf3 else 2)
+    bf16 = args.dense in ("bf16x3", "bf16x1")
+    # executed MMA flops per chunk: 2 (hi, lo) tf32 products, 3 bf16 parts, or 1 bf16 product
+    tc_flops = st["shard_chunks"] * 2 * 128 * 32 * npad * {"bf16x3": 3, "bf16x1": 1}.get(args.dense, 2)
     tc_tf = tc_flops / (t_tc * 1e-3) / 1e12 if t_tc > 0 else None
     try:
-        tc_peak = float(json.load(open(MEASURED_PEAKS))["bf16_tflops"]) / (1 if bf3 else 2)
+        tc_peak = float(json.load(open(MEASURED_PEAKS))["bf16_tflops"]) / (1 if bf16 else 2)
     except Exception:
-        tc_peak = 1590.0 / (1 if bf3 else 2)
+        tc_peak = 1590.0 / (1 if bf16 else 2)
     traffic = l2_read = lts_pct = dram_pct = None
     traffic_cfg = None
     tpath = os.path.join(ROOT, "profiles", "traffic.json")
@@ -890,7 +891,9 @@ def main():
         line = {
             "metric": "2-layer GCN epoch ms", "value": ms, "unit": "ms", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": False,
-            "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "scaling": "strong", "vs_baseline": None,
+            "dtype": "f32" if args.dense != "bf16x1" else "f32 (selective) + bf16 (full mode, fp32 accumulate)",
+            "data": "synthetic",
             "config": {
                 "workload": workload_str(w, g),
                 "P": P, "theta": theta, "theta_c": theta_c if theta_c else theta, "theta_source": theta_src, "optimizer": "adam",
@@ -944,16 +947,17 @@ def main():
                                                    "64 KB / 64 MB / 4 GB buffers, best of 3"}},
             "bytes_views": {
                 "aggregation": f"layer-1 forward, F={w.hidden} (selective + full mode)",
-                "B_min": bH, "B_pc": agg_bpc(st, rows, w.hidden, dense_rows, st["shard_chunks"], args.dense == "bf16x3"),
+                "B_min": bH, "B_pc": agg_bpc(st, rows, w.hidden, dense_rows, st["shard_chunks"], args.dense == "bf16x3",
+                                 args.dense == "bf16x1"),
                 "ncu_dram_selective": traffic,
                 "dram_over_B_min_selective": (traffic / b_sp) if traffic else None,
                 "src_rows_pc": st["shard_src_rows_pc"],
                 "note": "B_min = compulsory bytes; B_pc = each destination partition reads its distinct selective "
                         "sources once; ncu DRAM bytes of the selective kernels per launch (cold cache)"},
             "tensor_view": {"kernel": "tc_engine<A_BITS> full-mode tiles, layer-1 forward",
-                            "ms": t_tc, "achieved": tc_tf, "unit": "TFLOP/s (bf16)" if bf3 else "TFLOP/s (tf32)",
+                            "ms": t_tc, "achieved": tc_tf, "unit": "TFLOP/s (bf16)" if bf16 else "TFLOP/s (tf32)",
                             "peak": tc_peak, "frac": (tc_tf / tc_peak) if tc_tf else None,
-                            "peak_source": ("measured bf16 dense (MEASURED_PEAKS.json)" if bf3 else
+                            "peak_source": ("measured bf16 dense (MEASURED_PEAKS.json)" if bf16 else
                                             "measured bf16 dense (MEASURED_PEAKS.json) x 0.5 (tf32:bf16 nominal ratio)")},
             "agg_kernels_ms": kern,
             "agg_GBs": {"fwd_H": bH / (per["a5a6_agg_fwd_H"] * 1e-3) / 1e9,

@@ -75,9 +75,10 @@ enum { PCGCN_NORM_SYM = 0, PCGCN_NORM_NONE = 1 };     /* Â = D̃^-½ÃD̃^-½  
 enum {
   PCGCN_DENSE_TF32X2 = 0,    /* full mode on tcgen05 (kind::tf32): A∈{0,1} exact, Y = hi + lo, 2 MMAs */
   PCGCN_DENSE_FP32_SIMT = 1, /* full mode on CUDA cores in fp32 (the paper's §IV-C kernel, L183-L187) */
-  PCGCN_DENSE_BF16X1 = 2,    /* full mode on tcgen05 with the input rounded to bf16 (RN-even), one MMA per
-                                K-step, fp32 accumulation: the paper's 16-bit tensor-core policy (L191-L193,
-                                §V-E); error <= 2^-9 per term, gate 2e-2 (BASELINE.json north_star) */
+  PCGCN_DENSE_BF16X1 = 2,    /* full mode on tcgen05 kind::f16 with the input rounded to bf16 (RN-even):
+                                one bf16 part, 2 K=16 MMAs and 2·32·npad B bytes per 128x32 chunk, fp32
+                                accumulation: the paper's 16-bit tensor-core policy (L191-L193, §V-E);
+                                error <= 2^-9 per term, gate 2e-2 (BASELINE.json north_star) */
   PCGCN_DENSE_BF16X3 = 3     /* full mode on tcgen05 kind::f16: Y = b0 + b1 + b2, three bf16 parts
                                 (round to nearest, exact fp32 residuals: |Y - Σb| <= 2^-24|Y|), A∈{0,1}
                                 exact; 6 K=16 MMAs and 6·32·npad B bytes per 128x32 chunk against the

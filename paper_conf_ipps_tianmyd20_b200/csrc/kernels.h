@@ -44,6 +44,12 @@ struct AggArgs {
   float* seg_ws;             // [nseg x ldws] fp32 partial sums
   int64_t ldws;
   int* counter;              // dynamic row scheduler ticket (zeroed on the stream before each pass)
+  // inline segments: the row pass also claims the segments
+  const int32_t* seg_row = nullptr;  // [nseg] shard-local row of each segment
+  int* seg_cnt = nullptr;            // [nseg] completed segments per long row (at its first segment; self-resetting)
+  int* seg_ticket = nullptr;         // segment ticket (zeroed with the row ticket)
+  int seg_inline = 0;                // 1: no separate segment pass
+  int64_t seg_ahead = 0;             // row tickets ahead of the claiming warp within which segments are taken
   // device-initiated peer gather: sources of shard q are read from
   // shard q's own buffer (peer_base[q] = its row row0[q]; NVLink peer memory
   // on a multi-GPU node, CUDA IPC in the 1-GPU tests) instead of an exchanged copy
@@ -52,6 +58,7 @@ struct AggArgs {
   int64_t peer_row0[9];
   int phase = 0;             // 0: segment pass + row pass; 1: segment pass only; 2: row pass only
   int rows_per_ticket = 1;   // consecutive rows per scheduler ticket, 1..16
+  float mean_deg = 0.f;      // selective edges per row (layout choice: short rows -> multi-row warps)
 };
 // selective edges per long-row segment
 constexpr int SEG_EDGES = 1024;
@@ -83,10 +90,11 @@ struct DenseArgs {
   const float* blk = nullptr;  // source-window blocks (launch_split_windows); nullptr: hiT/loT maps
   int64_t blk_floats = 0;      // floats per window block
   int64_t n_src = 0;           // real source rows (vertices); rows [n_src, n) of the input are never read
-  int bf3 = 0;                 // PCGCN_DENSE_BF16X3: window blocks hold 3 bf16 parts (kind::f16 MMAs)
+  int bf3 = 0;                 // bf16 parts per window block (kind::f16 MMAs): 3 BF16X3, 1 BF16X1; 0 tf32
   int* dyn = nullptr;          // zeroed tile ticket: CTAs claim tiles dynamically in rt_order / plan order
 };
-// mode 0: tf32 hi/lo, 1: bf16 single (BF16X1), 2: three bf16 parts (BF16X3)
+// mode 0: tf32 hi/lo, 1: bf16-rounded tf32 single (unused since BF16X1 runs on kind::f16),
+// 2: three bf16 parts (BF16X3), 3: one bf16 part (BF16X1)
 cudaError_t launch_split_windows(const float* Y, int64_t ldy, int64_t n, int F, int npad, int mode, float* blk,
                                  int64_t nwin, cudaStream_t s);
 cudaError_t launch_dense_tc(const DenseArgs& a, cudaStream_t s);

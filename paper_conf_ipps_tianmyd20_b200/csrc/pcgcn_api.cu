@@ -166,7 +166,7 @@ pcgcn_status upload_plan(pcgcn_plan_s* p) {
   UP(&d.counter, (int*)nullptr, 32);
   {
     // long selective rows -> segments of SEG_EDGES edges (reading #22)
-    std::vector<int32_t> rs(d.rows, -1);
+    std::vector<int32_t> rs(d.rows, -1), srow;
     std::vector<int64_t> lo, hi;
     for (int64_t v = 0; v < d.rows; ++v) {
       if (rp[v + 1] - rp[v] <= SEG_EDGES) continue;
@@ -174,6 +174,7 @@ pcgcn_status upload_plan(pcgcn_plan_s* p) {
       for (int64_t e = rp[v]; e < rp[v + 1]; e += SEG_EDGES) {
         lo.push_back(e);
         hi.push_back(std::min<int64_t>(e + SEG_EDGES, rp[v + 1]));
+        srow.push_back(int32_t(v));
       }
     }
     d.nseg = int64_t(lo.size());
@@ -182,6 +183,9 @@ pcgcn_status upload_plan(pcgcn_plan_s* p) {
       UP(&d.seg_lo, lo.data(), d.nseg);
       UP(&d.seg_hi, hi.data(), d.nseg);
       UP(&d.seg_ws, (float*)nullptr, d.nseg * d.fpad_max);
+      UP(&d.seg_row, srow.data(), d.nseg);
+      UP(&d.seg_cnt, (int32_t*)nullptr, d.nseg);
+      if ((e = cudaMemset(d.seg_cnt, 0, d.nseg * sizeof(int32_t))) != cudaSuccess) return cuda_fail(e, "memset");
     }
   }
 #undef UP
@@ -279,8 +283,8 @@ bool window_out(pcgcn_plan_t p, int32_t F, WindowOut* wo) {
     return false;
   const int64_t npad = round_up(F, 16);
   wo->blk = d.yhi;
-  wo->mode = dp == PCGCN_DENSE_BF16X3 ? 3 : dp == PCGCN_DENSE_BF16X1 ? 2 : 1;
-  wo->blk_floats = dp == PCGCN_DENSE_BF16X3 ? npad * 48 : (dp == PCGCN_DENSE_BF16X1 ? 1 : 2) * npad * 32;
+  wo->mode = dp == PCGCN_DENSE_BF16X3 ? 3 : dp == PCGCN_DENSE_BF16X1 ? 4 : 1;
+  wo->blk_floats = dp == PCGCN_DENSE_BF16X3 ? npad * 48 : dp == PCGCN_DENSE_BF16X1 ? npad * 16 : 2 * npad * 32;
   wo->nwin = d.n_pad / 32;
   return true;
 }
@@ -349,9 +353,11 @@ pcgcn_status aggregate(pcgcn_plan_t p, const float* Y, int64_t ldy, float* Z, in
   a.relu = (flags & PCGCN_RELU) != 0;
   a.out_prescaled = (flags & PCGCN_OUT_PRESCALED) != 0;
   a.row_seg = d.row_seg; a.seg_lo = d.seg_lo; a.seg_hi = d.seg_hi; a.nseg = d.nseg;
+  a.seg_row = d.seg_row; a.seg_cnt = d.seg_cnt; a.seg_ticket = d.counter + 8;
   a.seg_ws = d.seg_ws; a.ldws = d.fpad_max;
   a.counter = d.counter;
   a.rows_per_ticket = rows_per_ticket(d.nnz_s, d.rows);
+  a.mean_deg = float(double(p->sp_rowptr[p->n]) / double(p->n));  // plan-global: every shard picks the same layout
   // the split + full-mode tiles run on the plan's high-priority side stream,
   // concurrently with the long-row segment pass on the caller's stream;
   // PROFILE calls stay serial so per-kernel times add up
@@ -369,13 +375,13 @@ pcgcn_status aggregate(pcgcn_plan_t p, const float* Y, int64_t ldy, float* Z, in
   // full mode's B: source-window blocks fetched by one bulk copy per chunk
   // (default), or the feature-major split read by strided TMA boxes (the
   // CTA-pair kernel, or PCGCN_DENSE_BLOCKED=0)
-  const bool blocked = bf3 || (tc && dense_blocked_enabled() && !dense_pair_eligible(npad));
+  const bool blocked = bf3 || bf16 || (tc && dense_blocked_enabled() && !dense_pair_eligible(npad));
   // IN_SPLIT: the producer already wrote the window blocks (pcgcn_gemm_*_split
   // writes them exactly when the full mode uses window blocks)
   const bool presplit = (flags & PCGCN_IN_SPLIT) && blocked;
   if (dense && tc && !presplit) {
     if (prof) d.ev_used[1] = true;
-    e = blocked ? launch_split_windows(src, ldsrc, p->n, F, npad, bf3 ? 2 : (bf16 ? 1 : 0), d.yhi, d.n_pad / 32, ms)
+    e = blocked ? launch_split_windows(src, ldsrc, p->n, F, npad, bf3 ? 2 : (bf16 ? 3 : 0), d.yhi, d.n_pad / 32, ms)
                 : launch_split_transpose(src, ldsrc, p->n, F, npad, d.yhi, bf16 ? nullptr : ylo, d.n_pad, ms);
     if (e != cudaSuccess) return cuda_fail(e, "split_transpose");
   }
@@ -395,8 +401,8 @@ pcgcn_status aggregate(pcgcn_plan_t p, const float* Y, int64_t ldy, float* Z, in
     }
     if (blocked) {
       da.blk = d.yhi;
-      da.blk_floats = bf3 ? int64_t(npad) * 48 : int64_t(bf16 ? 1 : 2) * npad * 32;
-      da.bf3 = bf3 ? 1 : 0;
+      da.blk_floats = bf3 ? int64_t(npad) * 48 : bf16 ? int64_t(npad) * 16 : int64_t(2) * npad * 32;
+      da.bf3 = bf3 ? 3 : (bf16 ? 1 : 0);  // bf16 parts of B (kind::f16)
     }
     e = tc ? launch_dense_tc(da, ms) : launch_dense_simt_y(da, src, ldsrc, F, ms);
     if (e != cudaSuccess) return cuda_fail(e, "dense-mode kernel");
@@ -597,9 +603,11 @@ static pcgcn_status aggregate_peer(pcgcn_plan_t p, const float* const* peer, int
   a.relu = (flags & PCGCN_RELU) != 0;
   a.out_prescaled = (flags & PCGCN_OUT_PRESCALED) != 0;
   a.row_seg = d.row_seg; a.seg_lo = d.seg_lo; a.seg_hi = d.seg_hi; a.nseg = d.nseg;
+  a.seg_row = d.seg_row; a.seg_cnt = d.seg_cnt; a.seg_ticket = d.counter + 8;
   a.seg_ws = d.seg_ws; a.ldws = d.fpad_max;
   a.counter = d.counter;
   a.rows_per_ticket = rows_per_ticket(d.nnz_s, d.rows);
+  a.mean_deg = float(double(p->sp_rowptr[p->n]) / double(p->n));  // plan-global: every shard picks the same layout
   a.peer_world = W;
   for (int q = 0; q < 8; ++q) a.peer_base[q] = q < W ? reinterpret_cast<const char*>(peer[q]) : nullptr;
   for (int q = 0; q <= 8; ++q)

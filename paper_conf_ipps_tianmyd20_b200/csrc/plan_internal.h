@@ -33,6 +33,8 @@ struct DevicePlan {
   int64_t* seg_lo = nullptr;      // [nseg] shard-local edge range of each segment
   int64_t* seg_hi = nullptr;
   float* seg_ws = nullptr;        // [nseg x fpad_max] segment partial sums
+  int32_t* seg_row = nullptr;     // [nseg] shard-local row of each segment
+  int32_t* seg_cnt = nullptr;     // [nseg] inline-segment completion counts (zero between calls)
   int* counter = nullptr;         // [32] selective-pass row ticket
   int32_t* halo_send = nullptr;   // [Σ_q send rows] plan rows of this shard, peers in rank order
   int32_t* halo_recv = nullptr;   // [Σ_q recv rows] plan rows of other shards, peers in rank order

@@ -38,6 +38,9 @@
 #include "kernels.h"
 
 namespace pcgcn {
+int knobs_mrow_gpt();   // PCGCN_MROW_GPT (multi-row groups per ticket)
+int knobs_seg_inline(); // PCGCN_SEG_INLINE (0: separate up-front segment pass)
+int knobs_seg_ahead();  // PCGCN_SEG_AHEAD (segment window, in row tickets per resident warp)
 namespace {
 
 __device__ __forceinline__ float4 ld_f4(const float* p) {
@@ -78,8 +81,18 @@ __device__ __forceinline__ const char* src_row(const char* yb, uint32_t j, uint3
 __device__ __forceinline__ uint32_t smem_addr(const void* p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
 }
+// a += b as two packed fp32 adds (add.rn.f32x2 = SASS FADD2, sm_100+): the
+// same two IEEE round-to-nearest adds per pair (bitwise equal to four FADDs)
+// at half the issue slots — the gather's FADDs are most of its instructions
+__device__ __forceinline__ void add2(float& ax, float& ay, float bx, float by) {
+  asm("{\n\t.reg .b64 pa, pb;\n\tmov.b64 pa, {%0, %1};\n\tmov.b64 pb, {%2, %3};\n\t"
+      "add.rn.f32x2 pa, pa, pb;\n\tmov.b64 {%0, %1}, pa;\n\t}"
+      : "+f"(ax), "+f"(ay)
+      : "f"(bx), "f"(by));
+}
 __device__ __forceinline__ void add4(float4& a, const float4& b) {
-  a.x += b.x; a.y += b.y; a.z += b.z; a.w += b.w;
+  add2(a.x, a.y, b.x, b.y);
+  add2(a.z, a.w, b.z, b.w);
 }
 // one lane vector of H float4 (H = 2: one 32-byte LDG.E.ENL2.256, sm_100's
 // widest load — half the load, shuffle and address instructions per gathered
@@ -289,6 +302,18 @@ __global__ void __launch_bounds__(128, 2 * Lay<G, V, H>::MINB) sparse_seg_kernel
   }
 }
 
+// Inline long-row segments (a.seg_inline): instead of a separate
+// up-front segment pass, the row pass's warps claim the segments of a long row
+// from a second ticket counter when the row-ticket frontier comes near the
+// row (segment s is taken once its row is within seg_ahead row tickets of the
+// claiming warp's next block), so a hub's segments gather while its community
+// is L2-resident.  A segment writes its partial sum, and the warp completing a
+// row's LAST segment (an atomic count per row, threadfence pattern) adds the
+// row's partials in segment order — the same fixed order as the two-pass
+// scheme, so results are bitwise identical — and runs the row's epilogue.
+// Block rows with segments are skipped by the block walk.
+__device__ __forceinline__ int peek_ticket(const int* t) { return *reinterpret_cast<const volatile int*>(t); }
+
 // Row pass: persistent warps claim destination rows in plan order from a
 // ticket counter (dynamic balance without losing the partition order's L2
 // locality); a row is gathered directly or, if long, summed from its
@@ -309,96 +334,9 @@ __global__ void __launch_bounds__(256, Lay<G, V, H>::MINB) sparse_row_kernel(Agg
   }
   const char* yb = (PEER ? nullptr : reinterpret_cast<const char*>(a.Y)) + 16 * H * (qv[0] < 0 ? 0 : qv[0]);
   const uint32_t rstride = uint32_t(a.ldy * 4);
-  // Rows are claimed in blocks of R consecutive rows per ticket (R >= 4 from
-  // the plan's mean selective degree: short rows would otherwise pay the
-  // ticket -> rowptr -> index dependency chain per row).  The next block's
-  // ticket is issued when a block starts and consumed three rows before its
-  // end; its R+1 row pointers are then copied global -> shared with cp.async
-  // (no registers held in flight) while those rows gather; and the first
-  // index batch of the next row is always in flight while the current row
-  // gathers: in steady state a row costs one gather round trip.
-  __shared__ long long s_rp[8][2][32];  // per warp: this block's / the next block's row pointers
-  const int wib = threadIdx.x >> 5;
-  const int R = a.rows_per_ticket;
-  const int nblk_total = int((a.rows + R - 1) / R);
-  auto fetch_rp = [&](int blk, int b) {  // async copy of rowptr[blk*R .. blk*R+R] into s_rp[wib][b]
-    if (blk < nblk_total && lane <= R) {
-      const int64_t r = int64_t(blk) * R + lane;
-      const long long* src = reinterpret_cast<const long long*>(a.rowptr + (r < a.rows ? r : a.rows));
-      asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_addr(&s_rp[wib][b][lane])), "l"(src)
-                   : "memory");
-    }
-    asm volatile("cp.async.commit_group;" ::: "memory");
-  };
-  auto wait_rp = [&]() {
-    asm volatile("cp.async.wait_group 0;" ::: "memory");
-    __syncwarp();
-  };
-  int blk;
-  {
-    int t = 0;
-    if (lane == 0) t = atomicAdd(a.counter, 1);
-    blk = __shfl_sync(0xffffffffu, t, 0);
-  }
-  int b = 0;
-  fetch_rp(blk, b);
-  wait_rp();
-  int pre = 0;
-  if (blk < nblk_total) {
-    const int64_t f0 = s_rp[wib][b][0], f1 = s_rp[wib][b][1];
-    pre = (f0 + lane < f1) ? ld_col<PEER>(a.col + f0 + lane, a) : 0;
-  }
-  while (blk < nblk_total) {
-    int tk = 0;
-    if (lane == 0) tk = atomicAdd(a.counter, 1);  // next block's ticket, consumed later
-    int nblk = nblk_total;
-    const int nr = int(a.rows - int64_t(blk) * R < R ? a.rows - int64_t(blk) * R : R);
-    const int ic = nr > 3 ? nr - 3 : 0;
-    for (int i = 0; i < nr; ++i) {
-    const int64_t row = int64_t(blk) * R + i;
-    if (i == ic) {
-      nblk = __shfl_sync(0xffffffffu, tk, 0);
-      fetch_rp(nblk, b ^ 1);
-    }
-    if (i + 1 == nr) wait_rp();
-    // edge ranges (re-read from shared memory, not kept live across the gather):
-    // this row [e0, e1) and the next row [n0, n1) (this block's, or the next block's first)
-    const int64_t e0 = s_rp[wib][b][i], e1 = s_rp[wib][b][i + 1];
-    int64_t n0 = 0, n1 = 0;
-    if (i + 1 < nr) {
-      n0 = e1;
-      n1 = s_rp[wib][b][i + 2];
-    } else if (nblk < nblk_total) {
-      n0 = s_rp[wib][b ^ 1][0];
-      n1 = s_rp[wib][b ^ 1][1];
-    }
-    float4 tot[V][H];
-    int pre_next;
-    // the epilogue's per-row scalars are loaded before the gather (in flight with it)
-    const float ri = a.r[a.row_lo + row];
-    const int zi = HAS_ZD ? a.zd_index[row] : -1;
-    const int sg = HAS_SEG ? a.row_seg[row] : -1;
-    if (HAS_SEG && sg >= 0) {
-      pre_next = (n0 + lane < n1) ? ld_col<PEER>(a.col + n0 + lane, a) : 0;
-      const int ns = int((e1 - e0 + SEG_EDGES - 1) / SEG_EDGES);
-#pragma unroll
-      for (int v = 0; v < V; ++v)
-#pragma unroll
-        for (int h = 0; h < H; ++h) tot[v][h] = make_float4(0.f, 0.f, 0.f, 0.f);
-      if (slot == 0) {
-        for (int k = 0; k < ns; ++k)
-#pragma unroll
-          for (int v = 0; v < V; ++v)
-#pragma unroll
-            for (int h = 0; h < H; ++h)
-              if (qv[v] >= 0 && H * qv[v] + h < nvec4)
-                add4(tot[v][h], __ldcg(reinterpret_cast<const float4*>(a.seg_ws + int64_t(sg + k) * a.ldws +
-                                                                        4 * (H * qv[v] + h))));
-      }
-    } else {
-      pre_next = gather_sum<G, V, H, PEER>(a.col + e0, int(e1 - e0), pre, a.col + n0, int(n1 - n0), yb, rstride,
-                                           lok, lane, tot, a);
-    }
+
+  // epilogue of one row (totals valid in slot-0 lanes): + Zd, x r_i, mask, ReLU, store
+  auto epilogue = [&](int64_t row, float4 (&tot)[V][H], int zi, float ri) {
     uint32_t bal[V][4];
     uint32_t mbyte[V];
 #pragma unroll
@@ -470,11 +408,456 @@ __global__ void __launch_bounds__(256, Lay<G, V, H>::MINB) sparse_row_kernel(Agg
         if (nvec + lane < 4 * ((a.F + 31) >> 5)) mrow[nvec + lane] = 0;
       }
     }
+  };
+  // one segment of a long row, gathered by this warp (inline segments)
+  auto run_segment = [&](int sgi) {
+    const int64_t lo = a.seg_lo[sgi], hi = a.seg_hi[sgi];
+    const int n = int(hi - lo);
+    const int first = lane < n ? ld_col<PEER>(a.col + lo + lane, a) : 0;
+    float4 tot[V][H];
+    gather_sum<G, V, H, PEER>(a.col + lo, n, first, nullptr, 0, yb, rstride, lok, lane, tot, a);
+    const int64_t row = a.seg_row[sgi];
+    const int s0 = a.row_seg[row];
+    const int ns = int((a.rowptr[row + 1] - a.rowptr[row] + SEG_EDGES - 1) / SEG_EDGES);
+    if (slot == 0) {
+#pragma unroll
+      for (int v = 0; v < V; ++v)
+#pragma unroll
+        for (int h = 0; h < H; ++h)
+          if (qv[v] >= 0 && H * qv[v] + h < nvec4)
+            __stcg(reinterpret_cast<float4*>(a.seg_ws + int64_t(sgi) * a.ldws + 4 * (H * qv[v] + h)), tot[v][h]);
+    }
+    __threadfence();
+    __syncwarp();
+    int last = 0;
+    if (lane == 0) last = atomicAdd(a.seg_cnt + s0, 1) == ns - 1;
+    if (__shfl_sync(0xffffffffu, last, 0)) {
+      __threadfence();
+#pragma unroll
+      for (int v = 0; v < V; ++v)
+#pragma unroll
+        for (int h = 0; h < H; ++h) tot[v][h] = make_float4(0.f, 0.f, 0.f, 0.f);
+      if (slot == 0) {
+        for (int k = 0; k < ns; ++k)
+#pragma unroll
+          for (int v = 0; v < V; ++v)
+#pragma unroll
+            for (int h = 0; h < H; ++h)
+              if (qv[v] >= 0 && H * qv[v] + h < nvec4)
+                add4(tot[v][h], __ldcg(reinterpret_cast<const float4*>(a.seg_ws + int64_t(s0 + k) * a.ldws +
+                                                                        4 * (H * qv[v] + h))));
+      }
+      epilogue(row, tot, HAS_ZD ? a.zd_index[row] : -1, a.r[a.row_lo + row]);
+      if (lane == 0) a.seg_cnt[s0] = 0;  // self-resetting for the next call
+    }
+  };
+  const bool inl = HAS_SEG && a.seg_inline;
+  // claim segments while the next unclaimed one belongs to a row before
+  // `limit` (warp-uniform; limit < 0: drain every remaining segment)
+  auto seg_loop = [&](int64_t limit) {
+    while (true) {
+      int sgi = 0;
+      if (lane == 0) sgi = atomicAdd(a.seg_ticket, 1);
+      sgi = __shfl_sync(0xffffffffu, sgi, 0);
+      if (sgi >= a.nseg) return;
+      run_segment(sgi);
+      if (limit >= 0) {
+        int go = 0;
+        if (lane == 0) {
+          const int pk = peek_ticket(a.seg_ticket);
+          go = pk < a.nseg && a.seg_row[pk] < limit;
+        }
+        if (!__shfl_sync(0xffffffffu, go, 0)) return;
+      }
+    }
+  };
+  // Rows are claimed in blocks of R consecutive rows per ticket (R >= 4 from
+  // the plan's mean selective degree: short rows would otherwise pay the
+  // ticket -> rowptr -> index dependency chain per row).  The next block's
+  // ticket is issued when a block starts and consumed three rows before its
+  // end; its R+1 row pointers are then copied global -> shared with cp.async
+  // (no registers held in flight) while those rows gather; and the first
+  // index batch of the next row is always in flight while the current row
+  // gathers: in steady state a row costs one gather round trip.
+  __shared__ long long s_rp[8][2][32];  // per warp: this block's / the next block's row pointers
+  const int wib = threadIdx.x >> 5;
+  const int R = a.rows_per_ticket;
+  const int nblk_total = int((a.rows + R - 1) / R);
+  auto fetch_rp = [&](int blk, int b) {  // async copy of rowptr[blk*R .. blk*R+R] into s_rp[wib][b]
+    if (blk < nblk_total && lane <= R) {
+      const int64_t r = int64_t(blk) * R + lane;
+      const long long* src = reinterpret_cast<const long long*>(a.rowptr + (r < a.rows ? r : a.rows));
+      asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_addr(&s_rp[wib][b][lane])), "l"(src)
+                   : "memory");
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+  };
+  auto wait_rp = [&]() {
+    asm volatile("cp.async.wait_group 0;" ::: "memory");
+    __syncwarp();
+  };
+  int blk;
+  {
+    int t = 0;
+    if (lane == 0) t = atomicAdd(a.counter, 1);
+    blk = __shfl_sync(0xffffffffu, t, 0);
+  }
+  int b = 0;
+  fetch_rp(blk, b);
+  wait_rp();
+  int pre = 0;
+  if (blk < nblk_total) {
+    const int64_t f0 = s_rp[wib][b][0], f1 = s_rp[wib][b][1];
+    pre = (f0 + lane < f1) ? ld_col<PEER>(a.col + f0 + lane, a) : 0;
+  }
+  while (blk < nblk_total) {
+    int tk = 0;
+    if (lane == 0) tk = atomicAdd(a.counter, 1);  // next block's ticket, consumed later
+    // inline segments: the next unclaimed segment (peeked now, its row read
+    // three rows before the block's end, decided at the end)
+    int speek = 0;
+    if (inl && lane == 0) speek = peek_ticket(a.seg_ticket);
+    int64_t srow = INT64_MAX;
+    int nblk = nblk_total;
+    const int nr = int(a.rows - int64_t(blk) * R < R ? a.rows - int64_t(blk) * R : R);
+    const int ic = nr > 3 ? nr - 3 : 0;
+    for (int i = 0; i < nr; ++i) {
+    const int64_t row = int64_t(blk) * R + i;
+    if (i == ic) {
+      nblk = __shfl_sync(0xffffffffu, tk, 0);
+      fetch_rp(nblk, b ^ 1);
+      if (inl && lane == 0 && speek < a.nseg) srow = a.seg_row[speek];
+    }
+    if (i + 1 == nr) wait_rp();
+    // edge ranges (re-read from shared memory, not kept live across the gather):
+    // this row [e0, e1) and the next row [n0, n1) (this block's, or the next block's first)
+    const int64_t e0 = s_rp[wib][b][i], e1 = s_rp[wib][b][i + 1];
+    int64_t n0 = 0, n1 = 0;
+    if (i + 1 < nr) {
+      n0 = e1;
+      n1 = s_rp[wib][b][i + 2];
+    } else if (nblk < nblk_total) {
+      n0 = s_rp[wib][b ^ 1][0];
+      n1 = s_rp[wib][b ^ 1][1];
+    }
+    float4 tot[V][H];
+    int pre_next;
+    // the epilogue's per-row scalars are loaded before the gather (in flight with it)
+    const float ri = a.r[a.row_lo + row];
+    const int zi = HAS_ZD ? a.zd_index[row] : -1;
+    const int sg = HAS_SEG ? a.row_seg[row] : -1;
+    bool skip = false;
+    if (HAS_SEG && sg >= 0) {
+      pre_next = (n0 + lane < n1) ? ld_col<PEER>(a.col + n0 + lane, a) : 0;
+      skip = inl;  // written by the warp that completes its last segment
+      const int ns = int((e1 - e0 + SEG_EDGES - 1) / SEG_EDGES);
+#pragma unroll
+      for (int v = 0; v < V; ++v)
+#pragma unroll
+        for (int h = 0; h < H; ++h) tot[v][h] = make_float4(0.f, 0.f, 0.f, 0.f);
+      if (slot == 0 && !inl) {
+        for (int k = 0; k < ns; ++k)
+#pragma unroll
+          for (int v = 0; v < V; ++v)
+#pragma unroll
+            for (int h = 0; h < H; ++h)
+              if (qv[v] >= 0 && H * qv[v] + h < nvec4)
+                add4(tot[v][h], __ldcg(reinterpret_cast<const float4*>(a.seg_ws + int64_t(sg + k) * a.ldws +
+                                                                        4 * (H * qv[v] + h))));
+      }
+    } else {
+      pre_next = gather_sum<G, V, H, PEER>(a.col + e0, int(e1 - e0), pre, a.col + n0, int(n1 - n0), yb, rstride,
+                                           lok, lane, tot, a);
+    }
+    if (!skip) epilogue(row, tot, zi, ri);
     pre = pre_next;
+    }
+    if (inl) {
+      const int64_t sr = __shfl_sync(0xffffffffu, srow, 0);
+      const int64_t limit = (int64_t(nblk) + a.seg_ahead) * R;
+      if (sr < limit) seg_loop(limit);
     }
     blk = nblk;
     b ^= 1;
   }
+  if (inl) seg_loop(-1);  // the row stream is done: drain the remaining segments
+}
+
+// Multi-row pass for short rows (C5's mean selective degree
+// 31): each of the warp's S = 32/G edge slots owns one destination row of a
+// group of S consecutive plan rows, so a row costs no cross-slot reduction
+// and the per-row work (row pointers, ticket, epilogue) is shared by S rows.
+// A slot walks its row's edges in CSR order with one running sum (lane g
+// holds columns [8g, 8g+8) as one 32-byte vector): the summation order is
+// fixed, bitwise run to run.  The warp steps max(deg) over its S rows, so the
+// layout wants rows of similar degree next to each other (degree vertex
+// order, reading #24).  Index batches: lane g of a slot loads edge base+g of
+// its row (G indices per slot per load), one batch ahead; the next group's
+// row pointers and segment ids are loaded while the current group gathers,
+// and its first index batch is issued by the current group's last step.
+template <int G, bool HAS_ZD, bool HAS_SEG, bool PEER>
+__global__ void __launch_bounds__(256, 4) sparse_mrow_kernel(AggArgs a) {
+  constexpr int H = 2;
+  constexpr int S = 32 / G;
+  static_assert(G >= 4 && G <= 16, "multi-row layout: 2..8 slots");
+  const int lane = threadIdx.x & 31;
+  const int slot = lane / G, g = lane % G;
+  const int nvec = (a.F + 7) >> 3;  // <= G
+  const int nvec4 = (a.F + 3) >> 2;
+  const bool lok = g < nvec;
+  const char* yb = (PEER ? nullptr : reinterpret_cast<const char*>(a.Y)) + 32 * (lok ? g : 0);
+  const uint32_t rstride = uint32_t(a.ldy * 4);
+  const int64_t ngrp = (a.rows + S - 1) / S;
+  const int GPT = a.rows_per_ticket;  // groups per ticket
+  const int64_t ntk = (ngrp + GPT - 1) / GPT;
+  auto ticket = [&]() {
+    int t = 0;
+    if (lane == 0) t = atomicAdd(a.counter, 1);
+    return __shfl_sync(0xffffffffu, t, 0);
+  };
+  // group q: lane l <= S holds rowptr[q*S + l] (clamped to rows), every lane
+  // the segment id of its slot's row
+  auto load_grp = [&](int64_t q, int64_t& rp, int& sgv) {
+    rp = 0;
+    sgv = -1;
+    if (q < ngrp) {
+      if (lane <= S) {
+        const int64_t r = q * S + lane;
+        rp = __ldg(a.rowptr + (r < a.rows ? r : a.rows));
+      }
+      if (HAS_SEG) {
+        const int64_t r = q * S + slot;
+        sgv = r < a.rows ? __ldg(a.row_seg + r) : -1;
+      }
+    }
+  };
+  auto range = [&](int64_t rp, int sgv, int64_t& e0, int64_t& e1) {
+    e0 = __shfl_sync(0xffffffffu, rp, slot);
+    e1 = __shfl_sync(0xffffffffu, rp, slot + 1);
+    return (HAS_SEG && sgv >= 0) ? 0 : int(e1 - e0);
+  };
+  // epilogue of one row held by this lane's slot: + Zd, x r_i (twice if prescaled output), mask byte, ReLU
+  auto epilogue = [&](int64_t row, float4 (&acc)[H], int zi, float ri) {
+      uint32_t mbyte = 0;
+#pragma unroll
+      for (int h = 0; h < H; ++h) {
+        const int q4 = H * g + h;
+        const bool own = lok && q4 < nvec4;
+        float4 z = acc[h];
+        if (HAS_ZD && own && zi >= 0) add4(z, ld_f4(a.zd + int64_t(zi) * a.ldzd + 4 * q4));
+        z.x *= ri; z.y *= ri; z.z *= ri; z.w *= ri;
+        if (a.out_prescaled) { z.x *= ri; z.y *= ri; z.z *= ri; z.w *= ri; }
+        const int c = 4 * q4;
+        mbyte |= (uint32_t(z.x > 0.f && c + 0 < a.F) | uint32_t(z.y > 0.f && c + 1 < a.F) << 1 |
+                  uint32_t(z.z > 0.f && c + 2 < a.F) << 2 | uint32_t(z.w > 0.f && c + 3 < a.F) << 3)
+                 << (4 * h);
+        if (a.relu) {
+          z.x = fmaxf(z.x, 0.f); z.y = fmaxf(z.y, 0.f); z.z = fmaxf(z.z, 0.f); z.w = fmaxf(z.w, 0.f);
+        }
+        if (own) *reinterpret_cast<float4*>(a.Z + row * a.ldz + 4 * q4) = z;
+      }
+      if (a.mask) {  // byte g of the little-endian mask row = columns 8g..8g+7
+        uint8_t* mrow = reinterpret_cast<uint8_t*>(a.mask + row * a.mask_ld);
+        if (lok) mrow[g] = uint8_t(mbyte);
+        if (nvec + g < 4 * ((a.F + 31) >> 5)) mrow[nvec + g] = 0;
+      }
+  };
+  const bool inl = HAS_SEG && a.seg_inline;
+  // inline segments (see sparse_row_kernel): one segment of a long row gathered
+  // by the whole warp in the one-row layout (G lanes per edge slot, S slots);
+  // the warp completing the row's last segment adds the partials in segment
+  // order and runs the epilogue in slot 0
+  auto run_segment = [&](int sgi) {
+    const int64_t lo = a.seg_lo[sgi], hi = a.seg_hi[sgi];
+    const int n = int(hi - lo);
+    const int first = lane < n ? ld_col<PEER>(a.col + lo + lane, a) : 0;
+    const bool lk[1] = {lok};
+    float4 tot[1][H];
+    gather_sum<G, 1, H, PEER>(a.col + lo, n, first, nullptr, 0, yb, rstride, lk, lane, tot, a);
+    const int64_t row = a.seg_row[sgi];
+    const int s0 = a.row_seg[row];
+    const int ns = int((a.rowptr[row + 1] - a.rowptr[row] + SEG_EDGES - 1) / SEG_EDGES);
+    if (slot == 0 && lok) {
+#pragma unroll
+      for (int h = 0; h < H; ++h)
+        if (H * g + h < nvec4)
+          __stcg(reinterpret_cast<float4*>(a.seg_ws + int64_t(sgi) * a.ldws + 4 * (H * g + h)), tot[0][h]);
+    }
+    __threadfence();
+    __syncwarp();
+    int last = 0;
+    if (lane == 0) last = atomicAdd(a.seg_cnt + s0, 1) == ns - 1;
+    if (__shfl_sync(0xffffffffu, last, 0)) {
+      __threadfence();
+      float4 acc[H];
+#pragma unroll
+      for (int h = 0; h < H; ++h) acc[h] = make_float4(0.f, 0.f, 0.f, 0.f);
+      if (slot == 0 && lok) {
+        for (int k = 0; k < ns; ++k)
+#pragma unroll
+          for (int h = 0; h < H; ++h)
+            if (H * g + h < nvec4)
+              add4(acc[h], __ldcg(reinterpret_cast<const float4*>(a.seg_ws + int64_t(s0 + k) * a.ldws +
+                                                                 4 * (H * g + h))));
+      }
+      if (slot == 0) epilogue(row, acc, HAS_ZD ? a.zd_index[row] : -1, a.r[a.row_lo + row]);
+      if (lane == 0) a.seg_cnt[s0] = 0;
+    }
+  };
+  auto seg_loop = [&](int64_t limit) {
+    while (true) {
+      int sgi = 0;
+      if (lane == 0) sgi = atomicAdd(a.seg_ticket, 1);
+      sgi = __shfl_sync(0xffffffffu, sgi, 0);
+      if (sgi >= a.nseg) return;
+      run_segment(sgi);
+      if (limit >= 0) {
+        int go = 0;
+        if (lane == 0) {
+          const int pk = peek_ticket(a.seg_ticket);
+          go = pk < a.nseg && a.seg_row[pk] < limit;
+        }
+        if (!__shfl_sync(0xffffffffu, go, 0)) return;
+      }
+    }
+  };
+  int t = ticket();
+  if (t >= ntk) { if (inl) seg_loop(-1); return; }
+  int64_t q = int64_t(t) * GPT;
+  int64_t qend = q + GPT < ngrp ? q + GPT : ngrp;
+  int tn = ticket();  // the next block's ticket, consumed when this block ends
+  int64_t rp;
+  int sgv;
+  load_grp(q, rp, sgv);
+  int64_t e0, e1;
+  int n = range(rp, sgv, e0, e1);
+  int idx = g < n ? ld_col<PEER>(a.col + e0 + g, a) : 0;
+  while (true) {
+    int64_t qn;
+    bool newblk = false;
+    if (q + 1 < qend) {
+      qn = q + 1;
+    } else {
+      qn = int64_t(tn) * GPT;
+      newblk = true;
+    }
+    int64_t rpn;
+    int sgn;
+    load_grp(qn, rpn, sgn);  // in flight while this group gathers
+    int speek = a.nseg;
+    if (inl && newblk && lane == 0) speek = peek_ticket(a.seg_ticket);
+    const int64_t row = q * S + slot;
+    const bool valid = row < a.rows;
+    const float ri = valid ? __ldg(a.r + a.row_lo + row) : 0.f;
+    const int zi = (HAS_ZD && valid) ? __ldg(a.zd_index + row) : -1;
+    float4 acc[H];
+#pragma unroll
+    for (int h = 0; h < H; ++h) acc[h] = make_float4(0.f, 0.f, 0.f, 0.f);
+    const int nmax = __reduce_max_sync(0xffffffffu, n);
+    int64_t e0n = 0, e1n = 0;
+    int nn = 0;
+    for (int base = 0; base < nmax; base += G) {
+      const int cur = idx;
+      if (base + G < nmax) {
+        idx = (base + G + g < n) ? ld_col<PEER>(a.col + e0 + base + G + g, a) : 0;
+      } else {  // last step: the next group's first batch
+        nn = range(rpn, sgn, e0n, e1n);
+        idx = g < nn ? ld_col<PEER>(a.col + e0n + g, a) : 0;
+      }
+#pragma unroll
+      for (int u0 = 0; u0 < G; u0 += 4) {
+        float4 buf[4][H];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const uint32_t j = uint32_t(__shfl_sync(0xffffffffu, cur, slot * G + u0 + u));
+          if (lok && base + u0 + u < n) {
+            ld_vec<H>(src_row<PEER>(yb, j, rstride, a), buf[u]);
+          } else {
+#pragma unroll
+            for (int h = 0; h < H; ++h) buf[u][h] = make_float4(0.f, 0.f, 0.f, 0.f);
+          }
+        }
+#pragma unroll
+        for (int u = 0; u < 4; ++u)
+#pragma unroll
+          for (int h = 0; h < H; ++h) add4(acc[h], buf[u][h]);
+        if (base + u0 + 4 >= nmax) break;  // warp-uniform: the rest of the batch is past every row
+      }
+    }
+    if (nmax == 0) {
+      nn = range(rpn, sgn, e0n, e1n);
+      idx = g < nn ? ld_col<PEER>(a.col + e0n + g, a) : 0;
+    }
+    if (HAS_SEG && !inl && sgv >= 0 && lok) {  // long row: its segment partials in segment order
+      const int ns = int((e1 - e0 + SEG_EDGES - 1) / SEG_EDGES);
+      for (int k = 0; k < ns; ++k)
+#pragma unroll
+        for (int h = 0; h < H; ++h)
+          if (H * g + h < nvec4)
+            add4(acc[h], __ldcg(reinterpret_cast<const float4*>(a.seg_ws + int64_t(sgv + k) * a.ldws +
+                                                               4 * (H * g + h))));
+    }
+    if (valid && !(inl && sgv >= 0)) epilogue(row, acc, zi, ri);  // inline: a long row is written by its last segment
+    if (inl && newblk) {
+      int64_t sr = INT64_MAX;
+      if (lane == 0 && speek < a.nseg) sr = a.seg_row[speek];
+      sr = __shfl_sync(0xffffffffu, sr, 0);
+      const int64_t limit = (qn / GPT + a.seg_ahead) * int64_t(GPT) * S;
+      if (sr < limit) seg_loop(limit);
+    }
+    if (qn >= ngrp) {
+      if (inl) seg_loop(-1);
+      break;
+    }
+    q = qn;
+    if (newblk) {
+      qend = q + GPT < ngrp ? q + GPT : ngrp;
+      tn = ticket();
+    }
+    rp = rpn;
+    sgv = sgn;
+    e0 = e0n;
+    e1 = e1n;
+    n = nn;
+  }
+}
+
+constexpr float MROW_MAX_DEG = 64.f;
+
+template <int G, bool PEER>
+cudaError_t launch_mrow(const AggArgs& a, cudaStream_t s) {
+  static int slots = 0;
+  if (!slots) {
+    int dev = 0, sms = 148, per = 4;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, sparse_mrow_kernel<G, true, true, PEER>, 256, 0);
+    slots = sms * (per > 0 ? per : 1);
+  }
+  const bool inl = a.nseg > 0 && a.phase == 0 && a.seg_row && knobs_seg_inline();
+  if (a.nseg > 0 && a.phase != 2 && !inl) {
+    sparse_seg_kernel<G, 1, 2, PEER><<<unsigned((a.nseg + 3) / 4), 128, 0, s>>>(a);
+    if (a.phase == 1) return cudaGetLastError();
+  }
+  // row ticket counter[0] and (inline segments) segment ticket counter[8]
+  cudaError_t e = cudaMemsetAsync(a.counter, 0, (inl ? 9 : 1) * sizeof(int), s);
+  if (e != cudaSuccess) return e;
+  constexpr int S = 32 / G;
+  AggArgs b = a;
+  b.rows_per_ticket = knobs_mrow_gpt();  // groups of S rows per ticket
+  const int64_t ntk = ((a.rows + S - 1) / S + b.rows_per_ticket - 1) / b.rows_per_ticket;
+  const int64_t want = (ntk + 7) / 8;
+  const unsigned grid = unsigned(want < slots ? want : slots);
+  b.seg_inline = inl ? 1 : 0;
+  b.seg_ahead = int64_t(grid) * 8 * knobs_seg_ahead();
+#define LAUNCH(ZD, SG) sparse_mrow_kernel<G, ZD, SG, PEER><<<grid, 256, 0, s>>>(b)
+  const bool zd = a.zd_index != nullptr, sg = a.nseg > 0;
+  if (zd && sg) LAUNCH(true, true);
+  else if (zd) LAUNCH(true, false);
+  else if (sg) LAUNCH(false, true);
+  else LAUNCH(false, false);
+#undef LAUNCH
+  return cudaGetLastError();
 }
 
 template <int G, int V, int H, bool PEER>
@@ -488,15 +871,20 @@ cudaError_t launch_gvp(const AggArgs& a, cudaStream_t s) {
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, sparse_row_kernel<G, V, H, true, true, PEER>, 256, 0);
     slots = sms * (per > 0 ? per : 1);
   }
-  if (a.nseg > 0 && a.phase != 2) {
+  const bool inl = a.nseg > 0 && a.phase == 0 && a.seg_row && knobs_seg_inline();
+  if (a.nseg > 0 && a.phase != 2 && !inl) {
     sparse_seg_kernel<G, V, H, PEER><<<unsigned((a.nseg + 3) / 4), 128, 0, s>>>(a);
     if (a.phase == 1) return cudaGetLastError();
   }
-  cudaError_t e = cudaMemsetAsync(a.counter, 0, sizeof(int), s);
+  // row ticket counter[0] and (inline segments) segment ticket counter[8]
+  cudaError_t e = cudaMemsetAsync(a.counter, 0, (inl ? 9 : 1) * sizeof(int), s);
   if (e != cudaSuccess) return e;
   const int64_t want = ((a.rows + a.rows_per_ticket - 1) / a.rows_per_ticket + 7) / 8;
   const unsigned grid = unsigned(want < slots ? want : slots);
-#define LAUNCH(ZD, SG) sparse_row_kernel<G, V, H, ZD, SG, PEER><<<grid, 256, 0, s>>>(a)
+  AggArgs b = a;
+  b.seg_inline = inl ? 1 : 0;
+  b.seg_ahead = int64_t(grid) * 8 * knobs_seg_ahead();
+#define LAUNCH(ZD, SG) sparse_row_kernel<G, V, H, ZD, SG, PEER><<<grid, 256, 0, s>>>(b)
   const bool zd = a.zd_index != nullptr, sg = a.nseg > 0;
   if (zd && sg) LAUNCH(true, true);
   else if (zd) LAUNCH(true, false);
@@ -596,8 +984,9 @@ __global__ void __launch_bounds__(256) split_window_kernel(const float* __restri
   }
   __syncthreads();
   const int k = tx;  // source within the window
-  if (mode == 2) {
-    uint16_t* out = reinterpret_cast<uint16_t*>(blk + w * int64_t(npad) * 48);  // 3 parts x npad x 64 B
+  if (mode == 2 || mode == 3) {  // 3 bf16 parts (BF16X3) or the first only (BF16X1)
+    const int parts = mode == 2 ? 3 : 1;
+    uint16_t* out = reinterpret_cast<uint16_t*>(blk + w * int64_t(npad) * 16 * parts);  // parts x npad x 64 B
     for (int ff = ty; ff < 32; ff += 8) {
       const int f = f0 + ff;
       if (f >= npad) continue;
@@ -608,8 +997,10 @@ __global__ void __launch_bounds__(256) split_window_kernel(const float* __restri
       const uint32_t h2 = bf16_rn_bits(r1 - __uint_as_float(h1));
       const int pos = f * 32 + ((((k >> 3) ^ ((f >> 1) & 3)) << 3) | (k & 7));  // bf16 element offset
       out[pos] = uint16_t(h0 >> 16);
-      out[npad * 32 + pos] = uint16_t(h1 >> 16);
-      out[2 * npad * 32 + pos] = uint16_t(h2 >> 16);
+      if (parts == 3) {
+        out[npad * 32 + pos] = uint16_t(h1 >> 16);
+        out[2 * npad * 32 + pos] = uint16_t(h2 >> 16);
+      }
     }
     return;
   }
@@ -653,17 +1044,31 @@ struct SparseKnobs {
   int fsplit = 0;
   bool v8 = true;
   bool g6 = true;  // PCGCN_SPARSE_G6=0: F = 41..48 keeps the 16-byte G = 16 layout (A/B)
+  // PCGCN_SPARSE_MROW: -1 (default) multi-row warps for 17..64 features when the
+  // plan's mean selective degree is <= MROW_MAX_DEG; 0 never; 1 wherever the layout fits
+  int mrow = -1;
+  int mrow_gpt = 4;  // PCGCN_MROW_GPT: groups per ticket
+  int seg_inline = 1;
+  int seg_ahead = 1;
   SparseKnobs() {
+    if (const char* e = getenv("PCGCN_SEG_INLINE")) seg_inline = atoi(e);
+    if (const char* e = getenv("PCGCN_SEG_AHEAD")) seg_ahead = std::max(1, atoi(e));
+    if (const char* e = getenv("PCGCN_SPARSE_MROW")) mrow = atoi(e);
+    if (const char* e = getenv("PCGCN_MROW_GPT")) mrow_gpt = std::max(1, atoi(e));
     if (const char* e = getenv("PCGCN_SPARSE_FSPLIT")) fsplit = atoi(e) / 32 * 32;
     if (const char* e = getenv("PCGCN_SPARSE_V8")) v8 = atoi(e) != 0;
     if (const char* e = getenv("PCGCN_SPARSE_G6")) g6 = atoi(e) != 0;
   }
 };
 
+
 static SparseKnobs& knobs() {
   static SparseKnobs k;
   return k;
 }
+int knobs_mrow_gpt() { return knobs().mrow_gpt; }
+int knobs_seg_inline() { return knobs().seg_inline; }
+int knobs_seg_ahead() { return knobs().seg_ahead; }
 
 bool sparse_fsplit_active(int F) { return knobs().fsplit > 0 && F > knobs().fsplit; }
 
@@ -699,6 +1104,12 @@ cudaError_t launch_sparse_pass(const AggArgs& a, cudaStream_t s) {
   // 32-byte vectors per row read the row's 192 bytes (6 sectors, as many as the
   // 44 floats of the 16-byte layout touch) with 5 rows per load instruction
   if (al32 && knobs().g6 && (a.F + 7) / 8 == 6) return launch_gv<6, 1, 2>(a, s);
+  // short rows (mean selective degree <= MROW_MAX_DEG): one row per edge slot
+  if (v8 && knobs().mrow != 0 && (knobs().mrow > 0 || a.mean_deg <= MROW_MAX_DEG)) {
+    const int nvec = (a.F + 7) / 8;
+    if (nvec >= 3 && nvec <= 4) return a.peer_world > 0 ? launch_mrow<4, true>(a, s) : launch_mrow<4, false>(a, s);
+    if (nvec >= 5 && nvec <= 8) return a.peer_world > 0 ? launch_mrow<8, true>(a, s) : launch_mrow<8, false>(a, s);
+  }
   if (v8) {
     const int nvec = (a.F + 7) / 8;
     if (nvec <= 1) return launch_gv<1, 1, 2>(a, s);

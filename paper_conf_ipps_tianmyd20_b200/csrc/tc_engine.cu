@@ -61,19 +61,19 @@ struct Layout {
   uint32_t tmem_cols, a_col0;
 };
 
-Layout make_layout(int mode, int npad, int max_stages, int max_u, bool b_raw = false, bool bf3 = false) {
+Layout make_layout(int mode, int npad, int max_stages, int max_u, bool b_raw = false, int bfp = 0) {
   Layout L;
   L.raw_bytes = (mode == A_TRANS && b_raw) ? uint32_t(npad) * BK * 4 : 0u;
   L.npad = npad;
   L.b_bytes = uint32_t(npad) * BK * 4;
-  // bf16x3 full mode: three K-major SW64 parts of npad rows x 64 B; else hi + lo tf32 (128 B rows)
-  L.bchunk = bf3 ? 3u * uint32_t(npad) * 64u : 2u * L.b_bytes;
+  // bf16 full modes: bfp (3: BF16X3, 1: BF16X1) K-major SW64 parts of npad rows x 64 B; else hi + lo tf32 (128 B rows)
+  L.bchunk = bfp ? uint32_t(bfp) * uint32_t(npad) * 64u : 2u * L.b_bytes;
   // transform GEMM outputs (N x npad rows, HBM-bound at scale) leave through a
   // shared-memory transpose so each store instruction writes whole row pieces
   L.out_bytes = (mode == A_ROWMAJOR && npad <= 128) ? 4u * 32u * (64u + 4u) * 4u : 0u;
   for (int U = (mode == A_BITS ? max_u : 1); U >= 1; U = U > 1 ? U / 2 : 0) {
     L.U = U;
-    L.a_cols = mode == A_BITS ? U * (bf3 ? BK / 2 : BK) : 2 * BK;
+    L.a_cols = mode == A_BITS ? U * (bfp ? BK / 2 : BK) : 2 * BK;
     L.a_bytes = mode == A_BITS ? uint32_t((U * BM * 4 + 1023) / 1024 * 1024) : BM * BK * 4;
     L.a_load_bytes = mode == A_BITS ? BM * 4 : BM * BK * 4;  // per chunk
     L.stage_bytes = L.a_bytes + uint32_t(U) * L.bchunk + L.raw_bytes;
@@ -126,14 +126,14 @@ struct Work {
   int64_t split_stride;
   int b_fused;       // B lo rows follow the hi rows in memory: one TMA box {32, 2*npad} per chunk
   int single;        // A_BITS: B hi only (bf16-rounded input), one MMA per K-step (PCGCN_DENSE_BF16X1)
-  int bf3;           // A_BITS: kind::f16, B = three bf16 parts (PCGCN_DENSE_BF16X3), window blocks only
+  int bf3;           // A_BITS: bf16 parts of B (kind::f16; 3: PCGCN_DENSE_BF16X3, 1: BF16X1; 0: tf32), window blocks only
   const int32_t* order;  // A_BITS: tile processed at position t (nullptr: t itself)
   int* dyn;              // A_BITS: tile ticket counter (zeroed before the launch): CTAs claim positions
                          // dynamically, in order, through a smem ring (nullptr: static round robin)
   const float* bblk;     // A_BITS: source-window blocks of B (pre-swizzled); nullptr: TMA boxes
   int64_t bblk_stride;   // floats per window block
   float* wblk;       // A_ROWMAJOR: also write the output as full-mode window blocks (fused split)
-  int wmode;         // 1: tf32 hi/lo (SW128, 2·npad rows), 2: bf16-rounded (BF16X1), 3: bf16x3 (SW64 parts)
+  int wmode;         // 1: tf32 hi/lo (SW128, 2·npad rows), 3: bf16x3 (three SW64 parts), 4: bf16x1 (one SW64 part)
   int64_t wblk_floats, wblk_nwin;  // floats per window block; windows in the buffer
   int b_raw;         // A_TRANS: B = row-major D box; the builders split + transpose it into the
                      // K-major SWIZZLE_128B hi/lo layout in smem (no feature-major pre-split pass)
@@ -340,14 +340,15 @@ __global__ void __launch_bounds__(NTHREADS, 1)
           const uint32_t sa = tmem + L.a_col0 + uint32_t(s) * uint32_t(L.a_cols);
           for (int u = 0; u < nu; ++u) {
             if (MODE == A_BITS && w.bf3) {
-              // A (0/1 as bf16, 16 TMEM columns) against the 3 bf16 parts of the
-              // window: 2 K=16 MMAs per part, fp32 accumulation in TMEM
+              // A (0/1 as bf16, 16 TMEM columns) against the bf16 parts of the
+              // window (3, or 1 for BF16X1): 2 K=16 MMAs per part, fp32 accumulation in TMEM
               const uint32_t b0 = sb + uint32_t(u) * L.bchunk;
               const uint32_t a0 = sa + uint32_t(u) * (BK / 2);
 #pragma unroll
               for (int part = 0; part < 3; ++part)
 #pragma unroll
                 for (int kk = 0; kk < 2; ++kk) {
+                  if (part >= w.bf3) break;
                   const uint64_t bd = sdesc_kmajor_sw64(b0 + uint32_t(part) * uint32_t(npad) * 64u + kk * 32u);
                   mma_ts_f16(d, a0 + kk * 8u, bd, idesc, acc);
                   acc = 1u;
@@ -583,7 +584,7 @@ __global__ void __launch_bounds__(NTHREADS, 1)
                 for (int fh = 0; fh < 64; fh += 32) {
                   const int f = h + fh + lane;
                   if (f >= npad) continue;
-                  if (w.wmode == 3) {
+                  if (w.wmode >= 3) {
                     uint16_t* b16 = reinterpret_cast<uint16_t*>(blk);
 #pragma unroll
                     for (int j = 0; j < 4; ++j) {  // sources 8j..8j+7: one 16-byte chunk per part
@@ -610,8 +611,10 @@ __global__ void __launch_bounds__(NTHREADS, 1)
                       }
                       const int pos = f * 32 + ((j ^ ((f >> 1) & 3)) << 3);
                       *reinterpret_cast<uint4*>(b16 + pos) = make_uint4(p0[0], p0[1], p0[2], p0[3]);
-                      *reinterpret_cast<uint4*>(b16 + npad * 32 + pos) = make_uint4(p1[0], p1[1], p1[2], p1[3]);
-                      *reinterpret_cast<uint4*>(b16 + 2 * npad * 32 + pos) = make_uint4(p2[0], p2[1], p2[2], p2[3]);
+                      if (w.wmode == 3) {
+                        *reinterpret_cast<uint4*>(b16 + npad * 32 + pos) = make_uint4(p1[0], p1[1], p1[2], p1[3]);
+                        *reinterpret_cast<uint4*>(b16 + 2 * npad * 32 + pos) = make_uint4(p2[0], p2[1], p2[2], p2[3]);
+                      }
                     }
                   } else {
 #pragma unroll
@@ -743,7 +746,7 @@ template <int MODE>
 cudaError_t launch_engine(const CUtensorMap& bhi, const CUtensorMap& blo, const CUtensorMap& amap, const Work& w,
                           int npad, cudaStream_t s) {
   if (w.ntiles <= 0) return cudaSuccess;
-  const Layout L = make_layout(MODE, npad, max_stages_env(), max_u_env(), w.b_raw != 0, w.bf3 != 0);
+  const Layout L = make_layout(MODE, npad, max_stages_env(), max_u_env(), w.b_raw != 0, w.bf3);
   const size_t smem = 1024 + size_t(L.stages) * L.stage_bytes + L.out_bytes + (3 * L.stages + 4 + 2 * TQ) * 8 + 16 +
                      TQ * 8;
   if (smem > 227 * 1024) return cudaErrorInvalidValue;

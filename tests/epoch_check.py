@@ -189,10 +189,25 @@ def check_gcnl_epoch(model, ref: OracleEpochL, perm, lr=None, report=None):
     return errs
 
 
-def check_gcn2_epoch(model, ref: OracleEpoch, perm, lr=None, Th0=None, Th1=None, report=None):
+# bf16x1 full mode (PCGCN_DENSE_BF16X1, the paper's 16-bit tensor-core policy,
+# L191-L193): each full-mode term carries the bf16 rounding of its input,
+# |δ| <= 2^-9 |Y'|, so every aggregation is within 2^-9 of its condition scale
+# and the epoch's outputs within a few of those (four aggregations compound):
+# the north star's stated 2e-2 gate; ReLU decisions within 2^-8·s_P1 of zero are
+# ambiguous at that error, and the band may hold a few percent of them.
+TOL_BF16 = 2e-2
+BAND_BF16 = 2.0 ** -8
+BAND_FRAC_BF16 = 0.05
+
+
+def check_gcn2_epoch(model, ref: OracleEpoch, perm, lr=None, Th0=None, Th1=None, report=None, tol=TOL,
+                     band_rel=BAND, band_frac=1e-3):
     """Compare a GCN2 (one epoch already run, eager or graph replay) with the
     oracle epoch.  ``lr``/``Th0``/``Th1``: also check the SGD update the model
-    applied, (Θ - Θ')/lr = ∇Θ.  Returns the dict of condition-scaled errors."""
+    applied, (Θ - Θ')/lr = ∇Θ.  ``tol``/``band_rel``/``band_frac``: the gate,
+    the ReLU ambiguity band and its non-vacuity cap (TOL_BF16 / BAND_BF16 /
+    BAND_FRAC_BF16 for the bf16x1 full mode).  Returns the dict of
+    condition-scaled errors."""
     inv = np.argsort(perm)
     H, C = ref.Th0.shape[1], ref.Th1.shape[1]
 
@@ -206,7 +221,7 @@ def check_gcn2_epoch(model, ref: OracleEpoch, perm, lr=None, Th0=None, Th1=None,
     errs["G1"] = cerr(up(model.G1, C), O.aggregate(ref.Ahat, ref.dL), ref.sG1)
     # ReLU decisions
     gbits = mask_bits(model.mask1, H, inv)
-    band = np.abs(ref.P1) <= BAND * ref.sP1
+    band = np.abs(ref.P1) <= band_rel * ref.sP1
     outside_ok = (gbits == (ref.P1 > 0)) | band
     assert outside_ok.all(), f"{int((~outside_ok).sum())} ReLU decisions differ outside the error band"
     amb = np.argwhere(band)
@@ -219,7 +234,7 @@ def check_gcn2_epoch(model, ref: OracleEpoch, perm, lr=None, Th0=None, Th1=None,
                 P1v[i, f] = 1e-300 if (bits >> t) & 1 else -1e-300
             variants.append(P1v)
     else:
-        assert band.mean() <= 1e-3, f"ReLU band holds {band.mean():.2e} of the decisions: vacuous check"
+        assert band.mean() <= band_frac, f"ReLU band holds {band.mean():.2e} of the decisions: vacuous check"
         variants.append(np.where(band, np.where(gbits, 1e-300, -1e-300), ref.P1))
     gTh1 = _np(model.gTh1)
     errs["gTh1"] = cerr(gTh1, ref.H1.T @ O.aggregate(ref.Ahat, ref.dL), ref.s_gTh1)
@@ -244,8 +259,9 @@ def check_gcn2_epoch(model, ref: OracleEpoch, perm, lr=None, Th0=None, Th1=None,
         errs["sgd_step"] = cerr((th - new) / lr, g, np.abs(th) / lr + np.abs(g))
     if report is not None:
         report.update(errs)
+    errs["relu_band_frac"] = float(band.mean())
     for k in ("H1", "L", "loss", "G1", "gTh1", "G0", "gTh0"):
-        assert errs[k] <= TOL, (k, errs)
+        assert errs[k] <= tol, (k, errs)
     if lr is not None:
         assert errs["sgd_step"] <= 1e-6, errs
     return errs

@@ -1,8 +1,8 @@
-"""Full (not extrapolated) fp64 oracle epoch on the host cores, once with BLAS
+"""Test infrastructure (imports oracle/, so it lives under tests/).  Full (not extrapolated) fp64 oracle epoch on the host cores, once with BLAS
 limited to 1 thread and once with all cores (SURVEY.md
 §8(d) "Oracle timing beside the GPU").  Prints one JSON line per workload.
 
-    python scripts/oracle_epoch_time.py [cora pubmed reddit]
+    python tests/oracle_epoch_time.py [cora pubmed reddit]
 """
 import json
 import os

@@ -83,7 +83,7 @@ SMALL = {
 @pytest.mark.parametrize("name", list(SMALL))
 @pytest.mark.parametrize("mode", ["sparse", "dense_tc", "dense_simt", "hybrid", "dense_bf16", "hybrid_tile",
                                   "dense_bf3", "hybrid_tile_bf3"])
-@pytest.mark.parametrize("F", [1, 7, 16, 33, 41, 48, 64, 128])
+@pytest.mark.parametrize("F", [1, 7, 16, 24, 32, 33, 40, 41, 48, 64, 128])
 def test_aggregation_parity(name, mode, F):
     g = SMALL[name]()
     P = max(1, min(8, g.n // 40))
@@ -614,13 +614,21 @@ np.savez(sys.argv[1], **out)
                                           ({"PCGCN_SPARSE_V8": "0"}, False),
                                           ({"PCGCN_SPARSE_FSPLIT": "32"}, False),
                                           ({"PCGCN_SPARSE_G6": "0"}, False),
-                                          ({"PCGCN_TC_DYN": "0"}, True)])
+                                          ({"PCGCN_TC_DYN": "0"}, True),
+                                          ({"PCGCN_SPARSE_MROW": "0"}, False),
+                                          ({"PCGCN_SPARSE_MROW": "1"}, False),
+                                          ({"PCGCN_MROW_GPT": "1"}, True),
+                                          ({"PCGCN_SEG_INLINE": "0"}, True),
+                                          ({"PCGCN_SEG_AHEAD": "64"}, True)])
 def test_scheduling_knobs_do_not_change_results(tmp_path, knob, bitwise):
-    """Row-block tickets, the full-mode/segment overlap, the in-kernel xtg B
+    """Row-block tickets, inline vs separate long-row segments (the same
+    partials added in the same order), the full-mode/segment overlap, the in-kernel xtg B
     conversion and the window-blocked full-mode B layout change only scheduling (every output row is still reduced by
     one warp in the same order; the MMA sequence and the hi/lo split are the
     same), so aggregation outputs, masks, gradients and the loss must be
-    bitwise identical to the default configuration."""
+    bitwise identical to the default configuration.  The lane-layout knobs
+    (16- vs 32-byte vectors, column slices, G = 6, multi-row warps) sum a row in
+    another fixed order: within 2e-6 of the largest output, masks self-consistent."""
     import os
     import subprocess
     import sys
@@ -653,7 +661,8 @@ def test_scheduling_knobs_do_not_change_results(tmp_path, knob, bitwise):
 
 
 @pytest.mark.parametrize("wname,theta,dense", [("cora", 0.01, "tf32x2"), ("pubmed", 0.0, "bf16x3"),
-                                               ("cora", 0.005, "bf16x3"), ("pubmed", 2.0, "tf32x2")])
+                                               ("cora", 0.005, "bf16x3"), ("pubmed", 2.0, "tf32x2"),
+                                               ("cora", 0.005, "bf16x1"), ("pubmed", 0.01, "bf16x1")])
 def test_fused_split_is_bitwise(wname, theta, dense):
     """pcgcn_gemm_xw_split / pcgcn_gemm_dwt_split write the full mode's window
     blocks in the GEMM epilogue and the aggregations then skip their split pass
@@ -666,7 +675,7 @@ def test_fused_split_is_bitwise(wname, theta, dense):
     Th0, Th1 = C.thetas(w)
     T = C.train_mask(g.n, w.theta_seed)
     kw = dict(order=L.ORDER_DEGREE, grain=L.GRAIN_TILE,
-              dense_prec=L.DENSE_BF16X3 if dense == "bf16x3" else L.DENSE_TF32X2)
+              dense_prec={"bf16x3": L.DENSE_BF16X3, "bf16x1": L.DENSE_BF16X1}.get(dense, L.DENSE_TF32X2))
     pl = L.Plan(g.n, g.rowptr, g.col, w.P, theta, **kw)
     pl_c = L.Plan(g.n, g.rowptr, g.col, w.P, theta * 2 if theta < 1 else theta, **kw)
     perm = pl.perm()

@@ -78,6 +78,35 @@ def test_c3_bench_epoch_all_rows(c3_epoch, theta, theta_c, cfg):
     print("c3 bench epoch", theta, theta_c, cfg, rep)
 
 
+@pytest.mark.parametrize("theta,theta_c", [(0.02, 0.03), (0.01, 0.015)])
+def test_c3_bench_epoch_bf16x1(c3_epoch, theta, theta_c):
+    """bench.py --dense bf16x1 (the paper's 16-bit full mode, L191-L193): the
+    same launch configuration with bf16-rounded full-mode inputs, all rows of
+    every epoch output vs the fp64 oracle at the north star's stated bf16 gate
+    (2e-2, condition-scaled; tests/epoch_check.py TOL_BF16) — and the fp32
+    selective part keeps the error well inside it."""
+    from paper_conf_ipps_tianmyd20_b200.gcn import GCN2
+    from epoch_check import check_gcn2_epoch, TOL_BF16, BAND_BF16, BAND_FRAC_BF16
+    w, g, X, Th0, Th1, y, T, ref = c3_epoch
+    kw = dict(f_max=max(w.hidden, w.classes), order=L.ORDER_DEGREE, grain=L.GRAIN_TILE,
+              dense_prec=L.DENSE_BF16X1)
+    pl = L.Plan(g.n, g.rowptr, g.col, w.P, theta, **kw)
+    pl_c = L.Plan(g.n, g.rowptr, g.col, w.P, theta_c, **kw)
+    assert pl.stats()["nnz_dense"] > 0 and pl_c.stats()["nnz_dense"] > 0
+    perm = pl.perm()
+    model = GCN2(pl, np.ascontiguousarray(X[perm]), y[perm], T[perm], Th0, Th1, optimizer="sgd", lr=0.1,
+                 plan_c=pl_c)
+    model.capture(warmup=0)
+    model.replay()
+    torch.cuda.synchronize()
+    rep = {}
+    check_gcn2_epoch(model, ref, perm, lr=0.1, Th0=Th0, Th1=Th1, report=rep, tol=TOL_BF16, band_rel=BAND_BF16,
+                     band_frac=BAND_FRAC_BF16)
+    print("c3 bench epoch bf16x1", theta, theta_c, rep)
+    # the bf16 rounding is the only error above fp32 level: it must show, and stay bounded
+    assert max(rep[k] for k in ("H1", "L", "G1", "G0")) <= 2.0 ** -6
+
+
 @pytest.fixture(scope="module")
 def c4s():
     """C4 (tiered SBM, BASELINE configs[3]) at 1/16 scale: 262K vertices,
