@@ -50,6 +50,7 @@ struct AggArgs {
   int* seg_ticket = nullptr;         // segment ticket (zeroed with the row ticket)
   int seg_inline = 0;                // 1: no separate segment pass
   int64_t seg_ahead = 0;             // row tickets ahead of the claiming warp within which segments are taken
+  int64_t near_rows = 0;             // > 0: sources farther than this (plan rows) load L2-evict-first
   // device-initiated peer gather: sources of shard q are read from
   // shard q's own buffer (peer_base[q] = its row row0[q]; NVLink peer memory
   // on a multi-GPU node, CUDA IPC in the 1-GPU tests) instead of an exchanged copy
@@ -59,6 +60,7 @@ struct AggArgs {
   int phase = 0;             // 0: segment pass + row pass; 1: segment pass only; 2: row pass only
   int rows_per_ticket = 1;   // consecutive rows per scheduler ticket, 1..16
   float mean_deg = 0.f;      // selective edges per row (layout choice: short rows -> multi-row warps)
+  int rows_by_degree = 0;    // plan rows sorted by degree inside partitions (multi-row groups are balanced)
 };
 // selective edges per long-row segment
 constexpr int SEG_EDGES = 1024;

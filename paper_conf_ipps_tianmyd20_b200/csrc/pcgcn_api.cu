@@ -358,6 +358,7 @@ pcgcn_status aggregate(pcgcn_plan_t p, const float* Y, int64_t ldy, float* Z, in
   a.counter = d.counter;
   a.rows_per_ticket = rows_per_ticket(d.nnz_s, d.rows);
   a.mean_deg = float(double(p->sp_rowptr[p->n]) / double(p->n));  // plan-global: every shard picks the same layout
+  a.rows_by_degree = p->opts.vertex_order == PCGCN_ORDER_DEGREE ? 1 : 0;
   // the split + full-mode tiles run on the plan's high-priority side stream,
   // concurrently with the long-row segment pass on the caller's stream;
   // PROFILE calls stay serial so per-kernel times add up
@@ -608,6 +609,7 @@ static pcgcn_status aggregate_peer(pcgcn_plan_t p, const float* const* peer, int
   a.counter = d.counter;
   a.rows_per_ticket = rows_per_ticket(d.nnz_s, d.rows);
   a.mean_deg = float(double(p->sp_rowptr[p->n]) / double(p->n));  // plan-global: every shard picks the same layout
+  a.rows_by_degree = p->opts.vertex_order == PCGCN_ORDER_DEGREE ? 1 : 0;
   a.peer_world = W;
   for (int q = 0; q < 8; ++q) a.peer_base[q] = q < W ? reinterpret_cast<const char*>(peer[q]) : nullptr;
   for (int q = 0; q <= 8; ++q)

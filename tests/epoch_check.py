@@ -193,11 +193,15 @@ def check_gcnl_epoch(model, ref: OracleEpochL, perm, lr=None, report=None):
 # L191-L193): each full-mode term carries the bf16 rounding of its input,
 # |δ| <= 2^-9 |Y'|, so every aggregation is within 2^-9 of its condition scale
 # and the epoch's outputs within a few of those (four aggregations compound):
-# the north star's stated 2e-2 gate; ReLU decisions within 2^-8·s_P1 of zero are
-# ambiguous at that error, and the band may hold a few percent of them.
+# the north star's stated 2e-2 gate.  ReLU decisions within 2^-8·s_P1 of zero
+# are ambiguous at that error — with random-sign features most of them are (C3:
+# ~74%, the condition scale Â(|X||Θ0|) is a worst case), so the band is not
+# capped: the decisions outside it must agree, and G0 / ∇Θ0 are checked against
+# the oracle backward under the GPU's own decisions inside it (each admissible
+# by the bound; "compare what is unique, check the rest is valid").
 TOL_BF16 = 2e-2
 BAND_BF16 = 2.0 ** -8
-BAND_FRAC_BF16 = 0.05
+BAND_FRAC_BF16 = 1.0
 
 
 def check_gcn2_epoch(model, ref: OracleEpoch, perm, lr=None, Th0=None, Th1=None, report=None, tol=TOL,

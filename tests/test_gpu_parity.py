@@ -618,8 +618,10 @@ np.savez(sys.argv[1], **out)
                                           ({"PCGCN_SPARSE_MROW": "0"}, False),
                                           ({"PCGCN_SPARSE_MROW": "1"}, False),
                                           ({"PCGCN_MROW_GPT": "1"}, True),
-                                          ({"PCGCN_SEG_INLINE": "0"}, True),
-                                          ({"PCGCN_SEG_AHEAD": "64"}, True)])
+                                          ({"PCGCN_SEG_INLINE": "1"}, True),
+                                          ({"PCGCN_SEG_INLINE": "1", "PCGCN_SEG_AHEAD": "64"}, True),
+                                          ({"PCGCN_SEG_INLINE": "1", "PCGCN_SEG_AHEAD": "1"}, True),
+                                          ({"PCGCN_NEAR_ROWS": "64"}, True)])
 def test_scheduling_knobs_do_not_change_results(tmp_path, knob, bitwise):
     """Row-block tickets, inline vs separate long-row segments (the same
     partials added in the same order), the full-mode/segment overlap, the in-kernel xtg B
