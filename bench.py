@@ -65,7 +65,43 @@ def parse():
     ap.add_argument("--f3-seeds", type=int, default=3, help="F3: initialisations")
     ap.add_argument("--table3", action="store_true",
                     help="Table III replica on RMAT-{0.1..10}: epoch ms of PCGCN-sel / -full / hybrid")
+    ap.add_argument("--calib-curve", default="",
+                    help="calibration curve (SURVEY §8(d)): 'F1,F2,..' widths; T_s(ρ), T_f per full-mode precision")
     return ap.parse_args()
+
+
+def run_calib_curve(args):
+    """The L161 calibration generalised to a curve: synthetic
+    2048-row partition blocks joined by random bipartite blocks of density ρ,
+    timed once all-selective (T_s) and once with the ρ-blocks in the full mode
+    (T_f), per width F and full-mode precision; the break-even density is where
+    T_s(ρ) = T_f (the θ L161 predicts from one point is T_f·p/T_s)."""
+    from paper_conf_ipps_tianmyd20_b200 import _lib as L
+    Fs = [int(x) for x in args.calib_curve.split(",")]
+    dens = (0.0025, 0.005, 0.01, 0.02, 0.03, 0.05, 0.1, 0.2, 0.5)
+    precs = {"bf16x3": L.DENSE_BF16X3, "bf16x1": L.DENSE_BF16X1, "tf32x2": L.DENSE_TF32X2}
+    rows = []
+    for pname in ("bf16x3", "bf16x1"):
+        for F in Fs:
+            pts = []
+            for rho in dens:
+                th, tf, ts = L.calibrate(F, 2048, rho, dense_prec=precs[pname])
+                pts.append({"rho": rho, "T_full_ms": tf, "T_sel_ms": ts, "theta_L161": th})
+                log(f"[calib] {pname} F={F} rho={rho} T_f={tf:.4f} T_s={ts:.4f} theta={th:.4f}")
+            # break-even: first density where the full mode is not slower (linear interpolation)
+            be = None
+            for a, b in zip(pts, pts[1:]):
+                da, db = a["T_sel_ms"] - a["T_full_ms"], b["T_sel_ms"] - b["T_full_ms"]
+                if da < 0 <= db:
+                    be = a["rho"] + (b["rho"] - a["rho"]) * (-da) / (db - da)
+                    break
+            if be is None and pts and pts[0]["T_sel_ms"] >= pts[0]["T_full_ms"]:
+                be = dens[0]
+            rows.append({"dense": pname, "F": F, "points": pts, "break_even_rho": be})
+    print(json.dumps({"calib_curve": rows, "block_rows": 2048,
+                      "note": "pcgcn_calibrate_prec: T_s = all-selective forward, T_f = the rho-blocks in the full "
+                              "mode (diagonal self-loop blocks selective in both); L161 theta = T_f*rho/T_s"}),
+          flush=True)
 
 
 def log(*a):
@@ -510,6 +546,9 @@ def main():
         return
     if args.table3:
         run_table3(args)
+        return
+    if args.calib_curve:
+        run_calib_curve(args)
         return
     if args.f2:
         run_f2(args)

@@ -348,6 +348,10 @@ pcgcn_status pcgcn_plan_export(pcgcn_plan_t p, int32_t which, void* host_buf, in
  * θ = T_f·p_ref/T_s in *theta_out.  Synchronises its own stream. */
 pcgcn_status pcgcn_calibrate(int32_t F, int32_t block_rows, float p_ref, float* theta_out,
                              float* t_full_ms, float* t_sel_ms);
+/* The same with the full mode in dense_prec (PCGCN_DENSE_*; pcgcn_calibrate = TF32X2): one point
+ * (p_ref, T_f, T_s) of the calibration curve T_s(ρ), T_f over densities and widths. */
+pcgcn_status pcgcn_calibrate_prec(int32_t F, int32_t block_rows, float p_ref, int32_t dense_prec,
+                                  float* theta_out, float* t_full_ms, float* t_sel_ms);
 
 /* In-situ refinement of θ for one feature width F (the L161 procedure applied
  * to the workload itself): times the plan's full-mode tiles and selective

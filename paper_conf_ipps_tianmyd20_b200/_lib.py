@@ -90,6 +90,8 @@ _sig("pcgcn_plan_export_bytes", c_i64, c_vp, c_i32)
 _sig("pcgcn_plan_export", c_i32, c_vp, c_i32, c_vp, c_i64)
 _sig("pcgcn_calibrate", c_i32, c_i32, c_i32, c_f32, ctypes.POINTER(c_f32), ctypes.POINTER(c_f32),
      ctypes.POINTER(c_f32))
+_sig("pcgcn_calibrate_prec", c_i32, c_i32, c_i32, c_f32, c_i32, ctypes.POINTER(c_f32), ctypes.POINTER(c_f32),
+     ctypes.POINTER(c_f32))
 _sig("pcgcn_plan_last_timings", c_i32, c_vp, ctypes.POINTER(c_f32))
 _sig("pcgcn_refine_theta", c_i32, c_vp, c_vp, c_i64, c_vp, c_i64, c_i32, ctypes.POINTER(c_f32),
      ctypes.POINTER(c_f32), ctypes.POINTER(c_f32))
@@ -397,10 +399,14 @@ def probe_read_gbs(nbytes, iters=20):
     return v.value
 
 
-def calibrate(F, block_rows=2048, p_ref=0.05):
+def calibrate(F, block_rows=2048, p_ref=0.05, dense_prec=None):
     th, tf, ts = c_f32(), c_f32(), c_f32()
-    check(lib.pcgcn_calibrate(F, block_rows, p_ref, ctypes.byref(th), ctypes.byref(tf), ctypes.byref(ts)),
-          "pcgcn_calibrate")
+    if dense_prec is None:
+        check(lib.pcgcn_calibrate(F, block_rows, p_ref, ctypes.byref(th), ctypes.byref(tf), ctypes.byref(ts)),
+              "pcgcn_calibrate")
+    else:
+        check(lib.pcgcn_calibrate_prec(F, block_rows, p_ref, dense_prec, ctypes.byref(th), ctypes.byref(tf),
+                                       ctypes.byref(ts)), "pcgcn_calibrate_prec")
     return th.value, tf.value, ts.value
 
 

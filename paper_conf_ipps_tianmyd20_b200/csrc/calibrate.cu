@@ -83,9 +83,10 @@ extern "C" pcgcn_status pcgcn_refine_theta(pcgcn_plan_t p, const float* Y, int64
   return PCGCN_OK;
 }
 
-extern "C" pcgcn_status pcgcn_calibrate(int32_t F, int32_t block_rows, float p_ref, float* theta_out,
-                                        float* t_full_ms, float* t_sel_ms) {
-  if (F < 1 || F > 256 || block_rows < 32 || !(p_ref > 0.f && p_ref <= 1.f) || !theta_out) {
+extern "C" pcgcn_status pcgcn_calibrate_prec(int32_t F, int32_t block_rows, float p_ref, int32_t dense_prec,
+                                             float* theta_out, float* t_full_ms, float* t_sel_ms) {
+  if (F < 1 || F > 256 || block_rows < 32 || !(p_ref > 0.f && p_ref <= 1.f) || !theta_out ||
+      dense_prec < PCGCN_DENSE_TF32X2 || dense_prec > PCGCN_DENSE_BF16X3) {
     pcgcn::set_error("calibrate: bad arguments");
     return PCGCN_EINVAL;
   }
@@ -120,6 +121,7 @@ extern "C" pcgcn_status pcgcn_calibrate(int32_t F, int32_t block_rows, float p_r
   pcgcn_opts_default(&o);
   o.part = part.data();
   o.f_max = F;
+  o.dense_prec = dense_prec;
   pcgcn_plan_t ps = nullptr, pf = nullptr;
   // diagonal blocks hold only the self-loops (density 1/B): keep them selective
   // in both plans so the two timings differ only in the mode of the p-blocks
@@ -155,4 +157,9 @@ extern "C" pcgcn_status pcgcn_calibrate(int32_t F, int32_t block_rows, float p_r
   if (t_full_ms) *t_full_ms = tf;
   if (t_sel_ms) *t_sel_ms = ts;
   return PCGCN_OK;
+}
+
+extern "C" pcgcn_status pcgcn_calibrate(int32_t F, int32_t block_rows, float p_ref, float* theta_out,
+                                        float* t_full_ms, float* t_sel_ms) {
+  return pcgcn_calibrate_prec(F, block_rows, p_ref, PCGCN_DENSE_TF32X2, theta_out, t_full_ms, t_sel_ms);
 }

@@ -50,7 +50,6 @@ struct AggArgs {
   int* seg_ticket = nullptr;         // segment ticket (zeroed with the row ticket)
   int seg_inline = 0;                // 1: no separate segment pass
   int64_t seg_ahead = 0;             // row tickets ahead of the claiming warp within which segments are taken
-  int64_t near_rows = 0;             // > 0: sources farther than this (plan rows) load L2-evict-first
   // device-initiated peer gather: sources of shard q are read from
   // shard q's own buffer (peer_base[q] = its row row0[q]; NVLink peer memory
   // on a multi-GPU node, CUDA IPC in the 1-GPU tests) instead of an exchanged copy

@@ -40,7 +40,6 @@
 namespace pcgcn {
 int knobs_mrow_gpt();   // PCGCN_MROW_GPT (multi-row groups per ticket)
 int knobs_seg_inline(); // PCGCN_SEG_INLINE (0: separate up-front segment pass)
-int64_t near_rows_for(const AggArgs& a);  // evict-first window (PCGCN_NEAR_ROWS)
 int knobs_seg_ahead();  // PCGCN_SEG_AHEAD (segment window, in quarters of the resident warps' row tickets)
 namespace {
 
@@ -110,27 +109,6 @@ __device__ __forceinline__ void ld_vec(const char* p, float4 (&o)[H]) {
   }
 }
 
-// ld_vec with an L2 eviction priority chosen per load: evict-first for a
-// `far` source row (outside the destination's neighbourhood in plan order:
-// an inter-community edge, read once), evict-normal otherwise — so the
-// random far rows stream through L2 without displacing the community slice
-// the near rows keep reusing (C5: Y' = 17 GB against a 126 MB L2)
-template <int H>
-__device__ __forceinline__ void ld_vec_ev(const char* p, float4 (&o)[H], bool far) {
-  const uint32_t f = far ? 1u : 0u;
-  if constexpr (H == 1) {  // (the eviction-priority form needs 32-byte vectors)
-    o[0] = ld_f4b(p);
-    (void)f;
-  } else {
-    asm("{\n\t.reg .pred pf;\n\tsetp.ne.u32 pf, %9, 0;\n\t"
-        "@pf ld.global.nc.L2::evict_first.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];\n\t"
-        "@!pf ld.global.nc.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];\n\t}"
-        : "=f"(o[0].x), "=f"(o[0].y), "=f"(o[0].z), "=f"(o[0].w), "=f"(o[1].x), "=f"(o[1].y), "=f"(o[1].z),
-          "=f"(o[1].w)
-        : "l"(p), "r"(f));
-  }
-}
-
 // Lane layout for a feature row of nvec lane vectors (H float4 each): the
 // warp's 32 lanes form S = 32/G edge slots of G lanes; lane l of a slot owns
 // vectors l, l+G, ..., l+(V-1)G.  A slot's G lanes read one contiguous piece
@@ -172,14 +150,11 @@ struct Lay {
 // (lane l: cp[l] if l < n), and the prefetch slot of the last batch loads the
 // first batch of the NEXT range (cpn, nn), which is returned — so a warp
 // walking rows never waits on a row's first index load.
-// EVF: per-load L2 eviction priority (ld_vec_ev): a source j is near iff
-// (j - nlo) mod 2^32 < nspan.
-template <int G, int V, int H, bool PEER = false, bool EVF = false>
+template <int G, int V, int H, bool PEER = false>
 __device__ __forceinline__ int gather_sum(const int* __restrict__ cp, int n, int first,
                                           const int* __restrict__ cpn, int nn, const char* __restrict__ yb,
                                           uint32_t rstride, const bool (&lok)[V], int lane,
-                                          float4 (&tot)[V][H], const AggArgs& a, uint32_t nlo = 0,
-                                          uint32_t nspan = 0) {
+                                          float4 (&tot)[V][H], const AggArgs& a) {
   using L = Lay<G, V, H>;
   constexpr int S = L::S, STEPS = L::STEPS, UNR = L::UNR, NACC = L::NACC, BATCH = L::BATCH;
   const int slot = lane / G;
@@ -211,8 +186,7 @@ __device__ __forceinline__ int gather_sum(const int* __restrict__ cp, int n, int
 #pragma unroll
           for (int v = 0; v < V; ++v) {
             if (active && (v == 0 || lok[v])) {
-              if constexpr (EVF) ld_vec_ev<H>(p + 16 * H * G * v, buf[u][v], j - nlo >= nspan);
-              else ld_vec<H>(p + 16 * H * G * v, buf[u][v]);
+              ld_vec<H>(p + 16 * H * G * v, buf[u][v]);
             } else {
 #pragma unroll
               for (int h = 0; h < H; ++h) buf[u][v][h] = make_float4(0.f, 0.f, 0.f, 0.f);
@@ -239,8 +213,7 @@ __device__ __forceinline__ int gather_sum(const int* __restrict__ cp, int n, int
 #pragma unroll
           for (int v = 0; v < V; ++v) {
             if (active && e < cnt && (v == 0 || lok[v])) {
-              if constexpr (EVF) ld_vec_ev<H>(p + 16 * H * G * v, buf[u][v], j - nlo >= nspan);
-              else ld_vec<H>(p + 16 * H * G * v, buf[u][v]);
+              ld_vec<H>(p + 16 * H * G * v, buf[u][v]);
             } else {
 #pragma unroll
               for (int h = 0; h < H; ++h) buf[u][v][h] = make_float4(0.f, 0.f, 0.f, 0.f);
@@ -346,7 +319,7 @@ __device__ __forceinline__ int peek_ticket(const int* t) { return *reinterpret_c
 // locality); a row is gathered directly or, if long, summed from its
 // segment partials in segment order.  Fused epilogue: + full-mode partial
 // sum Zd (mode combine, L193), x r_i (optionally twice), ReLU, bit mask.
-template <int G, int V, int H, bool HAS_ZD, bool HAS_SEG, bool PEER, bool EVF = false>
+template <int G, int V, int H, bool HAS_ZD, bool HAS_SEG, bool PEER>
 __global__ void __launch_bounds__(256, Lay<G, V, H>::MINB) sparse_row_kernel(AggArgs a) {
   const int lane = threadIdx.x & 31;
   const int slot = lane / G;
@@ -593,9 +566,8 @@ __global__ void __launch_bounds__(256, Lay<G, V, H>::MINB) sparse_row_kernel(Agg
                                                                         4 * (H * qv[v] + h))));
       }
     } else {
-      pre_next = gather_sum<G, V, H, PEER, EVF>(a.col + e0, int(e1 - e0), pre, a.col + n0, int(n1 - n0), yb,
-                                                rstride, lok, lane, tot, a,
-                                                uint32_t(a.row_lo + row - a.near_rows), uint32_t(2 * a.near_rows));
+      pre_next = gather_sum<G, V, H, PEER>(a.col + e0, int(e1 - e0), pre, a.col + n0, int(n1 - n0), yb, rstride,
+                                           lok, lane, tot, a);
     }
     if (!skip) epilogue(row, tot, zi, ri);
     pre = pre_next;
@@ -623,7 +595,7 @@ __global__ void __launch_bounds__(256, Lay<G, V, H>::MINB) sparse_row_kernel(Agg
 // its row (G indices per slot per load), one batch ahead; the next group's
 // row pointers and segment ids are loaded while the current group gathers,
 // and its first index batch is issued by the current group's last step.
-template <int G, bool HAS_ZD, bool HAS_SEG, bool PEER, bool EVF = false>
+template <int G, bool HAS_ZD, bool HAS_SEG, bool PEER>
 __global__ void __launch_bounds__(256, 4) sparse_mrow_kernel(AggArgs a) {
   constexpr int H = 2;
   constexpr int S = 32 / G;
@@ -776,7 +748,6 @@ __global__ void __launch_bounds__(256, 4) sparse_mrow_kernel(AggArgs a) {
     if (inl && newblk && lane == 0) speek = peek_ticket(a.seg_ticket);
     const int64_t row = q * S + slot;
     const bool valid = row < a.rows;
-    const uint32_t nlo = uint32_t(a.row_lo + row - a.near_rows), nspan = uint32_t(2 * a.near_rows);
     const float ri = valid ? __ldg(a.r + a.row_lo + row) : 0.f;
     const int zi = (HAS_ZD && valid) ? __ldg(a.zd_index + row) : -1;
     float4 acc[H];
@@ -800,8 +771,7 @@ __global__ void __launch_bounds__(256, 4) sparse_mrow_kernel(AggArgs a) {
         for (int u = 0; u < 4; ++u) {
           const uint32_t j = uint32_t(__shfl_sync(0xffffffffu, cur, slot * G + u0 + u));
           if (lok && base + u0 + u < n) {
-            if constexpr (EVF) ld_vec_ev<H>(src_row<PEER>(yb, j, rstride, a), buf[u], j - nlo >= nspan);
-            else ld_vec<H>(src_row<PEER>(yb, j, rstride, a), buf[u]);
+            ld_vec<H>(src_row<PEER>(yb, j, rstride, a), buf[u]);
           } else {
 #pragma unroll
             for (int h = 0; h < H; ++h) buf[u][h] = make_float4(0.f, 0.f, 0.f, 0.f);
@@ -880,15 +850,7 @@ cudaError_t launch_mrow(const AggArgs& a, cudaStream_t s) {
   const unsigned grid = unsigned(want < slots ? want : slots);
   b.seg_inline = inl ? 1 : 0;
   b.seg_ahead = int64_t(grid) * 8 * knobs_seg_ahead() / 4;
-  b.near_rows = PEER ? 0 : near_rows_for(a);
   const bool zd = a.zd_index != nullptr, sg = a.nseg > 0;
-  if constexpr (!PEER) {  // evict-first far rows: all-selective plans of inputs far larger than L2
-    if (b.near_rows > 0 && !zd) {
-      if (sg) sparse_mrow_kernel<G, false, true, false, true><<<grid, 256, 0, s>>>(b);
-      else sparse_mrow_kernel<G, false, false, false, true><<<grid, 256, 0, s>>>(b);
-      return cudaGetLastError();
-    }
-  }
 #define LAUNCH(ZD, SG) sparse_mrow_kernel<G, ZD, SG, PEER><<<grid, 256, 0, s>>>(b)
   if (zd && sg) LAUNCH(true, true);
   else if (zd) LAUNCH(true, false);
@@ -922,15 +884,7 @@ cudaError_t launch_gvp(const AggArgs& a, cudaStream_t s) {
   AggArgs b = a;
   b.seg_inline = inl ? 1 : 0;
   b.seg_ahead = int64_t(grid) * 8 * knobs_seg_ahead() / 4;
-  b.near_rows = PEER ? 0 : near_rows_for(a);
   const bool zd = a.zd_index != nullptr, sg = a.nseg > 0;
-  if constexpr (!PEER) {  // evict-first far rows: all-selective plans of inputs far larger than L2
-    if (b.near_rows > 0 && !zd) {
-      if (sg) sparse_row_kernel<G, V, H, false, true, false, true><<<grid, 256, 0, s>>>(b);
-      else sparse_row_kernel<G, V, H, false, false, false, true><<<grid, 256, 0, s>>>(b);
-      return cudaGetLastError();
-    }
-  }
 #define LAUNCH(ZD, SG) sparse_row_kernel<G, V, H, ZD, SG, PEER><<<grid, 256, 0, s>>>(b)
   if (zd && sg) LAUNCH(true, true);
   else if (zd) LAUNCH(true, false);
@@ -1096,13 +1050,9 @@ struct SparseKnobs {
   int mrow = -1;
   int mrow_gpt = 4;  // PCGCN_MROW_GPT: groups per ticket
   int seg_inline = 0;  // measured (B200, fixed θ, interleaved): C3 F=41 passes +5%, C5 neutral -> off
-  // PCGCN_NEAR_ROWS: -1 (default) auto — sources more than 16384 plan rows from the
-  // destination load evict-first when Y' exceeds 4x the L2; 0 never; > 0 that window
-  int64_t near_rows = -1;
   int seg_ahead = 4;  // quarters of (grid warps) row tickets
   SparseKnobs() {
     if (const char* e = getenv("PCGCN_SEG_INLINE")) seg_inline = atoi(e);
-    if (const char* e = getenv("PCGCN_NEAR_ROWS")) near_rows = atoll(e);
     if (const char* e = getenv("PCGCN_SEG_AHEAD")) seg_ahead = std::max(1, atoi(e));
     if (const char* e = getenv("PCGCN_SPARSE_MROW")) mrow = atoi(e);
     if (const char* e = getenv("PCGCN_MROW_GPT")) mrow_gpt = std::max(1, atoi(e));
@@ -1119,12 +1069,7 @@ static SparseKnobs& knobs() {
 }
 int knobs_mrow_gpt() { return knobs().mrow_gpt; }
 int knobs_seg_inline() { return knobs().seg_inline; }
-int64_t near_rows_for(const AggArgs& a) {
-  const int64_t k = knobs().near_rows;
-  if (k >= 0) return k;
-  const double ybytes = double(a.n_src) * double(a.ldy) * 4.0;
-  return ybytes > 4.0 * 126e6 ? 16384 : 0;
-}
+
 int knobs_seg_ahead() { return knobs().seg_ahead; }
 
 bool sparse_fsplit_active(int F) { return knobs().fsplit > 0 && F > knobs().fsplit; }

@@ -620,8 +620,7 @@ np.savez(sys.argv[1], **out)
                                           ({"PCGCN_MROW_GPT": "1"}, True),
                                           ({"PCGCN_SEG_INLINE": "1"}, True),
                                           ({"PCGCN_SEG_INLINE": "1", "PCGCN_SEG_AHEAD": "64"}, True),
-                                          ({"PCGCN_SEG_INLINE": "1", "PCGCN_SEG_AHEAD": "1"}, True),
-                                          ({"PCGCN_NEAR_ROWS": "64"}, True)])
+                                          ({"PCGCN_SEG_INLINE": "1", "PCGCN_SEG_AHEAD": "1"}, True)])
 def test_scheduling_knobs_do_not_change_results(tmp_path, knob, bitwise):
     """Row-block tickets, inline vs separate long-row segments (the same
     partials added in the same order), the full-mode/segment overlap, the in-kernel xtg B
