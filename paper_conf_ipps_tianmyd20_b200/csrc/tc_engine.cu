@@ -227,7 +227,9 @@ __global__ void __launch_bounds__(NTHREADS, 1)
   uint64_t* acc_empty = acc_full + 2;       // [2] (128 arrivals)
   uint64_t* tq_full = acc_empty + 2;        // [TQ] tile id written by the producer
   uint64_t* tq_empty = tq_full + TQ;        // [TQ] tile id read by the 3 consumer roles
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tq_empty + TQ);
+  uint64_t* bfull = tq_empty + TQ;          // [stages] A_BITS: the stage's bit tiles landed (A can be built
+                                            // while the B windows are still in flight)
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bfull + L.stages);
   int64_t* tq = reinterpret_cast<int64_t*>(tmem_slot + 4);  // [TQ] tile positions (-1: done)
   const int npad = L.npad;
 
@@ -235,6 +237,7 @@ __global__ void __launch_bounds__(NTHREADS, 1)
   if (threadIdx.x == 0) {
     for (int s = 0; s < L.stages; ++s) {
       mbar_init(&full[s], 1);
+      mbar_init(&bfull[s], 1);
       mbar_init(&a_full[s], 128);
       mbar_init(&empty[s], 1);
     }
@@ -269,19 +272,40 @@ __global__ void __launch_bounds__(NTHREADS, 1)
         const int64_t t = it.t;
         int64_t kb, nch, m0, sp;
         tile_range<MODE>(w, t, kb, nch, m0, sp);
+        // A_BITS: the source windows of a stage's chunks are loaded one stage
+        // ahead (independent loads, consumed after the next empty-slot wait),
+        // so the single producer thread never waits on a global load between
+        // two bulk copies (a load per chunk in the copy loop serialised ~1000
+        // cycles per chunk: the engine's cost per chunk was independent of N)
+        int c0_cur[4] = {0, 0, 0, 0}, c0_nxt[4] = {0, 0, 0, 0};
+        if (MODE == A_BITS) {
+#pragma unroll
+          for (int u = 0; u < 4; ++u)
+            if (u < L.U && u < nch) c0_nxt[u] = __ldg(w.ch_col0 + kb + u);
+        }
         for (int64_t i = 0; i < nch; i += L.U) {
           const int nu = int(nch - i < L.U ? nch - i : L.U);
+          if (MODE == A_BITS) {
+#pragma unroll
+            for (int u = 0; u < 4; ++u) {
+              c0_cur[u] = c0_nxt[u];
+              if (u < L.U && i + L.U + u < nch) c0_nxt[u] = __ldg(w.ch_col0 + kb + i + L.U + u);
+            }
+          }
           mbar_wait(&empty[s], ph ^ 1u);
           uint8_t* st = smem + s * L.stage_bytes;
-          mbar_expect_tx(&full[s], uint32_t(nu) * (L.a_load_bytes +
+          mbar_expect_tx(&full[s], uint32_t(nu) * ((MODE == A_BITS ? 0u : L.a_load_bytes) +
                                                    (w.b_raw ? L.raw_bytes
                                                             : w.bf3 ? L.bchunk : (w.single ? 1u : 2u) * L.b_bytes)));
-          // the bits of a tile's chunks are contiguous: one bulk copy per stage
-          if (MODE == A_BITS) bulk_load(st, w.bits + (kb + i) * BM, uint32_t(nu) * BM * 4, &full[s]);
+          // the bits of a tile's chunks are contiguous: one bulk copy per stage, on its own barrier
+          if (MODE == A_BITS) {
+            mbar_expect_tx(&bfull[s], uint32_t(nu) * BM * 4);
+            bulk_load(st, w.bits + (kb + i) * BM, uint32_t(nu) * BM * 4, &bfull[s]);
+          }
           for (int u = 0; u < nu; ++u) {
             int k0;
             if (MODE == A_BITS) {
-              k0 = w.ch_col0[kb + i + u];
+              k0 = c0_cur[u & 3];
             } else if (MODE == A_ROWMAJOR) {
               k0 = int(i * BK);
               tma_load_2d(&map_a, &full[s], st, k0, int(m0));
@@ -388,7 +412,8 @@ __global__ void __launch_bounds__(NTHREADS, 1)
       tile_range<MODE>(w, t, kb, nch, m0, sp);
       for (int64_t i = 0; i < nch; i += L.U) {
         const int nu = int(nch - i < L.U ? nch - i : L.U);
-        mbar_wait(&full[s], ph);  // data landed; stage and its TMEM A buffer are free
+        // data landed (A_BITS: the bits only); the stage and its TMEM A buffer are free
+        mbar_wait(MODE == A_BITS ? &bfull[s] : &full[s], ph);
         const uint8_t* st = smem + s * L.stage_bytes;
         const uint32_t taddr = tmem + lane_base + L.a_col0 + uint32_t(s) * uint32_t(L.a_cols);
         uint32_t v[32];
@@ -747,7 +772,7 @@ cudaError_t launch_engine(const CUtensorMap& bhi, const CUtensorMap& blo, const 
                           int npad, cudaStream_t s) {
   if (w.ntiles <= 0) return cudaSuccess;
   const Layout L = make_layout(MODE, npad, max_stages_env(), max_u_env(), w.b_raw != 0, w.bf3);
-  const size_t smem = 1024 + size_t(L.stages) * L.stage_bytes + L.out_bytes + (3 * L.stages + 4 + 2 * TQ) * 8 + 16 +
+  const size_t smem = 1024 + size_t(L.stages) * L.stage_bytes + L.out_bytes + (4 * L.stages + 4 + 2 * TQ) * 8 + 16 +
                      TQ * 8;
   if (smem > 227 * 1024) return cudaErrorInvalidValue;
   static int grid_cap = -1;  // PCGCN_TC_GRID: full-mode CTAs (tuning override, benchmarks only)
