@@ -139,6 +139,7 @@ pcgcn_status upload_plan(pcgcn_plan_s* p) {
         if (std::string(e) == "plan")
           for (int64_t i = 0; i < d.nrt; ++i) order[i] = int32_t(i);
       UP(&d.rt_order, order.data(), d.nrt);
+      UP(&d.rt_bysize, bysize.data(), d.nrt);
     }
     UP(&d.ch_col0, p->ch_col0.data() + ch_lo, d.nch);
     UP(&d.bits, p->bits.data() + ch_lo * TILE_M, d.nch * TILE_M);
@@ -248,6 +249,17 @@ bool tc_dyn_enabled() {
   if (v < 0) {
     const char* e = getenv("PCGCN_TC_DYN");
     v = e ? (atoi(e) != 0) : 1;
+  }
+  return v != 0;
+}
+
+// PCGCN_TC_DYN_ORDER=size (A/B knob): dynamic tile claims largest tile first
+// (longest-processing-time order; C3's largest tile holds ~the mean CTA share)
+bool tc_dyn_order_size() {
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("PCGCN_TC_DYN_ORDER");
+    v = (e && std::string(e) == "size") ? 1 : 0;
   }
   return v != 0;
 }
@@ -397,7 +409,7 @@ pcgcn_status aggregate(pcgcn_plan_t p, const float* Y, int64_t ldy, float* Z, in
       // tiles claimed dynamically, in plan order: neighbouring row tiles (and
       // their source windows) are in flight together, balance comes from the claims
       da.dyn = d.counter + 16;
-      da.rt_order = nullptr;
+      da.rt_order = tc_dyn_order_size() ? d.rt_bysize : nullptr;
       if ((e = cudaMemsetAsync(da.dyn, 0, sizeof(int), ms)) != cudaSuccess) return cuda_fail(e, "memset");
     }
     if (blocked) {

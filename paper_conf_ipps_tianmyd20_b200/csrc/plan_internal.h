@@ -22,6 +22,7 @@ struct DevicePlan {
   int32_t* rt_nrows = nullptr;    // [nrt shard]
   int64_t* rt_cptr = nullptr;     // [nrt+1] rebased
   int32_t* rt_order = nullptr;    // [nrt] full-mode engine tile order (balanced, see upload_plan)
+  int32_t* rt_bysize = nullptr;   // [nrt] tiles by descending chunk count (dynamic largest-first claims)
   int32_t* ch_col0 = nullptr;     // [nch shard]
   uint32_t* bits = nullptr;       // [nch*128]
   float* zd = nullptr;            // [nrt*128*fpad_max] dense partial sums

@@ -615,6 +615,7 @@ np.savez(sys.argv[1], **out)
                                           ({"PCGCN_SPARSE_FSPLIT": "32"}, False),
                                           ({"PCGCN_SPARSE_G6": "0"}, False),
                                           ({"PCGCN_TC_DYN": "0"}, True),
+                                          ({"PCGCN_TC_DYN_ORDER": "size"}, True),
                                           ({"PCGCN_SPARSE_MROW": "0"}, False),
                                           ({"PCGCN_SPARSE_MROW": "1"}, False),
                                           ({"PCGCN_MROW_GPT": "1"}, True),
