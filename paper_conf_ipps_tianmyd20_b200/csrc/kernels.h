@@ -60,6 +60,7 @@ struct AggArgs {
   int rows_per_ticket = 1;   // consecutive rows per scheduler ticket, 1..16
   float mean_deg = 0.f;      // selective edges per row (layout choice: short rows -> multi-row warps)
   int rows_by_degree = 0;    // plan rows sorted by degree inside partitions (multi-row groups are balanced)
+  int mrow_sort = 1;         // multi-row pass: group a ticket's 32 rows by degree
 };
 // selective edges per long-row segment
 constexpr int SEG_EDGES = 1024;

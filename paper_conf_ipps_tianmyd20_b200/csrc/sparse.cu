@@ -38,7 +38,7 @@
 #include "kernels.h"
 
 namespace pcgcn {
-int knobs_mrow_gpt();   // PCGCN_MROW_GPT (multi-row groups per ticket)
+int knobs_mrow_sort();  // PCGCN_MROW_SORT (0: multi-row groups in plan order)
 int knobs_seg_inline(); // PCGCN_SEG_INLINE (0: separate up-front segment pass)
 int knobs_seg_ahead();  // PCGCN_SEG_AHEAD (segment window, in quarters of the resident warps' row tickets)
 namespace {
@@ -607,33 +607,72 @@ __global__ void __launch_bounds__(256, 4) sparse_mrow_kernel(AggArgs a) {
   const bool lok = g < nvec;
   const char* yb = (PEER ? nullptr : reinterpret_cast<const char*>(a.Y)) + 32 * (lok ? g : 0);
   const uint32_t rstride = uint32_t(a.ldy * 4);
-  const int64_t ngrp = (a.rows + S - 1) / S;
-  const int GPT = a.rows_per_ticket;  // groups per ticket
-  const int64_t ntk = (ngrp + GPT - 1) / GPT;
+  // tickets of 32 consecutive plan rows, S-row groups inside a ticket
+  const int GPT = 32 / S;
+  const int64_t ntk = (a.rows + 31) / 32;
   auto ticket = [&]() {
     int t = 0;
     if (lane == 0) t = atomicAdd(a.counter, 1);
     return __shfl_sync(0xffffffffu, t, 0);
   };
-  // group q: lane l <= S holds rowptr[q*S + l] (clamped to rows), every lane
-  // the segment id of its slot's row
-  auto load_grp = [&](int64_t q, int64_t& rp, int& sgv) {
-    rp = 0;
-    sgv = -1;
-    if (q < ngrp) {
-      if (lane <= S) {
-        const int64_t r = q * S + lane;
-        rp = __ldg(a.rowptr + (r < a.rows ? r : a.rows));
+  // ticket tt's row pointers and segment ids -> this warp's shared-memory
+  // buffer b with cp.async (nothing held in registers while they travel)
+  __shared__ long long s_rp[8][2][34];
+  __shared__ int s_sg[8][2][32];
+  const int wib = threadIdx.x >> 5;
+  auto load_tk = [&](int tt, int b) {
+    if (tt < ntk) {
+      const int64_t r0 = int64_t(tt) * 32;
+      for (int l = lane; l <= 32; l += 32) {
+        const int64_t r = r0 + l < a.rows ? r0 + l : a.rows;
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_addr(&s_rp[wib][b][l])),
+                     "l"(reinterpret_cast<const long long*>(a.rowptr + r))
+                     : "memory");
       }
       if (HAS_SEG) {
-        const int64_t r = q * S + slot;
-        sgv = r < a.rows ? __ldg(a.row_seg + r) : -1;
+        if (r0 + lane < a.rows)
+          asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_addr(&s_sg[wib][b][lane])),
+                       "l"(a.row_seg + r0 + lane)
+                       : "memory");
+        else
+          s_sg[wib][b][lane] = -1;
       }
+    } else {  // past the last ticket: empty rows (the lookahead reads this buffer)
+      s_rp[wib][b][lane] = 0;
+      if (lane == 0) s_rp[wib][b][32] = 0;
+      if (HAS_SEG) s_sg[wib][b][lane] = -1;
     }
+    asm volatile("cp.async.commit_group;" ::: "memory");
   };
-  auto range = [&](int64_t rp, int sgv, int64_t& e0, int64_t& e1) {
-    e0 = __shfl_sync(0xffffffffu, rp, slot);
-    e1 = __shfl_sync(0xffffffffu, rp, slot + 1);
+  auto wait_tk = [&]() {
+    asm volatile("cp.async.wait_group 0;" ::: "memory");
+    __syncwarp();
+  };
+  // the ticket's rows ordered by gathered degree (bitonic sort across the warp,
+  // ties by row): each group of S rows then has rows of similar length, so a
+  // group costs about its mean row instead of its longest (the plan order
+  // stays as it is: only the 32-row window is reordered)
+  const bool sort_rows = a.mrow_sort != 0;
+  auto sort_tk = [&](int b) {
+    if (!sort_rows) return lane;
+    const bool sgd = HAS_SEG && s_sg[wib][b][lane] >= 0;
+    int x = ((sgd ? 0 : int(s_rp[wib][b][lane + 1] - s_rp[wib][b][lane])) << 5) | lane;
+#pragma unroll
+    for (int kk = 2; kk <= 32; kk <<= 1)
+#pragma unroll
+      for (int j = kk >> 1; j > 0; j >>= 1) {
+        const int o = __shfl_xor_sync(0xffffffffu, x, j);
+        const bool asc = (lane & kk) == 0, low = (lane & j) == 0;
+        x = (low == asc) ? min(x, o) : max(x, o);
+      }
+    return x & 31;
+  };
+  // group kq of the ticket in buffer b: this slot's row (index inside the ticket) and its range
+  auto slot_row = [&](int kq, int perm, int b, int& idx, int64_t& e0, int64_t& e1, int& sgv) {
+    idx = __shfl_sync(0xffffffffu, perm, kq * S + slot);
+    e0 = s_rp[wib][b][idx];
+    e1 = s_rp[wib][b][idx + 1];
+    sgv = HAS_SEG ? s_sg[wib][b][idx] : -1;
     return (HAS_SEG && sgv >= 0) ? 0 : int(e1 - e0);
   };
   // epilogue of one row held by this lane's slot: + Zd, x r_i (twice if prescaled output), mask byte, ReLU
@@ -723,45 +762,42 @@ __global__ void __launch_bounds__(256, 4) sparse_mrow_kernel(AggArgs a) {
   };
   int t = ticket();
   if (t >= ntk) { if (inl) seg_loop(-1); return; }
-  int64_t q = int64_t(t) * GPT;
-  int64_t qend = q + GPT < ngrp ? q + GPT : ngrp;
-  int tn = ticket();  // the next block's ticket, consumed when this block ends
-  int64_t rp;
-  int sgv;
-  load_grp(q, rp, sgv);
+  int tn = ticket();  // the next ticket, consumed when this one ends
+  int bt = 0;          // smem buffer of the current ticket
+  load_tk(t, bt);
+  wait_tk();
+  int perm = sort_tk(bt), permn = 0;
+  int kq = 0, ri_idx, sgv;
   int64_t e0, e1;
-  int n = range(rp, sgv, e0, e1);
+  int n = slot_row(0, perm, bt, ri_idx, e0, e1, sgv);
   int idx = g < n ? ld_col<PEER>(a.col + e0 + g, a) : 0;
   while (true) {
-    int64_t qn;
-    bool newblk = false;
-    if (q + 1 < qend) {
-      qn = q + 1;
-    } else {
-      qn = int64_t(tn) * GPT;
-      newblk = true;
+    const bool last = kq == GPT - 1;
+    if (kq == GPT - 2) load_tk(tn, bt ^ 1);  // the next ticket's rows, in flight for a group
+    if (last) {
+      wait_tk();
+      permn = sort_tk(bt ^ 1);
     }
-    int64_t rpn;
-    int sgn;
-    load_grp(qn, rpn, sgn);  // in flight while this group gathers
     int speek = a.nseg;
-    if (inl && newblk && lane == 0) speek = peek_ticket(a.seg_ticket);
-    const int64_t row = q * S + slot;
+    if (inl && last && lane == 0) speek = peek_ticket(a.seg_ticket);
+    const int64_t row = int64_t(t) * 32 + ri_idx;
     const bool valid = row < a.rows;
     const float ri = valid ? __ldg(a.r + a.row_lo + row) : 0.f;
     const int zi = (HAS_ZD && valid) ? __ldg(a.zd_index + row) : -1;
+    // the next group's row (this ticket, or the next one's first group)
+    int idxn, sgn;
+    int64_t e0n, e1n;
+    const int nn = last ? slot_row(0, permn, bt ^ 1, idxn, e0n, e1n, sgn)
+                        : slot_row(kq + 1, perm, bt, idxn, e0n, e1n, sgn);
     float4 acc[H];
 #pragma unroll
     for (int h = 0; h < H; ++h) acc[h] = make_float4(0.f, 0.f, 0.f, 0.f);
     const int nmax = __reduce_max_sync(0xffffffffu, n);
-    int64_t e0n = 0, e1n = 0;
-    int nn = 0;
     for (int base = 0; base < nmax; base += G) {
       const int cur = idx;
       if (base + G < nmax) {
         idx = (base + G + g < n) ? ld_col<PEER>(a.col + e0 + base + G + g, a) : 0;
       } else {  // last step: the next group's first batch
-        nn = range(rpn, sgn, e0n, e1n);
         idx = g < nn ? ld_col<PEER>(a.col + e0n + g, a) : 0;
       }
 #pragma unroll
@@ -784,10 +820,7 @@ __global__ void __launch_bounds__(256, 4) sparse_mrow_kernel(AggArgs a) {
         if (base + u0 + 4 >= nmax) break;  // warp-uniform: the rest of the batch is past every row
       }
     }
-    if (nmax == 0) {
-      nn = range(rpn, sgn, e0n, e1n);
-      idx = g < nn ? ld_col<PEER>(a.col + e0n + g, a) : 0;
-    }
+    if (nmax == 0) idx = g < nn ? ld_col<PEER>(a.col + e0n + g, a) : 0;
     if (HAS_SEG && !inl && sgv >= 0 && lok) {  // long row: its segment partials in segment order
       const int ns = int((e1 - e0 + SEG_EDGES - 1) / SEG_EDGES);
       for (int k = 0; k < ns; ++k)
@@ -798,26 +831,30 @@ __global__ void __launch_bounds__(256, 4) sparse_mrow_kernel(AggArgs a) {
                                                                4 * (H * g + h))));
     }
     if (valid && !(inl && sgv >= 0)) epilogue(row, acc, zi, ri);  // inline: a long row is written by its last segment
-    if (inl && newblk) {
-      int64_t sr = INT64_MAX;
-      if (lane == 0 && speek < a.nseg) sr = a.seg_row[speek];
-      sr = __shfl_sync(0xffffffffu, sr, 0);
-      const int64_t limit = (qn / GPT + a.seg_ahead) * int64_t(GPT) * S;
-      if (sr < limit) seg_loop(limit);
-    }
-    if (qn >= ngrp) {
-      if (inl) seg_loop(-1);
-      break;
-    }
-    q = qn;
-    if (newblk) {
-      qend = q + GPT < ngrp ? q + GPT : ngrp;
+    if (last) {
+      if (inl) {
+        int64_t sr = INT64_MAX;
+        if (lane == 0 && speek < a.nseg) sr = a.seg_row[speek];
+        sr = __shfl_sync(0xffffffffu, sr, 0);
+        const int64_t limit = (int64_t(tn) + a.seg_ahead) * 32;
+        if (sr < limit) seg_loop(limit);
+      }
+      if (tn >= ntk) {
+        if (inl) seg_loop(-1);
+        break;
+      }
+      t = tn;
       tn = ticket();
+      bt ^= 1;
+      perm = permn;
+      kq = 0;
+    } else {
+      ++kq;
     }
-    rp = rpn;
-    sgv = sgn;
+    ri_idx = idxn;
     e0 = e0n;
     e1 = e1n;
+    sgv = sgn;
     n = nn;
   }
 }
@@ -842,10 +879,9 @@ cudaError_t launch_mrow(const AggArgs& a, cudaStream_t s) {
   // row ticket counter[0] and (inline segments) segment ticket counter[8]
   cudaError_t e = cudaMemsetAsync(a.counter, 0, (inl ? 9 : 1) * sizeof(int), s);
   if (e != cudaSuccess) return e;
-  constexpr int S = 32 / G;
   AggArgs b = a;
-  b.rows_per_ticket = knobs_mrow_gpt();  // groups of S rows per ticket
-  const int64_t ntk = ((a.rows + S - 1) / S + b.rows_per_ticket - 1) / b.rows_per_ticket;
+  b.mrow_sort = knobs_mrow_sort();
+  const int64_t ntk = (a.rows + 31) / 32;  // tickets of 32 rows
   const int64_t want = (ntk + 7) / 8;
   const unsigned grid = unsigned(want < slots ? want : slots);
   b.seg_inline = inl ? 1 : 0;
@@ -1048,14 +1084,14 @@ struct SparseKnobs {
   // plan's mean selective degree is <= MROW_MAX_DEG and its rows are degree-ordered;
   // 0 never; 1 wherever the layout fits
   int mrow = -1;
-  int mrow_gpt = 4;  // PCGCN_MROW_GPT: groups per ticket
+  int mrow_sort = 1;  // PCGCN_MROW_SORT: rows of a 32-row ticket grouped by degree
   int seg_inline = 0;  // measured (B200, fixed θ, interleaved): C3 F=41 passes +5%, C5 neutral -> off
   int seg_ahead = 4;  // quarters of (grid warps) row tickets
   SparseKnobs() {
     if (const char* e = getenv("PCGCN_SEG_INLINE")) seg_inline = atoi(e);
     if (const char* e = getenv("PCGCN_SEG_AHEAD")) seg_ahead = std::max(1, atoi(e));
     if (const char* e = getenv("PCGCN_SPARSE_MROW")) mrow = atoi(e);
-    if (const char* e = getenv("PCGCN_MROW_GPT")) mrow_gpt = std::max(1, atoi(e));
+    if (const char* e = getenv("PCGCN_MROW_SORT")) mrow_sort = atoi(e);
     if (const char* e = getenv("PCGCN_SPARSE_FSPLIT")) fsplit = atoi(e) / 32 * 32;
     if (const char* e = getenv("PCGCN_SPARSE_V8")) v8 = atoi(e) != 0;
     if (const char* e = getenv("PCGCN_SPARSE_G6")) g6 = atoi(e) != 0;
@@ -1067,7 +1103,7 @@ static SparseKnobs& knobs() {
   static SparseKnobs k;
   return k;
 }
-int knobs_mrow_gpt() { return knobs().mrow_gpt; }
+int knobs_mrow_sort() { return knobs().mrow_sort; }
 int knobs_seg_inline() { return knobs().seg_inline; }
 
 int knobs_seg_ahead() { return knobs().seg_ahead; }
@@ -1106,10 +1142,12 @@ cudaError_t launch_sparse_pass(const AggArgs& a, cudaStream_t s) {
   // 32-byte vectors per row read the row's 192 bytes (6 sectors, as many as the
   // 44 floats of the 16-byte layout touch) with 5 rows per load instruction
   if (al32 && knobs().g6 && (a.F + 7) / 8 == 6) return launch_gv<6, 1, 2>(a, s);
-  // short rows (mean selective degree <= MROW_MAX_DEG) in degree-ordered plans
-  // (a group of S rows costs its longest row: in id order C5's F=32 pass went
-  // 19.6 -> 26.1 ms, in degree order 19.6 -> 16.3 ms): one row per edge slot
-  if (v8 && knobs().mrow != 0 && (knobs().mrow > 0 || (a.mean_deg <= MROW_MAX_DEG && a.rows_by_degree))) {
+  // short rows (mean selective degree <= MROW_MAX_DEG): one row per edge slot.
+  // A group of S rows costs its longest row, so the rows must come grouped by
+  // degree: degree-ordered plans, or the kernel's per-ticket grouping (in id
+  // order without it C5's F=32 pass went 19.6 -> 26.1 ms; degree order 16.3 ms)
+  if (v8 && knobs().mrow != 0 &&
+      (knobs().mrow > 0 || (a.mean_deg <= MROW_MAX_DEG && (a.rows_by_degree || knobs().mrow_sort)))) {
     const int nvec = (a.F + 7) / 8;
     if (nvec >= 3 && nvec <= 4) return a.peer_world > 0 ? launch_mrow<4, true>(a, s) : launch_mrow<4, false>(a, s);
     if (nvec >= 5 && nvec <= 8) return a.peer_world > 0 ? launch_mrow<8, true>(a, s) : launch_mrow<8, false>(a, s);

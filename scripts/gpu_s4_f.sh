@@ -10,3 +10,9 @@ timeout 1200 ncu --set full --clock-control none --import-source on -k regex:"tc
 PCGCN_TC_DYN_ORDER=size timeout 900 python bench.py --no-cpu-baseline --no-e2e --theta $TH --theta-c $TC > gpurun_out/s4f_c3_dynsize.json 2> /dev/null
 timeout 900 python bench.py --no-cpu-baseline --no-e2e --theta $TH --theta-c $TC > gpurun_out/s4f_c3_fixed.json 2> /dev/null
 PCGCN_TC_DYN_ORDER=size timeout 900 python bench.py --no-cpu-baseline --no-e2e --theta $TH --theta-c $TC > gpurun_out/s4f_c3_dynsize2.json 2> /dev/null
+timeout 900 python -m pytest tests/test_gpu_parity.py -m gpu -q -x -k "multirow or partial_warp or long_rows" > gpurun_out/s4f_pytest2.log 2>&1
+export PCGCN_GRAPH_CACHE=/tmp/pcgcn_graphs
+B5="python bench.py --workload pl32m --steps 5 --warmup 3 --no-cpu-baseline --no-e2e --theta 0.0583 --order id"
+timeout 1500 $B5 > gpurun_out/s4f_c5_mrowsort.json 2> gpurun_out/s4f_c5.err
+PCGCN_SPARSE_MROW=0 timeout 900 $B5 > gpurun_out/s4f_c5_nomrow.json 2> /dev/null
+timeout 900 $B5 > gpurun_out/s4f_c5_mrowsort2.json 2> /dev/null

@@ -618,11 +618,11 @@ np.savez(sys.argv[1], **out)
                                           ({"PCGCN_TC_DYN_ORDER": "size"}, True),
                                           ({"PCGCN_SPARSE_MROW": "0"}, False),
                                           ({"PCGCN_SPARSE_MROW": "1"}, False),
-                                          ({"PCGCN_MROW_GPT": "1"}, True),
+                                          ({"PCGCN_SPARSE_MROW": "1", "PCGCN_MROW_SORT": "0"}, False),
                                           ({"PCGCN_SEG_INLINE": "1"}, True),
                                           ({"PCGCN_SEG_INLINE": "1", "PCGCN_SEG_AHEAD": "64"}, True),
                                           ({"PCGCN_SEG_INLINE": "1", "PCGCN_SEG_AHEAD": "1"}, True)])
-def test_scheduling_knobs_do_not_change_results(tmp_path, knob, bitwise):
+def test_scheduling_knobs_do_not_change_results(tmp_path, knob, bitwise, base=None):
     """Row-block tickets, inline vs separate long-row segments (the same
     partials added in the same order), the full-mode/segment overlap, the in-kernel xtg B
     conversion and the window-blocked full-mode B layout change only scheduling (every output row is still reduced by
@@ -636,7 +636,7 @@ def test_scheduling_knobs_do_not_change_results(tmp_path, knob, bitwise):
     import sys
     root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
     res = {}
-    for tag, extra in (("default", {}), ("knob", knob)):
+    for tag, extra in (("default", base or {}), ("knob", {**(base or {}), **knob})):
         env = {k: v for k, v in os.environ.items() if not k.startswith("PCGCN_")}
         env.update(extra)
         f = str(tmp_path / f"{tag}.npz")
@@ -660,6 +660,15 @@ def test_scheduling_knobs_do_not_change_results(tmp_path, knob, bitwise):
         else:
             scale = max(float(np.max(np.abs(a))), 1e-30)
             assert float(np.max(np.abs(a.astype(np.float64) - b))) <= 2e-6 * scale, (knob, k)
+
+
+def test_multirow_degree_grouping_is_bitwise(tmp_path):
+    """Multi-row warps group a 32-row ticket's rows by degree (PCGCN_MROW_SORT):
+    which slot gathers a row changes, the row's own sequential sum does not —
+    outputs, masks, gradients and the loss are bitwise identical with and
+    without the grouping."""
+    test_scheduling_knobs_do_not_change_results(tmp_path, {"PCGCN_MROW_SORT": "0"}, True,
+                                                base={"PCGCN_SPARSE_MROW": "1"})
 
 
 @pytest.mark.parametrize("wname,theta,dense", [("cora", 0.01, "tf32x2"), ("pubmed", 0.0, "bf16x3"),
