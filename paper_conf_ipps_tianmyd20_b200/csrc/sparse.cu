@@ -1084,7 +1084,7 @@ struct SparseKnobs {
   // plan's mean selective degree is <= MROW_MAX_DEG and its rows are degree-ordered;
   // 0 never; 1 wherever the layout fits
   int mrow = -1;
-  int mrow_sort = 1;  // PCGCN_MROW_SORT: rows of a 32-row ticket grouped by degree
+  int mrow_sort = 0;  // PCGCN_MROW_SORT=1: rows of a 32-row ticket grouped by degree (id-ordered plans)
   int seg_inline = 0;  // measured (B200, fixed θ, interleaved): C3 F=41 passes +5%, C5 neutral -> off
   int seg_ahead = 4;  // quarters of (grid warps) row tickets
   SparseKnobs() {
@@ -1142,12 +1142,12 @@ cudaError_t launch_sparse_pass(const AggArgs& a, cudaStream_t s) {
   // 32-byte vectors per row read the row's 192 bytes (6 sectors, as many as the
   // 44 floats of the 16-byte layout touch) with 5 rows per load instruction
   if (al32 && knobs().g6 && (a.F + 7) / 8 == 6) return launch_gv<6, 1, 2>(a, s);
-  // short rows (mean selective degree <= MROW_MAX_DEG): one row per edge slot.
-  // A group of S rows costs its longest row, so the rows must come grouped by
-  // degree: degree-ordered plans, or the kernel's per-ticket grouping (in id
-  // order without it C5's F=32 pass went 19.6 -> 26.1 ms; degree order 16.3 ms)
+  // short rows (mean selective degree <= MROW_MAX_DEG) of degree-ordered plans:
+  // one row per edge slot (C5's F=32 pass: 19.6 -> 16.3 ms in degree order; in
+  // id order 26.1 ms, and 23.8 ms with the per-ticket degree grouping, against
+  // 20.0 ms for the warp-per-row pass — so id-ordered plans keep the latter)
   if (v8 && knobs().mrow != 0 &&
-      (knobs().mrow > 0 || (a.mean_deg <= MROW_MAX_DEG && (a.rows_by_degree || knobs().mrow_sort)))) {
+      (knobs().mrow > 0 || (a.mean_deg <= MROW_MAX_DEG && a.rows_by_degree))) {
     const int nvec = (a.F + 7) / 8;
     if (nvec >= 3 && nvec <= 4) return a.peer_world > 0 ? launch_mrow<4, true>(a, s) : launch_mrow<4, false>(a, s);
     if (nvec >= 5 && nvec <= 8) return a.peer_world > 0 ? launch_mrow<8, true>(a, s) : launch_mrow<8, false>(a, s);

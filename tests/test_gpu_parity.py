@@ -615,10 +615,10 @@ np.savez(sys.argv[1], **out)
                                           ({"PCGCN_SPARSE_FSPLIT": "32"}, False),
                                           ({"PCGCN_SPARSE_G6": "0"}, False),
                                           ({"PCGCN_TC_DYN": "0"}, True),
-                                          ({"PCGCN_TC_DYN_ORDER": "size"}, True),
+                                          ({"PCGCN_TC_DYN_ORDER": "plan"}, True),
                                           ({"PCGCN_SPARSE_MROW": "0"}, False),
                                           ({"PCGCN_SPARSE_MROW": "1"}, False),
-                                          ({"PCGCN_SPARSE_MROW": "1", "PCGCN_MROW_SORT": "0"}, False),
+                                          ({"PCGCN_SPARSE_MROW": "1", "PCGCN_MROW_SORT": "1"}, False),
                                           ({"PCGCN_SEG_INLINE": "1"}, True),
                                           ({"PCGCN_SEG_INLINE": "1", "PCGCN_SEG_AHEAD": "64"}, True),
                                           ({"PCGCN_SEG_INLINE": "1", "PCGCN_SEG_AHEAD": "1"}, True)])
@@ -667,7 +667,7 @@ def test_multirow_degree_grouping_is_bitwise(tmp_path):
     which slot gathers a row changes, the row's own sequential sum does not —
     outputs, masks, gradients and the loss are bitwise identical with and
     without the grouping."""
-    test_scheduling_knobs_do_not_change_results(tmp_path, {"PCGCN_MROW_SORT": "0"}, True,
+    test_scheduling_knobs_do_not_change_results(tmp_path, {"PCGCN_MROW_SORT": "1"}, True,
                                                 base={"PCGCN_SPARSE_MROW": "1"})
 
 
