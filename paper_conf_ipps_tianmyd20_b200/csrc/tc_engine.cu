@@ -188,6 +188,7 @@ __device__ __forceinline__ bool tile_next(const Work& w, TileIter& it, bool firs
   mbar_wait(&tq_full[slot], par);
   it.t = *reinterpret_cast<const volatile int64_t*>(&tq[slot]);
   if (bar_id > 0) asm volatile("bar.sync %0, 128;" ::"r"(bar_id) : "memory");
+  else __syncwarp();  // the MMA warp: every lane has read the slot before lane 0 releases it
   if (leader) mbar_arrive(&tq_empty[slot]);
   ++it.qi;
   return it.t >= 0;
@@ -334,13 +335,14 @@ __global__ void __launch_bounds__(NTHREADS, 1)
       }
     }
   } else if (warp == 1) {
-    if (lane == 0) {
-      // ---- MMA issuer ----
+    {
+      // ---- MMA issuer: the whole warp walks the schedule with warp-uniform
+      // operands, one elected lane issues each tcgen05.mma / commit ----
       const uint32_t idesc = (MODE == A_BITS && w.bf3) ? idesc_bf16(BM, npad) : idesc_tf32(BM, npad);
       int s = 0;
       uint32_t ph = 0, gc = 0;  // gc: accumulation-group counter (shared enumeration with the epilogue)
       TileIter it{0, 0};
-      for (bool f = true; tile_next(w, it, f, tq_full, tq_empty, tq, 0, true); f = false) {
+      for (bool f = true; tile_next(w, it, f, tq_full, tq_empty, tq, 0, lane == 0); f = false) {
         const int64_t t = it.t;
         int64_t kb, nch, m0, sp;
         tile_range<MODE>(w, t, kb, nch, m0, sp);
@@ -374,7 +376,7 @@ __global__ void __launch_bounds__(NTHREADS, 1)
                 for (int kk = 0; kk < 2; ++kk) {
                   if (part >= w.bf3) break;
                   const uint64_t bd = sdesc_kmajor_sw64(b0 + uint32_t(part) * uint32_t(npad) * 64u + kk * 32u);
-                  mma_ts_f16(d, a0 + kk * 8u, bd, idesc, acc);
+                  mma_ts_f16_w(d, a0 + kk * 8u, bd, idesc, acc);
                   acc = 1u;
                 }
               continue;
@@ -386,16 +388,16 @@ __global__ void __launch_bounds__(NTHREADS, 1)
             for (int kk = 0; kk < BK / 8; ++kk) {
               const uint64_t bh = sdesc_kmajor_sw128(bh0 + kk * 32u);
               const uint64_t bl = sdesc_kmajor_sw128(bl0 + kk * 32u);
-              mma_ts(d, a0 + kk * 8u, bh, idesc, acc);
-              if (!w.single) mma_ts(d, a0 + kk * 8u, bl, idesc, 1u);
-              if (MODE != A_BITS) mma_ts(d, a0 + BK + kk * 8u, bh, idesc, 1u);
+              mma_ts_w(d, a0 + kk * 8u, bh, idesc, acc);
+              if (!w.single) mma_ts_w(d, a0 + kk * 8u, bl, idesc, 1u);
+              if (MODE != A_BITS) mma_ts_w(d, a0 + BK + kk * 8u, bh, idesc, 1u);
               acc = 1u;
             }
           }
-          tc_commit(&empty[s]);
+          tc_commit_w(&empty[s]);
           if (++s == L.stages) { s = 0; ph ^= 1u; }
         }
-        tc_commit(&acc_full[ab]);
+        tc_commit_w(&acc_full[ab]);
         }
       }
     }
