@@ -21,7 +21,7 @@
 //             B = Gᵀ split hi/lo; split-K over rows into fixed slices.
 //
 // Roles (320 threads): warp 0 lane 0 = TMA producer, warp 1 = TMEM allocator
-// + single-thread MMA issuer, warps 2..5 = A builders (thread m owns tile row
+// + MMA issuer (the whole warp walks the schedule, one elected lane issues), warps 2..5 = A builders (thread m owns tile row
 // m = TMEM lane m), warps 6..9 = epilogue (tcgen05.ld -> global), with a
 // double-buffered accumulator so a tile's epilogue overlaps the next tile's
 // MMAs.  Split precision: for any fp32 v, hi = v with the low 13 mantissa
@@ -59,10 +59,28 @@ struct Layout {
   int gst;                            // stages per TMEM accumulation group (<= 8 chunks)
   uint32_t a_bytes, b_bytes, stage_bytes, a_load_bytes;  // b_bytes: ONE chunk of ONE operand
   uint32_t tmem_cols, a_col0;
+  int accw;                           // TMEM columns of one accumulator: npad, or 3·npad when the three
+                                      // bf16 parts are stacked along N (one MMA per K-step, see below)
 };
+
+// PCGCN_TC_STACK=0 (A/B knob): bf16x3 full mode with three N=npad MMAs per
+// K-step instead of one N=3·npad MMA over the stacked parts
+bool tc_stack_enabled() {
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("PCGCN_TC_STACK");
+    v = e ? (atoi(e) != 0) : 1;
+  }
+  return v != 0;
+}
 
 Layout make_layout(int mode, int npad, int max_stages, int max_u, bool b_raw = false, int bfp = 0) {
   Layout L;
+  // bf16x3 with npad <= 64 (F <= 64; the NPC = 64 epilogue): the window block's three parts are
+  // contiguous K-major SW64 row blocks, i.e. one B operand of 3·npad rows; one
+  // MMA per K-step writes A·b0 | A·b1 | A·b2 side by side in TMEM and the
+  // epilogue adds the three column blocks (a third of the MMA issues)
+  L.accw = (mode == A_BITS && bfp == 3 && npad <= 64 && tc_stack_enabled()) ? 3 * npad : npad;
   L.raw_bytes = (mode == A_TRANS && b_raw) ? uint32_t(npad) * BK * 4 : 0u;
   L.npad = npad;
   L.b_bytes = uint32_t(npad) * BK * 4;
@@ -80,7 +98,7 @@ Layout make_layout(int mode, int npad, int max_stages, int max_u, bool b_raw = f
     int st = int((200 * 1024 - L.out_bytes) / L.stage_bytes);
     st = st > max_stages ? max_stages : st;
     L.nacc = 2;
-    while (st >= 2 && L.nacc * npad + st * L.a_cols > 512) {
+    while (st >= 2 && L.nacc * L.accw + st * L.a_cols > 512) {
       if (st > 2) --st;
       else if (L.nacc == 2) L.nacc = 1;
       else st = 0;
@@ -89,11 +107,11 @@ Layout make_layout(int mode, int npad, int max_stages, int max_u, bool b_raw = f
     if (st >= 2 || U == 1) break;
   }
   if (L.stages < 2) L.stages = 2;
-  const uint32_t need = uint32_t(L.nacc * npad + L.stages * L.a_cols);
+  const uint32_t need = uint32_t(L.nacc * L.accw + L.stages * L.a_cols);
   uint32_t cols = 32;
   while (cols < need) cols <<= 1;
   L.tmem_cols = cols;
-  L.a_col0 = uint32_t(L.nacc * npad);
+  L.a_col0 = uint32_t(L.nacc * L.accw);
   static int group_chunks = -1;  // chunks per TMEM accumulation chain (PCGCN_TC_GROUP: tuning override)
   if (group_chunks < 0) {
     const char* e = getenv("PCGCN_TC_GROUP");
@@ -338,7 +356,8 @@ __global__ void __launch_bounds__(NTHREADS, 1)
     {
       // ---- MMA issuer: the whole warp walks the schedule with warp-uniform
       // operands, one elected lane issues each tcgen05.mma / commit ----
-      const uint32_t idesc = (MODE == A_BITS && w.bf3) ? idesc_bf16(BM, npad) : idesc_tf32(BM, npad);
+      const bool stacked = L.accw != npad;
+      const uint32_t idesc = (MODE == A_BITS && w.bf3) ? idesc_bf16(BM, L.accw) : idesc_tf32(BM, npad);
       int s = 0;
       uint32_t ph = 0, gc = 0;  // gc: accumulation-group counter (shared enumeration with the epilogue)
       TileIter it{0, 0};
@@ -354,7 +373,7 @@ __global__ void __launch_bounds__(NTHREADS, 1)
         const uint32_t aph = L.nacc == 2 ? ((gc >> 1) & 1u) : (gc & 1u);
         mbar_wait(&acc_empty[ab], aph ^ 1u);
         tc_fence_after();
-        const uint32_t d = tmem + ab * uint32_t(npad);
+        const uint32_t d = tmem + ab * uint32_t(L.accw);
         uint32_t acc = 0;
         const int64_t ge = (g0 + L.gst < nst ? g0 + L.gst : nst) * L.U;
         for (int64_t i = g0 * L.U; i < (ge < nch ? ge : nch); i += L.U) {
@@ -370,6 +389,14 @@ __global__ void __launch_bounds__(NTHREADS, 1)
               // window (3, or 1 for BF16X1): 2 K=16 MMAs per part, fp32 accumulation in TMEM
               const uint32_t b0 = sb + uint32_t(u) * L.bchunk;
               const uint32_t a0 = sa + uint32_t(u) * (BK / 2);
+              if (stacked) {  // one N = 3·npad MMA per K-step over the stacked parts
+#pragma unroll
+                for (int kk = 0; kk < 2; ++kk) {
+                  mma_ts_f16_w(d, a0 + kk * 8u, sdesc_kmajor_sw64(b0 + kk * 32u), idesc, acc);
+                  acc = 1u;
+                }
+                continue;
+              }
 #pragma unroll
               for (int part = 0; part < 3; ++part)
 #pragma unroll
@@ -525,7 +552,8 @@ __global__ void __launch_bounds__(NTHREADS, 1)
         const uint32_t ab = L.nacc == 2 ? (gc & 1u) : 0u;
         mbar_wait(&acc_full[ab], L.nacc == 2 ? ((gc >> 1) & 1u) : (gc & 1u));
         tc_fence_after();
-        const uint32_t src = tmem + lane_base + ab * uint32_t(npad);
+        const uint32_t src = tmem + lane_base + ab * uint32_t(L.accw);
+        const bool stacked = L.accw != npad;  // add the three part blocks (A·b0 + A·b1) + A·b2
 #pragma unroll
         for (int c0 = 0; c0 < (NPC > 0 ? NPC : 256); c0 += 16) {
           if (c0 < npad) {
@@ -538,6 +566,22 @@ __global__ void __launch_bounds__(NTHREADS, 1)
                   "=r"(r[15])
                 : "r"(src + uint32_t(c0)));
             asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+            if constexpr (MODE == A_BITS && NPC > 0 && NPC <= 64) if (stacked) {
+#pragma unroll
+              for (int part = 1; part < 3; ++part) {
+                uint32_t r2[16];
+                asm volatile(
+                    "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, "
+                    "[%16];"
+                    : "=r"(r2[0]), "=r"(r2[1]), "=r"(r2[2]), "=r"(r2[3]), "=r"(r2[4]), "=r"(r2[5]), "=r"(r2[6]),
+                      "=r"(r2[7]), "=r"(r2[8]), "=r"(r2[9]), "=r"(r2[10]), "=r"(r2[11]), "=r"(r2[12]), "=r"(r2[13]),
+                      "=r"(r2[14]), "=r"(r2[15])
+                    : "r"(src + uint32_t(part * npad + c0)));
+                asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+                for (int q = 0; q < 16; ++q) r[q] = __float_as_uint(__uint_as_float(r[q]) + __uint_as_float(r2[q]));
+              }
+            }
             if (NPC > 0) {
 #pragma unroll
               for (int q = 0; q < 16; ++q) racc[(c0 + q) % (NPC > 0 ? NPC : 1)] += __uint_as_float(r[q]);
