@@ -578,8 +578,10 @@ e = np.random.default_rng(7).integers(0, base, size=(3 * base, 2))
 edges += [tuple(x) for x in e.tolist() if x[0] != x[1]]
 g = G.from_edges(base, edges)
 rng = np.random.default_rng(11)
+import os
+dp = getattr(L, os.environ.get("PCGCN_TEST_DENSE", "DENSE_TF32X2"))
 for F, theta, ld in ((128, 0.02, 128), (41, 0.04, 44), (40, 0.04, 48), (32, 2.0, 32), (41, 0.03, 48)):
-    pl = L.Plan(g.n, g.rowptr, g.col, 8, theta)
+    pl = L.Plan(g.n, g.rowptr, g.col, 8, theta, dense_prec=dp)
     Y = torch.from_numpy(rng.standard_normal((g.n, ld)).astype(np.float32)).cuda()
     Y[:, F:] = 0
     Z = torch.zeros_like(Y)
@@ -669,6 +671,15 @@ def test_multirow_degree_grouping_is_bitwise(tmp_path):
     without the grouping."""
     test_scheduling_knobs_do_not_change_results(tmp_path, {"PCGCN_MROW_SORT": "1"}, True,
                                                 base={"PCGCN_SPARSE_MROW": "1"})
+
+
+def test_stacked_bf16x3_parts_match_three_mmas(tmp_path):
+    """bf16x3 full mode for F <= 64 stacks the three bf16 parts along N (one
+    MMA per K-step, the epilogue adds the three column blocks); PCGCN_TC_STACK=0
+    issues one MMA per part.  Same products, another fp32 association: within
+    2e-6 of the largest output, masks self-consistent."""
+    test_scheduling_knobs_do_not_change_results(tmp_path, {"PCGCN_TC_STACK": "0"}, False,
+                                                base={"PCGCN_TEST_DENSE": "DENSE_BF16X3"})
 
 
 @pytest.mark.parametrize("wname,theta,dense", [("cora", 0.01, "tf32x2"), ("pubmed", 0.0, "bf16x3"),
